@@ -1,0 +1,238 @@
+/*
+ * sknn.h -- C ABI of the B200-native Sweet KNN exact KNN join.
+ *
+ * Method: Chen, Ding, Shen, "Sweet KNN: An Efficient KNN on GPU through
+ * Reconciliation between Redundancy Removal and Regularity", ICDE 2017.
+ * Citations "P:L<n>" refer to line n of the paper transcript with
+ * the section / equation / algorithm / figure the line falls in.
+ *
+ * The operation (every entry point below computes or serves it):
+ *   KNN join ("KNN join problem"; Fig. 4 main procedure P:L271):
+ *   for every query point q in Q, the k points of the target set T closest
+ *   to q in Euclidean distance. Results are exact: the triangle-
+ *   inequality (TI) filters only skip targets that provably cannot be among
+ *   the k nearest. Ties are broken by the lowest
+ *   target index; every output row is sorted ascending by (distance, index)
+ *   (readings R2, R4). Squared distances are accumulated in fp32 in
+ *   the fixed dimension order c = 0..d-1; distances are IEEE sqrt of those.
+ *
+ * Memory conventions (all entry points):
+ *   - Point sets are row-major, contiguous, fp32: Q is [nq x d], T is [nt x d].
+ *   - Outputs: out_idx [nq x k] int32 original target row indices (plus
+ *     opt->index_base), out_dist [nq x k] fp32 Euclidean distances (or
+ *     squared distances when opt->out_squared != 0).
+ *   - Pointers may be DEVICE pointers (on the current CUDA device) or HOST
+ *     pointers (pageable or pinned). Host inputs are staged to the device and
+ *     host outputs copied back inside the call; in that case the call
+ *     synchronises `stream` before returning. With device pointers only, the
+ *     call is stream-ordered: it enqueues all work on `stream` and returns
+ *     without waiting (unless stats are requested); results are valid once
+ *     `stream` completes.
+ *   - The library never frees caller memory. Scratch is allocated with
+ *     cudaMallocAsync on `stream` and released (stream-ordered) before return.
+ *   - `stream` is a cudaStream_t (NULL = the legacy default stream).
+ *
+ * Errors: every function returns an sknn_status; no C++ exception crosses the
+ * ABI. On error the outputs are unspecified and sknn_last_error() (thread-
+ * local) holds a one-line description. Inputs must be finite (NaN/Inf are
+ * undefined behaviour).
+ */
+#ifndef SKNN_H_
+#define SKNN_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SKNN_VERSION_MAJOR 0
+#define SKNN_VERSION_MINOR 1
+
+/* cudaStream_t without pulling in the CUDA headers. */
+typedef struct CUstream_st* sknn_stream_t;
+
+typedef enum {
+    SKNN_OK = 0,
+    SKNN_ERR_INVALID_ARG = -1,    /* null pointer, nq < 0, nt <= 0, d <= 0, k <= 0, k > nt, nt >= 2^31, bad option */
+    SKNN_ERR_NOT_DEVICE_PTR = -2, /* pointer on another device / unrecognised memory */
+    SKNN_ERR_OOM = -3,            /* device or host allocation failed */
+    SKNN_ERR_CUDA = -4,           /* a CUDA runtime call or kernel launch failed */
+    SKNN_ERR_UNSUPPORTED = -5,    /* device is not sm_100, or k > SKNN_MAX_K */
+    SKNN_ERR_WRONG_DEVICE = -6    /* index used on a device other than the one that built it */
+} sknn_status;
+
+/* Largest k the register / warp top-k supports in this version (P:L529-535,
+ * Fig. 8 placement: on B200 k*4 <= th2 = 1020 B fits registers; the large-k
+ * partial filter of §IV-B1 is future work). */
+#define SKNN_MAX_K 32
+
+/* Execution-path override (sknn_options.force_path). */
+enum {
+    SKNN_PATH_AUTO = 0,   /* adaptive scheme (Fig. 8 re-derived for B200)                 */
+    SKNN_PATH_SPARSE = 1, /* TI filters + point-level scan only (Alg. 1 + Alg. 2)          */
+    SKNN_PATH_DENSE = 2,  /* TI filters; every surviving cluster pair on the dense tile path */
+    SKNN_PATH_BRUTE = 3   /* no filtering: every query against every target (the anchor)    */
+};
+
+/* Level-2 thread mapping override (sknn_options.mapping), §IV-B2 / §IV-D3. */
+enum {
+    SKNN_MAP_AUTO = 0,
+    SKNN_MAP_THREAD = 1,  /* one thread per query ("query level parallelism")       */
+    SKNN_MAP_WARP = 2     /* one warp per query ("multi-level parallelism")         */
+};
+
+/* Tunables. Zero-initialise and set struct_size = sizeof(sknn_options), or
+ * call sknn_options_default(). A NULL options pointer means all defaults. */
+typedef struct {
+    size_t struct_size;       /* ABI versioning: sizeof(sknn_options) of the caller              */
+    int32_t n_clusters_q;     /* 0 = auto floor(3*sqrt(nq)), clamped to [1, min(nq, 16384)] */
+    int32_t n_clusters_t;     /* 0 = auto floor(3*sqrt(nt)), same clamp                           */
+    int32_t landmark_trials;  /* 0 = 10 trials of the landmark sampler                   */
+    int32_t lloyd_iters;      /* -1 = default 2 (north_star "a few Lloyd iterations", reading R9); 0 = paper sampler only */
+    uint64_t seed;            /* landmark sampler seed (results never depend on it)               */
+    int32_t force_path;       /* SKNN_PATH_*                                                       */
+    int32_t mapping;          /* SKNN_MAP_*                                                        */
+    float dense_threshold;    /* elastic switch threshold (0 = auto)                               */
+    float r_factor;           /* cache-conflict factor r (0 = 0.25)                        */
+    int32_t out_squared;      /* 1: out_dist holds squared distances (for partial-list exchange)  */
+    int32_t pad0;
+    int64_t index_base;       /* added to every output index (target-sharded global indices)      */
+    int32_t shard_rank;       /* query sharding: only query clusters c with c % shard_count ==    */
+    int32_t shard_count;      /*   shard_rank are processed (0/1 = all); other output rows untouched */
+} sknn_options;
+
+/* Counters and per-stage times of one call (filled only when a non-NULL
+ * pointer is passed; the call then synchronises `stream` before returning). */
+typedef struct {
+    size_t struct_size;
+    uint64_t pairs_total;          /* nq * nt                                                         */
+    uint64_t dist_evals_sparse;    /* point distances evaluated by the level-2 scan ("count") */
+    uint64_t dist_evals_dense;     /* query-target pairs covered by dense tiles                       */
+    uint64_t dist_evals_brute;     /* pairs evaluated by the brute-force path                         */
+    uint64_t center_evals;         /* query-to-candidate-center distances in level-2 (Alg. 2 line 6)  */
+    uint64_t cand_pairs;           /* surviving (query cluster, target cluster) pairs after level-1  */
+    uint64_t dense_pairs;          /* of which processed as dense tiles                               */
+    float ms_total;                /* CUDA-event time of the whole call on `stream`                   */
+    float ms_build_t, ms_build_q, ms_level1, ms_sparse, ms_dense, ms_final;
+    int32_t mapping_used;          /* SKNN_MAP_THREAD or SKNN_MAP_WARP                               */
+    int32_t path_used;             /* SKNN_PATH_*                                                     */
+    int32_t mq, mt;                /* cluster counts used                                             */
+    int32_t kernel_launches;       /* kernels this call launched                                      */
+    int32_t pad0;
+} sknn_stats;
+
+/* Opaque resident target index (sknn_build / sknn_query). Owns device memory:
+ * the target points permuted into cluster order, padded to a multiple of 4
+ * floats, their distances to the cluster centers (descending within each
+ * cluster), original indices, cluster offsets, centers and radii. */
+typedef struct sknn_index sknn_index;
+
+/* Adaptive-scheme decisions (Fig. 8, §IV-D) for a problem on a device. */
+typedef struct {
+    int32_t num_sms, max_threads_per_sm, smem_per_sm, max_regs_per_thread;
+} sknn_device_props;
+
+typedef struct {
+    int32_t th1_bytes;        /* smem/SM / max threads/SM                   */
+    int32_t th2_bytes;        /* max regs/thread * 4                        */
+    int32_t placement;        /* 0 shared, 1 registers, 2 global (Fig. 8)            */
+    int32_t partial_filter;   /* 1 iff k/d > 8 (reading R13)                 */
+    int64_t r_max_cur;        /* r * max_cur total threads                  */
+    double tpq_raw;           /* r*max_cur/|Q| or 1                     */
+    int32_t threads_per_query;/* nearest power of two in log2 (reading R15), uncapped */
+    int32_t mapping;          /* SKNN_MAP_THREAD / SKNN_MAP_WARP chosen for B200      */
+    int32_t mq, mt;           /* cluster counts floor(3*sqrt(n)) clamped              */
+} sknn_config;
+
+/* ---------------------------------------------------------------- API --- */
+
+/* Fill *opt with defaults (struct_size set). */
+void sknn_options_default(sknn_options* opt);
+
+/* KNN join of Q against T (Fig. 4 main procedure): clusters both
+ * sets (Step 1; Q == T with nq == nt is a self-join and is
+ * clustered once, as in the paper's experiments P:L697), filters cluster
+ * pairs (Step 2, Alg. 1), filters and evaluates points
+ * (Step 3, Alg. 2), and writes the k nearest of every query.
+ * out_idx may be NULL ("w/ or w/o index information"). nq == 0 is a
+ * no-op returning SKNN_OK. */
+sknn_status sknn_join(const float* Q, int64_t nq, const float* T, int64_t nt,
+                      int32_t d, int32_t k, int32_t* out_idx, float* out_dist,
+                      sknn_stream_t stream);
+
+/* sknn_join with options (NULL = defaults) and optional stats (NULL = none). */
+sknn_status sknn_join_ex(const float* Q, int64_t nq, const float* T, int64_t nt,
+                         int32_t d, int32_t k, int32_t* out_idx, float* out_dist,
+                         const sknn_options* opt, sknn_stats* stats,
+                         sknn_stream_t stream);
+
+/* Build a resident target index (Step 1 for T). T may be device
+ * or host memory; the index keeps its own copy. The index records the value
+ * of the T pointer: a later sknn_query with Q == that pointer and nq == nt is
+ * treated as a self-join (the caller must not have changed the contents). */
+sknn_status sknn_build(const float* T, int64_t nt, int32_t d,
+                       const sknn_options* opt, sknn_index** out,
+                       sknn_stream_t stream);
+
+/* Query a resident index: Step 1 for Q, then Steps 2-3 (Fig. 4 lines 3-6).
+ * The index is read-only: concurrent queries on different streams are safe.
+ * Must run on the device that built the index (else SKNN_ERR_WRONG_DEVICE). */
+sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq,
+                       int32_t k, int32_t* out_idx, float* out_dist,
+                       const sknn_options* opt, sknn_stats* stats,
+                       sknn_stream_t stream);
+
+/* Merge P partial result lists into one (multi-GPU target-sharded mode;
+ * the paper's merge of per-thread sorted heaps, generalised to
+ * ranks). part_idx [P x nq x k] int32 global indices, part_d2 [P x nq x k]
+ * fp32 SQUARED distances, each row sorted ascending by (d2, idx) (as written
+ * by sknn_query with out_squared = 1). Output: the k smallest (d2, idx) keys
+ * of each query over all P lists; out_dist gets sqrt(d2) unless
+ * out_squared != 0. Device pointers only. */
+sknn_status sknn_merge_partials(const int32_t* part_idx, const float* part_d2,
+                                int32_t P, int64_t nq, int32_t k,
+                                int32_t* out_idx, float* out_dist,
+                                int32_t out_squared, sknn_stream_t stream);
+
+/* Free an index (after all queries using it completed). NULL is a no-op. */
+sknn_status sknn_index_free(sknn_index* index);
+
+/* Index geometry: points, dimension, padded dimension, clusters, device. */
+sknn_status sknn_index_info(const sknn_index* index, int64_t* nt, int32_t* d,
+                            int32_t* dp, int32_t* mt, int32_t* device);
+
+/* Copy index metadata to HOST buffers (any may be NULL; synchronous):
+ * off [mt+1] cluster offsets into the permuted order, orig [nt] original row
+ * of each permuted point, dist [nt] distance to its center (descending within
+ * a cluster, ties by index ascending, P:L241 / reading R11), centers
+ * [mt x dp], radius [mt] (max member distance, 0 for an empty cluster). */
+sknn_status sknn_index_export(const sknn_index* index, int32_t* off, int32_t* orig,
+                              float* dist, float* centers, float* radius);
+
+/* Level-1 products of a query against an index, to HOST buffers (testing):
+ * q_cluster [nq] cluster of each query, ub [mq] the inflated upper bound of
+ * each query cluster (calUB), cand_count [mq] surviving target
+ * clusters (groupFilter, Alg. 1), cand [mq x mt] candidate target clusters
+ * in ascending center distance (first cand_count[i] of row i valid). Any
+ * output may be NULL. mq_out receives the query cluster count. */
+sknn_status sknn_debug_level1(const sknn_index* index, const float* Q, int64_t nq,
+                              int32_t k, const sknn_options* opt, int32_t* mq_out,
+                              int32_t* q_cluster, float* ub, int32_t* cand_count,
+                              int32_t* cand, int64_t cand_capacity);
+
+/* Adaptive-scheme decisions (Fig. 8, §IV-D) -- pure host arithmetic.
+ * props == NULL queries the current device. */
+sknn_status sknn_config_decide(int64_t nq, int64_t nt, int32_t d, int32_t k,
+                               const sknn_device_props* props, float r_factor,
+                               sknn_config* out);
+
+const char* sknn_error_string(sknn_status status);
+const char* sknn_last_error(void);   /* thread-local message of the last failure */
+int32_t sknn_version(void);          /* (major << 16) | minor */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SKNN_H_ */

@@ -1,0 +1,615 @@
+// api.cu -- the C ABI (include/sknn.h): argument validation, the adaptive
+// configuration (Fig. 8, §IV-D re-derived for B200), host/device staging,
+// and the stage sequence of the Fig. 4 main procedure:
+//   detLmNum -> init (build both sides) -> calUB + groupFilter -> pointFilter.
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <mutex>
+#include <string>
+
+#include "../../include/sknn.h"
+#include "sknn_internal.cuh"
+#include "sknn_launch.h"
+
+namespace sknn {
+
+static thread_local std::string g_last_error;
+void set_last_error(const std::string& msg) { g_last_error = msg; }
+
+static sknn_status fail(sknn_status st, const std::string& msg) {
+    set_last_error(msg);
+    return st;
+}
+
+// detLmNum: floor(3*sqrt(n)), clamped (reading R10)
+static int det_lm_num(int64_t n, int32_t requested) {
+    int64_t m = requested > 0 ? requested : (int64_t)floor(3.0 * sqrt((double)n));
+    m = std::max<int64_t>(1, std::min<int64_t>(m, std::min<int64_t>(n, kMaxClusters)));
+    return (int)m;
+}
+
+// R7: eta = (d + 8) * 2^-24
+static float rounding_eta(int d) { return (float)((d + 8) * ldexp(1.0, -24)); }
+
+struct DevInfo {
+    int device = -1, num_sms = 0, max_threads_per_sm = 0, smem_per_sm = 0, regs_per_thread = 255, major = 0, minor = 0;
+};
+
+static sknn_status device_info(DevInfo& di) {
+    int dev = 0;
+    SKNN_CUDA(cudaGetDevice(&dev));
+    static std::mutex mu;
+    static DevInfo cache[64];
+    std::lock_guard<std::mutex> lk(mu);
+    if (dev >= 0 && dev < 64 && cache[dev].device == dev) {
+        di = cache[dev];
+        return SKNN_OK;
+    }
+    cudaDeviceProp p;
+    SKNN_CUDA(cudaGetDeviceProperties(&p, dev));
+    di.device = dev;
+    di.num_sms = p.multiProcessorCount;
+    di.max_threads_per_sm = p.maxThreadsPerMultiProcessor;
+    di.smem_per_sm = (int)p.sharedMemPerMultiprocessor;
+    di.major = p.major;
+    di.minor = p.minor;
+    if (di.major != 10 || di.minor != 0)
+        return fail(SKNN_ERR_UNSUPPORTED, "device " + std::to_string(dev) + " is sm_" + std::to_string(p.major) +
+                                              std::to_string(p.minor) + "; this library is built for sm_100a (B200)");
+    // keep freed scratch in the pool between calls
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    if (dev >= 0 && dev < 64) cache[dev] = di;
+    return SKNN_OK;
+}
+
+static sknn_options merge_options(const sknn_options* o) {
+    sknn_options d;
+    sknn_options_default(&d);
+    if (!o) return d;
+    size_t n = std::min(o->struct_size ? o->struct_size : sizeof(sknn_options), sizeof(sknn_options));
+    memcpy(&d, o, n);
+    d.struct_size = sizeof(sknn_options);
+    if (d.landmark_trials <= 0) d.landmark_trials = 10;
+    if (d.lloyd_iters < 0) d.lloyd_iters = 2;
+    if (d.r_factor <= 0.f) d.r_factor = 0.25f;
+    if (d.shard_count <= 1) { d.shard_count = 1; d.shard_rank = 0; }
+    return d;
+}
+
+enum PtrKind { PTR_DEVICE, PTR_HOST, PTR_BAD };
+
+static PtrKind classify(const void* p, int dev) {
+    cudaPointerAttributes at;
+    cudaError_t e = cudaPointerGetAttributes(&at, p);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return PTR_HOST;
+    }
+    if (at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged)
+        return at.device == dev ? PTR_DEVICE : PTR_BAD;
+    return PTR_HOST;
+}
+
+// Stage an input array on the device (copy when it is host memory).
+static sknn_status stage_in(Ctx& cx, const void* p, size_t bytes, const void** out, bool* was_host) {
+    PtrKind k = classify(p, cx.device);
+    if (k == PTR_BAD) return fail(SKNN_ERR_NOT_DEVICE_PTR, "input pointer lives on another device");
+    *was_host = (k == PTR_HOST);
+    if (k == PTR_DEVICE) {
+        *out = p;
+        return SKNN_OK;
+    }
+    void* d;
+    SKNN_TRY(cx.alloc_scratch(&d, bytes));
+    SKNN_CUDA(cudaMemcpyAsync(d, p, bytes, cudaMemcpyHostToDevice, cx.stream));
+    *out = d;
+    return SKNN_OK;
+}
+
+static sknn_status stage_out(Ctx& cx, void* p, size_t bytes, void** dev, bool* was_host) {
+    if (!p) {
+        *dev = nullptr;
+        *was_host = false;
+        return SKNN_OK;
+    }
+    PtrKind k = classify(p, cx.device);
+    if (k == PTR_BAD) return fail(SKNN_ERR_NOT_DEVICE_PTR, "output pointer lives on another device");
+    *was_host = (k == PTR_HOST);
+    if (k == PTR_DEVICE) {
+        *dev = p;
+        return SKNN_OK;
+    }
+    SKNN_TRY(cx.alloc_scratch(dev, bytes));
+    return SKNN_OK;
+}
+
+struct Timer {
+    bool on = false;
+    cudaEvent_t ev[8] = {};
+    int n = 0;
+    cudaStream_t s = nullptr;
+    void start(cudaStream_t st, bool enable) {
+        on = enable;
+        s = st;
+        if (!on) return;
+        for (int i = 0; i < 8; ++i) cudaEventCreate(&ev[i]);
+        mark();
+    }
+    int mark() {
+        if (!on) return -1;
+        cudaEventRecord(ev[n], s);
+        return n++;
+    }
+    float ms(int a, int b) const {
+        if (!on || a < 0 || b < 0) return 0.f;
+        float t = 0.f;
+        cudaEventElapsedTime(&t, ev[a], ev[b]);
+        return t;
+    }
+    ~Timer() {
+        if (on)
+            for (int i = 0; i < 8; ++i) cudaEventDestroy(ev[i]);
+    }
+};
+
+static int choose_mapping(const sknn_options& o, const DevInfo& di, int64_t nq, int dp) {
+    if (o.mapping == SKNN_MAP_THREAD || o.mapping == SKNN_MAP_WARP) return o.mapping;
+    // Fig. 8 bottom: |Q| >= r*max_cur -> query-level
+    // parallelism (thread per query); otherwise several threads per query.
+    double rmax = (double)o.r_factor * di.num_sms * di.max_threads_per_sm;
+    return ((double)nq >= rmax && dp <= 32) ? SKNN_MAP_THREAD : SKNN_MAP_WARP;
+}
+
+static sknn_status validate(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
+                            const float* out_dist) {
+    if (!Q || !T || !out_dist) return fail(SKNN_ERR_INVALID_ARG, "Q, T and out_dist must be non-NULL");
+    if (nq < 0) return fail(SKNN_ERR_INVALID_ARG, "nq < 0");
+    if (nt <= 0) return fail(SKNN_ERR_INVALID_ARG, "nt <= 0");
+    if (nt >= (int64_t(1) << 31) || nq >= (int64_t(1) << 31)) return fail(SKNN_ERR_INVALID_ARG, "nq, nt must be < 2^31");
+    if (d <= 0) return fail(SKNN_ERR_INVALID_ARG, "d <= 0");
+    if (k <= 0) return fail(SKNN_ERR_INVALID_ARG, "k <= 0");
+    if ((int64_t)k > nt) return fail(SKNN_ERR_INVALID_ARG, "k > nt");
+    if (k > SKNN_MAX_K) return fail(SKNN_ERR_UNSUPPORTED, "k > SKNN_MAX_K (large-k partial filter not built yet)");
+    return SKNN_OK;
+}
+
+// The query half of Fig. 4 (lines 3-6) given both clustered sides.
+static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, const sknn_options& o, int mapping,
+                              int32_t* out_idx, float* out_dist, Counters* counters, Timer& tm, int* mk_l1,
+                              int* mk_scan) {
+    const float eta = rounding_eta(ts.d);
+    Level1 l1;
+    const int srank = o.shard_count > 1 ? o.shard_rank : 0, scount = o.shard_count > 1 ? o.shard_count : 1;
+    SKNN_TRY(run_level1(cx, qs, ts, k, eta, srank, scount, l1, &counters->cand_pairs));
+    SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp), srank, scount, l1));
+    *mk_l1 = tm.mark();
+    ScanParams sp;
+    sp.k = k;
+    sp.eta = eta;
+    sp.mapping = mapping;
+    sp.out_squared = o.out_squared;
+    sp.index_base = o.index_base;
+    sp.out_idx = out_idx;
+    sp.out_dist = out_dist;
+    sp.counters = counters;
+    SKNN_TRY(run_scan(cx, qs, ts, l1, sp));
+    *mk_scan = tm.mark();
+    return SKNN_OK;
+}
+
+static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt, const Timer& tm, int m_bt, int m_bq,
+                       int m_l1, int m_scan, int m_end, int mapping, int path, int mq, int mt, int launches) {
+    size_t sz = st->struct_size ? std::min(st->struct_size, sizeof(sknn_stats)) : sizeof(sknn_stats);
+    sknn_stats s;
+    memset(&s, 0, sizeof(s));
+    s.struct_size = sizeof(sknn_stats);
+    s.pairs_total = (uint64_t)nq * (uint64_t)nt;
+    s.dist_evals_sparse = c.evals_sparse;
+    s.dist_evals_dense = c.evals_dense;
+    s.dist_evals_brute = c.evals_brute;
+    s.center_evals = c.center_evals;
+    s.cand_pairs = c.cand_pairs;
+    s.dense_pairs = c.dense_pairs;
+    s.ms_total = tm.ms(0, m_end);
+    s.ms_build_t = tm.ms(0, m_bt);
+    s.ms_build_q = m_bq >= 0 ? tm.ms(m_bt, m_bq) : 0.f;
+    int prev = m_bq >= 0 ? m_bq : m_bt;
+    s.ms_level1 = m_l1 >= 0 ? tm.ms(prev, m_l1) : 0.f;
+    s.ms_sparse = m_scan >= 0 ? tm.ms(m_l1, m_scan) : 0.f;
+    s.ms_final = 0.f;
+    s.mapping_used = mapping;
+    s.path_used = path;
+    s.mq = mq;
+    s.mt = mt;
+    s.kernel_launches = launches;
+    memcpy(st, &s, sz);
+}
+
+// Shared body of sknn_join_ex / sknn_query.
+static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
+                            int32_t* out_idx, float* out_dist, const sknn_options* opt_in, sknn_stats* stats,
+                            cudaStream_t stream, const sknn_index* index) {
+    SKNN_TRY(validate(Q, nq, T ? T : Q, nt, d, k, out_dist));
+    if (nq == 0) {
+        if (stats) {
+            memset(stats, 0, sizeof(sknn_stats));
+            stats->struct_size = sizeof(sknn_stats);
+        }
+        return SKNN_OK;
+    }
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    if (index && index->device != di.device) return fail(SKNN_ERR_WRONG_DEVICE, "index built on another device");
+    sknn_options o = merge_options(opt_in ? opt_in : (index ? &index->opt : nullptr));
+    if (opt_in && index) {  // clustering of the index side is fixed; query-side knobs come from opt_in
+        o.n_clusters_t = index->t.m;
+    }
+    Ctx cx;
+    cx.stream = stream;
+    cx.device = di.device;
+    cx.num_sms = di.num_sms;
+    Timer tm;
+    tm.start(stream, stats != nullptr);
+    sknn_status st = SKNN_OK;
+    const int dp = (d + 3) & ~3;
+    const bool self = index ? (Q == index->user_ptr && nq == index->t.n) : (Q == T && nq == nt);
+    int mapping = choose_mapping(o, di, nq, dp);
+    int path = o.force_path == SKNN_PATH_BRUTE ? SKNN_PATH_BRUTE : SKNN_PATH_SPARSE;
+    int m_bt = -1, m_bq = -1, m_l1 = -1, m_scan = -1, m_end = -1;
+    int mq = 0, mt = 0;
+    Counters host_c;
+    memset(&host_c, 0, sizeof(host_c));
+    bool q_host = false, t_host = false, oi_host = false, od_host = false;
+    const float* dQ = nullptr;
+    const float* dT = nullptr;
+    int32_t* d_oidx = nullptr;
+    float* d_odist = nullptr;
+    Counters* counters = nullptr;
+    do {
+        const void* tmp;
+        if ((st = stage_in(cx, Q, sizeof(float) * nq * d, &tmp, &q_host)) != SKNN_OK) break;
+        dQ = (const float*)tmp;
+        if (!index) {
+            if (self) {
+                dT = dQ;
+            } else {
+                if ((st = stage_in(cx, T, sizeof(float) * nt * d, &tmp, &t_host)) != SKNN_OK) break;
+                dT = (const float*)tmp;
+            }
+        }
+        void* vo;
+        if ((st = stage_out(cx, out_idx, sizeof(int32_t) * nq * k, &vo, &oi_host)) != SKNN_OK) break;
+        d_oidx = (int32_t*)vo;
+        if ((st = stage_out(cx, out_dist, sizeof(float) * nq * k, &vo, &od_host)) != SKNN_OK) break;
+        d_odist = (float*)vo;
+        if ((st = cx.alloc_scratch((void**)&counters, sizeof(Counters))) != SKNN_OK) break;
+        if (cudaMemsetAsync(counters, 0, sizeof(Counters), stream) != cudaSuccess) {
+            st = fail(SKNN_ERR_CUDA, "cudaMemsetAsync(counters) failed");
+            break;
+        }
+        if (path == SKNN_PATH_BRUTE) {
+            if (index) {
+                st = fail(SKNN_ERR_INVALID_ARG, "force_path = BRUTE is only available for sknn_join");
+                break;
+            }
+            ScanParams sp;
+            sp.k = k;
+            sp.out_squared = o.out_squared;
+            sp.index_base = o.index_base;
+            sp.out_idx = d_oidx;
+            sp.out_dist = d_odist;
+            sp.counters = counters;
+            mapping = SKNN_MAP_WARP;
+            st = run_brute(cx, dQ, nq, dT, nt, d, sp);
+            m_bt = tm.mark();
+            m_scan = m_bt;
+            break;
+        }
+        Side ts_local, qs_local;
+        const Side* ts;
+        if (index) {
+            ts = &index->t;
+        } else {
+            int m = det_lm_num(nt, o.n_clusters_t);
+            if ((st = build_side(cx, dT, nt, d, m, o.landmark_trials, o.lloyd_iters, o.seed, ts_local)) != SKNN_OK)
+                break;
+            ts = &ts_local;
+        }
+        m_bt = tm.mark();
+        const Side* qs;
+        if (self) {
+            qs = ts;
+        } else {
+            int m = det_lm_num(nq, o.n_clusters_q);
+            if ((st = build_side(cx, dQ, nq, d, m, o.landmark_trials, o.lloyd_iters, o.seed ^ 0x51ull, qs_local)) !=
+                SKNN_OK)
+                break;
+            qs = &qs_local;
+            m_bq = tm.mark();
+        }
+        mq = qs->m;
+        mt = ts->m;
+        st = query_core(cx, *qs, *ts, k, o, mapping, d_oidx, d_odist, counters, tm, &m_l1, &m_scan);
+    } while (0);
+    if (st == SKNN_OK) {
+        if (oi_host) {
+            cudaError_t e = cudaMemcpyAsync(out_idx, d_oidx, sizeof(int32_t) * nq * k, cudaMemcpyDeviceToHost, stream);
+            if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("D2H out_idx: ") + cudaGetErrorString(e));
+        }
+        if (od_host) {
+            cudaError_t e = cudaMemcpyAsync(out_dist, d_odist, sizeof(float) * nq * k, cudaMemcpyDeviceToHost, stream);
+            if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("D2H out_dist: ") + cudaGetErrorString(e));
+        }
+        if (stats && counters) cudaMemcpyAsync(&host_c, counters, sizeof(Counters), cudaMemcpyDeviceToHost, stream);
+        m_end = tm.mark();
+    }
+    int launches = cx.launches;
+    cx.free_all();
+    if (st == SKNN_OK && (stats || oi_host || od_host || q_host || t_host)) {
+        cudaError_t e = cudaStreamSynchronize(stream);
+        if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("kernel execution failed: ") + cudaGetErrorString(e));
+    }
+    if (st == SKNN_OK && stats)
+        fill_stats(stats, host_c, nq, nt, tm, m_bt, m_bq, m_l1, m_scan, m_end, mapping, path, mq, mt, launches);
+    return st;
+}
+
+}  // namespace sknn
+
+using namespace sknn;
+
+extern "C" {
+
+void sknn_options_default(sknn_options* o) {
+    if (!o) return;
+    memset(o, 0, sizeof(*o));
+    o->struct_size = sizeof(sknn_options);
+    o->landmark_trials = 10;
+    o->lloyd_iters = 2;
+    o->seed = 0x5eedull;
+    o->force_path = SKNN_PATH_AUTO;
+    o->mapping = SKNN_MAP_AUTO;
+    o->r_factor = 0.25f;
+}
+
+sknn_status sknn_join(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k, int32_t* out_idx,
+                      float* out_dist, sknn_stream_t stream) {
+    return run_join(Q, nq, T, nt, d, k, out_idx, out_dist, nullptr, nullptr, (cudaStream_t)stream, nullptr);
+}
+
+sknn_status sknn_join_ex(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
+                         int32_t* out_idx, float* out_dist, const sknn_options* opt, sknn_stats* stats,
+                         sknn_stream_t stream) {
+    return run_join(Q, nq, T, nt, d, k, out_idx, out_dist, opt, stats, (cudaStream_t)stream, nullptr);
+}
+
+sknn_status sknn_build(const float* T, int64_t nt, int32_t d, const sknn_options* opt, sknn_index** out,
+                       sknn_stream_t stream_) {
+    if (!out) return fail(SKNN_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    if (!T) return fail(SKNN_ERR_INVALID_ARG, "T is NULL");
+    if (nt <= 0 || nt >= (int64_t(1) << 31)) return fail(SKNN_ERR_INVALID_ARG, "nt must be in [1, 2^31)");
+    if (d <= 0) return fail(SKNN_ERR_INVALID_ARG, "d <= 0");
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    cudaStream_t stream = (cudaStream_t)stream_;
+    sknn_options o = merge_options(opt);
+    Ctx cx;
+    cx.stream = stream;
+    cx.device = di.device;
+    cx.num_sms = di.num_sms;
+    sknn_index* ix = new (std::nothrow) sknn_index();
+    if (!ix) return fail(SKNN_ERR_OOM, "host allocation of the index failed");
+    ix->device = di.device;
+    ix->user_ptr = T;
+    ix->opt = o;
+    sknn_status st;
+    do {
+        const void* dT;
+        bool th;
+        if ((st = stage_in(cx, T, sizeof(float) * nt * d, &dT, &th)) != SKNN_OK) break;
+        int m = det_lm_num(nt, o.n_clusters_t);
+        st = build_side(cx, (const float*)dT, nt, d, m, o.landmark_trials, o.lloyd_iters, o.seed, ix->t);
+    } while (0);
+    cx.free_scratch();
+    if (st == SKNN_OK) {
+        cudaError_t e = cudaStreamSynchronize(stream);  // the index is usable on any stream afterwards
+        if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("index build failed: ") + cudaGetErrorString(e));
+    }
+    if (st != SKNN_OK) {
+        cx.free_all();
+        delete ix;
+        return st;
+    }
+    *out = ix;
+    return SKNN_OK;
+}
+
+sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq, int32_t k, int32_t* out_idx,
+                       float* out_dist, const sknn_options* opt, sknn_stats* stats, sknn_stream_t stream) {
+    if (!index) return fail(SKNN_ERR_INVALID_ARG, "index is NULL");
+    return run_join(Q, nq, nullptr, index->t.n, index->t.d, k, out_idx, out_dist, opt, stats, (cudaStream_t)stream,
+                    index);
+}
+
+sknn_status sknn_merge_partials(const int32_t* part_idx, const float* part_d2, int32_t P, int64_t nq, int32_t k,
+                                int32_t* out_idx, float* out_dist, int32_t out_squared, sknn_stream_t stream) {
+    if (!part_idx || !part_d2 || !out_dist) return fail(SKNN_ERR_INVALID_ARG, "NULL pointer");
+    if (P <= 0 || nq < 0 || k <= 0) return fail(SKNN_ERR_INVALID_ARG, "P, k must be > 0 and nq >= 0");
+    if (k > SKNN_MAX_K) return fail(SKNN_ERR_UNSUPPORTED, "k > SKNN_MAX_K");
+    if (nq == 0) return SKNN_OK;
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    if (classify(part_idx, di.device) != PTR_DEVICE || classify(part_d2, di.device) != PTR_DEVICE ||
+        classify(out_dist, di.device) != PTR_DEVICE || (out_idx && classify(out_idx, di.device) != PTR_DEVICE))
+        return fail(SKNN_ERR_NOT_DEVICE_PTR, "sknn_merge_partials takes device pointers only");
+    Ctx cx;
+    cx.stream = (cudaStream_t)stream;
+    cx.device = di.device;
+    cx.num_sms = di.num_sms;
+    return run_merge(cx, part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared);
+}
+
+sknn_status sknn_index_free(sknn_index* ix) {
+    if (!ix) return SKNN_OK;
+    int cur = 0;
+    cudaGetDevice(&cur);
+    if (ix->device != cur) cudaSetDevice(ix->device);
+    void* ptrs[] = {ix->t.rows, ix->t.dist, ix->t.orig, ix->t.off, ix->t.centers, ix->t.radius};
+    for (void* p : ptrs)
+        if (p) cudaFree(p);
+    if (ix->device != cur) cudaSetDevice(cur);
+    delete ix;
+    return SKNN_OK;
+}
+
+sknn_status sknn_index_info(const sknn_index* ix, int64_t* nt, int32_t* d, int32_t* dp, int32_t* mt, int32_t* device) {
+    if (!ix) return fail(SKNN_ERR_INVALID_ARG, "index is NULL");
+    if (nt) *nt = ix->t.n;
+    if (d) *d = ix->t.d;
+    if (dp) *dp = ix->t.dp;
+    if (mt) *mt = ix->t.m;
+    if (device) *device = ix->device;
+    return SKNN_OK;
+}
+
+sknn_status sknn_index_export(const sknn_index* ix, int32_t* off, int32_t* orig, float* dist, float* centers,
+                              float* radius) {
+    if (!ix) return fail(SKNN_ERR_INVALID_ARG, "index is NULL");
+    const Side& t = ix->t;
+    if (off) SKNN_CUDA(cudaMemcpy(off, t.off, sizeof(int32_t) * (t.m + 1), cudaMemcpyDeviceToHost));
+    if (orig) SKNN_CUDA(cudaMemcpy(orig, t.orig, sizeof(int32_t) * t.n, cudaMemcpyDeviceToHost));
+    if (dist) SKNN_CUDA(cudaMemcpy(dist, t.dist, sizeof(float) * t.n, cudaMemcpyDeviceToHost));
+    if (centers) SKNN_CUDA(cudaMemcpy(centers, t.centers, sizeof(float) * t.m * t.dp, cudaMemcpyDeviceToHost));
+    if (radius) SKNN_CUDA(cudaMemcpy(radius, t.radius, sizeof(float) * t.m, cudaMemcpyDeviceToHost));
+    return SKNN_OK;
+}
+
+sknn_status sknn_debug_level1(const sknn_index* ix, const float* Q, int64_t nq, int32_t k, const sknn_options* opt,
+                              int32_t* mq_out, int32_t* q_cluster, float* ub, int32_t* cand_count, int32_t* cand,
+                              int64_t cand_capacity) {
+    if (!ix || !Q) return fail(SKNN_ERR_INVALID_ARG, "NULL pointer");
+    if (nq <= 0 || k <= 0 || k > ix->t.n || k > SKNN_MAX_K) return fail(SKNN_ERR_INVALID_ARG, "bad nq or k");
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    sknn_options o = merge_options(opt ? opt : &ix->opt);
+    Ctx cx;
+    cx.stream = nullptr;
+    cx.device = di.device;
+    cx.num_sms = di.num_sms;
+    sknn_status st = SKNN_OK;
+    const Side& ts = ix->t;
+    const bool self = (Q == ix->user_ptr && nq == ts.n);
+    Side qs_local;
+    const Side* qs = &ts;
+    Level1 l1;
+    do {
+        const void* dQ;
+        bool qh;
+        if ((st = stage_in(cx, Q, sizeof(float) * nq * ts.d, &dQ, &qh)) != SKNN_OK) break;
+        if (!self) {
+            int m = det_lm_num(nq, o.n_clusters_q);
+            if ((st = build_side(cx, (const float*)dQ, nq, ts.d, m, o.landmark_trials, o.lloyd_iters, o.seed ^ 0x51ull,
+                                 qs_local)) != SKNN_OK)
+                break;
+            qs = &qs_local;
+        }
+        if ((st = run_level1(cx, *qs, ts, k, rounding_eta(ts.d), 0, 1, l1, nullptr)) != SKNN_OK) break;
+        cudaError_t e = cudaStreamSynchronize(nullptr);
+        if (e != cudaSuccess) {
+            st = fail(SKNN_ERR_CUDA, std::string("level-1 failed: ") + cudaGetErrorString(e));
+            break;
+        }
+        const int mq = qs->m;
+        if (mq_out) *mq_out = mq;
+        if (ub) cudaMemcpy(ub, l1.ub, sizeof(float) * mq, cudaMemcpyDeviceToHost);
+        if (cand_count) cudaMemcpy(cand_count, l1.cand_count, sizeof(int32_t) * mq, cudaMemcpyDeviceToHost);
+        if (cand) {
+            if (cand_capacity < (int64_t)mq * ts.m) {
+                st = fail(SKNN_ERR_INVALID_ARG, "cand_capacity < mq * mt");
+                break;
+            }
+            cudaMemcpy(cand, l1.cand, sizeof(int32_t) * (size_t)mq * ts.m, cudaMemcpyDeviceToHost);
+        }
+        if (q_cluster) {
+            std::string err;
+            int32_t* hoff = new int32_t[mq + 1];
+            int32_t* horig = new int32_t[nq];
+            cudaMemcpy(hoff, qs->off, sizeof(int32_t) * (mq + 1), cudaMemcpyDeviceToHost);
+            cudaMemcpy(horig, qs->orig, sizeof(int32_t) * nq, cudaMemcpyDeviceToHost);
+            for (int c = 0; c < mq; ++c)
+                for (int p = hoff[c]; p < hoff[c + 1]; ++p) q_cluster[horig[p]] = c;
+            delete[] hoff;
+            delete[] horig;
+        }
+    } while (0);
+    cx.free_all();
+    cudaStreamSynchronize(nullptr);
+    return st;
+}
+
+sknn_status sknn_config_decide(int64_t nq, int64_t nt, int32_t d, int32_t k, const sknn_device_props* props,
+                               float r_factor, sknn_config* out) {
+    if (!out || nq < 0 || nt <= 0 || d <= 0 || k <= 0) return fail(SKNN_ERR_INVALID_ARG, "bad arguments");
+    sknn_device_props p;
+    if (props) {
+        p = *props;
+    } else {
+        int dev = 0;
+        cudaDeviceProp cp;
+        if (cudaGetDevice(&dev) != cudaSuccess || cudaGetDeviceProperties(&cp, dev) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(SKNN_ERR_CUDA, "no CUDA device to query; pass props");
+        }
+        p.num_sms = cp.multiProcessorCount;
+        p.max_threads_per_sm = cp.maxThreadsPerMultiProcessor;
+        p.smem_per_sm = (int)cp.sharedMemPerMultiprocessor;
+        p.max_regs_per_thread = 255;
+    }
+    if (r_factor <= 0.f) r_factor = 0.25f;
+    memset(out, 0, sizeof(*out));
+    out->th1_bytes = p.smem_per_sm / p.max_threads_per_sm;
+    out->th2_bytes = p.max_regs_per_thread * 4;
+    int bytes = k * 4;                                        // Fig. 8: k*4 <= th1 -> shared, > th2 -> global
+    out->placement = bytes <= out->th1_bytes ? 0 : (bytes > out->th2_bytes ? 2 : 1);
+    out->partial_filter = (k > 8 * d) ? 1 : 0;               // P:L615, reading R13
+    double maxcur = (double)p.num_sms * p.max_threads_per_sm;
+    double rmax = (double)r_factor * maxcur;
+    out->r_max_cur = (int64_t)rmax;
+    out->tpq_raw = ((double)nq >= rmax || nq == 0) ? 1.0 : rmax / (double)nq;
+    int tpq = 1;
+    if (out->tpq_raw > 1.0) tpq = 1 << (int)lround(log2(out->tpq_raw));       // reading R15
+    out->threads_per_query = tpq;
+    const int dp = (d + 3) & ~3;
+    out->mapping = ((double)nq >= rmax && dp <= 32) ? SKNN_MAP_THREAD : SKNN_MAP_WARP;
+    out->mq = det_lm_num(std::max<int64_t>(nq, 1), 0);
+    out->mt = det_lm_num(nt, 0);
+    return SKNN_OK;
+}
+
+const char* sknn_error_string(sknn_status s) {
+    switch (s) {
+        case SKNN_OK: return "SKNN_OK";
+        case SKNN_ERR_INVALID_ARG: return "SKNN_ERR_INVALID_ARG";
+        case SKNN_ERR_NOT_DEVICE_PTR: return "SKNN_ERR_NOT_DEVICE_PTR";
+        case SKNN_ERR_OOM: return "SKNN_ERR_OOM";
+        case SKNN_ERR_CUDA: return "SKNN_ERR_CUDA";
+        case SKNN_ERR_UNSUPPORTED: return "SKNN_ERR_UNSUPPORTED";
+        case SKNN_ERR_WRONG_DEVICE: return "SKNN_ERR_WRONG_DEVICE";
+    }
+    return "SKNN_ERR_UNKNOWN";
+}
+
+const char* sknn_last_error(void) { return g_last_error.c_str(); }
+
+int32_t sknn_version(void) { return (SKNN_VERSION_MAJOR << 16) | SKNN_VERSION_MINOR; }
+
+}  // extern "C"

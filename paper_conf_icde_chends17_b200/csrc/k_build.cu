@@ -1,0 +1,483 @@
+// k_build.cu -- Step 1 of the method: landmark/cluster construction
+// (§II-C Step 1; §III-A), re-designed for B200.
+//
+//   k_pad_rows         X [n x d] -> Xp [n x dp] zero padded (16-byte rows for float4 loads, Fig. 7b / P:L559)
+//   k_landmark_draw    10 trials x m distinct random candidate landmarks; a keyed Feistel
+//                      permutation of [0, n) gives distinct indices without a set
+//   k_landmark_sums    S = sum of pairwise distances of each trial's candidates
+//   k_landmark_pick    argmax_trial S (first trial on ties) and gather of the winning centers
+//   k_assign<DP>       nearest center of every point, ties -> lowest center;
+//                      optional Lloyd accumulation (north_star "a few Lloyd iterations", R9),
+//                      cluster histogram, and the exact fp32 distance to the chosen center
+//   k_lloyd_update     center = mean of members (empty cluster keeps its center)
+//   k_offsets          exclusive scan of cluster counts -> CSR offsets (replaces the paper's CPU
+//                      allocation between two kernels: no host round trip)
+//   k_scatter_keys     one sort key per point at its cluster slot
+//   k_segsort_small/big  members of every cluster sorted by distance descending, index ascending
+//                      ("sorts those points in descending order", reading R11)
+//   k_gather_side      permuted padded rows, member distances, original indices
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "sknn_internal.cuh"
+#include "sknn_launch.h"
+
+namespace sknn {
+
+typedef unsigned long long u64;
+
+__global__ void k_pad_rows(const float* __restrict__ X, int64_t n, int d, int dp, float* __restrict__ Xp) {
+    int64_t total = n * (int64_t)dp;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        int64_t r = e / dp;
+        int c = int(e - r * dp);
+        Xp[e] = (c < d) ? X[r * d + c] : 0.f;
+    }
+}
+
+// ---------------------------------------------------- landmark sampler --
+__device__ __forceinline__ uint32_t mix32(uint64_t x) {
+    x ^= x >> 30; x *= 0xbf58476d1ce4e5b9ull;
+    x ^= x >> 27; x *= 0x94d049bb133111ebull;
+    x ^= x >> 31;
+    return uint32_t(x >> 16);
+}
+
+// bijection on [0, n): 4-round Feistel network on 2*half bits + cycle walking
+__device__ uint32_t perm_index(uint32_t i, uint32_t n, uint64_t key) {
+    int bits = 2;
+    while ((1ull << bits) < n) ++bits;
+    if (bits & 1) ++bits;
+    int half = bits / 2;
+    uint32_t mask = (1u << half) - 1u;
+    uint32_t v = i;
+    do {
+        uint32_t L = v >> half, R = v & mask;
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            uint32_t F = mix32(key * 0x9e3779b97f4a7c15ull + (uint64_t(r) << 40) + R) & mask;
+            uint32_t nl = R;
+            R = L ^ F;
+            L = nl;
+        }
+        v = (L << half) | R;
+    } while (v >= n);
+    return v;
+}
+
+__global__ void k_landmark_draw(int64_t n, int m, int trials, uint64_t seed, int32_t* __restrict__ idx) {
+    int t = blockIdx.y;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < m; i += gridDim.x * blockDim.x)
+        idx[t * m + i] = (int32_t)perm_index((uint32_t)i, (uint32_t)n, seed * 1315423911ull + t + 1);
+}
+
+// partial[t * nblk + b] = sum over pairs (i<j) with i in block b of d(c_i, c_j)
+__global__ void k_landmark_sums(const float* __restrict__ Xp, int dp, int m, const int32_t* __restrict__ idx,
+                                double* __restrict__ partial) {
+    int t = blockIdx.y;
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    double s = 0.0;
+    if (i < m) {
+        const float* a = Xp + (int64_t)idx[t * m + i] * dp;
+        for (int j = i + 1; j < m; ++j) {
+            const float* b = Xp + (int64_t)idx[t * m + j] * dp;
+            s += (double)__fsqrt_rn(d2_rows(a, b, dp));
+        }
+    }
+    // fixed-order block reduction (deterministic)
+    __shared__ double red[256];
+    red[threadIdx.x] = s;
+    __syncthreads();
+    for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+        if (threadIdx.x < w) red[threadIdx.x] += red[threadIdx.x + w];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) partial[t * gridDim.x + blockIdx.x] = red[0];
+}
+
+__global__ void k_landmark_pick(const double* __restrict__ partial, int nblk, int trials, const int32_t* __restrict__ idx,
+                                int m, const float* __restrict__ Xp, int dp, float* __restrict__ centers) {
+    __shared__ int best;
+    if (threadIdx.x == 0) {
+        double bs = -1.0;
+        int bt = 0;
+        for (int t = 0; t < trials; ++t) {
+            double s = 0.0;
+            for (int b = 0; b < nblk; ++b) s += partial[t * nblk + b];
+            if (s > bs) { bs = s; bt = t; }  // first maximum
+        }
+        best = bt;
+    }
+    __syncthreads();
+    const int32_t* w = idx + best * m;
+    for (int e = threadIdx.x; e < m * dp; e += blockDim.x) {
+        int c = e / dp, col = e - c * dp;
+        centers[e] = Xp[(int64_t)w[c] * dp + col];
+    }
+}
+
+// -------------------------------------------------------------- assign --
+// Each thread owns one point; centers stream through shared memory. DP > 0:
+// the point lives in registers (compile-time padded dimension). DP == 0:
+// runtime dp, the point is re-read from L1 while 4 centers are scored at once.
+template <int DP>
+__global__ void __launch_bounds__(256) k_assign(const float* __restrict__ Xp, int64_t n, int dp_rt,
+                                                const float* __restrict__ centers, int m, int chunk,
+                                                int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
+                                                float* __restrict__ sums, int32_t* __restrict__ counts) {
+    extern __shared__ __align__(16) float s_c[];
+    const int dp = DP > 0 ? DP : dp_rt;
+    int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    bool active = i < n;
+    float best = __int_as_float(0x7f800000);
+    int bi = 0;
+    float4 q[DP > 0 ? DP / 4 : 1];
+    if constexpr (DP > 0) {
+        if (active) {
+#pragma unroll
+            for (int c = 0; c < DP / 4; ++c) q[c] = reinterpret_cast<const float4*>(Xp + i * DP)[c];
+        }
+    }
+    const float* xrow = Xp + (active ? i : 0) * dp;
+    for (int c0 = 0; c0 < m; c0 += chunk) {
+        int cn = min(chunk, m - c0);
+        __syncthreads();
+        for (int e = threadIdx.x; e < cn * dp / 4; e += blockDim.x)
+            reinterpret_cast<float4*>(s_c)[e] = reinterpret_cast<const float4*>(centers + (int64_t)c0 * dp)[e];
+        __syncthreads();
+        if (!active) continue;
+        if constexpr (DP > 0) {
+            for (int c = 0; c < cn; ++c) {
+                const float4* cc = reinterpret_cast<const float4*>(s_c + c * DP);
+                float s = 0.f;
+#pragma unroll
+                for (int j = 0; j < DP / 4; ++j) s = d2_acc4(s, q[j], cc[j]);
+                if (s < best) { best = s; bi = c0 + c; }
+            }
+        } else {
+            const float4* x4 = reinterpret_cast<const float4*>(xrow);
+            int c = 0;
+            for (; c + 4 <= cn; c += 4) {
+                float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+                const float4* c4 = reinterpret_cast<const float4*>(s_c + c * dp);
+                const int w = dp / 4;
+                for (int j = 0; j < w; ++j) {
+                    float4 xv = x4[j];
+                    s0 = d2_acc4(s0, xv, c4[j]);
+                    s1 = d2_acc4(s1, xv, c4[w + j]);
+                    s2 = d2_acc4(s2, xv, c4[2 * w + j]);
+                    s3 = d2_acc4(s3, xv, c4[3 * w + j]);
+                }
+                if (s0 < best) { best = s0; bi = c0 + c; }
+                if (s1 < best) { best = s1; bi = c0 + c + 1; }
+                if (s2 < best) { best = s2; bi = c0 + c + 2; }
+                if (s3 < best) { best = s3; bi = c0 + c + 3; }
+            }
+            for (; c < cn; ++c) {
+                const float4* c4 = reinterpret_cast<const float4*>(s_c + c * dp);
+                float s = 0.f;
+                for (int j = 0; j < dp / 4; ++j) s = d2_acc4(s, x4[j], c4[j]);
+                if (s < best) { best = s; bi = c0 + c; }
+            }
+        }
+    }
+    if (!active) return;
+    if (cid_out) cid_out[i] = bi;
+    if (dist_out) dist_out[i] = __fsqrt_rn(best);
+    if (counts) atomicAdd(counts + bi, 1);
+    if (sums) {
+        for (int c = 0; c < dp; ++c) atomicAdd(sums + (int64_t)bi * dp + c, xrow[c]);
+    }
+}
+
+__global__ void k_lloyd_update(float* __restrict__ centers, const float* __restrict__ sums,
+                               const int32_t* __restrict__ counts, int m, int dp) {
+    for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < m * dp; e += gridDim.x * blockDim.x) {
+        int c = e / dp;
+        int cnt = counts[c];
+        if (cnt > 0) centers[e] = sums[e] / (float)cnt;
+    }
+}
+
+// --------------------------------------------------------------- CSR -----
+// Single-CTA exclusive scan of cluster counts -> off[0..m]; zeroes cursor.
+__global__ void __launch_bounds__(1024) k_offsets(const int32_t* __restrict__ counts, int m, int32_t* __restrict__ off,
+                                                  int32_t* __restrict__ cursor) {
+    __shared__ int32_t s_sum[1024];
+    __shared__ int32_t s_carry;
+    if (threadIdx.x == 0) s_carry = 0;
+    __syncthreads();
+    for (int base = 0; base < m; base += 1024) {
+        int i = base + threadIdx.x;
+        int v = (i < m) ? counts[i] : 0;
+        s_sum[threadIdx.x] = v;
+        __syncthreads();
+        for (int w = 1; w < 1024; w <<= 1) {  // Hillis-Steele inclusive scan
+            int t = (threadIdx.x >= w) ? s_sum[threadIdx.x - w] : 0;
+            __syncthreads();
+            s_sum[threadIdx.x] += t;
+            __syncthreads();
+        }
+        if (i < m) {
+            off[i] = s_carry + s_sum[threadIdx.x] - v;
+            cursor[i] = 0;
+        }
+        __syncthreads();
+        if (threadIdx.x == 1023) s_carry += s_sum[1023];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) off[m] = s_carry;
+}
+
+// key: (~dist_bits) << 32 | index -> ascending key = descending distance, ascending index
+__global__ void k_scatter_keys(const int32_t* __restrict__ cid, const float* __restrict__ dist, int64_t n,
+                               const int32_t* __restrict__ off, int32_t* __restrict__ cursor, u64* __restrict__ keys) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        int c = cid[i];
+        int pos = off[c] + atomicAdd(cursor + c, 1);
+        keys[pos] = (u64(~__float_as_uint(dist[i])) << 32) | u64(uint32_t(i));
+    }
+}
+
+__device__ __forceinline__ float key_member_dist(u64 key) { return __uint_as_float(~uint32_t(key >> 32)); }
+
+// Ascending bitonic network in the "flip + half-cleaner" form: every
+// compare-exchange puts the minimum at the lower index, so virtual +inf
+// padding past the segment end never moves (no padding writes needed).
+__device__ __forceinline__ void cmpx(u64* s, int i, int p) {
+    u64 a = s[i], b = s[p];
+    if (b < a) { s[i] = b; s[p] = a; }
+}
+
+constexpr int kSmallSeg = 4096;
+
+__global__ void __launch_bounds__(512) k_segsort_small(u64* __restrict__ keys, const int32_t* __restrict__ off,
+                                                       float* __restrict__ radius) {
+    __shared__ u64 s[kSmallSeg];
+    int c = blockIdx.x;
+    int lo = off[c], size = off[c + 1] - lo;
+    if (size > kSmallSeg) return;
+    if (size <= 1) {
+        if (threadIdx.x == 0) radius[c] = size ? key_member_dist(keys[lo]) : 0.f;
+        return;
+    }
+    int S = 2;
+    while (S < size) S <<= 1;
+    for (int i = threadIdx.x; i < S; i += blockDim.x) s[i] = (i < size) ? keys[lo + i] : ~0ull;
+    __syncthreads();
+    for (int k = 2; k <= S; k <<= 1) {
+        for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {  // flip
+            int blk = t / (k / 2), r = t % (k / 2);
+            int i = blk * k + r, p = blk * k + k - 1 - r;
+            cmpx(s, i, p);
+        }
+        __syncthreads();
+        for (int j = k / 4; j > 0; j >>= 1) {  // half-cleaners
+            for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
+                int i = (t / j) * 2 * j + (t % j);
+                cmpx(s, i, i + j);
+            }
+            __syncthreads();
+        }
+    }
+    for (int i = threadIdx.x; i < size; i += blockDim.x) keys[lo + i] = s[i];
+    if (threadIdx.x == 0) radius[c] = key_member_dist(s[0]);
+}
+
+// Clusters larger than kSmallSeg: one CTA per cluster; stages whose partner
+// distance is < kSmallSeg run in shared memory chunk by chunk, the others
+// directly on global memory (virtual +inf padding beyond the segment).
+__global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, const int32_t* __restrict__ off,
+                                                      float* __restrict__ radius) {
+    __shared__ u64 s[kSmallSeg];
+    int c = blockIdx.x;
+    int lo = off[c], size = off[c + 1] - lo;
+    if (size <= kSmallSeg) return;
+    u64* g = keys + lo;
+    int S = 2;
+    while (S < size) S <<= 1;
+    auto gx = [&](int i, int p) {
+        if (p >= size) return;
+        u64 a = g[i], b = g[p];
+        if (b < a) { g[i] = b; g[p] = a; }
+    };
+    // phase A: fully sort every aligned chunk of kSmallSeg in smem
+    for (int base = 0; base < size; base += kSmallSeg) {
+        for (int i = threadIdx.x; i < kSmallSeg; i += blockDim.x) s[i] = (base + i < size) ? g[base + i] : ~0ull;
+        __syncthreads();
+        for (int k = 2; k <= kSmallSeg; k <<= 1) {
+            for (int t = threadIdx.x; t < kSmallSeg / 2; t += blockDim.x) {
+                int blk = t / (k / 2), r = t % (k / 2);
+                cmpx(s, blk * k + r, blk * k + k - 1 - r);
+            }
+            __syncthreads();
+            for (int j = k / 4; j > 0; j >>= 1) {
+                for (int t = threadIdx.x; t < kSmallSeg / 2; t += blockDim.x) {
+                    int i = (t / j) * 2 * j + (t % j);
+                    cmpx(s, i, i + j);
+                }
+                __syncthreads();
+            }
+        }
+        for (int i = threadIdx.x; i < kSmallSeg && base + i < size; i += blockDim.x) g[base + i] = s[i];
+        __syncthreads();
+    }
+    // phase B: merges of size > kSmallSeg
+    for (int k = 2 * kSmallSeg; k <= S; k <<= 1) {
+        for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
+            int blk = t / (k / 2), r = t % (k / 2);
+            int i = blk * k + r, p = blk * k + k - 1 - r;
+            if (i < size) gx(i, p);
+        }
+        __syncthreads();
+        int j = k / 4;
+        for (; j >= kSmallSeg; j >>= 1) {
+            for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
+                int i = (t / j) * 2 * j + (t % j);
+                if (i < size) gx(i, i + j);
+            }
+            __syncthreads();
+        }
+        // remaining half-cleaners (j < kSmallSeg) stay inside aligned chunks
+        for (int base = 0; base < size; base += kSmallSeg) {
+            for (int i = threadIdx.x; i < kSmallSeg; i += blockDim.x) s[i] = (base + i < size) ? g[base + i] : ~0ull;
+            __syncthreads();
+            for (int jj = kSmallSeg / 2; jj > 0; jj >>= 1) {
+                for (int t = threadIdx.x; t < kSmallSeg / 2; t += blockDim.x) {
+                    int i = (t / jj) * 2 * jj + (t % jj);
+                    cmpx(s, i, i + jj);
+                }
+                __syncthreads();
+            }
+            for (int i = threadIdx.x; i < kSmallSeg && base + i < size; i += blockDim.x) g[base + i] = s[i];
+            __syncthreads();
+        }
+    }
+    if (threadIdx.x == 0) radius[c] = key_member_dist(g[0]);
+}
+
+// rows_out[p] = Xp[idx(p)], dist_out[p], orig_out[p]; one thread per float4
+__global__ void k_gather_side(const u64* __restrict__ keys, const float* __restrict__ Xp, int64_t n, int dp,
+                              float* __restrict__ rows_out, float* __restrict__ dist_out, int32_t* __restrict__ orig_out) {
+    const int w = dp / 4;
+    int64_t total = n * w;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        int64_t p = e / w;
+        int c = int(e - p * w);
+        u64 key = keys[p];
+        uint32_t idx = uint32_t(key & 0xffffffffu);
+        reinterpret_cast<float4*>(rows_out)[e] = reinterpret_cast<const float4*>(Xp)[(int64_t)idx * w + c];
+        if (c == 0) {
+            dist_out[p] = key_member_dist(key);
+            orig_out[p] = (int32_t)idx;
+        }
+    }
+}
+
+// ------------------------------------------------------------ launcher --
+static int assign_chunk(int dp, int m, size_t* smem) {
+    int chunk = int((48 * 1024) / (dp * sizeof(float)));
+    if (chunk > m) chunk = m;
+    if (chunk < 1) chunk = 1;
+    *smem = size_t(chunk) * dp * sizeof(float);
+    return chunk;
+}
+
+static void launch_assign(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m,
+                          int32_t* cid, float* dist, float* sums, int32_t* counts) {
+    size_t smem;
+    int chunk = assign_chunk(dp, m, &smem);
+    dim3 grid((unsigned)((n + 255) / 256));
+    switch (dp) {
+#define SKNN_ASSIGN_CASE(D) \
+    case D: k_assign<D><<<grid, 256, smem, cx.stream>>>(Xp, n, dp, centers, m, chunk, cid, dist, sums, counts); break;
+        SKNN_ASSIGN_CASE(4) SKNN_ASSIGN_CASE(8) SKNN_ASSIGN_CASE(12) SKNN_ASSIGN_CASE(16)
+        SKNN_ASSIGN_CASE(20) SKNN_ASSIGN_CASE(24) SKNN_ASSIGN_CASE(28) SKNN_ASSIGN_CASE(32)
+#undef SKNN_ASSIGN_CASE
+        default: k_assign<0><<<grid, 256, smem, cx.stream>>>(Xp, n, dp, centers, m, chunk, cid, dist, sums, counts); break;
+    }
+    cx.launched();
+}
+
+// Build one clustered side (Step 1). X is a device pointer [n x d].
+sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int trials, int lloyd, uint64_t seed,
+                       Side& out) {
+    const int dp = (d + 3) & ~3;
+    out.n = n; out.d = d; out.dp = dp; out.m = m;
+    cudaStream_t s = cx.stream;
+    // owned outputs
+    SKNN_TRY(cx.alloc_persistent((void**)&out.rows, sizeof(float) * n * dp));
+    SKNN_TRY(cx.alloc_persistent((void**)&out.dist, sizeof(float) * n));
+    SKNN_TRY(cx.alloc_persistent((void**)&out.orig, sizeof(int32_t) * n));
+    SKNN_TRY(cx.alloc_persistent((void**)&out.off, sizeof(int32_t) * (m + 1)));
+    SKNN_TRY(cx.alloc_persistent((void**)&out.centers, sizeof(float) * m * dp));
+    SKNN_TRY(cx.alloc_persistent((void**)&out.radius, sizeof(float) * m));
+    out.owned = true;
+
+    // padded copy of X (skipped when X already has 16-byte rows)
+    const float* Xp = X;
+    if (dp != d || (reinterpret_cast<uintptr_t>(X) & 15u)) {
+        float* tmp;
+        SKNN_TRY(cx.alloc_scratch((void**)&tmp, sizeof(float) * n * dp));
+        int64_t tot = n * dp;
+        int blocks = (int)std::min<int64_t>((tot + 255) / 256, 148 * 16);
+        k_pad_rows<<<blocks, 256, 0, s>>>(X, n, d, dp, tmp);
+        cx.launched();
+        Xp = tmp;
+    }
+    // landmark sampler
+    int32_t* lidx;
+    SKNN_TRY(cx.alloc_scratch((void**)&lidx, sizeof(int32_t) * trials * m));
+    k_landmark_draw<<<dim3((m + 255) / 256, trials), 256, 0, s>>>(n, m, trials, seed, lidx);
+    cx.launched();
+    int nblk = (m + 255) / 256;
+    double* partial;
+    SKNN_TRY(cx.alloc_scratch((void**)&partial, sizeof(double) * trials * nblk));
+    k_landmark_sums<<<dim3(nblk, trials), 256, 0, s>>>(Xp, dp, m, lidx, partial);
+    cx.launched();
+    k_landmark_pick<<<1, 512, 0, s>>>(partial, nblk, trials, lidx, m, Xp, dp, out.centers);
+    cx.launched();
+
+    int32_t* cid;
+    float* pdist;
+    int32_t* counts;
+    int32_t* cursor;
+    SKNN_TRY(cx.alloc_scratch((void**)&cid, sizeof(int32_t) * n));
+    SKNN_TRY(cx.alloc_scratch((void**)&pdist, sizeof(float) * n));
+    SKNN_TRY(cx.alloc_scratch((void**)&counts, sizeof(int32_t) * m));
+    SKNN_TRY(cx.alloc_scratch((void**)&cursor, sizeof(int32_t) * m));
+    // Lloyd iterations (R9)
+    if (lloyd > 0) {
+        float* sums;
+        SKNN_TRY(cx.alloc_scratch((void**)&sums, sizeof(float) * m * dp));
+        for (int it = 0; it < lloyd; ++it) {
+            SKNN_CUDA(cudaMemsetAsync(sums, 0, sizeof(float) * m * dp, s));
+            SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
+            launch_assign(cx, Xp, n, dp, out.centers, m, nullptr, nullptr, sums, counts);
+            int blocks = std::max(1, std::min((m * dp + 255) / 256, 148 * 8));
+            k_lloyd_update<<<blocks, 256, 0, s>>>(out.centers, sums, counts, m, dp);
+            cx.launched();
+        }
+    }
+    // final assignment with exact member distances + histogram
+    SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
+    launch_assign(cx, Xp, n, dp, out.centers, m, cid, pdist, nullptr, counts);
+    k_offsets<<<1, 1024, 0, s>>>(counts, m, out.off, cursor);
+    cx.launched();
+    unsigned long long* keys;
+    SKNN_TRY(cx.alloc_scratch((void**)&keys, sizeof(unsigned long long) * n));
+    int sblocks = (int)std::min<int64_t>((n + 255) / 256, 148 * 16);
+    k_scatter_keys<<<sblocks, 256, 0, s>>>(cid, pdist, n, out.off, cursor, keys);
+    cx.launched();
+    k_segsort_small<<<m, 512, 0, s>>>(keys, out.off, out.radius);
+    cx.launched();
+    k_segsort_big<<<m, 1024, 0, s>>>(keys, out.off, out.radius);
+    cx.launched();
+    int64_t tot = n * (dp / 4);
+    int gblocks = (int)std::min<int64_t>((tot + 255) / 256, 148 * 16);
+    k_gather_side<<<gblocks, 256, 0, s>>>(keys, Xp, n, dp, out.rows, out.dist, out.orig);
+    cx.launched();
+    return cx.check_launch("build_side");
+}
+
+}  // namespace sknn

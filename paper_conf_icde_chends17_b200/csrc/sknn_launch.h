@@ -1,0 +1,118 @@
+// sknn_launch.h -- host-side launch context: stream, scratch allocations,
+// launch counting and error plumbing of one ABI call. Not part of the ABI.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+#include <string>
+#include <vector>
+
+#include "../../include/sknn.h"
+#include "sknn_internal.cuh"
+
+namespace sknn {
+
+void set_last_error(const std::string& msg);
+
+#define SKNN_TRY(expr)                      \
+    do {                                    \
+        sknn_status _st = (expr);           \
+        if (_st != SKNN_OK) return _st;     \
+    } while (0)
+
+#define SKNN_CUDA(call)                                                                    \
+    do {                                                                                   \
+        cudaError_t _e = (call);                                                           \
+        if (_e != cudaSuccess) {                                                           \
+            ::sknn::set_last_error(std::string(#call) + ": " + cudaGetErrorString(_e));   \
+            return _e == cudaErrorMemoryAllocation ? SKNN_ERR_OOM : SKNN_ERR_CUDA;         \
+        }                                                                                  \
+    } while (0)
+
+struct Ctx {
+    cudaStream_t stream = nullptr;
+    int device = 0;
+    int num_sms = 148;
+    int launches = 0;
+    std::vector<void*> scratch;     // freed (stream-ordered) when the call ends
+    std::vector<void*> persistent;  // handed to an index, or freed with scratch
+
+    void launched() { ++launches; }
+
+    sknn_status alloc_scratch(void** p, size_t bytes) {
+        if (bytes == 0) bytes = 16;
+        cudaError_t e = cudaMallocAsync(p, bytes, stream);
+        if (e != cudaSuccess) {
+            set_last_error(std::string("cudaMallocAsync(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+            return SKNN_ERR_OOM;
+        }
+        scratch.push_back(*p);
+        return SKNN_OK;
+    }
+    sknn_status alloc_persistent(void** p, size_t bytes) {
+        if (bytes == 0) bytes = 16;
+        cudaError_t e = cudaMallocAsync(p, bytes, stream);
+        if (e != cudaSuccess) {
+            set_last_error(std::string("cudaMallocAsync(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+            return SKNN_ERR_OOM;
+        }
+        persistent.push_back(*p);
+        return SKNN_OK;
+    }
+    sknn_status check_launch(const char* what) {
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) {
+            set_last_error(std::string(what) + ": kernel launch failed: " + cudaGetErrorString(e));
+            return SKNN_ERR_CUDA;
+        }
+        return SKNN_OK;
+    }
+    void free_scratch() {
+        for (void* p : scratch) cudaFreeAsync(p, stream);
+        scratch.clear();
+    }
+    void free_all() {
+        free_scratch();
+        for (void* p : persistent) cudaFreeAsync(p, stream);
+        persistent.clear();
+    }
+};
+
+// k_build.cu
+sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int trials, int lloyd, uint64_t seed,
+                       Side& out);
+
+// k_level1.cu
+struct Level1 {
+    float* ub = nullptr;          // [mq] inflated calUB per query cluster
+    int32_t* cand = nullptr;      // [mq x mt] candidate target clusters, ascending center distance
+    int32_t* cand_count = nullptr;  // [mq]
+    int2* tiles = nullptr;        // level-2 work tiles (query cluster, first member)
+    int* ntiles = nullptr;
+    int tile = 0;
+};
+sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, int k, float eta, int shard_rank, int shard_count,
+                       Level1& out, unsigned long long* cand_pairs_counter);
+// k_scan.cu: tiles of `tile` queries of one query cluster (thread-data remapping)
+sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int shard_rank, int shard_count, Level1& l1);
+int scan_tile_size(int mapping, int dp);
+
+// k_scan.cu
+struct ScanParams {
+    int k = 0;
+    float eta = 0.f;
+    int mapping = SKNN_MAP_THREAD;
+    int out_squared = 0;
+    int64_t index_base = 0;
+    int32_t* out_idx = nullptr;
+    float* out_dist = nullptr;
+    Counters* counters = nullptr;
+};
+sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p);
+sknn_status run_brute(Ctx& cx, const float* Q, int64_t nq, const float* T, int64_t nt, int d, const ScanParams& p);
+sknn_status run_merge(Ctx& cx, const int32_t* part_idx, const float* part_d2, int P, int64_t nq, int k,
+                      int32_t* out_idx, float* out_dist, int out_squared);
+
+}  // namespace sknn

@@ -1,0 +1,236 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar (SURVEY.md §8(c) c.2 / north_star): integer-valued inputs bit-exact
+(indices and fp32 distances); real-valued inputs within 1e-5 relative with
+neighbour sets equal up to ties (sknn_testutil.assert_knn_tolerant).
+Inputs come from datagen (seeded); expected values only from oracle/.
+"""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+from sknn_testutil import assert_knn_bitexact, assert_knn_tolerant
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def sknn():
+    import paper_conf_icde_chends17_b200 as s
+    from paper_conf_icde_chends17_b200 import buildlib
+    buildlib.build()
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    return s
+
+
+def dev(x):
+    return torch.from_numpy(np.ascontiguousarray(x, dtype=np.float32)).cuda()
+
+
+def run(sknn, Q, T, k, self_join, **opts):
+    dQ = dev(Q)
+    dT = dQ if self_join else dev(T)
+    idx, dist, st = sknn.join(dQ, dT, k, stats=True, **opts)
+    torch.cuda.synchronize()
+    return idx.cpu().numpy(), dist.cpu().numpy(), st
+
+
+CASES_INT = [
+    ("C1", 1.0), ("C3int", 0.05), ("C4", 0.004), ("C5", 0.0025),
+]
+
+
+@pytest.mark.parametrize("path,mapping", [("auto", "auto"), ("sparse", "thread"), ("sparse", "warp"),
+                                          ("brute", "auto")])
+def test_c1_bitexact_all_paths(sknn, path, mapping):
+    Q, T, k, sj = datagen.workload("C1")
+    idx, dist, st = run(sknn, Q, T, k, sj, force_path=path, mapping=mapping)
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    if path != "brute":
+        assert 0 < st["pruned_pct"] < 100
+
+
+@pytest.mark.parametrize("name,scale", CASES_INT)
+@pytest.mark.parametrize("mapping", ["auto", "thread", "warp"])
+def test_integer_workloads_bitexact(sknn, name, scale, mapping):
+    Q, T, k, sj = datagen.workload(name, scale)
+    idx, dist, st = run(sknn, Q, T, k, sj, mapping=mapping)
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    assert st["dist_evals"] >= Q.shape[0] * k
+
+
+@pytest.mark.parametrize("name,scale", [("C2", 0.05), ("C3", 0.1)])
+@pytest.mark.parametrize("mapping", ["thread", "warp"])
+def test_real_workloads_tolerant(sknn, name, scale, mapping):
+    Q, T, k, sj = datagen.workload(name, scale)
+    idx, dist, st = run(sknn, Q, T, k, sj, mapping=mapping)
+    _, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_tolerant(Q, T, idx, dist, rdist)
+
+
+def test_sphere_ties(sknn):
+    """P10: equal-norm sphere + origin, queries at the origin and at sphere points."""
+    X = datagen.sphere_ties()
+    Q = np.concatenate([np.zeros((3, 4), np.float32), X[:40]], axis=0)
+    for k in (1, 5, 17, 32):
+        for path in ("auto", "brute"):
+            for mapping in ("thread", "warp"):
+                idx, dist, _ = run(sknn, Q, X, k, False, force_path=path, mapping=mapping)
+                ridx, rdist = oracle.knn_join(Q, X, k)
+                assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+@pytest.mark.parametrize("d", [1, 2, 3, 5, 7, 13, 33, 64])
+def test_odd_dimensions(sknn, d):
+    rng = np.random.default_rng(d)
+    T = rng.integers(0, 40, size=(3000, d)).astype(np.float32)
+    Q = rng.integers(0, 40, size=(700, d)).astype(np.float32)
+    for k in (1, 9, 32):
+        for mapping in ("thread", "warp"):
+            idx, dist, _ = run(sknn, Q, T, k, False, mapping=mapping)
+            ridx, rdist = oracle.knn_join(Q, T, k)
+            assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+@pytest.mark.parametrize("n,k", [(1, 1), (2, 2), (5, 5), (33, 32), (100, 32), (257, 3)])
+def test_tiny_and_k_equals_n(sknn, n, k):
+    rng = np.random.default_rng(n)
+    X = rng.integers(0, 5, size=(n, 3)).astype(np.float32)
+    for mapping in ("thread", "warp"):
+        idx, dist, _ = run(sknn, X, X, k, True, mapping=mapping)
+        ridx, rdist = oracle.knn_join(X, X, k)
+        assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+def test_all_duplicates(sknn):
+    """Degenerate: every point identical -> one cluster, all distances 0, lowest indices."""
+    X = np.full((2000, 4), 7.0, np.float32)
+    idx, dist, _ = run(sknn, X, X, 16, True)
+    assert np.all(dist == 0)
+    assert np.all(idx == np.arange(16)[None, :])
+
+
+def test_big_cluster_sort_path(sknn):
+    """A cluster larger than the 4096-key shared-memory sort (k_segsort_big)."""
+    rng = np.random.default_rng(5)
+    big = rng.integers(0, 3, size=(20000, 2)).astype(np.float32)   # dense blob
+    far = rng.integers(1000, 1100, size=(500, 2)).astype(np.float32)
+    X = np.concatenate([big, far])
+    idx, dist, _ = run(sknn, X, X, 8, True, n_clusters_t=4)
+    ridx, rdist = oracle.knn_join(X, X, 8)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+def test_host_pointers_match_device(sknn):
+    Q, T, k, sj = datagen.workload("C1")
+    hidx, hdist = sknn.join(Q, Q, k)     # numpy host buffers: staged inside the call
+    didx, ddist, _ = run(sknn, Q, T, k, sj)
+    np.testing.assert_array_equal(hidx, didx)
+    np.testing.assert_array_equal(hdist, ddist)
+
+
+def test_without_indices(sknn):
+    Q, T, k, sj = datagen.workload("C1")
+    dQ = dev(Q)
+    idx, dist = sknn.join(dQ, dQ, k, with_index=False)
+    assert idx is None
+    _, rdist = oracle.knn_join(Q, T, k)
+    np.testing.assert_array_equal(dist.cpu().numpy(), rdist)
+
+
+def test_seed_and_lloyd_do_not_change_results(sknn):
+    Q, T, k, sj = datagen.workload("C3int", 0.03)
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    for seed, lloyd, ncl in [(1, 0, 0), (2, 1, 0), (3, 4, 0), (4, 2, 7), (5, 2, 1)]:
+        idx, dist, _ = run(sknn, Q, T, k, sj, seed=seed, lloyd_iters=lloyd, n_clusters_t=ncl)
+        assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+def test_index_build_query_and_invariants(sknn):
+    """sknn_build / sknn_query, plus index invariants P6."""
+    T = datagen.c5_blobs(30000, which="T")
+    Q = datagen.c5_blobs(5000, which="Q")
+    k = 32
+    ix = sknn.build(dev(T))
+    e = ix.export()
+    off, orig, dist, cent, rad = e["off"], e["orig"], e["dist"], e["centers"], e["radius"]
+    m = len(rad)
+    assert off[0] == 0 and off[-1] == T.shape[0] and np.all(np.diff(off) >= 0)
+    assert np.array_equal(np.sort(orig), np.arange(T.shape[0]))   # every point exactly once
+    for c in range(m):
+        seg = dist[off[c]:off[c + 1]]
+        if len(seg) == 0:
+            assert rad[c] == 0
+            continue
+        assert np.all(np.diff(seg) <= 0)                         # descending (R11)
+        assert rad[c] == seg[0]
+        mem = orig[off[c]:off[c + 1]]
+        rec = np.sqrt(((T[mem].astype(np.float64) - cent[c, :16].astype(np.float64)) ** 2).sum(1))
+        np.testing.assert_allclose(seg, rec, rtol=2e-6)           # recorded distances are exact-ish
+        eq = seg[1:] == seg[:-1]
+        assert np.all(mem[1:][eq] > mem[:-1][eq])                 # ties by index ascending
+    idx, dd, st = ix.query(dev(Q), k, stats=True)
+    torch.cuda.synchronize()
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx.cpu().numpy(), dd.cpu().numpy(), ridx, rdist)
+    ix.close()
+
+
+def test_level1_soundness(sknn):
+    """P7: UB_qc >= the true k-th distance of every member query; the cluster of
+    every true neighbour is a candidate of the query's cluster."""
+    T = datagen.c5_blobs(20000, which="T")
+    Q = datagen.c5_blobs(3000, which="Q")
+    k = 32
+    ix = sknn.build(dev(T))
+    e = ix.export()
+    tcl = np.empty(T.shape[0], np.int64)
+    for c in range(len(e["radius"])):
+        tcl[e["orig"][e["off"][c]:e["off"][c + 1]]] = c
+    l1 = ix.debug_level1(dev(Q), k)
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    qc = l1["q_cluster"]
+    assert np.all(l1["ub"][qc] >= rdist[:, -1])
+    for i in range(Q.shape[0]):
+        cands = set(l1["cand"][qc[i], :l1["cand_count"][qc[i]]].tolist())
+        assert set(tcl[ridx[i]].tolist()) <= cands
+    ix.close()
+
+
+def test_merge_partials_equals_unsharded(sknn):
+    """Simulated target sharding on one GPU (P11): per-shard partial lists with
+    global indices merged by sknn_merge_partials == the unsharded join."""
+    T = datagen.c5_blobs(24000, which="T")
+    Q = datagen.c5_blobs(4000, which="Q")
+    k = 32
+    dQ = dev(Q)
+    parts_i, parts_d = [], []
+    P = 3
+    bounds = np.linspace(0, T.shape[0], P + 1).astype(int)
+    for r in range(P):
+        Ts = dev(T[bounds[r]:bounds[r + 1]])
+        i, d = sknn.join(dQ, Ts, k, out_squared=1, index_base=int(bounds[r]))
+        parts_i.append(i)
+        parts_d.append(d)
+    idx, dist = sknn.merge_partials(torch.stack(parts_i), torch.stack(parts_d), k)
+    torch.cuda.synchronize()
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx.cpu().numpy(), dist.cpu().numpy(), ridx, rdist)
+
+
+@pytest.mark.slow
+def test_c2_full_size_sampled(sknn):
+    """C2 at BASELINE size in the launch configuration bench.py times; the oracle
+    checks a seeded sample of queries one by one."""
+    Q, T, k, sj = datagen.workload("C2")
+    idx, dist, st = run(sknn, Q, T, k, sj)
+    rng = np.random.default_rng(99)
+    s = rng.choice(Q.shape[0], 2000, replace=False)
+    _, rdist = oracle.knn_join(Q[s], T, k)
+    assert_knn_tolerant(Q[s], T, idx[s], dist[s], rdist)
+    assert st["pruned_pct"] > 99.0
