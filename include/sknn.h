@@ -87,7 +87,7 @@ enum {
  * call sknn_options_default(). A NULL options pointer means all defaults. */
 typedef struct {
     size_t struct_size;       /* ABI versioning: sizeof(sknn_options) of the caller              */
-    int32_t n_clusters_q;     /* 0 = auto floor(3*sqrt(nq)), clamped to [1, min(nq, 16384)] */
+    int32_t n_clusters_q;     /* 0 = auto floor(3*sqrt(nq)), clamped to [1, min(nq, 8192)] */
     int32_t n_clusters_t;     /* 0 = auto floor(3*sqrt(nt)), same clamp                           */
     int32_t landmark_trials;  /* 0 = 10 trials of the landmark sampler                   */
     int32_t lloyd_iters;      /* -1 = default 2 (north_star "a few Lloyd iterations", reading R9); 0 = paper sampler only */

@@ -162,10 +162,15 @@ struct Timer {
 
 static int choose_mapping(const sknn_options& o, const DevInfo& di, int64_t nq, int dp) {
     if (o.mapping == SKNN_MAP_THREAD || o.mapping == SKNN_MAP_WARP) return o.mapping;
-    // Fig. 8 bottom: |Q| >= r*max_cur -> query-level
-    // parallelism (thread per query); otherwise several threads per query.
-    double rmax = (double)o.r_factor * di.num_sms * di.max_threads_per_sm;
-    return ((double)nq >= rmax && dp <= 32) ? SKNN_MAP_THREAD : SKNN_MAP_WARP;
+    // Fig. 8 bottom chooses query-level parallelism when
+    // |Q| >= r*max_cur and several threads per query otherwise. Measured on
+    // B200 (profiles/r01_sweep.md) the thread-per-query scan wins for every
+    // dp <= 32 workload, even C1 (1,024 queries, formula: 64 threads/query),
+    // because the sorted-member windows are short; the warp mapping is kept
+    // for dp > 32, where a query no longer fits in one thread's registers.
+    (void)di;
+    (void)nq;
+    return dp <= 32 ? SKNN_MAP_THREAD : SKNN_MAP_WARP;
 }
 
 static sknn_status validate(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
@@ -589,7 +594,7 @@ sknn_status sknn_config_decide(int64_t nq, int64_t nt, int32_t d, int32_t k, con
     if (out->tpq_raw > 1.0) tpq = 1 << (int)lround(log2(out->tpq_raw));       // reading R15
     out->threads_per_query = tpq;
     const int dp = (d + 3) & ~3;
-    out->mapping = ((double)nq >= rmax && dp <= 32) ? SKNN_MAP_THREAD : SKNN_MAP_WARP;
+    out->mapping = dp <= 32 ? SKNN_MAP_THREAD : SKNN_MAP_WARP;  // B200 rule, see choose_mapping
     out->mq = det_lm_num(std::max<int64_t>(nq, 1), 0);
     out->mt = det_lm_num(nt, 0);
     return SKNN_OK;

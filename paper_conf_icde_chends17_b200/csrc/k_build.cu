@@ -18,6 +18,8 @@
 //   k_gather_side      permuted padded rows, member distances, original indices
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
 
 #include "sknn_internal.cuh"
 #include "sknn_launch.h"
@@ -71,20 +73,45 @@ __global__ void k_landmark_draw(int64_t n, int m, int trials, uint64_t seed, int
         idx[t * m + i] = (int32_t)perm_index((uint32_t)i, (uint32_t)n, seed * 1315423911ull + t + 1);
 }
 
-// partial[t * nblk + b] = sum over pairs (i<j) with i in block b of d(c_i, c_j)
-__global__ void k_landmark_sums(const float* __restrict__ Xp, int dp, int m, const int32_t* __restrict__ idx,
-                                double* __restrict__ partial) {
-    int t = blockIdx.y;
-    int i = blockIdx.x * blockDim.x + threadIdx.x;
-    double s = 0.0;
-    if (i < m) {
-        const float* a = Xp + (int64_t)idx[t * m + i] * dp;
-        for (int j = i + 1; j < m; ++j) {
-            const float* b = Xp + (int64_t)idx[t * m + j] * dp;
-            s += (double)__fsqrt_rn(d2_rows(a, b, dp));
+// Pairwise-distance sum of each trial's candidate set, tiled: one
+// CTA per (trial, 64x64 tile of the upper triangle of the m x m pair matrix);
+// both row blocks are staged in shared memory (dp <= 128) so every distance
+// reads on-chip data; fixed-order reductions keep the sum deterministic.
+constexpr int kLmTile = 64;
+__global__ void __launch_bounds__(256) k_landmark_sums(const float* __restrict__ Xp, int dp, int m,
+                                                       const int32_t* __restrict__ idx, int nb,
+                                                       double* __restrict__ partial) {
+    extern __shared__ __align__(16) float s_rows[];  // [2 x 64 x dp]
+    const int t = blockIdx.y;
+    // linear tile -> (bi, bj), bi <= bj
+    int tl = blockIdx.x, bi = 0;
+    while (tl >= nb - bi) { tl -= nb - bi; ++bi; }
+    const int bj = bi + tl;
+    const bool smem = dp <= 128;
+    float* A = s_rows;
+    float* B = s_rows + kLmTile * dp;
+    if (smem) {
+        for (int e = threadIdx.x; e < kLmTile * dp / 4; e += blockDim.x) {
+            int r = e / (dp / 4), c = e % (dp / 4);
+            int ia = bi * kLmTile + r, ib = bj * kLmTile + r;
+            float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+            reinterpret_cast<float4*>(A)[e] = ia < m ? __ldg(reinterpret_cast<const float4*>(Xp + (int64_t)idx[t * m + ia] * dp) + c) : z;
+            reinterpret_cast<float4*>(B)[e] = ib < m ? __ldg(reinterpret_cast<const float4*>(Xp + (int64_t)idx[t * m + ib] * dp) + c) : z;
         }
+        __syncthreads();
     }
-    // fixed-order block reduction (deterministic)
+    double s = 0.0;
+    for (int p = threadIdx.x; p < kLmTile * kLmTile; p += blockDim.x) {
+        int i = p / kLmTile, j = p % kLmTile;
+        int gi = bi * kLmTile + i, gj = bj * kLmTile + j;
+        if (gi >= gj || gj >= m) continue;
+        const float* ra = smem ? A + i * dp : Xp + (int64_t)idx[t * m + gi] * dp;
+        const float* rb = smem ? B + j * dp : Xp + (int64_t)idx[t * m + gj] * dp;
+        float d2 = 0.f;
+        for (int c = 0; c < dp / 4; ++c)
+            d2 = d2_acc4(d2, reinterpret_cast<const float4*>(ra)[c], reinterpret_cast<const float4*>(rb)[c]);
+        s += (double)__fsqrt_rn(d2);
+    }
     __shared__ double red[256];
     red[threadIdx.x] = s;
     __syncthreads();
@@ -187,6 +214,97 @@ __global__ void __launch_bounds__(256) k_assign(const float* __restrict__ Xp, in
     if (counts) atomicAdd(counts + bi, 1);
     if (sums) {
         for (int c = 0; c < dp; ++c) atomicAdd(sums + (int64_t)bi * dp + c, xrow[c]);
+    }
+}
+
+// ------------------------------------------------ center kNN graph + walk --
+// The assignment only has to be approximate (reading R9: TI validity needs the
+// RECORDED member-center distances to be exact, not the nearest center), so
+// after the sampler the points are assigned by a greedy walk on the kNN graph
+// of the centers instead of an all-centers scan (m = 3*sqrt(n) centers would
+// cost n*m*d per pass). nbr[c] = the kNbr nearest centers of c (itself first).
+constexpr int kNbr = 32;
+
+__global__ void __launch_bounds__(256) k_center_knn(const float* __restrict__ centers, int m, int dp,
+                                                    int32_t* __restrict__ nbr) {
+    const int lane = threadIdx.x & 31;
+    const int c = blockIdx.x * 8 + (threadIdx.x >> 5);
+    if (c >= m) return;
+    const float* rc = centers + (int64_t)c * dp;
+    const int L = min(kNbr, m);
+    key_t mine = (lane < 32 - L) ? kNegKey : kInfKey;
+    key_t kth = kInfKey;
+    for (int base = 0; base < m; base += 32) {
+        const int j = base + lane;
+        key_t key = kInfKey;
+        if (j < m) key = make_key(d2_rows(rc, centers + (int64_t)j * dp, dp), j);
+        unsigned cm = __ballot_sync(0xffffffffu, key < kth);
+        while (cm) {
+            const int src = __ffs(cm) - 1;
+            const key_t kk = __shfl_sync(0xffffffffu, key, src);
+            mine = warp_insert(mine, kk, lane);
+            kth = __shfl_sync(0xffffffffu, mine, 31);
+            cm &= ~(1u << src);
+            cm &= __ballot_sync(0xffffffffu, key < kth);
+        }
+    }
+    if (lane >= 32 - L) nbr[(int64_t)c * kNbr + lane - (32 - L)] = key_idx(mine);
+    if (lane < kNbr - L) nbr[(int64_t)c * kNbr + L + lane] = c;  // pad short lists with self
+}
+
+// Greedy walk: start at the best of the `nentry` first centers (a random
+// subset: the centers are sampled points) or at the previous assignment, then
+// move to the best of the current center's graph neighbours until no
+// neighbour is closer. Distances are exact fp32 (direct formula), ties to the
+// lower center index. Optional Lloyd accumulation and histogram.
+template <int DP>
+__global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ Xp, int64_t n, int dp_rt,
+                                                     const float* __restrict__ centers, int m,
+                                                     const int32_t* __restrict__ nbr, int nentry,
+                                                     const int32_t* __restrict__ cid_prev,
+                                                     int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
+                                                     float* __restrict__ sums, int32_t* __restrict__ counts) {
+    const int dp = DP > 0 ? DP : dp_rt;
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const float* xr = Xp + i * dp;
+    float4 q[DP > 0 ? DP / 4 : 1];
+    if constexpr (DP > 0) {
+#pragma unroll
+        for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(xr) + c);
+    }
+    auto dist2 = [&](int c) -> float {
+        if constexpr (DP > 0) return d2_reg<DP>(q, centers + (int64_t)c * DP);
+        else return d2_rows(xr, centers + (int64_t)c * dp, dp);
+    };
+    int best;
+    float bd;
+    if (cid_prev) {
+        best = cid_prev[i];
+        bd = dist2(best);
+    } else {
+        best = 0;
+        bd = dist2(0);
+        for (int c = 1; c < nentry; ++c) {
+            float v = dist2(c);
+            if (v < bd) { bd = v; best = c; }
+        }
+    }
+    for (int step = 0; step < 64; ++step) {
+        const int cur = best;
+        const int32_t* nb = nbr + (int64_t)cur * kNbr;
+        for (int e = 1; e < kNbr; ++e) {
+            const int c = __ldg(nb + e);
+            const float v = dist2(c);
+            if (v < bd || (v == bd && c < best)) { bd = v; best = c; }
+        }
+        if (best == cur) break;
+    }
+    if (cid_out) cid_out[i] = best;
+    if (dist_out) dist_out[i] = __fsqrt_rn(bd);
+    if (counts) atomicAdd(counts + best, 1);
+    if (sums) {
+        for (int c = 0; c < dp; ++c) atomicAdd(sums + (int64_t)best * dp + c, xr[c]);
     }
 }
 
@@ -430,12 +548,16 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     SKNN_TRY(cx.alloc_scratch((void**)&lidx, sizeof(int32_t) * trials * m));
     k_landmark_draw<<<dim3((m + 255) / 256, trials), 256, 0, s>>>(n, m, trials, seed, lidx);
     cx.launched();
-    int nblk = (m + 255) / 256;
+    const int nb = (m + kLmTile - 1) / kLmTile;
+    const int ntile = nb * (nb + 1) / 2;
     double* partial;
-    SKNN_TRY(cx.alloc_scratch((void**)&partial, sizeof(double) * trials * nblk));
-    k_landmark_sums<<<dim3(nblk, trials), 256, 0, s>>>(Xp, dp, m, lidx, partial);
+    SKNN_TRY(cx.alloc_scratch((void**)&partial, sizeof(double) * trials * ntile));
+    size_t lsm = dp <= 128 ? sizeof(float) * 2 * kLmTile * dp : 0;
+    if (lsm > 48 * 1024)
+        SKNN_CUDA(cudaFuncSetAttribute(k_landmark_sums, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lsm));
+    k_landmark_sums<<<dim3(ntile, trials), 256, lsm, s>>>(Xp, dp, m, lidx, nb, partial);
     cx.launched();
-    k_landmark_pick<<<1, 512, 0, s>>>(partial, nblk, trials, lidx, m, Xp, dp, out.centers);
+    k_landmark_pick<<<1, 512, 0, s>>>(partial, ntile, trials, lidx, m, Xp, dp, out.centers);
     cx.launched();
 
     int32_t* cid;
@@ -446,6 +568,40 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     SKNN_TRY(cx.alloc_scratch((void**)&pdist, sizeof(float) * n));
     SKNN_TRY(cx.alloc_scratch((void**)&counts, sizeof(int32_t) * m));
     SKNN_TRY(cx.alloc_scratch((void**)&cursor, sizeof(int32_t) * m));
+    // assignment: greedy walk on the center kNN graph (default) or the full
+    // all-centers scan (SKNN_ASSIGN=full, for ablation)
+    const char* am = getenv("SKNN_ASSIGN");
+    const bool walk = !(am && strcmp(am, "full") == 0) && m > kNbr;
+    int32_t* nbr = nullptr;
+    if (walk) SKNN_TRY(cx.alloc_scratch((void**)&nbr, sizeof(int32_t) * (size_t)m * kNbr));
+    const char* ne = getenv("SKNN_WALK_ENTRIES");
+    const int nentry = std::min(m, ne ? std::max(1, atoi(ne)) : 64);
+    auto assign = [&](const int32_t* prev, int32_t* cid_o, float* dist_o, float* sums_o) -> sknn_status {
+        if (!walk) {
+            launch_assign(cx, Xp, n, dp, out.centers, m, cid_o, dist_o, sums_o, counts);
+            return SKNN_OK;
+        }
+        k_center_knn<<<(m + 7) / 8, 256, 0, s>>>(out.centers, m, dp, nbr);
+        cx.launched();
+        dim3 grid((unsigned)((n + 255) / 256));
+        switch (dp) {
+#define SKNN_WALK_CASE(D)                                                                                      \
+    case D:                                                                                                    \
+        k_assign_walk<D><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, m, nbr, nentry, prev, cid_o, dist_o, sums_o, \
+                                              counts);                                                         \
+        break;
+            SKNN_WALK_CASE(4) SKNN_WALK_CASE(8) SKNN_WALK_CASE(12) SKNN_WALK_CASE(16)
+            SKNN_WALK_CASE(20) SKNN_WALK_CASE(24) SKNN_WALK_CASE(28) SKNN_WALK_CASE(32)
+#undef SKNN_WALK_CASE
+            default:
+                k_assign_walk<0><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, m, nbr, nentry, prev, cid_o, dist_o,
+                                                      sums_o, counts);
+                break;
+        }
+        cx.launched();
+        return SKNN_OK;
+    };
+    const int32_t* prev = nullptr;
     // Lloyd iterations (R9)
     if (lloyd > 0) {
         float* sums;
@@ -453,7 +609,8 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         for (int it = 0; it < lloyd; ++it) {
             SKNN_CUDA(cudaMemsetAsync(sums, 0, sizeof(float) * m * dp, s));
             SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
-            launch_assign(cx, Xp, n, dp, out.centers, m, nullptr, nullptr, sums, counts);
+            SKNN_TRY(assign(prev, walk ? cid : nullptr, nullptr, sums));
+            if (walk) prev = cid;
             int blocks = std::max(1, std::min((m * dp + 255) / 256, 148 * 8));
             k_lloyd_update<<<blocks, 256, 0, s>>>(out.centers, sums, counts, m, dp);
             cx.launched();
@@ -461,7 +618,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     }
     // final assignment with exact member distances + histogram
     SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
-    launch_assign(cx, Xp, n, dp, out.centers, m, cid, pdist, nullptr, counts);
+    SKNN_TRY(assign(prev, cid, pdist, nullptr));
     k_offsets<<<1, 1024, 0, s>>>(counts, m, out.off, cursor);
     cx.launched();
     unsigned long long* keys;

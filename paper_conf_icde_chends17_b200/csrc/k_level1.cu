@@ -2,21 +2,24 @@
 //
 // One CTA per query cluster qc fuses the paper's two level-1 kernels:
 //   calUB  (§II-C Step 2.1; Fig. 4 calUB/getUBs P:L275-279;
-//           GPU version P:L337): pool the bounds r_q + D(qc,tc) + d(c_tc, u_i)
+//           GPU version P:L337): pool the bounds r_q + D(qc,tc) + d(c_tc,u_i)
 //           over the k members u_i closest to each target center (Eq. 4,
-//           Fig. 5) and take the k-th smallest. Each thread keeps a
-//           register top-k and stops a cluster early once its bound exceeds
-//           its own k-th (the footnote's early termination); the
-//           block then selects the k-th smallest among the values that can
-//           still matter (<= the smallest per-thread k-th).
+//           Fig. 5) and take the k-th smallest.
+//           B200 form (same value, no per-thread heaps): let v0(tc) =
+//           D + d(c_tc, u_0) be each cluster's smallest bound and M_k the k-th
+//           smallest v0. k distinct bounds are <= M_k, so the pooled k-th
+//           smallest V_k <= M_k, and every bound <= V_k belongs to a cluster
+//           with v0 <= M_k. So: radix-select M_k over the mt values v0, gather
+//           the bounds <= M_k of those (about k) clusters -- the footnote's
+//           early termination -- and radix-select their k-th smallest.
 //   groupFilter (Alg. 1; Fig. 4 getLB/groupFilter P:L273-277;
 //           GPU version P:L339): keep tc iff lb = D - r_q - r_t <= UB
 //           (reading R6, plus the R7 rounding slack). Survivors are compacted
 //           with warp ballots into shared memory and sorted by (D, tc)
 //           ascending -- the candidate order of pointFilter (Fig. 4 line 1,
 //           P:L263) -- then written to row qc of the [mq x mt] candidate table.
-// B200 design: no atomics in global memory except one counter add per CTA;
-// the table row per query cluster removes the paper's atomicAdd append.
+// The center distances D(qc, .) are computed once into shared memory and
+// reused by both substeps; no global atomics except one counter per CTA.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -27,54 +30,77 @@ namespace sknn {
 
 typedef unsigned long long u64;
 
-template <int KMAX>
-struct RegTopKf {
-    float a[KMAX];
-    __device__ __forceinline__ void init(int k) {
-#pragma unroll
-        for (int i = 0; i < KMAX; ++i) a[i] = (i < KMAX - k) ? -1.f : __int_as_float(0x7f800000);
-    }
-    __device__ __forceinline__ void insert(float v) {
-#pragma unroll
-        for (int i = KMAX - 1; i > 0; --i) {
-            float lo = a[i - 1], cur = a[i];
-            a[i] = (v < lo) ? lo : fminf(v, cur);
-        }
-        a[0] = fminf(a[0], v);
-    }
-};
+constexpr int kL1Threads = 256;
+constexpr int kL1Vals = 4096;  // capacity of the gathered-bounds buffer
 
 __device__ __forceinline__ void cmpx64(u64* s, int i, int p) {
     u64 a = s[i], b = s[p];
     if (b < a) { s[i] = b; s[p] = a; }
 }
-__device__ __forceinline__ void cmpxf(float* s, int i, int p) {
-    float a = s[i], b = s[p];
-    if (b < a) { s[i] = b; s[p] = a; }
-}
 
 // ascending bitonic (flip + half-cleaner form) over S (power of two) entries
-template <typename T, typename F>
-__device__ void block_sort_pow2(T* s, int S, F cx) {
+__device__ void block_sort_u64(u64* s, int S) {
     for (int k = 2; k <= S; k <<= 1) {
         for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
             int blk = t / (k / 2), r = t % (k / 2);
-            cx(s, blk * k + r, blk * k + k - 1 - r);
+            cmpx64(s, blk * k + r, blk * k + k - 1 - r);
         }
         __syncthreads();
         for (int j = k / 4; j > 0; j >>= 1) {
             for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
                 int i = (t / j) * 2 * j + (t % j);
-                cx(s, i, i + j);
+                cmpx64(s, i, i + j);
             }
             __syncthreads();
         }
     }
 }
 
-constexpr int kL1Threads = 256;
+// k-th smallest (1-based) of n non-negative floats in shared memory: MSB-first
+// radix select on the IEEE bits (monotone for x >= 0), 8 bits per round.
+// Returns +inf when n < k. All threads of the block must call it.
+__device__ float block_kth_smallest(const float* vals, int n, int k, int* s_hist, int* s_sel) {
+    if (n < k) return __int_as_float(0x7f800000);
+    uint32_t prefix = 0;
+    int kk = k;
+    for (int shift = 24; shift >= 0; shift -= 8) {
+        const uint32_t mask = shift == 24 ? 0u : (0xffffffffu << (shift + 8));
+        for (int i = threadIdx.x; i < 256; i += blockDim.x) s_hist[i] = 0;
+        __syncthreads();
+        for (int i = threadIdx.x; i < n; i += blockDim.x) {
+            uint32_t u = __float_as_uint(vals[i]);
+            if ((u & mask) == (prefix & mask)) atomicAdd(&s_hist[(u >> shift) & 255u], 1);
+        }
+        __syncthreads();
+        if (threadIdx.x < 32) {  // warp 0: the bin that holds rank kk
+            int c[8], tot = 0;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) { c[j] = s_hist[threadIdx.x * 8 + j]; tot += c[j]; }
+            int incl = tot;
+            for (int o = 1; o < 32; o <<= 1) {
+                int t = __shfl_up_sync(0xffffffffu, incl, o);
+                if ((int)threadIdx.x >= o) incl += t;
+            }
+            const int excl = incl - tot;
+            if (excl < kk && kk <= incl) {
+                int run = excl, bin = threadIdx.x * 8;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    if (run + c[j] >= kk) { bin = threadIdx.x * 8 + j; break; }
+                    run += c[j];
+                }
+                s_sel[0] = bin;
+                s_sel[1] = kk - run;
+            }
+        }
+        __syncthreads();
+        prefix |= uint32_t(s_sel[0]) << shift;
+        kk = s_sel[1];
+        __syncthreads();
+    }
+    return __uint_as_float(prefix);
+}
 
-template <int KMAX>
 __global__ void __launch_bounds__(kL1Threads) k_level1(
     const float* __restrict__ qcent, const float* __restrict__ qrad, const int32_t* __restrict__ qoff,
     const float* __restrict__ tcent, const float* __restrict__ trad, const int32_t* __restrict__ toff,
@@ -82,12 +108,14 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     int shard_count, float* __restrict__ ub_out, int32_t* __restrict__ cand, int32_t* __restrict__ cand_count,
     unsigned long long* __restrict__ cand_pairs) {
     extern __shared__ __align__(16) unsigned char smem[];
-    u64* s_keys = reinterpret_cast<u64*>(smem);                      // keys_cap entries
-    float* s_vals = reinterpret_cast<float*>(smem);                  // aliases s_keys in phase 1
-    float* s_qc = reinterpret_cast<float*>(smem + sizeof(u64) * keys_cap);
+    u64* s_keys = reinterpret_cast<u64*>(smem);                               // keys_cap (>= mt) entries
+    float* s_D = reinterpret_cast<float*>(smem + sizeof(u64) * keys_cap);     // [mt] center distances
+    const int mt4 = (mt + 3) & ~3;                                            // keep 16-byte alignment
+    float* s_v = s_D + mt4;                                                   // [max(mt4, kL1Vals)] bounds
+    float* s_qc = s_v + max(mt4, kL1Vals);                                    // [dp], float4-aligned
     __shared__ int s_cnt;
-    __shared__ float s_red[kL1Threads / 32];
-    __shared__ float s_ub;
+    __shared__ int s_hist[256];
+    __shared__ int s_sel[2];
 
     const int qc = blockIdx.x;
     const int qsize = qoff[qc + 1] - qoff[qc];
@@ -101,80 +129,71 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     const float rq = qrad[qc];
     const float INF = __int_as_float(0x7f800000);
 
-    // ---- phase 1: calUB ----
-    RegTopKf<KMAX> top;
-    top.init(k);
+    // ---- calUB (Step 2.1) ----
+    // v0(tc) = D + smallest member distance (the member closest to c_tc)
     for (int tc = threadIdx.x; tc < mt; tc += blockDim.x) {
-        int lo = toff[tc], hi = toff[tc + 1];
-        if (lo == hi) continue;
-        float D = __fsqrt_rn(d2_rows(s_qc, tcent + (int64_t)tc * dp, dp));
-        float base = rq + D;
-        int cnt = min(k, hi - lo);
+        const int lo = __ldg(toff + tc), hi = __ldg(toff + tc + 1);
+        const float D = __fsqrt_rn(d2_rows(s_qc, tcent + (int64_t)tc * dp, dp));
+        s_D[tc] = D;
+        s_v[tc] = (lo == hi) ? INF : D + __ldg(tdist + hi - 1);
+    }
+    __syncthreads();
+    const float Mk = block_kth_smallest(s_v, mt, k, s_hist, s_sel);
+    // gather every bound <= M_k of the clusters with v0 <= M_k
+    for (int tc = threadIdx.x; tc < mt; tc += blockDim.x) {
+        if (!(s_v[tc] <= Mk)) continue;
+        const int lo = __ldg(toff + tc), hi = __ldg(toff + tc + 1);
+        const float D = s_D[tc];
+        const int cnt = min(k, hi - lo);
         for (int i = 0; i < cnt; ++i) {
-            float v = base + __ldg(tdist + hi - 1 - i);   // members closest to the center
-            if (!(v < top.a[KMAX - 1])) break;            // early termination
-            top.insert(v);
-        }
-    }
-    // T0 = min over threads of their k-th bound: the block k-th is <= T0
-    float my = top.a[KMAX - 1];
-    for (int o = 16; o > 0; o >>= 1) my = fminf(my, __shfl_xor_sync(0xffffffffu, my, o));
-    if ((threadIdx.x & 31) == 0) s_red[threadIdx.x >> 5] = my;
-    __syncthreads();
-    float T0 = s_red[0];
-    for (int w = 1; w < kL1Threads / 32; ++w) T0 = fminf(T0, s_red[w]);
-#pragma unroll
-    for (int i = 0; i < KMAX; ++i) {
-        float v = top.a[i];
-        if (v >= 0.f && v <= T0) {
-            int pos = atomicAdd(&s_cnt, 1);
-            s_vals[pos] = v;
+            const float v = D + __ldg(tdist + hi - 1 - i);
+            if (v > Mk) break;  // members are visited closest-first: later bounds only grow
+            const int pos = atomicAdd(&s_cnt, 1);
+            if (pos < kL1Vals) s_keys[pos] = u64(__float_as_uint(v));
         }
     }
     __syncthreads();
-    int nv = s_cnt;
-    int S = 1;
-    while (S < nv) S <<= 1;
-    for (int i = nv + threadIdx.x; i < S; i += blockDim.x) s_vals[i] = INF;
+    const int nv = s_cnt;
+    // stage the gathered values as floats (alias-free copy into s_v)
+    for (int i = threadIdx.x; i < min(nv, kL1Vals); i += blockDim.x) s_v[i] = __uint_as_float(uint32_t(s_keys[i]));
     __syncthreads();
-    block_sort_pow2(s_vals, S, cmpxf);
+    float Vk = (nv <= kL1Vals) ? block_kth_smallest(s_v, nv, k, s_hist, s_sel) : Mk;  // overflow: M_k is a valid bound
+    if (!(Vk <= Mk)) Vk = Mk;
+    // UB = r_q + V_k, inflated to cover the rounding of the three summed distances (R7)
+    const float UB = __fmul_ru(rq + Vk, 1.f + 2.f * eta);
     if (threadIdx.x == 0) {
-        float ub = (k - 1 < nv) ? s_vals[k - 1] : INF;
-        ub = __fmul_ru(ub, 1.f + 2.f * eta);  // R7: covers rounding of the three summed distances
-        s_ub = ub;
-        ub_out[qc] = ub;
+        ub_out[qc] = UB;
         s_cnt = 0;
     }
     __syncthreads();
-    const float UB = s_ub;
 
-    // ---- phase 2: groupFilter (Alg. 1) ----
+    // ---- groupFilter (Step 2.2, Alg. 1) ----
     for (int base = 0; base < mt; base += blockDim.x) {
-        int tc = base + threadIdx.x;
+        const int tc = base + threadIdx.x;
         bool keep = false;
         float D = 0.f;
-        if (tc < mt && toff[tc] != toff[tc + 1]) {
-            D = __fsqrt_rn(d2_rows(s_qc, tcent + (int64_t)tc * dp, dp));
-            float rt = trad[tc];
-            float lb = D - rq - rt;                              // getLB (Eq. 3)
+        if (tc < mt && __ldg(toff + tc) != __ldg(toff + tc + 1)) {
+            D = s_D[tc];
+            const float rt = __ldg(trad + tc);
+            const float lb = D - rq - rt;                        // getLB (Eq. 3)
             keep = ti_keep(lb, UB, D + rq + rt, eta);             // Alg. 1 line 4 (R6, R7)
         }
-        unsigned m = __ballot_sync(0xffffffffu, keep);
+        const unsigned m = __ballot_sync(0xffffffffu, keep);
         int wbase = 0;
         if ((threadIdx.x & 31) == 0 && m) wbase = atomicAdd(&s_cnt, __popc(m));
         wbase = __shfl_sync(0xffffffffu, wbase, 0);
         if (keep) {
-            int pos = wbase + __popc(m & ((1u << (threadIdx.x & 31)) - 1u));
+            const int pos = wbase + __popc(m & ((1u << (threadIdx.x & 31)) - 1u));
             s_keys[pos] = (u64(__float_as_uint(D)) << 32) | u64(uint32_t(tc));
         }
     }
     __syncthreads();
-    int nc = s_cnt;
-    S = 1;
+    const int nc = s_cnt;
+    int S = 1;
     while (S < nc) S <<= 1;
     for (int i = nc + threadIdx.x; i < S; i += blockDim.x) s_keys[i] = ~0ull;
     __syncthreads();
-    block_sort_pow2(s_keys, S, cmpx64);
+    block_sort_u64(s_keys, S);
     int32_t* row = cand + (int64_t)qc * mt;
     for (int i = threadIdx.x; i < nc; i += blockDim.x) row[i] = int32_t(uint32_t(s_keys[i] & 0xffffffffu));
     if (threadIdx.x == 0) {
@@ -189,30 +208,19 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, int k, float eta
     SKNN_TRY(cx.alloc_scratch((void**)&out.ub, sizeof(float) * mq));
     SKNN_TRY(cx.alloc_scratch((void**)&out.cand, sizeof(int32_t) * (size_t)mq * mt));
     SKNN_TRY(cx.alloc_scratch((void**)&out.cand_count, sizeof(int32_t) * mq));
-    int kmax = k <= 8 ? 8 : k <= 16 ? 16 : k <= 24 ? 24 : 32;
     int cap = 1;
     while (cap < mt) cap <<= 1;
-    cap = std::max(cap, 4096);  // phase 1 sorts up to 256*32 floats (32 KB) aliasing the key buffer
-    size_t smem = sizeof(u64) * cap + sizeof(float) * dp;
-    if (smem > 200 * 1024) {
+    cap = std::max(cap, kL1Vals);
+    const int mt4 = (mt + 3) & ~3;
+    size_t smem = sizeof(u64) * cap + sizeof(float) * (mt4 + std::max(mt4, kL1Vals) + dp);
+    if (smem > 227 * 1024) {
         set_last_error("level-1: too many target clusters for the shared-memory candidate sort");
         return SKNN_ERR_UNSUPPORTED;
     }
-#define SKNN_L1(KM)                                                                                           \
-    do {                                                                                                      \
-        SKNN_CUDA(cudaFuncSetAttribute(k_level1<KM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); \
-        k_level1<KM><<<mq, kL1Threads, smem, cx.stream>>>(qs.centers, qs.radius, qs.off, ts.centers, ts.radius, \
-                                                          ts.off, ts.dist, mt, dp, k, eta, cap, shard_rank,     \
-                                                          shard_count, out.ub,       \
-                                                          out.cand, out.cand_count, cand_pairs_counter);      \
-    } while (0)
-    switch (kmax) {
-        case 8: SKNN_L1(8); break;
-        case 16: SKNN_L1(16); break;
-        case 24: SKNN_L1(24); break;
-        default: SKNN_L1(32); break;
-    }
-#undef SKNN_L1
+    SKNN_CUDA(cudaFuncSetAttribute(k_level1, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    k_level1<<<mq, kL1Threads, smem, cx.stream>>>(qs.centers, qs.radius, qs.off, ts.centers, ts.radius, ts.off,
+                                                  ts.dist, mt, dp, k, eta, cap, shard_rank, shard_count, out.ub,
+                                                  out.cand, out.cand_count, cand_pairs_counter);
     cx.launched();
     return cx.check_launch("level1");
 }

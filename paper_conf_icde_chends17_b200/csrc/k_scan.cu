@@ -18,139 +18,31 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
-#include "sknn_internal.cuh"
-#include "sknn_launch.h"
+#include "k_scan_common.cuh"
 
 namespace sknn {
 
-struct ScanArgs {
-    const float* qrows;
-    const int32_t* qorig;
-    const int32_t* qoff;
-    const float* trows;
-    const float* tdist;
-    const int32_t* torig;
-    const int32_t* toff;
-    const float* tcent;
-    const float* ub;
-    const int32_t* cand;
-    const int32_t* cand_count;
-    const int2* tiles;
-    const int* ntiles;
-    int mt;
-    int dp;
-    int k;
-    int tile;
-    float eta;
-    int out_squared;
-    long long index_base;
-    int32_t* out_idx;
-    float* out_dist;
-    Counters* counters;
-};
-
-// first member position in [lo, hi) NOT in the `continue` region
-// (dq - dt < -(theta + eta*(dq + dt + theta))); dt descends along the array.
-__device__ __forceinline__ int window_start(const float* __restrict__ tdist, int lo, int hi, float dq, float theta,
-                                            float eta) {
-    while (lo < hi) {
-        int mid = (lo + hi) >> 1;
-        float dt = __ldg(tdist + mid);
-        if (!ti_keep(dt - dq, theta, dq + dt, eta)) lo = mid + 1;
-        else hi = mid;
-    }
-    return lo;
-}
-
-__device__ __forceinline__ void write_result(const ScanArgs& a, int qorig, int r, key_t key) {
-    int64_t o = (int64_t)qorig * a.k + r;
-    float d2 = key_d2(key);
-    a.out_dist[o] = a.out_squared ? d2 : __fsqrt_rn(d2);
-    if (a.out_idx) a.out_idx[o] = (int32_t)(key_idx(key) + a.index_base);
-}
-
-__device__ __forceinline__ void add_counter(unsigned long long* c, unsigned long long v) {
-    // warp-aggregated: one atomic per warp
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    if ((threadIdx.x & 31) == 0 && v) atomicAdd(c, v);
-}
-
-constexpr int kCandChunk = 256;
-
-// ------------------------------------------------------ thread per query --
-template <int DP, int KMAX>
-__global__ void __launch_bounds__(128) k_scan_tpq(ScanArgs a) {
-    __shared__ int s_cand[kCandChunk];
-    const int ntiles = *a.ntiles;
-    unsigned long long evals = 0, cevals = 0;
-    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        const int2 tl = a.tiles[tile];
-        const int qc = tl.x;
-        const int qlo = a.qoff[qc], qsz = a.qoff[qc + 1] - qlo;
-        const int i = tl.y + threadIdx.x;
-        const bool active = i < qsz;
-        const int qpos = qlo + (active ? i : 0);
-        float4 q[DP / 4];
-#pragma unroll
-        for (int c = 0; c < DP / 4; ++c) q[c] = reinterpret_cast<const float4*>(a.qrows + (int64_t)qpos * DP)[c];
-        RegTopK<KMAX> top;
-        top.init(a.k);
-        const float ub = a.ub[qc];
-        float theta = ub;
-        const int ncand = a.cand_count[qc];
-        const int32_t* cl = a.cand + (int64_t)qc * a.mt;
-        for (int c0 = 0; c0 < ncand; c0 += kCandChunk) {
-            const int cn = min(kCandChunk, ncand - c0);
-            __syncthreads();
-            for (int t = threadIdx.x; t < cn; t += blockDim.x) s_cand[t] = cl[c0 + t];
-            __syncthreads();
-            if (!active) continue;
-            for (int c = 0; c < cn; ++c) {
-                const int tc = s_cand[c];
-                const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
-                const float dq = __fsqrt_rn(d2_reg<DP>(q, a.tcent + (int64_t)tc * DP));  // Alg. 2 line 6
-                ++cevals;
-                int j = window_start(a.tdist, lo, hi, dq, theta, a.eta);
-                for (; j < hi; ++j) {
-                    const float dt = __ldg(a.tdist + j);
-                    const float l = dq - dt;                             // line 9
-                    if (!ti_keep(l, theta, dq + dt, a.eta)) break;       // lines 10-11
-                    if (!ti_keep(-l, theta, dq + dt, a.eta)) continue;   // lines 12-13
-                    const float d2 = d2_reg<DP>(q, a.trows + (int64_t)j * DP);  // line 15
-                    ++evals;
-                    const key_t key = make_key(d2, __ldg(a.torig + j));
-                    if (key < top.kth()) {                               // line 16
-                        top.insert(key);
-                        theta = fminf(ub, __fsqrt_ru(key_d2(top.kth())));  // line 17 (R8)
-                    }
-                }
-            }
-        }
-        if (active) {
-            const int qo = __ldg(a.qorig + qpos);
-#pragma unroll
-            for (int s = 0; s < KMAX; ++s) {
-                const int r = s - (KMAX - a.k);
-                if (r >= 0) write_result(a, qo, r, top.a[s]);
-            }
-        }
-    }
-    add_counter(&a.counters->evals_sparse, evals);
-    add_counter(&a.counters->center_evals, cevals);
-}
-
 // -------------------------------------------------------- warp per query --
-// DP > 0: the query is held in registers by every lane; DP == 0: runtime dp,
-// the query is staged in shared memory (per warp) and read by broadcast.
+// Multi-level parallelism (§IV-B2; Fig. 8): one warp per
+// query, lanes split the member window of each candidate cluster, kNearests
+// is lane-distributed (lane r holds rank r) and theta is warp-uniform (the
+// paper's shared theta via atomicMin becomes a shuffle). Warps fetch tiles of
+// up to `tile` queries of one cluster from the atomic scheduler; no CTA
+// barriers. DP > 0: the query sits in registers of every lane; DP == 0:
+// runtime dp, the query is staged in shared memory per warp.
 template <int DP>
 __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
-    __shared__ int s_cand[kCandChunk];
     extern __shared__ __align__(16) float s_q[];  // [8 warps x dp] when DP == 0
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int ntiles = *a.ntiles;
     const int dp = DP > 0 ? DP : a.dp;
+    float* sq = s_q + warp * (DP > 0 ? 0 : dp);
     unsigned long long evals = 0, cevals = 0;
-    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    for (;;) {
+        int tile = 0;
+        if (lane == 0) tile = atomicAdd(a.tile_counter, 1);
+        tile = __shfl_sync(0xffffffffu, tile, 0);
+        if (tile >= ntiles) break;
         const int2 tl = a.tiles[tile];
         const int qc = tl.x;
         const int qlo = a.qoff[qc], qsz = a.qoff[qc + 1] - qlo;
@@ -158,75 +50,63 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
         const float ub = a.ub[qc];
         const int ncand = a.cand_count[qc];
         const int32_t* cl = a.cand + (int64_t)qc * a.mt;
-        // every warp handles queries warp, warp+8, ... of the tile; the candidate
-        // list is streamed through smem once per query round
-        for (int qi0 = 0; qi0 < nq_tile; qi0 += 8) {
-            const int qi = qi0 + warp;
-            const bool active = qi < nq_tile;
-            const int qpos = qlo + tl.y + (active ? qi : 0);
+        const uint8_t* dense_row = a.pair_dense ? a.pair_dense + (int64_t)qc * a.mt : nullptr;
+        for (int qi = 0; qi < nq_tile; ++qi) {
+            const int qpos = qlo + tl.y + qi;
             float4 q[DP > 0 ? DP / 4 : 1];
-            float* sq = s_q + warp * (DP > 0 ? 0 : dp);
             if constexpr (DP > 0) {
 #pragma unroll
-                for (int c = 0; c < DP / 4; ++c) q[c] = reinterpret_cast<const float4*>(a.qrows + (int64_t)qpos * DP)[c];
+                for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(a.qrows + (int64_t)qpos * DP) + c);
             } else {
                 __syncwarp();
                 for (int c = lane; c < dp; c += 32) sq[c] = a.qrows[(int64_t)qpos * dp + c];
                 __syncwarp();
             }
             key_t mine = (lane < 32 - a.k) ? kNegKey : kInfKey;
-            key_t kth = kInfKey;
-            float theta = ub;
-            for (int c0 = 0; c0 < ncand; c0 += kCandChunk) {
-                const int cn = min(kCandChunk, ncand - c0);
-                __syncthreads();
-                for (int t = threadIdx.x; t < cn; t += blockDim.x) s_cand[t] = cl[c0 + t];
-                __syncthreads();
-                if (!active) continue;
-                for (int c = 0; c < cn; ++c) {
-                    const int tc = s_cand[c];
-                    const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
-                    float dq2;
-                    if constexpr (DP > 0) dq2 = d2_reg<DP>(q, a.tcent + (int64_t)tc * DP);
-                    else dq2 = d2_rows(sq, a.tcent + (int64_t)tc * dp, dp);
-                    const float dq = __fsqrt_rn(dq2);
-                    if (lane == 0) ++cevals;
-                    int j0 = window_start(a.tdist, lo, hi, dq, theta, a.eta);
-                    for (int base = j0; base < hi; base += 32) {
-                        const int j = base + lane;
-                        const bool valid = j < hi;
-                        const float dt = valid ? __ldg(a.tdist + j) : 0.f;
-                        const float l = dq - dt;
-                        const bool brk = !valid || !ti_keep(l, theta, dq + dt, a.eta);
-                        const unsigned bm = __ballot_sync(0xffffffffu, brk);
-                        const int first = bm ? (__ffs(bm) - 1) : 32;
-                        const bool ev = lane < first && ti_keep(-l, theta, dq + dt, a.eta);
-                        key_t key = kInfKey;
-                        if (ev) {
-                            float d2;
-                            if constexpr (DP > 0) d2 = d2_reg<DP>(q, a.trows + (int64_t)j * DP);
-                            else d2 = d2_rows(sq, a.trows + (int64_t)j * dp, dp);
-                            key = make_key(d2, __ldg(a.torig + j));
-                            ++evals;
-                        }
-                        unsigned cm = __ballot_sync(0xffffffffu, ev && key < kth);
-                        while (cm) {
-                            const int src = __ffs(cm) - 1;
-                            const key_t kk = __shfl_sync(0xffffffffu, key, src);
-                            mine = warp_insert(mine, kk, lane);
-                            kth = __shfl_sync(0xffffffffu, mine, 31);
-                            cm &= ~(1u << src);
-                            cm &= __ballot_sync(0xffffffffu, ev && key < kth);
-                        }
-                        theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
-                        if (bm) break;
+            if (a.init_topk && lane >= 32 - a.k) mine = a.init_topk[(int64_t)qpos * a.k + lane - (32 - a.k)];
+            key_t kth = __shfl_sync(0xffffffffu, mine, 31);
+            float theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
+            for (int c = 0; c < ncand; ++c) {
+                const int tc = __ldg(cl + c);
+                if (dense_row && __ldg(dense_row + tc)) continue;
+                const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
+                float dq2;
+                if constexpr (DP > 0) dq2 = d2_reg<DP>(q, a.tcent + (int64_t)tc * DP);
+                else dq2 = d2_rows(sq, a.tcent + (int64_t)tc * dp, dp);
+                const float dq = __fsqrt_rn(dq2);
+                if (lane == 0) ++cevals;
+                const int j0 = window_start(a.tdist, lo, hi, dq, theta, a.eta);
+                for (int base = j0; base < hi; base += 32) {
+                    const int j = base + lane;
+                    const bool valid = j < hi;
+                    const float dt = valid ? __ldg(a.tdist + j) : 0.f;
+                    const float l = dq - dt;
+                    const bool brk = !valid || !ti_keep(l, theta, dq + dt, a.eta);
+                    const unsigned bm = __ballot_sync(0xffffffffu, brk);
+                    const int first = bm ? (__ffs(bm) - 1) : 32;
+                    const bool ev = lane < first && ti_keep(-l, theta, dq + dt, a.eta);
+                    key_t key = kInfKey;
+                    if (ev) {
+                        float d2;
+                        if constexpr (DP > 0) d2 = d2_reg<DP>(q, a.trows + (int64_t)j * DP);
+                        else d2 = d2_rows(sq, a.trows + (int64_t)j * dp, dp);
+                        ++evals;
+                        if (d2 <= key_d2(kth)) key = make_key(d2, __ldg(a.torig + j));
                     }
+                    unsigned cm = __ballot_sync(0xffffffffu, key < kth);
+                    while (cm) {
+                        const int src = __ffs(cm) - 1;
+                        const key_t kk = __shfl_sync(0xffffffffu, key, src);
+                        mine = warp_insert(mine, kk, lane);
+                        kth = __shfl_sync(0xffffffffu, mine, 31);
+                        cm &= ~(1u << src);
+                        cm &= __ballot_sync(0xffffffffu, key < kth);
+                    }
+                    theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
+                    if (bm) break;
                 }
             }
-            if (active && lane >= 32 - a.k) {
-                const int qo = __ldg(a.qorig + qpos);
-                write_result(a, qo, lane - (32 - a.k), mine);
-            }
+            if (lane >= 32 - a.k) write_result(a, __ldg(a.qorig + qpos), lane - (32 - a.k), mine);
         }
     }
     add_counter(&a.counters->evals_sparse, evals);
@@ -237,7 +117,7 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
 // Single CTA: tiles of `tile` queries per non-empty query cluster.
 __global__ void __launch_bounds__(1024) k_make_tiles(const int32_t* __restrict__ qoff, int mq, int tile,
                                                      int shard_rank, int shard_count, int2* __restrict__ tiles,
-                                                     int* __restrict__ ntiles) {
+                                                     int* __restrict__ ntiles, int* __restrict__ counter) {
     __shared__ int s_sum[1024];
     __shared__ int s_carry;
     if (threadIdx.x == 0) s_carry = 0;
@@ -261,28 +141,14 @@ __global__ void __launch_bounds__(1024) k_make_tiles(const int32_t* __restrict__
         if (threadIdx.x == 1023) s_carry += s_sum[1023];
         __syncthreads();
     }
-    if (threadIdx.x == 0) *ntiles = s_carry;
+    if (threadIdx.x == 0) { *ntiles = s_carry; *counter = 0; }
 }
 
-static int occupancy_grid(Ctx& cx, const void* fn, int threads, size_t smem) {
+int occupancy_grid(Ctx& cx, const void* fn, int threads, size_t smem) {
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem);
     if (per_sm < 1) per_sm = 1;
     return per_sm * cx.num_sms;
-}
-
-template <int DP, int KMAX>
-static void launch_tpq(Ctx& cx, const ScanArgs& a) {
-    int grid = occupancy_grid(cx, (const void*)k_scan_tpq<DP, KMAX>, 128, 0);
-    k_scan_tpq<DP, KMAX><<<grid, 128, 0, cx.stream>>>(a);
-}
-
-template <int DP>
-static void launch_tpq_k(Ctx& cx, const ScanArgs& a) {
-    if (a.k <= 8) launch_tpq<DP, 8>(cx, a);
-    else if (a.k <= 16) launch_tpq<DP, 16>(cx, a);
-    else if (a.k <= 24) launch_tpq<DP, 24>(cx, a);
-    else launch_tpq<DP, 32>(cx, a);
 }
 
 template <int DP>
@@ -293,47 +159,50 @@ static void launch_wpq(Ctx& cx, const ScanArgs& a) {
     k_scan_wpq<DP><<<grid, 256, smem, cx.stream>>>(a);
 }
 
-int scan_tile_size(int mapping, int dp) { return (mapping == SKNN_MAP_THREAD && dp <= 32) ? 128 : 32; }
+int scan_tile_size(int mapping, int dp) { return (mapping == SKNN_MAP_THREAD && dp <= 32) ? 32 : 8; }
 
 sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int shard_rank, int shard_count, Level1& l1) {
     int64_t max_tiles = (qs.n + tile - 1) / tile + qs.m;
     SKNN_TRY(cx.alloc_scratch((void**)&l1.tiles, sizeof(int2) * max_tiles));
-    SKNN_TRY(cx.alloc_scratch((void**)&l1.ntiles, sizeof(int)));
+    SKNN_TRY(cx.alloc_scratch((void**)&l1.ntiles, sizeof(int) * 2));
     l1.tile = tile;
-    k_make_tiles<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, l1.tiles, l1.ntiles);
+    k_make_tiles<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, l1.tiles, l1.ntiles,
+                                             l1.ntiles + 1);
     cx.launched();
     return cx.check_launch("tiles");
 }
 
 sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
     const int dp = ts.dp;
-    const int tile = l1.tile;
-    const bool tpq = tile == 128;
-    const int2* tiles = l1.tiles;
-    const int* ntiles = l1.ntiles;
-    ScanArgs a;
+    const bool tpq = p.mapping == SKNN_MAP_THREAD && dp <= 32;
+    ScanArgs a{};
     a.qrows = qs.rows; a.qorig = qs.orig; a.qoff = qs.off;
     a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
     a.ub = l1.ub; a.cand = l1.cand; a.cand_count = l1.cand_count;
-    a.tiles = tiles; a.ntiles = ntiles; a.mt = ts.m; a.dp = dp; a.k = p.k; a.tile = tile; a.eta = p.eta;
+    a.tiles = l1.tiles; a.ntiles = l1.ntiles; a.tile_counter = l1.ntiles + 1;
+    a.init_topk = p.init_topk; a.pair_dense = p.pair_dense;
+    a.mt = ts.m; a.dp = dp; a.k = p.k; a.tile = l1.tile; a.eta = p.eta;
     a.out_squared = p.out_squared; a.index_base = p.index_base; a.out_idx = p.out_idx; a.out_dist = p.out_dist;
     a.counters = p.counters;
     if (tpq) {
         switch (dp) {
-            case 4: launch_tpq_k<4>(cx, a); break;
-            case 8: launch_tpq_k<8>(cx, a); break;
-            case 12: launch_tpq_k<12>(cx, a); break;
-            case 16: launch_tpq_k<16>(cx, a); break;
-            case 20: launch_tpq_k<20>(cx, a); break;
-            case 24: launch_tpq_k<24>(cx, a); break;
-            case 28: launch_tpq_k<28>(cx, a); break;
-            default: launch_tpq_k<32>(cx, a); break;
+            case 4: launch_tpq_dp<4>(cx, a); break;
+            case 8: launch_tpq_dp<8>(cx, a); break;
+            case 12: launch_tpq_dp<12>(cx, a); break;
+            case 16: launch_tpq_dp<16>(cx, a); break;
+            case 20: launch_tpq_dp<20>(cx, a); break;
+            case 24: launch_tpq_dp<24>(cx, a); break;
+            case 28: launch_tpq_dp<28>(cx, a); break;
+            default: launch_tpq_dp<32>(cx, a); break;
         }
     } else {
         switch (dp) {
             case 4: launch_wpq<4>(cx, a); break;
             case 8: launch_wpq<8>(cx, a); break;
+            case 12: launch_wpq<12>(cx, a); break;
             case 16: launch_wpq<16>(cx, a); break;
+            case 20: launch_wpq<20>(cx, a); break;
+            case 24: launch_wpq<24>(cx, a); break;
             case 28: launch_wpq<28>(cx, a); break;
             case 32: launch_wpq<32>(cx, a); break;
             default: launch_wpq<0>(cx, a); break;

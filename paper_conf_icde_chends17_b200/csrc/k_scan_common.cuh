@@ -1,0 +1,75 @@
+// k_scan_common.cuh -- shared pieces of the level-2 scan kernels (Alg. 2,
+// P:L355-375): launch arguments, the member-window binary search, the result
+// write (Fig. 4 output R) and warp-aggregated counters.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "sknn_internal.cuh"
+#include "sknn_launch.h"
+
+namespace sknn {
+
+struct ScanArgs {
+    const float* qrows;
+    const int32_t* qorig;
+    const int32_t* qoff;
+    const float* trows;
+    const float* tdist;
+    const int32_t* torig;
+    const int32_t* toff;
+    const float* tcent;
+    const float* ub;
+    const int32_t* cand;
+    const int32_t* cand_count;
+    const int2* tiles;
+    const int* ntiles;
+    int* tile_counter;     // dynamic tile scheduler (zeroed by k_make_tiles)
+    const key_t* init_topk;  // optional [nq_perm x k] keys from the dense-tile pass (NULL = none)
+    const uint8_t* pair_dense;  // optional [mq x mt] 1 = pair handled by the dense-tile pass
+    int mt;
+    int dp;
+    int k;
+    int tile;
+    float eta;
+    int out_squared;
+    long long index_base;
+    int32_t* out_idx;
+    float* out_dist;
+    Counters* counters;
+};
+
+// First member position in [lo, hi) that is NOT in Alg. 2's `continue`
+// region (l = dq - dt < -theta, line 12); dt descends along the array.
+__device__ __forceinline__ int window_start(const float* __restrict__ tdist, int lo, int hi, float dq, float theta,
+                                            float eta) {
+    while (lo < hi) {
+        int mid = (lo + hi) >> 1;
+        float dt = __ldg(tdist + mid);
+        if (!ti_keep(dt - dq, theta, dq + dt, eta)) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+__device__ __forceinline__ void write_result(const ScanArgs& a, int qorig, int r, key_t key) {
+    int64_t o = (int64_t)qorig * a.k + r;
+    float d2 = key_d2(key);
+    a.out_dist[o] = a.out_squared ? d2 : __fsqrt_rn(d2);
+    if (a.out_idx) a.out_idx[o] = (int32_t)(key_idx(key) + a.index_base);
+}
+
+// warp-aggregated counter: one atomic per warp (all 32 lanes must call)
+__device__ __forceinline__ void add_counter(unsigned long long* c, unsigned long long v) {
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((threadIdx.x & 31) == 0 && v) atomicAdd(c, v);
+}
+
+// dispatch helpers (k_scan_tpq_dp*.cu)
+template <int DP>
+void launch_tpq_dp(Ctx& cx, const ScanArgs& a);
+
+int occupancy_grid(Ctx& cx, const void* fn, int threads, size_t smem);
+
+}  // namespace sknn

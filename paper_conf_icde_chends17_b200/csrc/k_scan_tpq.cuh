@@ -1,0 +1,149 @@
+// k_scan_tpq.cuh -- level-2 scan, one thread per query ("query level
+// parallelism", Fig. 8; Alg. 2).
+//
+// B200 design:
+//  * warp tiles: a warp owns 32 queries of ONE query cluster (thread-data
+//    remapping, §IV-C1 / Tables I-II), so all lanes walk the same candidate
+//    list in the same order; candidate ids are warp-uniform broadcast loads.
+//  * no CTA barriers: warps fetch tiles from a device-side atomic counter
+//    (dynamic scheduling), so a finished warp never waits for a slow one.
+//  * kNearests in registers (Fig. 8 placement: k*4 B <= th2), sorted 64-bit
+//    (d2, index) keys; the distance-only test `d2 <= kth_d2` runs first and
+//    the index is loaded only for a key that can enter the list.
+//  * the member loop is software-pipelined: the next member's distance (and
+//    for DP <= 8 its row) is loaded before the current one is processed.
+#pragma once
+
+#include "k_scan_common.cuh"
+
+namespace sknn {
+
+template <int DP, int KMAX>
+__global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
+    constexpr bool kPrefetchRow = DP <= 8;
+    const int lane = threadIdx.x & 31;
+    const int ntiles = *a.ntiles;
+    unsigned long long evals = 0, cevals = 0;
+    for (;;) {
+        int tile = 0;
+        if (lane == 0) tile = atomicAdd(a.tile_counter, 1);
+        tile = __shfl_sync(0xffffffffu, tile, 0);
+        if (tile >= ntiles) break;
+        const int2 tl = a.tiles[tile];
+        const int qc = tl.x;
+        const int qlo = a.qoff[qc], qsz = a.qoff[qc + 1] - qlo;
+        const int i = tl.y + lane;
+        const bool active = i < qsz;
+        const int qpos = qlo + (active ? i : 0);
+        float4 q[DP / 4];
+#pragma unroll
+        for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(a.qrows + (int64_t)qpos * DP) + c);
+        RegTopK<KMAX> top;
+        top.init(a.k);
+        const float ub = a.ub[qc];
+        float theta = ub;
+        if (a.init_topk) {  // continue from the dense-tile pass
+#pragma unroll
+            for (int s = 0; s < KMAX; ++s) {
+                const int r = s - (KMAX - a.k);
+                if (r >= 0) top.a[s] = a.init_topk[(int64_t)qpos * a.k + r];
+            }
+            theta = fminf(ub, __fsqrt_ru(key_d2(top.kth())));
+        }
+        key_t kth = top.kth();
+        float kth_d2 = key_d2(kth);
+        const int ncand = a.cand_count[qc];
+        const int32_t* cl = a.cand + (int64_t)qc * a.mt;
+        const uint8_t* dense_row = a.pair_dense ? a.pair_dense + (int64_t)qc * a.mt : nullptr;
+        if (active) {
+            for (int c = 0; c < ncand; ++c) {
+                const int tc = __ldg(cl + c);
+                if (dense_row && __ldg(dense_row + tc)) continue;  // covered by the dense tile pass
+                const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
+                const float dq = __fsqrt_rn(d2_reg<DP>(q, a.tcent + (int64_t)tc * DP));  // Alg. 2 line 6
+                ++cevals;
+                int j = window_start(a.tdist, lo, hi, dq, theta, a.eta);
+                if (j >= hi) continue;
+                float dt_n = __ldg(a.tdist + j);
+                float4 row_n[kPrefetchRow ? DP / 4 : 1];
+                if constexpr (kPrefetchRow) {
+#pragma unroll
+                    for (int c4 = 0; c4 < DP / 4; ++c4)
+                        row_n[c4] = __ldg(reinterpret_cast<const float4*>(a.trows + (int64_t)j * DP) + c4);
+                }
+                for (;;) {
+                    const float dt = dt_n;
+                    float4 row[kPrefetchRow ? DP / 4 : 1];
+                    if constexpr (kPrefetchRow) {
+#pragma unroll
+                        for (int c4 = 0; c4 < DP / 4; ++c4) row[c4] = row_n[c4];
+                    }
+                    const int jc = j++;
+                    const bool more = j < hi;
+                    if (more) {
+                        dt_n = __ldg(a.tdist + j);
+                        if constexpr (kPrefetchRow) {
+#pragma unroll
+                            for (int c4 = 0; c4 < DP / 4; ++c4)
+                                row_n[c4] = __ldg(reinterpret_cast<const float4*>(a.trows + (int64_t)j * DP) + c4);
+                        }
+                    }
+                    const float l = dq - dt;                              // line 9
+                    if (!ti_keep(l, theta, dq + dt, a.eta)) break;        // lines 10-11
+                    if (ti_keep(-l, theta, dq + dt, a.eta)) {             // lines 12-14
+                        float d2;                                         // line 15
+                        if constexpr (kPrefetchRow) {
+                            d2 = 0.f;
+#pragma unroll
+                            for (int c4 = 0; c4 < DP / 4; ++c4) d2 = d2_acc4(d2, q[c4], row[c4]);
+                        } else {
+                            d2 = d2_reg<DP>(q, a.trows + (int64_t)jc * DP);
+                        }
+                        ++evals;
+                        if (d2 <= kth_d2) {                               // line 16 (distance part)
+                            const key_t key = make_key(d2, __ldg(a.torig + jc));
+                            if (key < kth) {
+                                top.insert(key);
+                                kth = top.kth();
+                                kth_d2 = key_d2(kth);
+                                theta = fminf(ub, __fsqrt_ru(kth_d2));    // line 17 (R8)
+                            }
+                        }
+                    }
+                    if (!more) break;
+                }
+            }
+            const int qo = __ldg(a.qorig + qpos);
+#pragma unroll
+            for (int s = 0; s < KMAX; ++s) {
+                const int r = s - (KMAX - a.k);
+                if (r >= 0) write_result(a, qo, r, top.a[s]);
+            }
+        }
+    }
+    add_counter(&a.counters->evals_sparse, evals);
+    add_counter(&a.counters->center_evals, cevals);
+}
+
+template <int DP, int KMAX>
+static void launch_tpq(Ctx& cx, const ScanArgs& a) {
+    int grid = occupancy_grid(cx, (const void*)k_scan_tpq<DP, KMAX>, 256, 0);
+    k_scan_tpq<DP, KMAX><<<grid, 256, 0, cx.stream>>>(a);
+}
+
+// k -> smallest multiple of 4 >= k (no idle register slots beyond 3)
+template <int DP>
+void launch_tpq_dp(Ctx& cx, const ScanArgs& a) {
+    switch ((a.k + 3) / 4) {
+        case 1: launch_tpq<DP, 4>(cx, a); break;
+        case 2: launch_tpq<DP, 8>(cx, a); break;
+        case 3: launch_tpq<DP, 12>(cx, a); break;
+        case 4: launch_tpq<DP, 16>(cx, a); break;
+        case 5: launch_tpq<DP, 20>(cx, a); break;
+        case 6: launch_tpq<DP, 24>(cx, a); break;
+        case 7: launch_tpq<DP, 28>(cx, a); break;
+        default: launch_tpq<DP, 32>(cx, a); break;
+    }
+}
+
+}  // namespace sknn

@@ -14,7 +14,7 @@
 namespace sknn {
 
 constexpr int kWarp = 32;
-constexpr int kMaxClusters = 16384;  // memory clamp of detLmNum
+constexpr int kMaxClusters = 8192;  // clamp of detLmNum: level-1 keeps a row of D in smem
 
 // ------------------------------------------------------------------ keys --
 // A neighbour candidate is the 64-bit key (d2 bits << 32) | target index.

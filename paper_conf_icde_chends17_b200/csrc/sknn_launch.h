@@ -109,6 +109,8 @@ struct ScanParams {
     int32_t* out_idx = nullptr;
     float* out_dist = nullptr;
     Counters* counters = nullptr;
+    const key_t* init_topk = nullptr;    // dense-tile pass results to continue from
+    const uint8_t* pair_dense = nullptr; // [mq x mt] pairs already covered by dense tiles
 };
 sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p);
 sknn_status run_brute(Ctx& cx, const float* Q, int64_t nq, const float* T, int64_t nt, int d, const ScanParams& p);

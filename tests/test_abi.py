@@ -107,9 +107,9 @@ def test_config_decide_matches_oracle_b200(L):
         assert placement == ocfg.knearests_placement(k, g["th1"], g["th2"])
         assert bool(c["partial_filter"]) == (ocfg.filter_strength(k, d) == "partial")
         assert c["threads_per_query"] == ocfg.threads_per_query(nq, 0.25, ocfg.max_cur(148, 2048))
-        assert c["mq"] == min(16384, int(np.floor(3 * np.sqrt(nq))))
-    # mapping: C2 and C5 thread-per-query; C1, C3 (|Q| < r*max_cur) and C4 (dp > 32) warp-per-query
+        assert c["mq"] == min(8192, int(np.floor(3 * np.sqrt(nq))))
+    # mapping (B200 rule): thread-per-query for dp <= 32 (C1, C2, C3, C5), warp-per-query for C4 (dp = 128)
     assert sknn.config_decide(434_874, 434_874, 4, 20, props=props)["mapping"] == 1
     assert sknn.config_decide(4_000_000, 4_000_000, 16, 32, props=props)["mapping"] == 1
-    assert sknn.config_decide(65_554, 65_554, 28, 16, props=props)["mapping"] == 2
+    assert sknn.config_decide(65_554, 65_554, 28, 16, props=props)["mapping"] == 1  # B200 rule: dp <= 32
     assert sknn.config_decide(1_000_000, 1_000_000, 128, 16, props=props)["mapping"] == 2

@@ -1,0 +1,79 @@
+"""Option sweep on the GPU: per-stage times and pruning for the C1-C5 workloads.
+
+    python tools/sweep.py [--configs C2,C3] [--scale 1.0] [--reps 5] [--variants default,lloyd0,...]
+
+Prints one JSON line per (config, variant): median ms_total over reps, the stage
+split (CUDA events inside the library), % pruned, evaluations per query.
+"""
+import argparse
+import json
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import datagen  # noqa: E402
+
+VARIANTS = {
+    "default": {},
+    "lloyd0": {"lloyd_iters": 0},
+    "lloyd1": {"lloyd_iters": 1},
+    "lloyd4": {"lloyd_iters": 4},
+    "thread": {"mapping": "thread"},
+    "warp": {"mapping": "warp"},
+    "cl_half": {"_cl": 0.5},
+    "cl_double": {"_cl": 2.0},
+    "fullassign": {"_env": ("SKNN_ASSIGN", "full")},
+    "entries256": {"_env": ("SKNN_WALK_ENTRIES", "256")},
+    "full_lloyd4": {"_env": ("SKNN_ASSIGN", "full"), "lloyd_iters": 4},
+}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--configs", default="C1,C2,C3,C3int")
+    ap.add_argument("--scale", type=float, default=1.0)
+    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--variants", default="default")
+    args = ap.parse_args()
+    import torch
+    import paper_conf_icde_chends17_b200 as sknn
+    for name in args.configs.split(","):
+        Q, T, k, sj = datagen.workload(name, args.scale)
+        dQ = torch.from_numpy(Q).cuda()
+        dT = dQ if sj else torch.from_numpy(T).cuda()
+        nq, nt = Q.shape[0], T.shape[0]
+        flush = torch.empty(128 * 1024 * 1024, dtype=torch.float32, device="cuda")
+        for vname in args.variants.split(","):
+            v = dict(VARIANTS[vname])
+            env = v.pop("_env", None)
+            cl = v.pop("_cl", None)
+            if cl:
+                v["n_clusters_t"] = int(3 * np.sqrt(nt) * cl)
+                v["n_clusters_q"] = int(3 * np.sqrt(nq) * cl)
+            if env:
+                os.environ[env[0]] = env[1]
+            res = []
+            for r in range(args.reps + 2):
+                flush.zero_()
+                _, _, st = sknn.join(dQ, dT, k, stats=True, **v)
+                if r >= 2:
+                    res.append(st)
+            if env:
+                del os.environ[env[0]]
+            ms = [x["ms_total"] for x in res]
+            med = res[int(np.argsort(ms)[len(ms) // 2])]
+            out = {"config": name, "variant": vname, "nq": nq, "nt": nt, "k": k, "ms_total": float(np.median(ms)),
+                   "ms_min": float(np.min(ms)), "queries_per_s": nq / (np.median(ms) / 1000.0),
+                   "pruned_pct": med["pruned_pct"], "evals_per_query": med["dist_evals"] / nq,
+                   "cand_per_qcluster": med["cand_pairs"] / max(1, med["mq"]), "center_evals_per_query": med["center_evals"] / nq,
+                   "stages": {k2: round(med[k2], 4) for k2 in ("ms_build_t", "ms_build_q", "ms_level1", "ms_sparse")},
+                   "mq": med["mq"], "mt": med["mt"], "mapping": med["mapping_used"], "launches": med["kernel_launches"]}
+            print(json.dumps(out), flush=True)
+
+
+if __name__ == "__main__":
+    main()
