@@ -114,6 +114,7 @@ typedef struct {
     uint64_t center_evals;         /* query-to-candidate-center distances in level-2 (Alg. 2 line 6)  */
     uint64_t cand_pairs;           /* surviving (query cluster, target cluster) pairs after level-1  */
     uint64_t dense_pairs;          /* of which processed as dense tiles                               */
+    uint64_t dist_recompute;       /* dense-tile survivors recomputed with the exact fp32 formula     */
     float ms_total;                /* CUDA-event time of the whole call on `stream`                   */
     float ms_build_t, ms_build_q, ms_level1, ms_sparse, ms_dense, ms_final;
     int32_t mapping_used;          /* SKNN_MAP_THREAD or SKNN_MAP_WARP                               */

@@ -56,6 +56,7 @@ class Stats(ctypes.Structure):
                 ("dist_evals_sparse", ctypes.c_uint64), ("dist_evals_dense", ctypes.c_uint64),
                 ("dist_evals_brute", ctypes.c_uint64), ("center_evals", ctypes.c_uint64),
                 ("cand_pairs", ctypes.c_uint64), ("dense_pairs", ctypes.c_uint64),
+                ("dist_recompute", ctypes.c_uint64),
                 ("ms_total", ctypes.c_float), ("ms_build_t", ctypes.c_float), ("ms_build_q", ctypes.c_float),
                 ("ms_level1", ctypes.c_float), ("ms_sparse", ctypes.c_float), ("ms_dense", ctypes.c_float),
                 ("ms_final", ctypes.c_float), ("mapping_used", ctypes.c_int32), ("path_used", ctypes.c_int32),

@@ -186,16 +186,50 @@ static sknn_status validate(const float* Q, int64_t nq, const float* T, int64_t 
     return SKNN_OK;
 }
 
-// The query half of Fig. 4 (lines 3-6) given both clustered sides.
+struct Marks {
+    int bt = -1, bq = -1, l1 = -1, dense = -1, scan = -1, end = -1;
+};
+
+// Elastic switch mode for level-1 (S8): 2 = every pair dense, 1 = none, 0 = cost model.
+static int dense_mode_for(const sknn_options& o, int dp) {
+    if (o.force_path == SKNN_PATH_DENSE) return 2;
+    if (o.force_path == SKNN_PATH_SPARSE) return 1;
+    // tensor cores pay once a distance costs more than the screen (dp >= 16)
+    return (dp >= 16 && dense_supported(dp)) ? 0 : 1;
+}
+
+// The query half of Fig. 4 (lines 3-6) given both clustered sides:
+// calUB + groupFilter (+ the elastic switch) -> dense tiles -> pointFilter.
 static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, const sknn_options& o, int mapping,
-                              int32_t* out_idx, float* out_dist, Counters* counters, Timer& tm, int* mk_l1,
-                              int* mk_scan) {
+                              int32_t* out_idx, float* out_dist, Counters* counters, Timer& tm, Marks& mk) {
     const float eta = rounding_eta(ts.d);
     Level1 l1;
-    const int srank = o.shard_count > 1 ? o.shard_rank : 0, scount = o.shard_count > 1 ? o.shard_count : 1;
-    SKNN_TRY(run_level1(cx, qs, ts, k, eta, srank, scount, l1, &counters->cand_pairs));
-    SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp), srank, scount, l1));
-    *mk_l1 = tm.mark();
+    Level1Params lp;
+    lp.k = k;
+    lp.eta = eta;
+    lp.shard_rank = o.shard_count > 1 ? o.shard_rank : 0;
+    lp.shard_count = o.shard_count > 1 ? o.shard_count : 1;
+    lp.dense_mode = dense_mode_for(o, ts.dp);
+    lp.dense_tau = o.dense_threshold > 0.f ? o.dense_threshold : 1.f;
+    if (lp.dense_mode == 2 && !dense_supported(ts.dp)) {
+        set_last_error("force_path = DENSE needs d <= 256");
+        return SKNN_ERR_UNSUPPORTED;
+    }
+    SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
+    SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp), lp.shard_rank, lp.shard_count, l1));
+    mk.l1 = tm.mark();
+    key_t* init_topk = nullptr;
+    if (lp.dense_mode != 1) {
+        SKNN_TRY(cx.alloc_scratch((void**)&init_topk, sizeof(key_t) * (size_t)qs.n * k));
+        SKNN_TRY(run_dense_tiles(cx, qs, l1));
+        DenseParams dpar;
+        dpar.k = k;
+        dpar.eta = eta;
+        dpar.topk_out = init_topk;
+        dpar.counters = counters;
+        SKNN_TRY(run_dense(cx, qs, ts, l1, dpar));
+        mk.dense = tm.mark();
+    }
     ScanParams sp;
     sp.k = k;
     sp.eta = eta;
@@ -205,13 +239,14 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     sp.out_idx = out_idx;
     sp.out_dist = out_dist;
     sp.counters = counters;
+    sp.init_topk = init_topk;
     SKNN_TRY(run_scan(cx, qs, ts, l1, sp));
-    *mk_scan = tm.mark();
+    mk.scan = tm.mark();
     return SKNN_OK;
 }
 
-static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt, const Timer& tm, int m_bt, int m_bq,
-                       int m_l1, int m_scan, int m_end, int mapping, int path, int mq, int mt, int launches) {
+static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt, const Timer& tm, const Marks& mk,
+                       int mapping, int path, int mq, int mt, int launches) {
     size_t sz = st->struct_size ? std::min(st->struct_size, sizeof(sknn_stats)) : sizeof(sknn_stats);
     sknn_stats s;
     memset(&s, 0, sizeof(s));
@@ -223,15 +258,17 @@ static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt
     s.center_evals = c.center_evals;
     s.cand_pairs = c.cand_pairs;
     s.dense_pairs = c.dense_pairs;
-    s.ms_total = tm.ms(0, m_end);
-    s.ms_build_t = tm.ms(0, m_bt);
-    s.ms_build_q = m_bq >= 0 ? tm.ms(m_bt, m_bq) : 0.f;
-    int prev = m_bq >= 0 ? m_bq : m_bt;
-    s.ms_level1 = m_l1 >= 0 ? tm.ms(prev, m_l1) : 0.f;
-    s.ms_sparse = m_scan >= 0 ? tm.ms(m_l1, m_scan) : 0.f;
+    s.dist_recompute = c.dist_recompute;
+    s.ms_total = tm.ms(0, mk.end);
+    s.ms_build_t = tm.ms(0, mk.bt);
+    s.ms_build_q = mk.bq >= 0 ? tm.ms(mk.bt, mk.bq) : 0.f;
+    const int prev = mk.bq >= 0 ? mk.bq : mk.bt;
+    s.ms_level1 = mk.l1 >= 0 ? tm.ms(prev, mk.l1) : 0.f;
+    s.ms_dense = mk.dense >= 0 ? tm.ms(mk.l1, mk.dense) : 0.f;
+    s.ms_sparse = mk.scan >= 0 ? tm.ms(mk.dense >= 0 ? mk.dense : mk.l1, mk.scan) : 0.f;
     s.ms_final = 0.f;
     s.mapping_used = mapping;
-    s.path_used = path;
+    s.path_used = (path == SKNN_PATH_BRUTE) ? path : (c.dense_pairs ? SKNN_PATH_DENSE : SKNN_PATH_SPARSE);
     s.mq = mq;
     s.mt = mt;
     s.kernel_launches = launches;
@@ -268,7 +305,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     const bool self = index ? (Q == index->user_ptr && nq == index->t.n) : (Q == T && nq == nt);
     int mapping = choose_mapping(o, di, nq, dp);
     int path = o.force_path == SKNN_PATH_BRUTE ? SKNN_PATH_BRUTE : SKNN_PATH_SPARSE;
-    int m_bt = -1, m_bq = -1, m_l1 = -1, m_scan = -1, m_end = -1;
+    Marks mk;
     int mq = 0, mt = 0;
     Counters host_c;
     memset(&host_c, 0, sizeof(host_c));
@@ -314,8 +351,8 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
             sp.counters = counters;
             mapping = SKNN_MAP_WARP;
             st = run_brute(cx, dQ, nq, dT, nt, d, sp);
-            m_bt = tm.mark();
-            m_scan = m_bt;
+            mk.bt = tm.mark();
+            mk.scan = mk.bt;
             break;
         }
         Side ts_local, qs_local;
@@ -328,7 +365,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
                 break;
             ts = &ts_local;
         }
-        m_bt = tm.mark();
+        mk.bt = tm.mark();
         const Side* qs;
         if (self) {
             qs = ts;
@@ -338,11 +375,11 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
                 SKNN_OK)
                 break;
             qs = &qs_local;
-            m_bq = tm.mark();
+            mk.bq = tm.mark();
         }
         mq = qs->m;
         mt = ts->m;
-        st = query_core(cx, *qs, *ts, k, o, mapping, d_oidx, d_odist, counters, tm, &m_l1, &m_scan);
+        st = query_core(cx, *qs, *ts, k, o, mapping, d_oidx, d_odist, counters, tm, mk);
     } while (0);
     if (st == SKNN_OK) {
         if (oi_host) {
@@ -354,7 +391,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
             if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("D2H out_dist: ") + cudaGetErrorString(e));
         }
         if (stats && counters) cudaMemcpyAsync(&host_c, counters, sizeof(Counters), cudaMemcpyDeviceToHost, stream);
-        m_end = tm.mark();
+        mk.end = tm.mark();
     }
     int launches = cx.launches;
     cx.free_all();
@@ -363,7 +400,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
         if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("kernel execution failed: ") + cudaGetErrorString(e));
     }
     if (st == SKNN_OK && stats)
-        fill_stats(stats, host_c, nq, nt, tm, m_bt, m_bq, m_l1, m_scan, m_end, mapping, path, mq, mt, launches);
+        fill_stats(stats, host_c, nq, nt, tm, mk, mapping, path, mq, mt, launches);
     return st;
 }
 
@@ -527,7 +564,11 @@ sknn_status sknn_debug_level1(const sknn_index* ix, const float* Q, int64_t nq, 
                 break;
             qs = &qs_local;
         }
-        if ((st = run_level1(cx, *qs, ts, k, rounding_eta(ts.d), 0, 1, l1, nullptr)) != SKNN_OK) break;
+        Level1Params lp;
+        lp.k = k;
+        lp.eta = rounding_eta(ts.d);
+        lp.dense_mode = 1;  // report the full candidate list in `cand`
+        if ((st = run_level1(cx, *qs, ts, lp, l1, nullptr)) != SKNN_OK) break;
         cudaError_t e = cudaStreamSynchronize(nullptr);
         if (e != cudaSuccess) {
             st = fail(SKNN_ERR_CUDA, std::string("level-1 failed: ") + cudaGetErrorString(e));

@@ -105,8 +105,9 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     const float* __restrict__ qcent, const float* __restrict__ qrad, const int32_t* __restrict__ qoff,
     const float* __restrict__ tcent, const float* __restrict__ trad, const int32_t* __restrict__ toff,
     const float* __restrict__ tdist, int mt, int dp, int k, float eta, int keys_cap, int shard_rank,
-    int shard_count, float* __restrict__ ub_out, int32_t* __restrict__ cand, int32_t* __restrict__ cand_count,
-    unsigned long long* __restrict__ cand_pairs) {
+    int shard_count, int dense_mode, float dense_tau, float* __restrict__ ub_out, int32_t* __restrict__ cand,
+    int32_t* __restrict__ cand_count, int32_t* __restrict__ dcand, int32_t* __restrict__ dcount,
+    Counters* __restrict__ counters) {
     extern __shared__ __align__(16) unsigned char smem[];
     u64* s_keys = reinterpret_cast<u64*>(smem);                               // keys_cap (>= mt) entries
     float* s_D = reinterpret_cast<float*>(smem + sizeof(u64) * keys_cap);     // [mt] center distances
@@ -120,7 +121,7 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     const int qc = blockIdx.x;
     const int qsize = qoff[qc + 1] - qoff[qc];
     if (qsize == 0 || (shard_count > 1 && qc % shard_count != shard_rank)) {
-        if (threadIdx.x == 0) { ub_out[qc] = 0.f; cand_count[qc] = 0; }
+        if (threadIdx.x == 0) { ub_out[qc] = 0.f; cand_count[qc] = 0; dcount[qc] = 0; }
         return;
     }
     for (int i = threadIdx.x; i < dp; i += blockDim.x) s_qc[i] = qcent[(int64_t)qc * dp + i];
@@ -194,20 +195,69 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     for (int i = nc + threadIdx.x; i < S; i += blockDim.x) s_keys[i] = ~0ull;
     __syncthreads();
     block_sort_u64(s_keys, S);
+    // elastic switch (S8): split the sorted candidates into the sparse list
+    // (point-level scan, Alg. 2) and the dense-tile list (tensor cores),
+    // stable in ascending D. auto: a pair is dense when the cluster-level
+    // window 2*UB covers at least tau of the member-distance range r_t and the
+    // cluster is big enough to fill tiles (cost model in DESIGN.md §6).
     int32_t* row = cand + (int64_t)qc * mt;
-    for (int i = threadIdx.x; i < nc; i += blockDim.x) row[i] = int32_t(uint32_t(s_keys[i] & 0xffffffffu));
+    int32_t* drow = dcand + (int64_t)qc * mt;
+    __shared__ int s_wcnt[2][kL1Threads / 32];
+    __shared__ int s_base[2];
+    if (threadIdx.x == 0) { s_base[0] = 0; s_base[1] = 0; }
+    __syncthreads();
+    for (int base = 0; base < nc; base += blockDim.x) {
+        const int i = base + threadIdx.x;
+        int tc = -1;
+        bool dense = false;
+        if (i < nc) {
+            tc = int32_t(uint32_t(s_keys[i] & 0xffffffffu));
+            if (dense_mode == 2) {
+                dense = true;
+            } else if (dense_mode == 0) {
+                const int sz = __ldg(toff + tc + 1) - __ldg(toff + tc);
+                dense = sz >= 16 && 2.f * UB >= dense_tau * __ldg(trad + tc);
+            }
+        }
+        const unsigned md = __ballot_sync(0xffffffffu, i < nc && dense);
+        const unsigned ms = __ballot_sync(0xffffffffu, i < nc && !dense);
+        const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+        if (lane == 0) { s_wcnt[0][w] = __popc(ms); s_wcnt[1][w] = __popc(md); }
+        __syncthreads();
+        int offs = 0, offd = 0;
+        for (int ww = 0; ww < w; ++ww) { offs += s_wcnt[0][ww]; offd += s_wcnt[1][ww]; }
+        const unsigned below = (1u << lane) - 1u;
+        if (i < nc) {
+            if (dense) drow[s_base[1] + offd + __popc(md & below)] = tc;
+            else row[s_base[0] + offs + __popc(ms & below)] = tc;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int ts = 0, td = 0;
+            for (int ww = 0; ww < kL1Threads / 32; ++ww) { ts += s_wcnt[0][ww]; td += s_wcnt[1][ww]; }
+            s_base[0] += ts;
+            s_base[1] += td;
+        }
+        __syncthreads();
+    }
     if (threadIdx.x == 0) {
-        cand_count[qc] = nc;
-        if (cand_pairs) atomicAdd(cand_pairs, (unsigned long long)nc);
+        cand_count[qc] = s_base[0];
+        dcount[qc] = s_base[1];
+        if (counters) {
+            atomicAdd(&counters->cand_pairs, (unsigned long long)nc);
+            if (s_base[1]) atomicAdd(&counters->dense_pairs, (unsigned long long)s_base[1]);
+        }
     }
 }
 
-sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, int k, float eta, int shard_rank, int shard_count,
-                       Level1& out, unsigned long long* cand_pairs_counter) {
+sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Params& p, Level1& out,
+                       Counters* counters) {
     const int mq = qs.m, mt = ts.m, dp = ts.dp;
     SKNN_TRY(cx.alloc_scratch((void**)&out.ub, sizeof(float) * mq));
     SKNN_TRY(cx.alloc_scratch((void**)&out.cand, sizeof(int32_t) * (size_t)mq * mt));
     SKNN_TRY(cx.alloc_scratch((void**)&out.cand_count, sizeof(int32_t) * mq));
+    SKNN_TRY(cx.alloc_scratch((void**)&out.dcand, sizeof(int32_t) * (size_t)mq * mt));
+    SKNN_TRY(cx.alloc_scratch((void**)&out.dcount, sizeof(int32_t) * mq));
     int cap = 1;
     while (cap < mt) cap <<= 1;
     cap = std::max(cap, kL1Vals);
@@ -219,8 +269,9 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, int k, float eta
     }
     SKNN_CUDA(cudaFuncSetAttribute(k_level1, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     k_level1<<<mq, kL1Threads, smem, cx.stream>>>(qs.centers, qs.radius, qs.off, ts.centers, ts.radius, ts.off,
-                                                  ts.dist, mt, dp, k, eta, cap, shard_rank, shard_count, out.ub,
-                                                  out.cand, out.cand_count, cand_pairs_counter);
+                                                  ts.dist, mt, dp, p.k, p.eta, cap, p.shard_rank, p.shard_count,
+                                                  p.dense_mode, p.dense_tau, out.ub, out.cand, out.cand_count,
+                                                  out.dcand, out.dcount, counters);
     cx.launched();
     return cx.check_launch("level1");
 }

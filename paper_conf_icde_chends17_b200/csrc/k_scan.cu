@@ -50,7 +50,6 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
         const float ub = a.ub[qc];
         const int ncand = a.cand_count[qc];
         const int32_t* cl = a.cand + (int64_t)qc * a.mt;
-        const uint8_t* dense_row = a.pair_dense ? a.pair_dense + (int64_t)qc * a.mt : nullptr;
         for (int qi = 0; qi < nq_tile; ++qi) {
             const int qpos = qlo + tl.y + qi;
             float4 q[DP > 0 ? DP / 4 : 1];
@@ -63,12 +62,11 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
                 __syncwarp();
             }
             key_t mine = (lane < 32 - a.k) ? kNegKey : kInfKey;
-            if (a.init_topk && lane >= 32 - a.k) mine = a.init_topk[(int64_t)qpos * a.k + lane - (32 - a.k)];
+            if (a.init_topk && a.dcount[qc] > 0 && lane >= 32 - a.k) mine = a.init_topk[(int64_t)qpos * a.k + lane - (32 - a.k)];
             key_t kth = __shfl_sync(0xffffffffu, mine, 31);
             float theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
             for (int c = 0; c < ncand; ++c) {
                 const int tc = __ldg(cl + c);
-                if (dense_row && __ldg(dense_row + tc)) continue;
                 const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
                 float dq2;
                 if constexpr (DP > 0) dq2 = d2_reg<DP>(q, a.tcent + (int64_t)tc * DP);
@@ -116,8 +114,9 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
 // ---------------------------------------------------------------- tiles --
 // Single CTA: tiles of `tile` queries per non-empty query cluster.
 __global__ void __launch_bounds__(1024) k_make_tiles(const int32_t* __restrict__ qoff, int mq, int tile,
-                                                     int shard_rank, int shard_count, int2* __restrict__ tiles,
-                                                     int* __restrict__ ntiles, int* __restrict__ counter) {
+                                                     int shard_rank, int shard_count, const int32_t* __restrict__ need,
+                                                     int2* __restrict__ tiles, int* __restrict__ ntiles,
+                                                     int* __restrict__ counter) {
     __shared__ int s_sum[1024];
     __shared__ int s_carry;
     if (threadIdx.x == 0) s_carry = 0;
@@ -126,6 +125,7 @@ __global__ void __launch_bounds__(1024) k_make_tiles(const int32_t* __restrict__
         int c = base + threadIdx.x;
         int sz = (c < mq) ? qoff[c + 1] - qoff[c] : 0;
         if (shard_count > 1 && c % shard_count != shard_rank) sz = 0;
+        if (need && c < mq && need[c] == 0) sz = 0;
         int nt = (sz + tile - 1) / tile;
         s_sum[threadIdx.x] = nt;
         __syncthreads();
@@ -166,10 +166,22 @@ sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int shard_rank, int sha
     SKNN_TRY(cx.alloc_scratch((void**)&l1.tiles, sizeof(int2) * max_tiles));
     SKNN_TRY(cx.alloc_scratch((void**)&l1.ntiles, sizeof(int) * 2));
     l1.tile = tile;
-    k_make_tiles<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, l1.tiles, l1.ntiles,
-                                             l1.ntiles + 1);
+    k_make_tiles<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, nullptr, l1.tiles,
+                                             l1.ntiles, l1.ntiles + 1);
     cx.launched();
     return cx.check_launch("tiles");
+}
+
+// dense-tile work list: tiles of 128 queries of the clusters with dense pairs
+sknn_status run_dense_tiles(Ctx& cx, const Side& qs, Level1& l1) {
+    const int tile = 128;
+    int64_t max_tiles = (qs.n + tile - 1) / tile + qs.m;
+    SKNN_TRY(cx.alloc_scratch((void**)&l1.dtiles, sizeof(int2) * max_tiles));
+    SKNN_TRY(cx.alloc_scratch((void**)&l1.dntiles, sizeof(int) * 2));
+    k_make_tiles<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, 0, 1, l1.dcount, l1.dtiles, l1.dntiles,
+                                             l1.dntiles + 1);
+    cx.launched();
+    return cx.check_launch("dense tiles list");
 }
 
 sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
@@ -180,7 +192,7 @@ sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, 
     a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
     a.ub = l1.ub; a.cand = l1.cand; a.cand_count = l1.cand_count;
     a.tiles = l1.tiles; a.ntiles = l1.ntiles; a.tile_counter = l1.ntiles + 1;
-    a.init_topk = p.init_topk; a.pair_dense = p.pair_dense;
+    a.init_topk = p.init_topk; a.dcount = l1.dcount;
     a.mt = ts.m; a.dp = dp; a.k = p.k; a.tile = l1.tile; a.eta = p.eta;
     a.out_squared = p.out_squared; a.index_base = p.index_base; a.out_idx = p.out_idx; a.out_dist = p.out_dist;
     a.counters = p.counters;

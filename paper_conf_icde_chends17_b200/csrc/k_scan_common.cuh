@@ -27,7 +27,7 @@ struct ScanArgs {
     const int* ntiles;
     int* tile_counter;     // dynamic tile scheduler (zeroed by k_make_tiles)
     const key_t* init_topk;  // optional [nq_perm x k] keys from the dense-tile pass (NULL = none)
-    const uint8_t* pair_dense;  // optional [mq x mt] 1 = pair handled by the dense-tile pass
+    const int32_t* dcount;   // optional [mq] dense pairs per query cluster (init_topk valid iff > 0)
     int mt;
     int dp;
     int k;

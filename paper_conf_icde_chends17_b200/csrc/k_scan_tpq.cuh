@@ -42,7 +42,7 @@ __global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
         top.init(a.k);
         const float ub = a.ub[qc];
         float theta = ub;
-        if (a.init_topk) {  // continue from the dense-tile pass
+        if (a.init_topk && a.dcount[qc] > 0) {  // continue from the dense-tile pass
 #pragma unroll
             for (int s = 0; s < KMAX; ++s) {
                 const int r = s - (KMAX - a.k);
@@ -54,11 +54,9 @@ __global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
         float kth_d2 = key_d2(kth);
         const int ncand = a.cand_count[qc];
         const int32_t* cl = a.cand + (int64_t)qc * a.mt;
-        const uint8_t* dense_row = a.pair_dense ? a.pair_dense + (int64_t)qc * a.mt : nullptr;
         if (active) {
             for (int c = 0; c < ncand; ++c) {
                 const int tc = __ldg(cl + c);
-                if (dense_row && __ldg(dense_row + tc)) continue;  // covered by the dense tile pass
                 const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
                 const float dq = __fsqrt_rn(d2_reg<DP>(q, a.tcent + (int64_t)tc * DP));  // Alg. 2 line 6
                 ++cevals;

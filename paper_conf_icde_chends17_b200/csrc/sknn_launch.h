@@ -90,11 +90,33 @@ struct Level1 {
     int32_t* cand = nullptr;      // [mq x mt] candidate target clusters, ascending center distance
     int32_t* cand_count = nullptr;  // [mq]
     int2* tiles = nullptr;        // level-2 work tiles (query cluster, first member)
-    int* ntiles = nullptr;
+    int* ntiles = nullptr;        // [2]: tile count, scheduler counter
     int tile = 0;
+    int32_t* dcand = nullptr;     // [mq x mt] dense-tile candidates (elastic switch), ascending D
+    int32_t* dcount = nullptr;    // [mq]
+    int2* dtiles = nullptr;       // dense work tiles (128 queries of one cluster)
+    int* dntiles = nullptr;       // [2]
 };
-sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, int k, float eta, int shard_rank, int shard_count,
-                       Level1& out, unsigned long long* cand_pairs_counter);
+struct Level1Params {
+    int k = 0;
+    float eta = 0.f;
+    int shard_rank = 0, shard_count = 1;
+    int dense_mode = 0;           // 0 auto (cost model), 1 never, 2 every candidate pair
+    float dense_tau = 1.f;        // auto: dense iff |tc| >= 16 and 2*UB >= tau * r_t
+};
+sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Params& p, Level1& out,
+                       Counters* counters);
+// k_dense.cu
+struct DenseParams {
+    int k = 0;
+    float eta = 0.f;
+    key_t* topk_out = nullptr;
+    Counters* counters = nullptr;
+};
+int dense_kp(int dp);
+bool dense_supported(int dp);
+sknn_status run_dense_tiles(Ctx& cx, const Side& qs, Level1& l1);
+sknn_status run_dense(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const DenseParams& p);
 // k_scan.cu: tiles of `tile` queries of one query cluster (thread-data remapping)
 sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int shard_rank, int shard_count, Level1& l1);
 int scan_tile_size(int mapping, int dp);
@@ -110,7 +132,6 @@ struct ScanParams {
     float* out_dist = nullptr;
     Counters* counters = nullptr;
     const key_t* init_topk = nullptr;    // dense-tile pass results to continue from
-    const uint8_t* pair_dense = nullptr; // [mq x mt] pairs already covered by dense tiles
 };
 sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p);
 sknn_status run_brute(Ctx& cx, const float* Q, int64_t nq, const float* T, int64_t nt, int d, const ScanParams& p);

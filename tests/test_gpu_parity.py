@@ -234,3 +234,52 @@ def test_c2_full_size_sampled(sknn):
     _, rdist = oracle.knn_join(Q[s], T, k)
     assert_knn_tolerant(Q[s], T, idx[s], dist[s], rdist)
     assert st["pruned_pct"] > 99.0
+
+
+# ------------------------------------------------------------ dense tiles --
+@pytest.mark.parametrize("name,scale", [("C1", 1.0), ("C3int", 0.05), ("C4", 0.004), ("C5", 0.0025)])
+@pytest.mark.parametrize("mapping", ["thread", "warp"])
+def test_dense_tiles_bitexact(sknn, name, scale, mapping):
+    """S11: every surviving cluster pair through the tcgen05 dense-tile screen
+    (force_path=dense) -- results must stay bit-identical to the oracle."""
+    Q, T, k, sj = datagen.workload(name, scale)
+    idx, dist, st = run(sknn, Q, T, k, sj, force_path="dense", mapping=mapping)
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    assert st["dense_pairs"] > 0 and st["dist_evals_dense"] > 0
+    assert st["dist_evals_sparse"] == 0
+
+
+@pytest.mark.parametrize("name,scale", [("C2", 0.05), ("C3", 0.1)])
+def test_dense_tiles_real_tolerant(sknn, name, scale):
+    Q, T, k, sj = datagen.workload(name, scale)
+    idx, dist, st = run(sknn, Q, T, k, sj, force_path="dense")
+    _, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_tolerant(Q, T, idx, dist, rdist)
+    assert st["dense_pairs"] > 0
+
+
+def test_dense_tiles_ties_and_dims(sknn):
+    X = datagen.sphere_ties()
+    Q = np.concatenate([np.zeros((3, 4), np.float32), X[:40]], axis=0)
+    for k in (1, 17, 32):
+        idx, dist, _ = run(sknn, Q, X, k, False, force_path="dense")
+        ridx, rdist = oracle.knn_join(Q, X, k)
+        assert_knn_bitexact(idx, dist, ridx, rdist)
+    rng = np.random.default_rng(17)
+    for d in (3, 16, 33, 100, 130):
+        T = rng.integers(0, 40, size=(2500, d)).astype(np.float32)
+        Qd = rng.integers(0, 40, size=(300, d)).astype(np.float32)
+        idx, dist, _ = run(sknn, Qd, T, 9, False, force_path="dense")
+        ridx, rdist = oracle.knn_join(Qd, T, 9)
+        assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+def test_auto_switch_mixes_paths(sknn):
+    """The elastic switch (auto) on a dp >= 16 workload sends some pairs to
+    dense tiles and the rest to the sparse scan; results stay exact."""
+    Q, T, k, sj = datagen.workload("C5", 0.0025)
+    idx, dist, st = run(sknn, Q, T, k, sj)
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    assert st["dense_pairs"] > 0

@@ -23,6 +23,9 @@ VARIANTS = {
     "lloyd1": {"lloyd_iters": 1},
     "lloyd4": {"lloyd_iters": 4},
     "thread": {"mapping": "thread"},
+    "sparse": {"force_path": "sparse"},
+    "dense": {"force_path": "dense"},
+    "tau4": {"dense_threshold": 4.0},
     "warp": {"mapping": "warp"},
     "cl_half": {"_cl": 0.5},
     "cl_double": {"_cl": 2.0},
@@ -70,7 +73,8 @@ def main():
                    "ms_min": float(np.min(ms)), "queries_per_s": nq / (np.median(ms) / 1000.0),
                    "pruned_pct": med["pruned_pct"], "evals_per_query": med["dist_evals"] / nq,
                    "cand_per_qcluster": med["cand_pairs"] / max(1, med["mq"]), "center_evals_per_query": med["center_evals"] / nq,
-                   "stages": {k2: round(med[k2], 4) for k2 in ("ms_build_t", "ms_build_q", "ms_level1", "ms_sparse")},
+                   "stages": {k2: round(med[k2], 4) for k2 in ("ms_build_t", "ms_build_q", "ms_level1", "ms_dense", "ms_sparse")},
+                   "dense_pairs": med["dense_pairs"], "evals_dense": med["dist_evals_dense"], "recompute": med["dist_recompute"],
                    "mq": med["mq"], "mt": med["mt"], "mapping": med["mapping_used"], "launches": med["kernel_launches"]}
             print(json.dumps(out), flush=True)
 
