@@ -3,9 +3,10 @@
 // dense, regularity beats per-point TI checks).
 //
 // For a tile of up to 128 queries of one query cluster and each of its dense
-// candidate target clusters, the member window (union of the rows' Alg. 2
-// windows) is streamed through shared memory in chunks of NCH targets and the
-// 128 x NCH dot products run on the 5th-generation tensor cores:
+// candidate target clusters, the whole target cluster (no per-point TI checks:
+// the regular path of the elastic switch) is streamed through shared memory in
+// chunks of NCH targets and the 128 x NCH dot products run on the
+// 5th-generation tensor cores:
 //
 //   a = q - c_r, b = t - c_r            (c_r = query-cluster center rounded to
 //                                        integers: re-centring avoids the
@@ -134,18 +135,6 @@ __device__ __forceinline__ bool split8(const float (&v)[8], uint4& hi, uint4& lo
     return nz;
 }
 
-// first position in [lo, hi) where Alg. 2 breaks (l = dq - dt > theta, line 10)
-__device__ __forceinline__ int window_end(const float* __restrict__ tdist, int lo, int hi, float dq, float theta,
-                                          float eta) {
-    while (lo < hi) {
-        int mid = (lo + hi) >> 1;
-        float dt = __ldg(tdist + mid);
-        if (ti_keep(dq - dt, theta, dq + dt, eta)) lo = mid + 1;
-        else hi = mid;
-    }
-    return lo;
-}
-
 template <int KMAX, int NCH>
 __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
     extern __shared__ __align__(128) unsigned char smem[];
@@ -160,7 +149,7 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
     float* s_cr = s_tn + NCH;                                             // [KP]
     __shared__ uint64_t s_bar;
     __shared__ uint32_t s_tmem;
-    __shared__ int s_tile, s_w0, s_w1, s_loA, s_loB;
+    __shared__ int s_tile, s_loA, s_loB;
 
     const int tid = threadIdx.x, warp = tid >> 5;
     if (warp == 0) {
@@ -238,35 +227,38 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
         for (int ci = 0; ci < nd; ++ci) {
             const int tc = __ldg(dl + ci);
             const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
-            // the tile's member window: union of the rows' Alg. 2 windows
-            int w0 = hi, w1 = lo;
-            if (active) {
-                const float dq = __fsqrt_rn(d2_rows(qrow, a.tcent + (int64_t)tc * dp, dp));
-                w0 = window_start(a.tdist, lo, hi, dq, theta, a.eta);
-                w1 = window_end(a.tdist, w0, hi, dq, theta, a.eta);
-            }
-            if (tid == 0) { s_w0 = hi; s_w1 = lo; }
-            __syncthreads();
-            if (w0 < w1) { atomicMin(&s_w0, w0); atomicMax(&s_w1, w1); }
-            __syncthreads();
-            const int W0 = s_w0, W1 = s_w1;
+            // dense pair: the whole target cluster is screened (no per-point TI
+            // checks -- the regular tiled path of the elastic switch)
+            const int W0 = lo, W1 = hi;
             for (int j0 = W0; j0 < W1; j0 += NCH) {
                 const int nb = min(NCH, W1 - j0);
                 // stage B = t - c_r and ||b||^2 (1 - eps)
                 if (tid == 0) s_loB = 0;
                 __syncthreads();
                 {
-                    const int c8n = KP / 8;
+                    // TPR threads per target row; each converts a contiguous K range
+                    constexpr int TPR = kDenseM / NCH;
+                    const int row = tid / TPR, part = tid % TPR;
+                    const int c8n = KP / 8, c8per = c8n / TPR;
+                    const bool rv = row < nb;
+                    const float4* src4 = reinterpret_cast<const float4*>(a.trows + (int64_t)(j0 + (rv ? row : 0)) * dp);
+                    const float4* cr4 = reinterpret_cast<const float4*>(s_cr);
                     bool nz = false;
-                    for (int w = tid; w < NCH * c8n; w += blockDim.x) {
-                        const int row = w / c8n, c8 = w % c8n;
-                        const bool rv = row < nb;
-                        const float* src = a.trows + (int64_t)(j0 + (rv ? row : 0)) * dp;
+                    float tn = 0.f;
+#pragma unroll 4
+                    for (int c8 = part * c8per; c8 < (part + 1) * c8per; ++c8) {
                         float v[8];
 #pragma unroll
-                        for (int i = 0; i < 8; ++i) {
-                            const int kk = c8 * 8 + i;
-                            v[i] = (rv && kk < dp) ? __ldg(src + kk) - s_cr[kk] : 0.f;
+                        for (int h = 0; h < 2; ++h) {
+                            const int k4 = c8 * 2 + h;
+                            float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+                            if (rv && k4 * 4 < dp) {
+                                const float4 t4 = __ldg(src4 + k4), c4 = cr4[k4];
+                                x = make_float4(t4.x - c4.x, t4.y - c4.y, t4.z - c4.z, t4.w - c4.w);
+                            }
+                            v[4 * h + 0] = x.x; v[4 * h + 1] = x.y; v[4 * h + 2] = x.z; v[4 * h + 3] = x.w;
+                            tn = __fmaf_rn(x.x, x.x, tn); tn = __fmaf_rn(x.y, x.y, tn);
+                            tn = __fmaf_rn(x.z, x.z, tn); tn = __fmaf_rn(x.w, x.w, tn);
                         }
                         uint4 hi4, lo4;
                         nz |= split8(v, hi4, lo4);
@@ -274,19 +266,9 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
                         *reinterpret_cast<uint4*>(sB_hi + off) = hi4;
                         *reinterpret_cast<uint4*>(sB_lo + off) = lo4;
                     }
-                    for (int row = tid; row < NCH; row += blockDim.x) {
-                        float tn = INF;
-                        if (row < nb) {
-                            const float* src = a.trows + (int64_t)(j0 + row) * dp;
-                            tn = 0.f;
-                            for (int c = 0; c < dp; ++c) {
-                                const float x = __ldg(src + c) - s_cr[c];
-                                tn = __fmaf_rn(x, x, tn);
-                            }
-                            tn *= (1.f - a.eps_tc);
-                        }
-                        s_tn[row] = tn;
-                    }
+#pragma unroll
+                    for (int o = 1; o < TPR; o <<= 1) tn += __shfl_xor_sync(0xffffffffu, tn, o);
+                    if (part == 0) s_tn[row] = rv ? tn * (1.f - a.eps_tc) : INF;
                     if (__syncthreads_or(nz) && tid == 0) s_loB = 1;
                 }
                 fence_async_smem();

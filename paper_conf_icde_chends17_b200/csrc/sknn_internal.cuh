@@ -50,6 +50,7 @@ __device__ __forceinline__ float d2_rows(const float* __restrict__ a, const floa
     const float4* a4 = reinterpret_cast<const float4*>(a);
     const float4* b4 = reinterpret_cast<const float4*>(b);
     float s = 0.f;
+#pragma unroll 8
     for (int c = 0; c < dp / 4; ++c) s = d2_acc4(s, a4[c], __ldg(b4 + c));
     return s;
 }
