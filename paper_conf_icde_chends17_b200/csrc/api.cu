@@ -210,7 +210,7 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     lp.shard_rank = o.shard_count > 1 ? o.shard_rank : 0;
     lp.shard_count = o.shard_count > 1 ? o.shard_count : 1;
     lp.dense_mode = dense_mode_for(o, ts.dp);
-    lp.dense_tau = o.dense_threshold > 0.f ? o.dense_threshold : 1.f;
+    lp.dense_tau = o.dense_threshold > 0.f ? o.dense_threshold : 0.5f;
     if (lp.dense_mode == 2 && !dense_supported(ts.dp)) {
         set_last_error("force_path = DENSE needs d <= 256");
         return SKNN_ERR_UNSUPPORTED;

@@ -1,0 +1,279 @@
+// k_assign_tc.cu -- Step 1 assignment screen on the tensor cores (SURVEY §8(a)
+// S3: "argmin_c ||x - c|| ... screen: tensor cores"; P:L323-331 assign every
+// point to its closest landmark).
+//
+// The assignment only has to be approximate (reading R9: TI validity needs the
+// RECORDED member-center distance to be exact, not the nearest center), so the
+// nearest center is chosen from
+//     score_j = ||b_j||^2 - 2 a.b_j,   a = x - o, b_j = c_j - o   (o = mean center)
+// with a and b rounded to bf16 and a.b_j accumulated in fp32 by tcgen05.mma
+// (kind::f16, M = 128 points x N = 128 centers per MMA, K = d padded to 16);
+// ||a||^2 is the same for every j and drops out of the argmin. The exact fp32
+// distance to the chosen center (the shared d2 formula) is then recomputed.
+//
+// Data movement: the centers are pre-converted once per pass into the UMMA
+// canonical K-major layout (8-row x 16-byte core matrices), chunk by chunk, so a
+// CTA streams them with 1-D bulk async copies (cp.async.bulk, the TMA engine)
+// into a double-buffered shared-memory ring while the previous chunk's MMA
+// result is reduced from TMEM (tcgen05.ld) by the four epilogue warps.
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "sknn_internal.cuh"
+#include "sknn_launch.h"
+
+namespace sknn {
+
+constexpr int kTcM = 128;   // points per CTA (TMEM lanes)
+constexpr int kTcN = 128;   // centers per chunk (TMEM columns per accumulator)
+
+__device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ uint64_t desc_kmajor(uint32_t saddr, uint32_t sbo) {
+    return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)(128u >> 4) << 16) | ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) |
+           ((uint64_t)1 << 46);
+}
+
+__device__ __forceinline__ void mma_bf16_f32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+
+__device__ __forceinline__ void wait_parity(uint32_t bar, uint32_t ph) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\tW_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@!P1 bra W_%=;\n\t}\n" ::"r"(bar),
+        "r"(ph)
+        : "memory");
+}
+
+__device__ __forceinline__ void ld32(uint32_t taddr, uint32_t (&r)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+__host__ __device__ constexpr uint32_t idesc_bf16_m128(int n) {
+    return (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(n >> 3) << 17) | (uint32_t(kTcM >> 4) << 24);
+}
+
+// o = mean of the m centers (one CTA, fixed order per column)
+__global__ void k_center_mean(const float* __restrict__ centers, int m, int dp, float* __restrict__ o) {
+    for (int c = threadIdx.x; c < dp; c += blockDim.x) {
+        double s = 0.0;
+        for (int j = 0; j < m; ++j) s += centers[(int64_t)j * dp + c];
+        o[c] = (float)(s / m);
+    }
+}
+
+// centers -> bf16 (c - o) in chunked core-matrix layout + ||b||^2 of the rounded values
+__global__ void k_centers_to_tc(const float* __restrict__ centers, int m, int mpad, int dp, int kp,
+                                const float* __restrict__ o, __nv_bfloat16* __restrict__ out, float* __restrict__ bn) {
+    const int c8n = kp / 8;
+    const int64_t total = (int64_t)mpad * c8n;
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < total; w += (int64_t)gridDim.x * blockDim.x) {
+        const int j = (int)(w / c8n), c8 = (int)(w % c8n);
+        uint32_t h[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            float v0 = 0.f, v1 = 0.f;
+            const int k0 = c8 * 8 + 2 * i;
+            if (j < m && k0 < dp) v0 = centers[(int64_t)j * dp + k0] - o[k0];
+            if (j < m && k0 + 1 < dp) v1 = centers[(int64_t)j * dp + k0 + 1] - o[k0 + 1];
+            h[i] = (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v0)) |
+                   ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v1)) << 16);
+        }
+        const int chunk = j / kTcN, r = j % kTcN;
+        const size_t off = (size_t)chunk * kTcN * kp * 2 + (size_t)(r >> 3) * kp * 16 + (size_t)c8 * 128 + (size_t)(r & 7) * 16;
+        *reinterpret_cast<uint4*>(reinterpret_cast<unsigned char*>(out) + off) = make_uint4(h[0], h[1], h[2], h[3]);
+    }
+    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < mpad; j += gridDim.x * blockDim.x) {
+        float s = __int_as_float(0x7f800000);
+        if (j < m) {
+            s = 0.f;
+            for (int k = 0; k < dp; ++k) {
+                const float v = __bfloat162float(__float2bfloat16_rn(centers[(int64_t)j * dp + k] - o[k]));
+                s = __fmaf_rn(v, v, s);
+            }
+        }
+        bn[j] = s;
+    }
+}
+
+// One CTA = 128 points; streams every center chunk through a 2-deep bulk-copy ring.
+__global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__ Xp, int64_t n, int dp, int kp,
+                                                       const float* __restrict__ o,
+                                                       const __nv_bfloat16* __restrict__ cbf,
+                                                       const float* __restrict__ bn, int m, int nchunks,
+                                                       const float* __restrict__ centers,
+                                                       int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
+                                                       float* __restrict__ sums, int32_t* __restrict__ counts) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t a_bytes = (uint32_t)kTcM * kp * 2, b_bytes = (uint32_t)kTcN * kp * 2;
+    unsigned char* sA = smem;
+    auto sB = [&](int b) { return smem + a_bytes + (uint32_t)b * b_bytes; };
+    auto sBn = [&](int b) { return reinterpret_cast<float*>(smem + a_bytes + 2 * b_bytes) + b * kTcN; };
+    __shared__ __align__(8) uint64_t bar_full[2], bar_mma[2];
+    __shared__ uint32_t s_tmem;
+    const int tid = threadIdx.x, warp = tid >> 5;
+    const uint32_t sbo = (uint32_t)kp * 16u;
+
+    if (warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(&s_tmem)),
+                     "r"(2u * kTcN));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (tid == 0) {
+        for (int i = 0; i < 2; ++i) {
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar_full[i])));
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar_mma[i])));
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    // stage A = x - o (bf16) for the CTA's 128 points
+    const int64_t row0 = (int64_t)blockIdx.x * kTcM;
+    {
+        const int c8n = kp / 8;
+        for (int w = tid; w < kTcM * c8n; w += blockDim.x) {
+            const int r = w / c8n, c8 = w % c8n;
+            const int64_t i = row0 + r;
+            uint32_t h[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                float v0 = 0.f, v1 = 0.f;
+                const int k0 = c8 * 8 + 2 * e;
+                if (i < n && k0 < dp) v0 = Xp[i * dp + k0] - o[k0];
+                if (i < n && k0 + 1 < dp) v1 = Xp[i * dp + k0 + 1] - o[k0 + 1];
+                h[e] = (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v0)) |
+                       ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v1)) << 16);
+            }
+            const uint32_t off = (uint32_t)(r >> 3) * sbo + (uint32_t)c8 * 128u + (uint32_t)(r & 7) * 16u;
+            *reinterpret_cast<uint4*>(sA + off) = make_uint4(h[0], h[1], h[2], h[3]);
+        }
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = s_tmem;
+    const uint32_t idesc = idesc_bf16_m128(kTcN);
+
+    auto issue_copy = [&](int chunk, int buf) {
+        const uint32_t bar = su32(&bar_full[buf]);
+        const uint32_t bytes = b_bytes + kTcN * 4;
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+        const unsigned char* src = reinterpret_cast<const unsigned char*>(cbf) + (size_t)chunk * b_bytes;
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(su32(sB(buf))),
+            "l"(src), "r"(b_bytes), "r"(bar)
+            : "memory");
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(su32(sBn(buf))),
+            "l"(bn + (size_t)chunk * kTcN), "r"((uint32_t)(kTcN * 4)), "r"(bar)
+            : "memory");
+    };
+    auto issue_mma = [&](int buf) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const uint32_t aB = su32(sA), bB = su32(sB(buf));
+        for (int s = 0; s < kp / 16; ++s)
+            mma_bf16_f32(tmem + (uint32_t)(buf * kTcN), desc_kmajor(aB + s * 256u, sbo), desc_kmajor(bB + s * 256u, sbo),
+                         idesc, s > 0);
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                         su32(&bar_mma[buf]))
+                     : "memory");
+    };
+
+    uint32_t ph_full[2] = {0, 0}, ph_mma[2] = {0, 0};
+    if (tid == 0) {
+        issue_copy(0, 0);
+        if (nchunks > 1) issue_copy(1, 1);
+        wait_parity(su32(&bar_full[0]), 0);
+        issue_mma(0);
+    }
+    ph_full[0] = 1;
+    float best = __int_as_float(0x7f800000);
+    int bi = 0;
+    const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
+    for (int c = 0; c < nchunks; ++c) {
+        const int buf = c & 1;
+        // issue the next chunk's MMA as soon as its copy landed (overlaps this epilogue)
+        if (tid == 0 && c + 1 < nchunks) {
+            const int nb = (c + 1) & 1;
+            wait_parity(su32(&bar_full[nb]), ph_full[nb]);
+            issue_mma(nb);
+        }
+        if (c + 1 < nchunks) ph_full[(c + 1) & 1] ^= 1u;
+        wait_parity(su32(&bar_mma[buf]), ph_mma[buf]);
+        ph_mma[buf] ^= 1u;
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const float* bnv = sBn(buf);
+#pragma unroll 1
+        for (int cb = 0; cb < kTcN / 32; ++cb) {
+            uint32_t v[32];
+            ld32(trow + (uint32_t)(buf * kTcN + cb * 32), v);
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+                const float sc = __fmaf_rn(-2.f, __uint_as_float(v[j]), bnv[cb * 32 + j]);
+                if (sc < best) { best = sc; bi = c * kTcN + cb * 32 + j; }
+            }
+        }
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncthreads();  // buffer `buf` (smem + TMEM) is free again
+        if (tid == 0 && c + 2 < nchunks) issue_copy(c + 2, buf);
+    }
+    const int64_t i = row0 + tid;
+    if (i < n) {
+        bi = min(bi, m - 1);
+        const float* xr = Xp + i * dp;
+        const float d2 = d2_rows(xr, centers + (int64_t)bi * dp, dp);  // exact fp32, shared formula
+        if (cid_out) cid_out[i] = bi;
+        if (dist_out) dist_out[i] = __fsqrt_rn(d2);
+        if (counts) atomicAdd(counts + bi, 1);
+        if (sums)
+            for (int c = 0; c < dp; ++c) atomicAdd(sums + (int64_t)bi * dp + c, xr[c]);
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(2u * kTcN));
+}
+
+bool assign_tc_supported(int dp) { return dp >= 8 && ((dp + 15) & ~15) <= 256; }
+
+sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m, int32_t* cid,
+                          float* dist, float* sums, int32_t* counts) {
+    const int kp = (dp + 15) & ~15;
+    const int nchunks = (m + kTcN - 1) / kTcN;
+    const int mpad = nchunks * kTcN;
+    float* o;
+    __nv_bfloat16* cbf;
+    float* bn;
+    SKNN_TRY(cx.alloc_scratch((void**)&o, sizeof(float) * dp));
+    SKNN_TRY(cx.alloc_scratch((void**)&cbf, (size_t)mpad * kp * 2));
+    SKNN_TRY(cx.alloc_scratch((void**)&bn, sizeof(float) * mpad));
+    k_center_mean<<<1, 128, 0, cx.stream>>>(centers, m, dp, o);
+    cx.launched();
+    const int64_t work = (int64_t)mpad * (kp / 8);
+    k_centers_to_tc<<<(int)std::min<int64_t>((work + 255) / 256, 148 * 8), 256, 0, cx.stream>>>(centers, m, mpad, dp, kp,
+                                                                                                o, cbf, bn);
+    cx.launched();
+    // >= 90 KB keeps at most two CTAs per SM: each holds 256 of the 512 TMEM columns
+    const size_t smem = std::max<size_t>((size_t)kTcM * kp * 2 + 2 * (size_t)kTcN * kp * 2 + 2 * kTcN * 4, 90 * 1024);
+    SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const int64_t grid = (n + kTcM - 1) / kTcM;
+    k_assign_tc<<<(unsigned)grid, kTcM, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, bn, m, nchunks, centers, cid, dist,
+                                                          sums, counts);
+    cx.launched();
+    return cx.check_launch("assign (tensor cores)");
+}
+
+}  // namespace sknn

@@ -308,6 +308,57 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
     }
 }
 
+// ------------------------------------------------------------ D^2 seeding --
+__global__ void k_sum_sq(const float* __restrict__ dist, int64_t n, double* __restrict__ out) {
+    double s = 0.0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double v = dist[i];
+        s += v * v;
+    }
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    __shared__ double red[32];
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
+        atomicAdd(out, t);
+    }
+}
+
+// point i becomes a center with probability min(1, m1 * d2_i / S) (at most m1 kept)
+__global__ void k_d2_sample(const float* __restrict__ Xp, int64_t n, int dp, const float* __restrict__ dist,
+                            const double* __restrict__ S, int m1, uint64_t seed, float* __restrict__ centers,
+                            int* __restrict__ cnt) {
+    const double tot = *S;
+    if (!(tot > 0.0)) return;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double v = dist[i];
+        const double p = (double)m1 * v * v / tot;
+        const double u = (double)mix32(seed * 0x2545f4914f6cdd1dull + (uint64_t)i) * (1.0 / 4294967296.0);
+        if (u < p) {
+            const int pos = atomicAdd(cnt, 1);
+            if (pos < m1) {
+                const float4* src = reinterpret_cast<const float4*>(Xp + i * dp);
+                float4* dst = reinterpret_cast<float4*>(centers + (int64_t)pos * dp);
+                for (int c = 0; c < dp / 4; ++c) dst[c] = src[c];
+            }
+        }
+    }
+}
+
+// slots the sampling left empty get random points
+__global__ void k_d2_fill(const float* __restrict__ Xp, int64_t n, int dp, int m1, uint64_t seed,
+                          float* __restrict__ centers, const int* __restrict__ cnt) {
+    const int start = min(*cnt, m1);
+    for (int j = start + blockIdx.x * blockDim.x + threadIdx.x; j < m1; j += gridDim.x * blockDim.x) {
+        const uint32_t i = perm_index((uint32_t)j, (uint32_t)n, seed ^ 0xd2d2d2d2ull);
+        const float4* src = reinterpret_cast<const float4*>(Xp + (int64_t)i * dp);
+        float4* dst = reinterpret_cast<float4*>(centers + (int64_t)j * dp);
+        for (int c = 0; c < dp / 4; ++c) dst[c] = src[c];
+    }
+}
+
 __global__ void k_lloyd_update(float* __restrict__ centers, const float* __restrict__ sums,
                                const int32_t* __restrict__ counts, int m, int dp) {
     for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < m * dp; e += gridDim.x * blockDim.x) {
@@ -543,21 +594,28 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         cx.launched();
         Xp = tmp;
     }
+    // D^2 seeding split (reading R9): m0 landmarks from the paper's sampler
+    // (P:L321), the other m - m0 drawn with probability ~ squared distance to
+    // the nearest landmark (one k-means|| round), so small or far groups of
+    // points get a center instead of inflating a far cluster's radius.
+    const char* sd = getenv("SKNN_SEEDING");
+    const bool d2seed = !(sd && strcmp(sd, "paper") == 0) && m >= 64;
+    const int m0 = d2seed ? (m + 1) / 2 : m;
     // landmark sampler
     int32_t* lidx;
-    SKNN_TRY(cx.alloc_scratch((void**)&lidx, sizeof(int32_t) * trials * m));
-    k_landmark_draw<<<dim3((m + 255) / 256, trials), 256, 0, s>>>(n, m, trials, seed, lidx);
+    SKNN_TRY(cx.alloc_scratch((void**)&lidx, sizeof(int32_t) * trials * m0));
+    k_landmark_draw<<<dim3((m0 + 255) / 256, trials), 256, 0, s>>>(n, m0, trials, seed, lidx);
     cx.launched();
-    const int nb = (m + kLmTile - 1) / kLmTile;
+    const int nb = (m0 + kLmTile - 1) / kLmTile;
     const int ntile = nb * (nb + 1) / 2;
     double* partial;
     SKNN_TRY(cx.alloc_scratch((void**)&partial, sizeof(double) * trials * ntile));
     size_t lsm = dp <= 128 ? sizeof(float) * 2 * kLmTile * dp : 0;
     if (lsm > 48 * 1024)
         SKNN_CUDA(cudaFuncSetAttribute(k_landmark_sums, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lsm));
-    k_landmark_sums<<<dim3(ntile, trials), 256, lsm, s>>>(Xp, dp, m, lidx, nb, partial);
+    k_landmark_sums<<<dim3(ntile, trials), 256, lsm, s>>>(Xp, dp, m0, lidx, nb, partial);
     cx.launched();
-    k_landmark_pick<<<1, 512, 0, s>>>(partial, ntile, trials, lidx, m, Xp, dp, out.centers);
+    k_landmark_pick<<<1, 512, 0, s>>>(partial, ntile, trials, lidx, m0, Xp, dp, out.centers);
     cx.launched();
 
     int32_t* cid;
@@ -568,33 +626,40 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     SKNN_TRY(cx.alloc_scratch((void**)&pdist, sizeof(float) * n));
     SKNN_TRY(cx.alloc_scratch((void**)&counts, sizeof(int32_t) * m));
     SKNN_TRY(cx.alloc_scratch((void**)&cursor, sizeof(int32_t) * m));
-    // assignment: greedy walk on the center kNN graph (default) or the full
-    // all-centers scan (SKNN_ASSIGN=full, for ablation)
+    // assignment (approximate is enough, R9): tensor-core screen over all
+    // centers for dp >= 16 (k_assign_tc), greedy walk on the center kNN graph
+    // for low dp, exact all-centers SIMT scan otherwise. SKNN_ASSIGN=
+    // tc|walk|full overrides (ablation).
     const char* am = getenv("SKNN_ASSIGN");
-    const bool walk = !(am && strcmp(am, "full") == 0) && m > kNbr;
+    const bool force_full = am && strcmp(am, "full") == 0;
+    const bool force_walk = am && strcmp(am, "walk") == 0;
+    const bool force_tc = am && strcmp(am, "tc") == 0;
+    const bool use_tc = !force_full && !force_walk && assign_tc_supported(dp) && (force_tc || dp >= 16);
+    const bool walk = !use_tc && !force_full && m > kNbr;
     int32_t* nbr = nullptr;
     if (walk) SKNN_TRY(cx.alloc_scratch((void**)&nbr, sizeof(int32_t) * (size_t)m * kNbr));
     const char* ne = getenv("SKNN_WALK_ENTRIES");
-    const int nentry = std::min(m, ne ? std::max(1, atoi(ne)) : 64);
-    auto assign = [&](const int32_t* prev, int32_t* cid_o, float* dist_o, float* sums_o) -> sknn_status {
-        if (!walk) {
-            launch_assign(cx, Xp, n, dp, out.centers, m, cid_o, dist_o, sums_o, counts);
+    const int nentry = std::min(m0, ne ? std::max(1, atoi(ne)) : 64);
+    auto assign = [&](const int32_t* prev, int32_t* cid_o, float* dist_o, float* sums_o, int mc) -> sknn_status {
+        if (use_tc) return run_assign_tc(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, counts);
+        if (!walk || mc <= kNbr) {
+            launch_assign(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, counts);
             return SKNN_OK;
         }
-        k_center_knn<<<(m + 7) / 8, 256, 0, s>>>(out.centers, m, dp, nbr);
+        k_center_knn<<<(mc + 7) / 8, 256, 0, s>>>(out.centers, mc, dp, nbr);
         cx.launched();
         dim3 grid((unsigned)((n + 255) / 256));
         switch (dp) {
 #define SKNN_WALK_CASE(D)                                                                                      \
     case D:                                                                                                    \
-        k_assign_walk<D><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, m, nbr, nentry, prev, cid_o, dist_o, sums_o, \
+        k_assign_walk<D><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, mc, nbr, nentry, prev, cid_o, dist_o, sums_o, \
                                               counts);                                                         \
         break;
             SKNN_WALK_CASE(4) SKNN_WALK_CASE(8) SKNN_WALK_CASE(12) SKNN_WALK_CASE(16)
             SKNN_WALK_CASE(20) SKNN_WALK_CASE(24) SKNN_WALK_CASE(28) SKNN_WALK_CASE(32)
 #undef SKNN_WALK_CASE
             default:
-                k_assign_walk<0><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, m, nbr, nentry, prev, cid_o, dist_o,
+                k_assign_walk<0><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, mc, nbr, nentry, prev, cid_o, dist_o,
                                                       sums_o, counts);
                 break;
         }
@@ -602,6 +667,24 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         return SKNN_OK;
     };
     const int32_t* prev = nullptr;
+    if (m0 < m) {
+        SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
+        SKNN_TRY(assign(nullptr, cid, pdist, nullptr, m0));
+        prev = cid;
+        double* ssum;
+        int* scnt;
+        SKNN_TRY(cx.alloc_scratch((void**)&ssum, sizeof(double) + sizeof(int) * 2));
+        scnt = reinterpret_cast<int*>(ssum + 1);
+        SKNN_CUDA(cudaMemsetAsync(ssum, 0, sizeof(double) + sizeof(int) * 2, s));
+        int rb = (int)std::min<int64_t>((n + 255) / 256, 148 * 8);
+        k_sum_sq<<<rb, 256, 0, s>>>(pdist, n, ssum);
+        cx.launched();
+        k_d2_sample<<<rb, 256, 0, s>>>(Xp, n, dp, pdist, ssum, m - m0, seed, out.centers + (int64_t)m0 * dp, scnt);
+        cx.launched();
+        k_d2_fill<<<std::max(1, (m - m0 + 255) / 256), 256, 0, s>>>(Xp, n, dp, m - m0, seed, out.centers + (int64_t)m0 * dp,
+                                                                   scnt);
+        cx.launched();
+    }
     // Lloyd iterations (R9)
     if (lloyd > 0) {
         float* sums;
@@ -609,7 +692,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         for (int it = 0; it < lloyd; ++it) {
             SKNN_CUDA(cudaMemsetAsync(sums, 0, sizeof(float) * m * dp, s));
             SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
-            SKNN_TRY(assign(prev, walk ? cid : nullptr, nullptr, sums));
+            SKNN_TRY(assign(prev, cid, nullptr, sums, m));
             if (walk) prev = cid;
             int blocks = std::max(1, std::min((m * dp + 255) / 256, 148 * 8));
             k_lloyd_update<<<blocks, 256, 0, s>>>(out.centers, sums, counts, m, dp);
@@ -618,7 +701,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     }
     // final assignment with exact member distances + histogram
     SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
-    SKNN_TRY(assign(prev, cid, pdist, nullptr));
+    SKNN_TRY(assign(prev, cid, pdist, nullptr, m));
     k_offsets<<<1, 1024, 0, s>>>(counts, m, out.off, cursor);
     cx.launched();
     unsigned long long* keys;

@@ -197,8 +197,8 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     block_sort_u64(s_keys, S);
     // elastic switch (S8): split the sorted candidates into the sparse list
     // (point-level scan, Alg. 2) and the dense-tile list (tensor cores),
-    // stable in ascending D. auto: a pair is dense when the cluster-level
-    // window 2*UB covers at least tau of the member-distance range r_t and the
+    // stable in ascending D. auto: a pair is dense when a typical query's
+    // member window is expected to cover at least tau of the cluster and the
     // cluster is big enough to fill tiles (cost model in DESIGN.md §6).
     int32_t* row = cand + (int64_t)qc * mt;
     int32_t* drow = dcand + (int64_t)qc * mt;
@@ -215,8 +215,14 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
             if (dense_mode == 2) {
                 dense = true;
             } else if (dense_mode == 0) {
+                // expected share of tc's members inside a typical query's Alg. 2
+                // window [dq - th, dq + th] with dq ~ D and th ~ V_k (the k-th
+                // nearest target bound of the cluster center, without r_q)
                 const int sz = __ldg(toff + tc + 1) - __ldg(toff + tc);
-                dense = sz >= 16 && 2.f * UB >= dense_tau * __ldg(trad + tc);
+                const float rt = __ldg(trad + tc);
+                const float Dp = s_D[tc];
+                const float ov = fminf(rt, Dp + Vk) - fmaxf(0.f, Dp - Vk);
+                dense = sz >= 32 && ov >= dense_tau * fmaxf(rt, 1e-30f);
             }
         }
         const unsigned md = __ballot_sync(0xffffffffu, i < nc && dense);

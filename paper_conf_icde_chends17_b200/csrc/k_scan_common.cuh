@@ -53,6 +53,30 @@ __device__ __forceinline__ int window_start(const float* __restrict__ tdist, int
     return lo;
 }
 
+// First position in [lo, hi) whose member distance dt <= dq (members are
+// sorted by distance descending): the split point of the bidirectional scan.
+__device__ __forceinline__ int window_start_geq(const float* __restrict__ tdist, int lo, int hi, float dq) {
+    while (lo < hi) {
+        int mid = (lo + hi) >> 1;
+        if (__ldg(tdist + mid) > dq) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// First position in [lo, hi) where Alg. 2 breaks (l = dq - dt > theta,
+// line 10): l grows along the distance-descending member array.
+__device__ __forceinline__ int window_end(const float* __restrict__ tdist, int lo, int hi, float dq, float theta,
+                                          float eta) {
+    while (lo < hi) {
+        int mid = (lo + hi) >> 1;
+        float dt = __ldg(tdist + mid);
+        if (ti_keep(dq - dt, theta, dq + dt, eta)) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
 __device__ __forceinline__ void write_result(const ScanArgs& a, int qorig, int r, key_t key) {
     int64_t o = (int64_t)qorig * a.k + r;
     float d2 = key_d2(key);

@@ -20,7 +20,7 @@ namespace sknn {
 
 template <int DP, int KMAX>
 __global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
-    constexpr bool kPrefetchRow = DP <= 8;
+    const float INF = __int_as_float(0x7f800000);
     const int lane = threadIdx.x & 31;
     const int ntiles = *a.ntiles;
     unsigned long long evals = 0, cevals = 0;
@@ -60,55 +60,42 @@ __global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
                 const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
                 const float dq = __fsqrt_rn(d2_reg<DP>(q, a.tcent + (int64_t)tc * DP));  // Alg. 2 line 6
                 ++cevals;
-                int j = window_start(a.tdist, lo, hi, dq, theta, a.eta);
-                if (j >= hi) continue;
-                float dt_n = __ldg(a.tdist + j);
-                float4 row_n[kPrefetchRow ? DP / 4 : 1];
-                if constexpr (kPrefetchRow) {
-#pragma unroll
-                    for (int c4 = 0; c4 < DP / 4; ++c4)
-                        row_n[c4] = __ldg(reinterpret_cast<const float4*>(a.trows + (int64_t)j * DP) + c4);
-                }
+                // Alg. 2 lines 7-17, visited in order of the 1-landmark lower bound
+                // |l| = |dq - dt| (Eq. 1): start where dt ~ dq and walk outward on
+                // both sides, always taking the side with the smaller bound, until
+                // both bounds exceed theta (lines 10-13). Every member with
+                // |l| <= theta is still evaluated, but near targets come first so
+                // theta (line 17) tightens after a few evaluations.
+                int R = window_start_geq(a.tdist, lo, hi, dq);  // first member with dt <= dq
+                int L = R - 1;
+                float dtL = L >= lo ? __ldg(a.tdist + L) : 0.f;
+                float dtR = R < hi ? __ldg(a.tdist + R) : 0.f;
                 for (;;) {
-                    const float dt = dt_n;
-                    float4 row[kPrefetchRow ? DP / 4 : 1];
-                    if constexpr (kPrefetchRow) {
-#pragma unroll
-                        for (int c4 = 0; c4 < DP / 4; ++c4) row[c4] = row_n[c4];
+                    const float bL = L >= lo ? dtL - dq : INF;       // -l on the left (dt > dq)
+                    const float bR = R < hi ? dq - dtR : INF;        // l on the right (dt <= dq)
+                    const bool takeL = bL < bR;
+                    const float bmin = takeL ? bL : bR;
+                    const float dtc = takeL ? dtL : dtR;
+                    if (!ti_keep(bmin, theta, dq + dtc, a.eta)) break;  // both sides beyond theta
+                    const int jc = takeL ? L : R;
+                    if (takeL) {
+                        --L;
+                        if (L >= lo) dtL = __ldg(a.tdist + L);
+                    } else {
+                        ++R;
+                        if (R < hi) dtR = __ldg(a.tdist + R);
                     }
-                    const int jc = j++;
-                    const bool more = j < hi;
-                    if (more) {
-                        dt_n = __ldg(a.tdist + j);
-                        if constexpr (kPrefetchRow) {
-#pragma unroll
-                            for (int c4 = 0; c4 < DP / 4; ++c4)
-                                row_n[c4] = __ldg(reinterpret_cast<const float4*>(a.trows + (int64_t)j * DP) + c4);
+                    const float d2 = d2_reg<DP>(q, a.trows + (int64_t)jc * DP);  // line 15
+                    ++evals;
+                    if (d2 <= kth_d2) {                                         // line 16 (distance part)
+                        const key_t key = make_key(d2, __ldg(a.torig + jc));
+                        if (key < kth) {
+                            top.insert(key);
+                            kth = top.kth();
+                            kth_d2 = key_d2(kth);
+                            theta = fminf(ub, __fsqrt_ru(kth_d2));              // line 17 (R8)
                         }
                     }
-                    const float l = dq - dt;                              // line 9
-                    if (!ti_keep(l, theta, dq + dt, a.eta)) break;        // lines 10-11
-                    if (ti_keep(-l, theta, dq + dt, a.eta)) {             // lines 12-14
-                        float d2;                                         // line 15
-                        if constexpr (kPrefetchRow) {
-                            d2 = 0.f;
-#pragma unroll
-                            for (int c4 = 0; c4 < DP / 4; ++c4) d2 = d2_acc4(d2, q[c4], row[c4]);
-                        } else {
-                            d2 = d2_reg<DP>(q, a.trows + (int64_t)jc * DP);
-                        }
-                        ++evals;
-                        if (d2 <= kth_d2) {                               // line 16 (distance part)
-                            const key_t key = make_key(d2, __ldg(a.torig + jc));
-                            if (key < kth) {
-                                top.insert(key);
-                                kth = top.kth();
-                                kth_d2 = key_d2(kth);
-                                theta = fminf(ub, __fsqrt_ru(kth_d2));    // line 17 (R8)
-                            }
-                        }
-                    }
-                    if (!more) break;
                 }
             }
             const int qo = __ldg(a.qorig + qpos);

@@ -85,14 +85,16 @@ struct RegTopK {
         for (int i = 0; i < KMAX; ++i) a[i] = (i < KMAX - k) ? kNegKey : kInfKey;
     }
     __device__ __forceinline__ key_t kth() const { return a[KMAX - 1]; }
-    // precondition: key < a[KMAX-1]
+    // precondition: key < a[KMAX-1]. The comparisons c[i] = key < a[i] are
+    // evaluated once (a monotone mask), then every slot is one select chain:
+    // a[i] = c[i-1] ? a[i-1] : (c[i] ? key : a[i]).
     __device__ __forceinline__ void insert(key_t key) {
+        bool c[KMAX];
 #pragma unroll
-        for (int i = KMAX - 1; i > 0; --i) {
-            key_t lo = a[i - 1], cur = a[i];
-            a[i] = (key < lo) ? lo : ((key < cur) ? key : cur);
-        }
-        a[0] = (key < a[0]) ? key : a[0];
+        for (int i = 0; i < KMAX; ++i) c[i] = key < a[i];
+#pragma unroll
+        for (int i = KMAX - 1; i > 0; --i) a[i] = c[i - 1] ? a[i - 1] : (c[i] ? key : a[i]);
+        a[0] = c[0] ? key : a[0];
     }
 };
 

@@ -84,6 +84,11 @@ struct Ctx {
 sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int trials, int lloyd, uint64_t seed,
                        Side& out);
 
+// k_assign_tc.cu: nearest-center screen on the tensor cores
+bool assign_tc_supported(int dp);
+sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m, int32_t* cid,
+                          float* dist, float* sums, int32_t* counts);
+
 // k_level1.cu
 struct Level1 {
     float* ub = nullptr;          // [mq] inflated calUB per query cluster
@@ -102,7 +107,7 @@ struct Level1Params {
     float eta = 0.f;
     int shard_rank = 0, shard_count = 1;
     int dense_mode = 0;           // 0 auto (cost model), 1 never, 2 every candidate pair
-    float dense_tau = 1.f;        // auto: dense iff |tc| >= 16 and 2*UB >= tau * r_t
+    float dense_tau = 0.5f;       // auto: dense iff |tc| >= 32 and the expected window share >= tau
 };
 sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Params& p, Level1& out,
                        Counters* counters);

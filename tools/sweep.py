@@ -26,11 +26,17 @@ VARIANTS = {
     "sparse": {"force_path": "sparse"},
     "dense": {"force_path": "dense"},
     "tau4": {"dense_threshold": 4.0},
+    "tau25": {"dense_threshold": 0.25},
+    "tau75": {"dense_threshold": 0.75},
+    "tau95": {"dense_threshold": 0.95},
     "warp": {"mapping": "warp"},
     "cl_half": {"_cl": 0.5},
     "cl_double": {"_cl": 2.0},
     "fullassign": {"_env": ("SKNN_ASSIGN", "full")},
+    "walkassign": {"_env": ("SKNN_ASSIGN", "walk")},
+    "tcassign": {"_env": ("SKNN_ASSIGN", "tc")},
     "entries256": {"_env": ("SKNN_WALK_ENTRIES", "256")},
+    "paperseed": {"_env": ("SKNN_SEEDING", "paper")},
     "full_lloyd4": {"_env": ("SKNN_ASSIGN", "full"), "lloyd_iters": 4},
 }
 
