@@ -117,7 +117,8 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
                                                        const float* __restrict__ bn, int m, int nchunks,
                                                        const float* __restrict__ centers,
                                                        int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
-                                                       float* __restrict__ sums, int32_t* __restrict__ counts) {
+                                                       long long* __restrict__ sums, const double* __restrict__ fx,
+                                                       int32_t* __restrict__ counts) {
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t a_bytes = (uint32_t)kTcM * kp * 2, b_bytes = (uint32_t)kTcN * kp * 2;
     unsigned char* sA = smem;
@@ -239,8 +240,7 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
         if (cid_out) cid_out[i] = bi;
         if (dist_out) dist_out[i] = __fsqrt_rn(d2);
         if (counts) atomicAdd(counts + bi, 1);
-        if (sums)
-            for (int c = 0; c < dp; ++c) atomicAdd(sums + (int64_t)bi * dp + c, xr[c]);
+        if (sums) fx_accumulate(sums + (int64_t)bi * dp, xr, dp, *fx);
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
@@ -250,7 +250,7 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
 bool assign_tc_supported(int dp) { return dp >= 8 && ((dp + 15) & ~15) <= 256; }
 
 sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m, int32_t* cid,
-                          float* dist, float* sums, int32_t* counts) {
+                          float* dist, long long* sums, const double* fx, int32_t* counts) {
     const int kp = (dp + 15) & ~15;
     const int nchunks = (m + kTcN - 1) / kTcN;
     const int mpad = nchunks * kTcN;
@@ -271,7 +271,7 @@ sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int64_t grid = (n + kTcM - 1) / kTcM;
     k_assign_tc<<<(unsigned)grid, kTcM, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, bn, m, nchunks, centers, cid, dist,
-                                                          sums, counts);
+                                                          sums, fx, counts);
     cx.launched();
     return cx.check_launch("assign (tensor cores)");
 }

@@ -151,7 +151,8 @@ template <int DP>
 __global__ void __launch_bounds__(256) k_assign(const float* __restrict__ Xp, int64_t n, int dp_rt,
                                                 const float* __restrict__ centers, int m, int chunk,
                                                 int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
-                                                float* __restrict__ sums, int32_t* __restrict__ counts) {
+                                                long long* __restrict__ sums, const double* __restrict__ fx,
+                                                int32_t* __restrict__ counts) {
     extern __shared__ __align__(16) float s_c[];
     const int dp = DP > 0 ? DP : dp_rt;
     int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -213,7 +214,7 @@ __global__ void __launch_bounds__(256) k_assign(const float* __restrict__ Xp, in
     if (dist_out) dist_out[i] = __fsqrt_rn(best);
     if (counts) atomicAdd(counts + bi, 1);
     if (sums) {
-        for (int c = 0; c < dp; ++c) atomicAdd(sums + (int64_t)bi * dp + c, xrow[c]);
+        fx_accumulate(sums + (int64_t)bi * dp, xrow, dp, *fx);
     }
 }
 
@@ -263,7 +264,8 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
                                                      const int32_t* __restrict__ nbr, int nentry,
                                                      const int32_t* __restrict__ cid_prev,
                                                      int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
-                                                     float* __restrict__ sums, int32_t* __restrict__ counts) {
+                                                     long long* __restrict__ sums, const double* __restrict__ fx,
+                                                     int32_t* __restrict__ counts) {
     const int dp = DP > 0 ? DP : dp_rt;
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i >= n) return;
@@ -304,53 +306,101 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
     if (dist_out) dist_out[i] = __fsqrt_rn(bd);
     if (counts) atomicAdd(counts + best, 1);
     if (sums) {
-        for (int c = 0; c < dp; ++c) atomicAdd(sums + (int64_t)best * dp + c, xr[c]);
+        fx_accumulate(sums + (int64_t)best * dp, xr, dp, *fx);
     }
 }
 
 // ------------------------------------------------------------ D^2 seeding --
-__global__ void k_sum_sq(const float* __restrict__ dist, int64_t n, double* __restrict__ out) {
+// sum of squared distances, deterministic: per-block partials + ordered final sum
+__global__ void k_sum_sq(const float* __restrict__ dist, int64_t n, double* __restrict__ partial) {
     double s = 0.0;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const double v = dist[i];
         s += v * v;
     }
-    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    __shared__ double red[32];
-    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+    __shared__ double red[256];
+    red[threadIdx.x] = s;
+    __syncthreads();
+    for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+        if (threadIdx.x < w) red[threadIdx.x] += red[threadIdx.x + w];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) partial[blockIdx.x] = red[0];
+}
+
+__global__ void k_sum_final(const double* __restrict__ partial, int nb, double* __restrict__ out) {
+    double s = 0.0;
+    for (int b = 0; b < nb; ++b) s += partial[b];
+    *out = s;
+}
+
+// point i becomes a center with probability min(1, m1 * d2_i / S); the picks
+// are compacted in point order (count -> scan -> write), so the sampled set
+// and its slot order are deterministic.
+constexpr int kSampleBlocks = 1024;
+
+__device__ __forceinline__ bool d2_pick(const float* __restrict__ dist, int64_t i, double tot, int m1, uint64_t seed) {
+    const double v = dist[i];
+    const double p = (double)m1 * v * v / tot;
+    const double u = (double)mix32(seed * 0x2545f4914f6cdd1dull + (uint64_t)i) * (1.0 / 4294967296.0);
+    return u < p;
+}
+
+__global__ void __launch_bounds__(256) k_d2_count(const float* __restrict__ dist, int64_t n, const double* __restrict__ S,
+                                                  int m1, uint64_t seed, int32_t* __restrict__ bcount) {
+    const double tot = *S;
+    const int64_t per = (n + gridDim.x - 1) / gridDim.x;
+    const int64_t lo = blockIdx.x * per, hi = min(n, lo + per);
+    int c = 0;
+    if (tot > 0.0)
+        for (int64_t i = lo + threadIdx.x; i < hi; i += blockDim.x) c += d2_pick(dist, i, tot, m1, seed) ? 1 : 0;
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    __shared__ int red[8];
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
     __syncthreads();
     if (threadIdx.x == 0) {
-        double t = 0.0;
-        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
-        atomicAdd(out, t);
+        int t = 0;
+        for (int w = 0; w < 8; ++w) t += red[w];
+        bcount[blockIdx.x] = t;
     }
 }
 
-// point i becomes a center with probability min(1, m1 * d2_i / S) (at most m1 kept)
-__global__ void k_d2_sample(const float* __restrict__ Xp, int64_t n, int dp, const float* __restrict__ dist,
-                            const double* __restrict__ S, int m1, uint64_t seed, float* __restrict__ centers,
-                            int* __restrict__ cnt) {
+__global__ void __launch_bounds__(256) k_d2_write(const float* __restrict__ Xp, int64_t n, int dp,
+                                                  const float* __restrict__ dist, const double* __restrict__ S, int m1,
+                                                  uint64_t seed, const int32_t* __restrict__ boff,
+                                                  float* __restrict__ centers) {
     const double tot = *S;
     if (!(tot > 0.0)) return;
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const double v = dist[i];
-        const double p = (double)m1 * v * v / tot;
-        const double u = (double)mix32(seed * 0x2545f4914f6cdd1dull + (uint64_t)i) * (1.0 / 4294967296.0);
-        if (u < p) {
-            const int pos = atomicAdd(cnt, 1);
-            if (pos < m1) {
+    const int64_t per = (n + gridDim.x - 1) / gridDim.x;
+    const int64_t lo = blockIdx.x * per, hi = min(n, lo + per);
+    __shared__ int wc[8];
+    int run = boff[blockIdx.x];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int64_t base = lo; base < hi; base += blockDim.x) {
+        const int64_t i = base + threadIdx.x;
+        const bool pick = i < hi && d2_pick(dist, i, tot, m1, seed);
+        const unsigned bm = __ballot_sync(0xffffffffu, pick);
+        if (lane == 0) wc[w] = __popc(bm);
+        __syncthreads();
+        int off = run;
+        for (int ww = 0; ww < w; ++ww) off += wc[ww];
+        if (pick) {
+            const int slot = off + __popc(bm & ((1u << lane) - 1u));
+            if (slot < m1) {
                 const float4* src = reinterpret_cast<const float4*>(Xp + i * dp);
-                float4* dst = reinterpret_cast<float4*>(centers + (int64_t)pos * dp);
+                float4* dst = reinterpret_cast<float4*>(centers + (int64_t)slot * dp);
                 for (int c = 0; c < dp / 4; ++c) dst[c] = src[c];
             }
         }
+        for (int ww = 0; ww < 8; ++ww) run += wc[ww];
+        __syncthreads();
     }
 }
 
 // slots the sampling left empty get random points
 __global__ void k_d2_fill(const float* __restrict__ Xp, int64_t n, int dp, int m1, uint64_t seed,
-                          float* __restrict__ centers, const int* __restrict__ cnt) {
-    const int start = min(*cnt, m1);
+                          float* __restrict__ centers, const int32_t* __restrict__ total) {
+    const int start = min(*total, m1);
     for (int j = start + blockIdx.x * blockDim.x + threadIdx.x; j < m1; j += gridDim.x * blockDim.x) {
         const uint32_t i = perm_index((uint32_t)j, (uint32_t)n, seed ^ 0xd2d2d2d2ull);
         const float4* src = reinterpret_cast<const float4*>(Xp + (int64_t)i * dp);
@@ -359,13 +409,30 @@ __global__ void k_d2_fill(const float* __restrict__ Xp, int64_t n, int dp, int m
     }
 }
 
-__global__ void k_lloyd_update(float* __restrict__ centers, const float* __restrict__ sums,
-                               const int32_t* __restrict__ counts, int m, int dp) {
+// Lloyd update from the fixed-point sums (deterministic: integer adds commute)
+__global__ void k_lloyd_update(float* __restrict__ centers, const long long* __restrict__ sums,
+                               const double* __restrict__ fx, const int32_t* __restrict__ counts, int m, int dp) {
+    const double inv = 1.0 / *fx;
     for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < m * dp; e += gridDim.x * blockDim.x) {
-        int c = e / dp;
-        int cnt = counts[c];
-        if (cnt > 0) centers[e] = sums[e] / (float)cnt;
+        const int c = e / dp;
+        const int cnt = counts[c];
+        if (cnt > 0) centers[e] = (float)((double)sums[e] * inv / (double)cnt);
     }
+}
+
+// fixed-point scale for the Lloyd sums: 2^s with max|x| * n * 2^s < 2^61
+__global__ void k_absmax(const float* __restrict__ Xp, int64_t total, unsigned int* __restrict__ out) {
+    float mx = 0.f;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x)
+        mx = fmaxf(mx, fabsf(Xp[e]));
+    for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if ((threadIdx.x & 31) == 0) atomicMax(out, __float_as_uint(mx));
+}
+
+__global__ void k_fx_scale(const unsigned int* __restrict__ amax, int64_t n, double* __restrict__ fx) {
+    const double mx = fmax((double)__uint_as_float(*amax), 1e-30);
+    const double e = floor(61.0 - log2(mx * (double)n));
+    *fx = exp2(fmin(e, 1000.0));
 }
 
 // --------------------------------------------------------------- CSR -----
@@ -553,17 +620,17 @@ static int assign_chunk(int dp, int m, size_t* smem) {
 }
 
 static void launch_assign(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m,
-                          int32_t* cid, float* dist, float* sums, int32_t* counts) {
+                          int32_t* cid, float* dist, long long* sums, const double* fx, int32_t* counts) {
     size_t smem;
     int chunk = assign_chunk(dp, m, &smem);
     dim3 grid((unsigned)((n + 255) / 256));
     switch (dp) {
 #define SKNN_ASSIGN_CASE(D) \
-    case D: k_assign<D><<<grid, 256, smem, cx.stream>>>(Xp, n, dp, centers, m, chunk, cid, dist, sums, counts); break;
+    case D: k_assign<D><<<grid, 256, smem, cx.stream>>>(Xp, n, dp, centers, m, chunk, cid, dist, sums, fx, counts); break;
         SKNN_ASSIGN_CASE(4) SKNN_ASSIGN_CASE(8) SKNN_ASSIGN_CASE(12) SKNN_ASSIGN_CASE(16)
         SKNN_ASSIGN_CASE(20) SKNN_ASSIGN_CASE(24) SKNN_ASSIGN_CASE(28) SKNN_ASSIGN_CASE(32)
 #undef SKNN_ASSIGN_CASE
-        default: k_assign<0><<<grid, 256, smem, cx.stream>>>(Xp, n, dp, centers, m, chunk, cid, dist, sums, counts); break;
+        default: k_assign<0><<<grid, 256, smem, cx.stream>>>(Xp, n, dp, centers, m, chunk, cid, dist, sums, fx, counts); break;
     }
     cx.launched();
 }
@@ -640,10 +707,23 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     if (walk) SKNN_TRY(cx.alloc_scratch((void**)&nbr, sizeof(int32_t) * (size_t)m * kNbr));
     const char* ne = getenv("SKNN_WALK_ENTRIES");
     const int nentry = std::min(m0, ne ? std::max(1, atoi(ne)) : 64);
-    auto assign = [&](const int32_t* prev, int32_t* cid_o, float* dist_o, float* sums_o, int mc) -> sknn_status {
-        if (use_tc) return run_assign_tc(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, counts);
+    // fixed-point scale of the Lloyd sums (deterministic centers, hence a
+    // deterministic clustering: query-sharded ranks agree on cluster ids)
+    double* fx;
+    unsigned int* amax;
+    SKNN_TRY(cx.alloc_scratch((void**)&fx, sizeof(double) + sizeof(unsigned int)));
+    amax = reinterpret_cast<unsigned int*>(fx + 1);
+    if (lloyd > 0) {
+        SKNN_CUDA(cudaMemsetAsync(amax, 0, sizeof(unsigned int), s));
+        k_absmax<<<(int)std::min<int64_t>((n * dp + 255) / 256, 148 * 8), 256, 0, s>>>(Xp, n * dp, amax);
+        k_fx_scale<<<1, 1, 0, s>>>(amax, n, fx);
+        cx.launched();
+        cx.launched();
+    }
+    auto assign = [&](const int32_t* prev, int32_t* cid_o, float* dist_o, long long* sums_o, int mc) -> sknn_status {
+        if (use_tc) return run_assign_tc(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, fx, counts);
         if (!walk || mc <= kNbr) {
-            launch_assign(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, counts);
+            launch_assign(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, fx, counts);
             return SKNN_OK;
         }
         k_center_knn<<<(mc + 7) / 8, 256, 0, s>>>(out.centers, mc, dp, nbr);
@@ -653,14 +733,14 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
 #define SKNN_WALK_CASE(D)                                                                                      \
     case D:                                                                                                    \
         k_assign_walk<D><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, mc, nbr, nentry, prev, cid_o, dist_o, sums_o, \
-                                              counts);                                                         \
+                                              fx, counts);                                                     \
         break;
             SKNN_WALK_CASE(4) SKNN_WALK_CASE(8) SKNN_WALK_CASE(12) SKNN_WALK_CASE(16)
             SKNN_WALK_CASE(20) SKNN_WALK_CASE(24) SKNN_WALK_CASE(28) SKNN_WALK_CASE(32)
 #undef SKNN_WALK_CASE
             default:
                 k_assign_walk<0><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, mc, nbr, nentry, prev, cid_o, dist_o,
-                                                      sums_o, counts);
+                                                      sums_o, fx, counts);
                 break;
         }
         cx.launched();
@@ -672,30 +752,39 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         SKNN_TRY(assign(nullptr, cid, pdist, nullptr, m0));
         prev = cid;
         double* ssum;
-        int* scnt;
-        SKNN_TRY(cx.alloc_scratch((void**)&ssum, sizeof(double) + sizeof(int) * 2));
-        scnt = reinterpret_cast<int*>(ssum + 1);
-        SKNN_CUDA(cudaMemsetAsync(ssum, 0, sizeof(double) + sizeof(int) * 2, s));
-        int rb = (int)std::min<int64_t>((n + 255) / 256, 148 * 8);
-        k_sum_sq<<<rb, 256, 0, s>>>(pdist, n, ssum);
+        int32_t* bcnt;
+        int32_t* boff;
+        const int rb = (int)std::min<int64_t>((n + 255) / 256, 148 * 8);
+        SKNN_TRY(cx.alloc_scratch((void**)&ssum, sizeof(double) * (rb + 1)));
+        SKNN_TRY(cx.alloc_scratch((void**)&bcnt, sizeof(int32_t) * (3 * kSampleBlocks + 8)));
+        boff = bcnt + kSampleBlocks;                   // kSampleBlocks + 1 entries
+        int32_t* dummy = bcnt + 2 * kSampleBlocks + 1;  // cursor scratch of k_offsets
+        k_sum_sq<<<rb, 256, 0, s>>>(pdist, n, ssum + 1);
         cx.launched();
-        k_d2_sample<<<rb, 256, 0, s>>>(Xp, n, dp, pdist, ssum, m - m0, seed, out.centers + (int64_t)m0 * dp, scnt);
+        k_sum_final<<<1, 1, 0, s>>>(ssum + 1, rb, ssum);
+        cx.launched();
+        k_d2_count<<<kSampleBlocks, 256, 0, s>>>(pdist, n, ssum, m - m0, seed, bcnt);
+        cx.launched();
+        k_offsets<<<1, 1024, 0, s>>>(bcnt, kSampleBlocks, boff, dummy);
+        cx.launched();
+        k_d2_write<<<kSampleBlocks, 256, 0, s>>>(Xp, n, dp, pdist, ssum, m - m0, seed, boff,
+                                                 out.centers + (int64_t)m0 * dp);
         cx.launched();
         k_d2_fill<<<std::max(1, (m - m0 + 255) / 256), 256, 0, s>>>(Xp, n, dp, m - m0, seed, out.centers + (int64_t)m0 * dp,
-                                                                   scnt);
+                                                                   boff + kSampleBlocks);
         cx.launched();
     }
     // Lloyd iterations (R9)
     if (lloyd > 0) {
-        float* sums;
-        SKNN_TRY(cx.alloc_scratch((void**)&sums, sizeof(float) * m * dp));
+        long long* sums;
+        SKNN_TRY(cx.alloc_scratch((void**)&sums, sizeof(long long) * m * dp));
         for (int it = 0; it < lloyd; ++it) {
-            SKNN_CUDA(cudaMemsetAsync(sums, 0, sizeof(float) * m * dp, s));
+            SKNN_CUDA(cudaMemsetAsync(sums, 0, sizeof(long long) * m * dp, s));
             SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
             SKNN_TRY(assign(prev, cid, nullptr, sums, m));
             if (walk) prev = cid;
             int blocks = std::max(1, std::min((m * dp + 255) / 256, 148 * 8));
-            k_lloyd_update<<<blocks, 256, 0, s>>>(out.centers, sums, counts, m, dp);
+            k_lloyd_update<<<blocks, 256, 0, s>>>(out.centers, sums, fx, counts, m, dp);
             cx.launched();
         }
     }

@@ -64,6 +64,13 @@ __device__ __forceinline__ float d2_reg(const float4 (&q)[DP / 4], const float* 
     return s;
 }
 
+// Fixed-point accumulation of a row into int64 sums (Lloyd update): integer
+// atomics commute, so the centers do not depend on the order of the adds.
+__device__ __forceinline__ void fx_accumulate(long long* dst, const float* x, int dp, double scale) {
+    for (int c = 0; c < dp; ++c)
+        atomicAdd(reinterpret_cast<unsigned long long*>(dst + c), (unsigned long long)__double2ll_rn((double)x[c] * scale));
+}
+
 // ------------------------------------------------------- rounding slack --
 // Reading R7: every TI prune test keeps a pair unless its lower bound exceeds
 // theta by more than eta * (sum of the magnitudes involved), eta = (d+8)*2^-24

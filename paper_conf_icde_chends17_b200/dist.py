@@ -1,0 +1,92 @@
+"""Multi-GPU KNN join over torch.distributed (one process per GPU, NCCL).
+
+SURVEY.md §8(e). Two modes:
+
+* Query sharding (default; north_star "sharding queries, with the target
+  index and cluster metadata replicated"): every rank holds all of T. For a
+  self-join every rank clusters T identically (seeded, deterministic sizes)
+  and processes the query clusters c with c % P == rank
+  (``sknn_options.shard_rank/shard_count``); otherwise rank r takes the
+  contiguous query rows [r*nq/P, (r+1)*nq/P). No data-path collective; the
+  optional result assembly is one all-reduce outside the join.
+* Target sharding: rank r owns T[r*nt/P, (r+1)*nt/P), computes partial k-lists
+  of ALL queries with squared distances and global indices (``out_squared``,
+  ``index_base``), the partial lists are exchanged with one all-gather over
+  NVLink and merged exactly by ``sknn_merge_partials`` (the paper's merge of
+  sorted per-thread heaps, across ranks). The (d2, index) keys are
+  global and the merge is a selection on their total order, so the result is
+  bit-identical to the single-GPU join.
+
+The local join and merge default to the CUDA library; tests may inject other
+callables to exercise the orchestration on CPU with the gloo backend.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+from . import join as _cuda_join
+from . import merge_partials as _cuda_merge
+
+
+def shard_bounds(n: int, world: int, rank: int):
+    """Contiguous, balanced [lo, hi) of rank among world over n items."""
+    base, rem = divmod(n, world)
+    lo = rank * base + min(rank, rem)
+    return lo, lo + base + (1 if rank < rem else 0)
+
+
+def _world(group):
+    return dist.get_world_size(group), dist.get_rank(group)
+
+
+def join_query_sharded(Q, T, k: int, *, group=None, self_join: bool | None = None, gather: bool = True,
+                       local_join=None, **opts):
+    """Query-sharded join. Returns (idx, dist) for the rank's rows (gather=False:
+    full-size buffers with -1 / 0 in rows of other ranks) or the assembled
+    full result on every rank (gather=True, one all-reduce)."""
+    world, rank = _world(group)
+    local_join = local_join or _cuda_join
+    if self_join is None:
+        self_join = Q is T
+    nq = Q.shape[0]
+    if self_join:
+        idx = torch.full((nq, k), -1, dtype=torch.int32, device=Q.device)
+        dst = torch.zeros((nq, k), dtype=torch.float32, device=Q.device)
+        local_join(Q, Q, k, out=(idx, dst), shard_rank=rank, shard_count=world, **opts)
+    else:
+        lo, hi = shard_bounds(nq, world, rank)
+        idx = torch.full((nq, k), -1, dtype=torch.int32, device=Q.device)
+        dst = torch.zeros((nq, k), dtype=torch.float32, device=Q.device)
+        if hi > lo:
+            i, d = local_join(Q[lo:hi].contiguous(), T, k, **opts)[:2]
+            idx[lo:hi] = i
+            dst[lo:hi] = d
+    if not gather or world == 1:
+        return idx, dst
+    # rows are disjoint across ranks: -1 / 0 elsewhere, so MAX / SUM assemble them
+    dist.all_reduce(idx, op=dist.ReduceOp.MAX, group=group)
+    dist.all_reduce(dst, op=dist.ReduceOp.SUM, group=group)
+    return idx, dst
+
+
+def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, local_join=None, merge=None,
+                        out_squared: bool = False, **opts):
+    """Target-sharded join: local partial lists of every query against this
+    rank's T_shard (global indices), all-gathered and merged exactly."""
+    world, rank = _world(group)
+    local_join = local_join or _cuda_join
+    merge = merge or _cuda_merge
+    nq = Q.shape[0]
+    kk = min(k, T_shard.shape[0])
+    pidx, pd2 = local_join(Q, T_shard, kk, out_squared=1, index_base=int(shard_offset), **opts)[:2]
+    if kk < k:  # a shard smaller than k: pad with +inf keys (never selected over real ones)
+        pad_i = torch.full((nq, k - kk), -1, dtype=torch.int32, device=Q.device)
+        pad_d = torch.full((nq, k - kk), float("inf"), dtype=torch.float32, device=Q.device)
+        pidx = torch.cat([pidx, pad_i], 1)
+        pd2 = torch.cat([pd2, pad_d], 1)
+    all_i = torch.empty((world * nq, k), dtype=torch.int32, device=Q.device)
+    all_d = torch.empty((world * nq, k), dtype=torch.float32, device=Q.device)
+    dist.all_gather_into_tensor(all_i, pidx.contiguous(), group=group)
+    dist.all_gather_into_tensor(all_d, pd2.contiguous(), group=group)
+    return merge(all_i.view(world, nq, k), all_d.view(world, nq, k), k, out_squared=out_squared)

@@ -1,0 +1,110 @@
+"""Multi-process (world_size 2, gloo, CPU) tests of the multi-GPU orchestration
+in paper_conf_icde_chends17_b200/dist.py: shard bounds, query-sharded result
+assembly, target-sharded partial-list exchange with global indices and the
+exact merge. The per-rank join is injected (the CPU oracle restricted to the
+rank's shard) and so is the merge (a host reference), because the CUDA
+library needs a GPU; the same orchestration code runs with NCCL on B200s.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import datagen
+import oracle
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def oracle_local_join(Q, T, k, out=None, out_squared=0, index_base=0, shard_rank=0, shard_count=1, **_):
+    """CPU stand-in for sknn.join with the same calling convention (tests only)."""
+    Qn, Tn = Q.numpy(), T.numpy()
+    idx, dist_, d2 = oracle.knn_join(Qn, Tn, k, return_d2=True)
+    vals = d2.astype(np.float32) if out_squared else dist_
+    idx = idx + index_base
+    if out is not None:
+        # query sharding of a self-join: rows of this rank's "clusters" (here: i % count)
+        rows = np.arange(Qn.shape[0]) % shard_count == shard_rank
+        out[0][torch.from_numpy(rows)] = torch.from_numpy(idx[rows].astype(np.int32))
+        out[1][torch.from_numpy(rows)] = torch.from_numpy(vals[rows])
+        return out
+    return torch.from_numpy(idx.astype(np.int32)), torch.from_numpy(vals)
+
+
+def host_merge(all_i, all_d, k, out_squared=False):
+    P, nq, _ = all_d.shape
+    I = all_i.numpy().transpose(1, 0, 2).reshape(nq, -1)
+    D = all_d.numpy().transpose(1, 0, 2).reshape(nq, -1)
+    oi = np.empty((nq, k), np.int32)
+    od = np.empty((nq, k), np.float32)
+    for q in range(nq):
+        order = np.lexsort((I[q], D[q]))[:k]
+        oi[q] = I[q][order]
+        od[q] = D[q][order] if out_squared else np.sqrt(D[q][order].astype(np.float64)).astype(np.float32)
+    return torch.from_numpy(oi), torch.from_numpy(od)
+
+
+def _worker(rank, world, port, results):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icde_chends17_b200 import dist as sdist
+    try:
+        X = datagen.c1_uniform_int(600)
+        Q = datagen.c1_uniform_int(150, seed=9)
+        k = 8
+        # target sharding
+        lo, hi = sdist.shard_bounds(X.shape[0], world, rank)
+        i, d = sdist.join_target_sharded(torch.from_numpy(Q), torch.from_numpy(X[lo:hi]).contiguous(), k, lo,
+                                         local_join=oracle_local_join, merge=host_merge)
+        # query sharding, non-self join (contiguous rows)
+        qi, qd = sdist.join_query_sharded(torch.from_numpy(Q), torch.from_numpy(X), k, self_join=False,
+                                          local_join=oracle_local_join)
+        # query sharding, self join (cluster-interleaved rows, assembled by all-reduce)
+        Xt = torch.from_numpy(X)
+        si, sd = sdist.join_query_sharded(Xt, Xt, k, local_join=oracle_local_join)
+        results[rank] = (i.numpy(), d.numpy(), qi.numpy(), qd.numpy(), si.numpy(), sd.numpy())
+    finally:
+        dist.destroy_process_group()
+
+
+def test_shard_bounds():
+    from paper_conf_icde_chends17_b200.dist import shard_bounds
+    for n in (0, 1, 7, 100, 101):
+        for w in (1, 2, 3, 8):
+            parts = [shard_bounds(n, w, r) for r in range(w)]
+            assert parts[0][0] == 0 and parts[-1][1] == n
+            assert all(parts[r][1] == parts[r + 1][0] for r in range(w - 1))
+            sizes = [b - a for a, b in parts]
+            assert max(sizes) - min(sizes) <= 1
+
+
+def test_two_rank_gloo_matches_single_join():
+    world = 2
+    port = _free_port()
+    mgr = mp.Manager()
+    results = mgr.dict()
+    mp.spawn(_worker, args=(world, port, results), nprocs=world, join=True)
+    X = datagen.c1_uniform_int(600)
+    Q = datagen.c1_uniform_int(150, seed=9)
+    k = 8
+    ridx, rdist = oracle.knn_join(Q, X, k)
+    sidx, sdist_ = oracle.knn_join(X, X, k)
+    for r in range(world):
+        i, d, qi, qd, si, sd = results[r]
+        np.testing.assert_array_equal(i, ridx)       # target-sharded == single join (bit-exact)
+        np.testing.assert_array_equal(d, rdist)
+        np.testing.assert_array_equal(qi, ridx)      # query-sharded, assembled
+        np.testing.assert_array_equal(qd, rdist)
+        np.testing.assert_array_equal(si, sidx)      # self-join, cluster-interleaved shards
+        np.testing.assert_array_equal(sd, sdist_)

@@ -283,3 +283,62 @@ def test_auto_switch_mixes_paths(sknn):
     ridx, rdist = oracle.knn_join(Q, T, k)
     assert_knn_bitexact(idx, dist, ridx, rdist)
     assert st["dense_pairs"] > 0
+
+
+# ------------------------------------------------------------ multi-GPU --
+def test_query_shard_option_covers_all_rows(sknn):
+    """Query sharding of a self-join (sknn_options.shard_rank/count): P ranks'
+    cluster-interleaved shards, run one after the other into the same output,
+    reproduce the single join bit-exactly (P11)."""
+    Q, T, k, sj = datagen.workload("C3int", 0.05)
+    dX = dev(Q)
+    idx = torch.full((Q.shape[0], k), -1, dtype=torch.int32, device="cuda")
+    dst = torch.zeros((Q.shape[0], k), dtype=torch.float32, device="cuda")
+    for r in range(3):
+        sknn.join(dX, dX, k, out=(idx, dst), shard_rank=r, shard_count=3)
+    torch.cuda.synchronize()
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx.cpu().numpy(), dst.cpu().numpy(), ridx, rdist)
+
+
+def test_dist_nccl_world1(sknn):
+    """The torch.distributed orchestration on the NCCL backend (world size 1 on
+    the one GPU the driver provides): both sharding modes equal the join."""
+    import os
+    import socket
+    import torch.distributed as tdist
+    from paper_conf_icde_chends17_b200 import dist as sdist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    tdist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        T = datagen.c5_blobs(20000, which="T")
+        Q = datagen.c5_blobs(3000, which="Q")
+        k = 32
+        ridx, rdist = oracle.knn_join(Q, T, k)
+        i, d = sdist.join_target_sharded(dev(Q), dev(T), k, 0)
+        assert_knn_bitexact(i.cpu().numpy(), d.cpu().numpy(), ridx, rdist)
+        i, d = sdist.join_query_sharded(dev(Q), dev(T), k, self_join=False)
+        assert_knn_bitexact(i.cpu().numpy(), d.cpu().numpy(), ridx, rdist)
+    finally:
+        tdist.destroy_process_group()
+
+
+def test_build_is_deterministic(sknn):
+    """The clustering is deterministic (fixed-point Lloyd sums, ordered sampling
+    compaction): two builds export identical indexes and two joins report
+    identical counters -- query-sharded ranks rely on agreeing cluster ids."""
+    for name, scale in (("C2", 0.05), ("C5", 0.005), ("C4", 0.004)):
+        Q, T, k, sj = datagen.workload(name, scale)
+        a = sknn.build(dev(T)).export()
+        b = sknn.build(dev(T)).export()
+        for key in a:
+            np.testing.assert_array_equal(a[key], b[key])
+        _, _, s1 = run(sknn, Q, T, k, sj)
+        _, _, s2 = run(sknn, Q, T, k, sj)
+        for key in ("dist_evals", "cand_pairs", "center_evals", "dense_pairs"):
+            assert s1[key] == s2[key], key
