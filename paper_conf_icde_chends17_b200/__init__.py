@@ -20,7 +20,7 @@ import threading
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsweetknn.so")
+LIB_PATH = os.environ.get("SKNN_LIB") or os.path.join(_HERE, "libsweetknn.so")
 
 SKNN_OK = 0
 STATUS = {0: "SKNN_OK", -1: "SKNN_ERR_INVALID_ARG", -2: "SKNN_ERR_NOT_DEVICE_PTR", -3: "SKNN_ERR_OOM",

@@ -78,6 +78,7 @@ static sknn_options merge_options(const sknn_options* o) {
     memcpy(&d, o, n);
     d.struct_size = sizeof(sknn_options);
     if (d.landmark_trials <= 0) d.landmark_trials = 10;
+    if (d.landmark_trials > 64) d.landmark_trials = 64;
     if (d.lloyd_iters < 0) d.lloyd_iters = 2;
     if (d.r_factor <= 0.f) d.r_factor = 0.25f;
     if (d.shard_count <= 1) { d.shard_count = 1; d.shard_rank = 0; }

@@ -124,15 +124,22 @@ __global__ void __launch_bounds__(256) k_landmark_sums(const float* __restrict__
 
 __global__ void k_landmark_pick(const double* __restrict__ partial, int nblk, int trials, const int32_t* __restrict__ idx,
                                 int m, const float* __restrict__ Xp, int dp, float* __restrict__ centers) {
+    __shared__ double s_tr[64];
     __shared__ int best;
+    // warp w sums trial w's partials: fixed lane strides + a fixed shuffle tree (deterministic)
+    const int lane = threadIdx.x & 31;
+    for (int t = threadIdx.x >> 5; t < trials; t += blockDim.x >> 5) {
+        double v = 0.0;
+        for (int b = lane; b < nblk; b += 32) v += partial[t * nblk + b];
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (lane == 0) s_tr[t] = v;
+    }
+    __syncthreads();
     if (threadIdx.x == 0) {
         double bs = -1.0;
         int bt = 0;
-        for (int t = 0; t < trials; ++t) {
-            double s = 0.0;
-            for (int b = 0; b < nblk; ++b) s += partial[t * nblk + b];
-            if (s > bs) { bs = s; bt = t; }  // first maximum
-        }
+        for (int t = 0; t < trials; ++t)
+            if (s_tr[t] > bs) { bs = s_tr[t]; bt = t; }  // first maximum
         best = bt;
     }
     __syncthreads();
@@ -329,9 +336,16 @@ __global__ void k_sum_sq(const float* __restrict__ dist, int64_t n, double* __re
 }
 
 __global__ void k_sum_final(const double* __restrict__ partial, int nb, double* __restrict__ out) {
-    double s = 0.0;
-    for (int b = 0; b < nb; ++b) s += partial[b];
-    *out = s;
+    __shared__ double red[256];
+    double v = 0.0;
+    for (int b = threadIdx.x; b < nb; b += blockDim.x) v += partial[b];
+    red[threadIdx.x] = v;
+    __syncthreads();
+    for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+        if (threadIdx.x < w) red[threadIdx.x] += red[threadIdx.x + w];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) *out = red[0];
 }
 
 // point i becomes a center with probability min(1, m1 * d2_i / S); the picks
@@ -720,14 +734,20 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         cx.launched();
         cx.launched();
     }
+    int graph_m = -1;
     auto assign = [&](const int32_t* prev, int32_t* cid_o, float* dist_o, long long* sums_o, int mc) -> sknn_status {
         if (use_tc) return run_assign_tc(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, fx, counts);
         if (!walk || mc <= kNbr) {
             launch_assign(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, fx, counts);
             return SKNN_OK;
         }
-        k_center_knn<<<(mc + 7) / 8, 256, 0, s>>>(out.centers, mc, dp, nbr);
-        cx.launched();
+        // the walk may use a slightly stale graph (the assignment only has to be
+        // approximate): build it for the first pass and after seeding only
+        if (graph_m != mc) {
+            k_center_knn<<<(mc + 7) / 8, 256, 0, s>>>(out.centers, mc, dp, nbr);
+            cx.launched();
+            graph_m = mc;
+        }
         dim3 grid((unsigned)((n + 255) / 256));
         switch (dp) {
 #define SKNN_WALK_CASE(D)                                                                                      \
@@ -761,7 +781,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         int32_t* dummy = bcnt + 2 * kSampleBlocks + 1;  // cursor scratch of k_offsets
         k_sum_sq<<<rb, 256, 0, s>>>(pdist, n, ssum + 1);
         cx.launched();
-        k_sum_final<<<1, 1, 0, s>>>(ssum + 1, rb, ssum);
+        k_sum_final<<<1, 256, 0, s>>>(ssum + 1, rb, ssum);
         cx.launched();
         k_d2_count<<<kSampleBlocks, 256, 0, s>>>(pdist, n, ssum, m - m0, seed, bcnt);
         cx.launched();
