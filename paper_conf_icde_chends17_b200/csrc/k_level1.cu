@@ -31,7 +31,7 @@ namespace sknn {
 typedef unsigned long long u64;
 
 constexpr int kL1Threads = 256;
-constexpr int kL1Vals = 4096;  // capacity of the gathered-bounds buffer
+constexpr int kL1Vals = 1024;  // capacity of the gathered-bounds buffer (overflow: M_k is used)
 
 __device__ __forceinline__ void cmpx64(u64* s, int i, int p) {
     u64 a = s[i], b = s[p];
@@ -146,11 +146,20 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
         const int lo = __ldg(toff + tc), hi = __ldg(toff + tc + 1);
         const float D = s_D[tc];
         const int cnt = min(k, hi - lo);
-        for (int i = 0; i < cnt; ++i) {
-            const float v = D + __ldg(tdist + hi - 1 - i);
-            if (v > Mk) break;  // members are visited closest-first: later bounds only grow
-            const int pos = atomicAdd(&s_cnt, 1);
-            if (pos < kL1Vals) s_keys[pos] = u64(__float_as_uint(v));
+        // members closest to the center first; batches of 8 independent loads
+        for (int i0 = 0; i0 < cnt; i0 += 8) {
+            float dv[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) dv[u] = (i0 + u < cnt) ? __ldg(tdist + hi - 1 - i0 - u) : __int_as_float(0x7f800000);
+            bool stop = false;
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                const float v = D + dv[u];
+                if (v > Mk) { stop = true; break; }  // later bounds only grow
+                const int pos = atomicAdd(&s_cnt, 1);
+                if (pos < kL1Vals) s_keys[pos] = u64(__float_as_uint(v));
+            }
+            if (stop) break;
         }
     }
     __syncthreads();
@@ -267,7 +276,7 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
     int cap = 1;
     while (cap < mt) cap <<= 1;
     cap = std::max(cap, kL1Vals);
-    const int mt4 = (mt + 3) & ~3;
+    const int mt4 = (mt + 3) & ~3;  // s_keys holds the gathered bounds (<= kL1Vals) before phase 2
     size_t smem = sizeof(u64) * cap + sizeof(float) * (mt4 + std::max(mt4, kL1Vals) + dp);
     if (smem > 227 * 1024) {
         set_last_error("level-1: too many target clusters for the shared-memory candidate sort");
