@@ -14,12 +14,44 @@
 //    for DP <= 8 its row) is loaded before the current one is processed.
 #pragma once
 
+#include <stdlib.h>
+
 #include "k_scan_common.cuh"
 
 namespace sknn {
 
-template <int DP, int KMAX>
-__global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
+// kNearests in shared memory (Fig. 8: k*4 <= th1 = smem/SM / threads/SM,
+// P:L629), laid out like the paper's Layout 2 (Fig. 6b): slot r of
+// thread t at [r][t], so a warp's accesses to one slot are contiguous. Sorted
+// ascending; an insertion shifts only the slots above the insertion point.
+constexpr int kTpqThreads = 256;
+struct SmemTopK {
+    key_t* s;
+    int k;
+    __device__ __forceinline__ void init(key_t* col, int k_) {
+        s = col;
+        k = k_;
+        for (int r = 0; r < k; ++r) s[r * kTpqThreads] = kInfKey;
+    }
+    __device__ __forceinline__ key_t get(int r) const { return s[r * kTpqThreads]; }
+    __device__ __forceinline__ void set(int r, key_t v) { s[r * kTpqThreads] = v; }
+    // precondition: key < current k-th; returns the new k-th
+    __device__ __forceinline__ key_t insert(key_t key) {
+        int i = k - 1;
+        while (i > 0) {
+            const key_t v = s[(i - 1) * kTpqThreads];
+            if (!(key < v)) break;
+            s[i * kTpqThreads] = v;
+            --i;
+        }
+        s[i * kTpqThreads] = key;
+        return s[(k - 1) * kTpqThreads];
+    }
+};
+
+template <int DP, int KMAX, bool SMEM>
+__global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
+    extern __shared__ __align__(16) key_t s_topk[];  // [k][256] when SMEM
     const float INF = __int_as_float(0x7f800000);
     const int lane = threadIdx.x & 31;
     const int ntiles = *a.ntiles;
@@ -38,19 +70,32 @@ __global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
         float4 q[DP / 4];
 #pragma unroll
         for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(a.qrows + (int64_t)qpos * DP) + c);
-        RegTopK<KMAX> top;
-        top.init(a.k);
+        RegTopK<SMEM ? 1 : KMAX> top;
+        SmemTopK stop;
+        key_t kth;
+        if constexpr (SMEM) {
+            stop.init(s_topk + threadIdx.x, a.k);
+            kth = kInfKey;
+        } else {
+            top.init(a.k);
+            kth = top.kth();
+        }
         const float ub = a.ub[qc];
         float theta = ub;
         if (a.init_topk && a.dcount[qc] > 0) {  // continue from the dense-tile pass
+            if constexpr (SMEM) {
+                for (int r = 0; r < a.k; ++r) stop.set(r, a.init_topk[(int64_t)qpos * a.k + r]);
+                kth = stop.get(a.k - 1);
+            } else {
 #pragma unroll
-            for (int s = 0; s < KMAX; ++s) {
-                const int r = s - (KMAX - a.k);
-                if (r >= 0) top.a[s] = a.init_topk[(int64_t)qpos * a.k + r];
+                for (int s = 0; s < KMAX; ++s) {
+                    const int r = s - (KMAX - a.k);
+                    if (r >= 0) top.a[s] = a.init_topk[(int64_t)qpos * a.k + r];
+                }
+                kth = top.kth();
             }
-            theta = fminf(ub, __fsqrt_ru(key_d2(top.kth())));
+            theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
         }
-        key_t kth = top.kth();
         float kth_d2 = key_d2(kth);
         const int ncand = a.cand_count[qc];
         const int32_t* cl = a.cand + (int64_t)qc * a.mt;
@@ -90,8 +135,12 @@ __global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
                     if (d2 <= kth_d2) {                                         // line 16 (distance part)
                         const key_t key = make_key(d2, __ldg(a.torig + jc));
                         if (key < kth) {
-                            top.insert(key);
-                            kth = top.kth();
+                            if constexpr (SMEM) {
+                                kth = stop.insert(key);
+                            } else {
+                                top.insert(key);
+                                kth = top.kth();
+                            }
                             kth_d2 = key_d2(kth);
                             theta = fminf(ub, __fsqrt_ru(kth_d2));              // line 17 (R8)
                         }
@@ -99,10 +148,14 @@ __global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
                 }
             }
             const int qo = __ldg(a.qorig + qpos);
+            if constexpr (SMEM) {
+                for (int r = 0; r < a.k; ++r) write_result(a, qo, r, stop.get(r));
+            } else {
 #pragma unroll
-            for (int s = 0; s < KMAX; ++s) {
-                const int r = s - (KMAX - a.k);
-                if (r >= 0) write_result(a, qo, r, top.a[s]);
+                for (int s = 0; s < KMAX; ++s) {
+                    const int r = s - (KMAX - a.k);
+                    if (r >= 0) write_result(a, qo, r, top.a[s]);
+                }
             }
         }
     }
@@ -110,24 +163,35 @@ __global__ void __launch_bounds__(256) k_scan_tpq(ScanArgs a) {
     add_counter(&a.counters->center_evals, cevals);
 }
 
-template <int DP, int KMAX>
+template <int DP, int KMAX, bool SMEM>
 static void launch_tpq(Ctx& cx, const ScanArgs& a) {
-    int grid = occupancy_grid(cx, (const void*)k_scan_tpq<DP, KMAX>, 256, 0);
-    k_scan_tpq<DP, KMAX><<<grid, 256, 0, cx.stream>>>(a);
+    const size_t smem = SMEM ? sizeof(key_t) * (size_t)a.k * kTpqThreads : 0;
+    if (smem > 48 * 1024)
+        cudaFuncSetAttribute(k_scan_tpq<DP, KMAX, SMEM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int grid = occupancy_grid(cx, (const void*)k_scan_tpq<DP, KMAX, SMEM>, kTpqThreads, smem);
+    k_scan_tpq<DP, KMAX, SMEM><<<grid, kTpqThreads, smem, cx.stream>>>(a);
 }
 
-// k -> smallest multiple of 4 >= k (no idle register slots beyond 3)
+// kNearests placement (Fig. 8, P:L587-609 re-derived for B200 in DESIGN.md):
+// shared memory when k*4 <= th1 (k <= 28 on B200), registers otherwise;
+// SKNN_TOPK=reg|smem overrides for ablation.
 template <int DP>
 void launch_tpq_dp(Ctx& cx, const ScanArgs& a) {
+    const char* ov = getenv("SKNN_TOPK");
+    const bool smem = ov ? (ov[0] == 's') : (a.k * 4 <= 114);
+    if (smem) {
+        launch_tpq<DP, 1, true>(cx, a);
+        return;
+    }
     switch ((a.k + 3) / 4) {
-        case 1: launch_tpq<DP, 4>(cx, a); break;
-        case 2: launch_tpq<DP, 8>(cx, a); break;
-        case 3: launch_tpq<DP, 12>(cx, a); break;
-        case 4: launch_tpq<DP, 16>(cx, a); break;
-        case 5: launch_tpq<DP, 20>(cx, a); break;
-        case 6: launch_tpq<DP, 24>(cx, a); break;
-        case 7: launch_tpq<DP, 28>(cx, a); break;
-        default: launch_tpq<DP, 32>(cx, a); break;
+        case 1: launch_tpq<DP, 4, false>(cx, a); break;
+        case 2: launch_tpq<DP, 8, false>(cx, a); break;
+        case 3: launch_tpq<DP, 12, false>(cx, a); break;
+        case 4: launch_tpq<DP, 16, false>(cx, a); break;
+        case 5: launch_tpq<DP, 20, false>(cx, a); break;
+        case 6: launch_tpq<DP, 24, false>(cx, a); break;
+        case 7: launch_tpq<DP, 28, false>(cx, a); break;
+        default: launch_tpq<DP, 32, false>(cx, a); break;
     }
 }
 

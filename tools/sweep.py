@@ -37,6 +37,8 @@ VARIANTS = {
     "tcassign": {"_env": ("SKNN_ASSIGN", "tc")},
     "entries256": {"_env": ("SKNN_WALK_ENTRIES", "256")},
     "paperseed": {"_env": ("SKNN_SEEDING", "paper")},
+    "topk_reg": {"_env": ("SKNN_TOPK", "reg")},
+    "topk_smem": {"_env": ("SKNN_TOPK", "smem")},
     "full_lloyd4": {"_env": ("SKNN_ASSIGN", "full"), "lloyd_iters": 4},
 }
 
