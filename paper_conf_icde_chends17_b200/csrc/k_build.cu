@@ -501,7 +501,7 @@ __device__ __forceinline__ void cmpx(u64* s, int i, int p) {
 
 constexpr int kSmallSeg = 4096;
 
-__global__ void __launch_bounds__(512) k_segsort_small(u64* __restrict__ keys, const int32_t* __restrict__ off,
+__global__ void __launch_bounds__(128) k_segsort_small(u64* __restrict__ keys, const int32_t* __restrict__ off,
                                                        float* __restrict__ radius) {
     __shared__ u64 s[kSmallSeg];
     int c = blockIdx.x;
@@ -680,7 +680,9 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     // the nearest landmark (one k-means|| round), so small or far groups of
     // points get a center instead of inflating a far cluster's radius.
     const char* sd = getenv("SKNN_SEEDING");
-    const bool d2seed = !(sd && strcmp(sd, "paper") == 0) && m >= 64;
+    // (measured: helps dp >= 16 -- C3 202 -> 137 candidate clusters -- and is
+    // neutral for the low-dimensional C1/C2, where it only costs a pass)
+    const bool d2seed = !(sd && strcmp(sd, "paper") == 0) && m >= 64 && (dp >= 16 || (sd && strcmp(sd, "d2") == 0));
     const int m0 = d2seed ? (m + 1) / 2 : m;
     // landmark sampler
     int32_t* lidx;
@@ -818,7 +820,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     int sblocks = (int)std::min<int64_t>((n + 255) / 256, 148 * 16);
     k_scatter_keys<<<sblocks, 256, 0, s>>>(cid, pdist, n, out.off, cursor, keys);
     cx.launched();
-    k_segsort_small<<<m, 512, 0, s>>>(keys, out.off, out.radius);
+    k_segsort_small<<<m, 128, 0, s>>>(keys, out.off, out.radius);
     cx.launched();
     k_segsort_big<<<m, 1024, 0, s>>>(keys, out.off, out.radius);
     cx.launched();
