@@ -106,7 +106,8 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     const float* __restrict__ tcent, const float* __restrict__ trad, const int32_t* __restrict__ toff,
     const float* __restrict__ tdist, int mt, int dp, int k, float eta, int keys_cap, int shard_rank,
     int shard_count, int dense_mode, float dense_tau, float* __restrict__ ub_out, int32_t* __restrict__ cand,
-    int32_t* __restrict__ cand_count, int32_t* __restrict__ dcand, int32_t* __restrict__ dcount,
+    int32_t* __restrict__ cand_count, float* __restrict__ cand_D, int32_t* __restrict__ dcand,
+    int32_t* __restrict__ dcount,
     Counters* __restrict__ counters) {
     extern __shared__ __align__(16) unsigned char smem[];
     u64* s_keys = reinterpret_cast<u64*>(smem);                               // keys_cap (>= mt) entries
@@ -211,6 +212,7 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     // cluster is big enough to fill tiles (cost model in DESIGN.md §6).
     int32_t* row = cand + (int64_t)qc * mt;
     int32_t* drow = dcand + (int64_t)qc * mt;
+    float* Drow = cand_D + (int64_t)qc * mt;
     __shared__ int s_wcnt[2][kL1Threads / 32];
     __shared__ int s_base[2];
     if (threadIdx.x == 0) { s_base[0] = 0; s_base[1] = 0; }
@@ -244,7 +246,11 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
         const unsigned below = (1u << lane) - 1u;
         if (i < nc) {
             if (dense) drow[s_base[1] + offd + __popc(md & below)] = tc;
-            else row[s_base[0] + offs + __popc(ms & below)] = tc;
+            else {
+                const int pos = s_base[0] + offs + __popc(ms & below);
+                row[pos] = tc;
+                Drow[pos] = __uint_as_float(uint32_t(s_keys[i] >> 32));  // center distance D (Eq. 3 per query)
+            }
         }
         __syncthreads();
         if (threadIdx.x == 0) {
@@ -271,6 +277,7 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
     SKNN_TRY(cx.alloc_scratch((void**)&out.ub, sizeof(float) * mq));
     SKNN_TRY(cx.alloc_scratch((void**)&out.cand, sizeof(int32_t) * (size_t)mq * mt));
     SKNN_TRY(cx.alloc_scratch((void**)&out.cand_count, sizeof(int32_t) * mq));
+    SKNN_TRY(cx.alloc_scratch((void**)&out.cand_D, sizeof(float) * (size_t)mq * mt));
     SKNN_TRY(cx.alloc_scratch((void**)&out.dcand, sizeof(int32_t) * (size_t)mq * mt));
     SKNN_TRY(cx.alloc_scratch((void**)&out.dcount, sizeof(int32_t) * mq));
     int cap = 1;
@@ -285,7 +292,7 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
     SKNN_CUDA(cudaFuncSetAttribute(k_level1, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     k_level1<<<mq, kL1Threads, smem, cx.stream>>>(qs.centers, qs.radius, qs.off, ts.centers, ts.radius, ts.off,
                                                   ts.dist, mt, dp, p.k, p.eta, cap, p.shard_rank, p.shard_count,
-                                                  p.dense_mode, p.dense_tau, out.ub, out.cand, out.cand_count,
+                                                  p.dense_mode, p.dense_tau, out.ub, out.cand, out.cand_count, out.cand_D,
                                                   out.dcand, out.dcount, counters);
     cx.launched();
     return cx.check_launch("level1");

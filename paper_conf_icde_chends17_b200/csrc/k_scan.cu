@@ -190,7 +190,8 @@ sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, 
     ScanArgs a{};
     a.qrows = qs.rows; a.qorig = qs.orig; a.qoff = qs.off;
     a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
-    a.ub = l1.ub; a.cand = l1.cand; a.cand_count = l1.cand_count;
+    a.ub = l1.ub; a.cand = l1.cand; a.cand_count = l1.cand_count; a.cand_D = l1.cand_D;
+    a.qdist = qs.dist; a.trad = ts.radius;
     a.tiles = l1.tiles; a.ntiles = l1.ntiles; a.tile_counter = l1.ntiles + 1;
     a.init_topk = p.init_topk; a.dcount = l1.dcount;
     a.mt = ts.m; a.dp = dp; a.k = p.k; a.tile = l1.tile; a.eta = p.eta;

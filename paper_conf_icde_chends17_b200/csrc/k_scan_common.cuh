@@ -23,6 +23,9 @@ struct ScanArgs {
     const float* ub;
     const int32_t* cand;
     const int32_t* cand_count;
+    const float* cand_D;
+    const float* qdist;   // query's own member distance d(q, c_q)
+    const float* trad;    // target cluster radius
     const int2* tiles;
     const int* ntiles;
     int* tile_counter;     // dynamic tile scheduler (zeroed by k_make_tiles)

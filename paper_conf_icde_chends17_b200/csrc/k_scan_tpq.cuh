@@ -99,12 +99,22 @@ __global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
         float kth_d2 = key_d2(kth);
         const int ncand = a.cand_count[qc];
         const int32_t* cl = a.cand + (int64_t)qc * a.mt;
+        const float* cD = a.cand_D + (int64_t)qc * a.mt;
+        const float rown = __ldg(a.qdist + qpos);  // d(q, c_q)
         if (active) {
             for (int c = 0; c < ncand; ++c) {
                 const int tc = __ldg(cl + c);
+                // per-query 2-landmark bound (Eq. 3 with the query itself in place of
+                // the query cluster's farthest member): D - d(q,c_q) - r_t <= d(q,t)
+                const float D = __ldg(cD + c), rt = __ldg(a.trad + tc);
+                if (!ti_keep(D - rown - rt, theta, D + rown + rt, a.eta)) continue;
                 const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
                 const float dq = __fsqrt_rn(d2_reg<DP>(q, a.tcent + (int64_t)tc * DP));  // Alg. 2 line 6
                 ++cevals;
+                // empty window: every member distance lies in [dt_min, r_t]
+                if (!ti_keep(dq - rt, theta, dq + rt, a.eta)) continue;
+                const float dtmin = __ldg(a.tdist + hi - 1);
+                if (!ti_keep(dtmin - dq, theta, dq + dtmin, a.eta)) continue;
                 // Alg. 2 lines 7-17, visited in order of the 1-landmark lower bound
                 // |l| = |dq - dt| (Eq. 1): start where dt ~ dq and walk outward on
                 // both sides, always taking the side with the smaller bound, until

@@ -94,6 +94,7 @@ struct Level1 {
     float* ub = nullptr;          // [mq] inflated calUB per query cluster
     int32_t* cand = nullptr;      // [mq x mt] candidate target clusters, ascending center distance
     int32_t* cand_count = nullptr;  // [mq]
+    float* cand_D = nullptr;      // [mq x mt] center distance D(qc, tc) of each sparse candidate
     int2* tiles = nullptr;        // level-2 work tiles (query cluster, first member)
     int* ntiles = nullptr;        // [2]: tile count, scheduler counter
     int tile = 0;
