@@ -65,14 +65,22 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
             if (a.init_topk && a.dcount[qc] > 0 && lane >= 32 - a.k) mine = a.init_topk[(int64_t)qpos * a.k + lane - (32 - a.k)];
             key_t kth = __shfl_sync(0xffffffffu, mine, 31);
             float theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
+            const float rown = __ldg(a.qdist + qpos);  // d(q, c_q)
+            const float* cD = a.cand_D + (int64_t)qc * a.mt;
             for (int c = 0; c < ncand; ++c) {
                 const int tc = __ldg(cl + c);
+                // per-query 2-landmark bound (Eq. 3), then the empty-window checks
+                const float D = __ldg(cD + c), rt = __ldg(a.trad + tc);
+                if (!ti_keep(D - rown - rt, theta, D + rown + rt, a.eta)) continue;
                 const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
                 float dq2;
                 if constexpr (DP > 0) dq2 = d2_reg<DP>(q, a.tcent + (int64_t)tc * DP);
                 else dq2 = d2_rows(sq, a.tcent + (int64_t)tc * dp, dp);
                 const float dq = __fsqrt_rn(dq2);
                 if (lane == 0) ++cevals;
+                if (!ti_keep(dq - rt, theta, dq + rt, a.eta)) continue;
+                const float dtmin = __ldg(a.tdist + hi - 1);
+                if (!ti_keep(dtmin - dq, theta, dq + dtmin, a.eta)) continue;
                 const int j0 = window_start(a.tdist, lo, hi, dq, theta, a.eta);
                 for (int base = j0; base < hi; base += 32) {
                     const int j = base + lane;
