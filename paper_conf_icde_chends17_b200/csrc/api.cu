@@ -195,8 +195,17 @@ struct Marks {
 static int dense_mode_for(const sknn_options& o, int dp) {
     if (o.force_path == SKNN_PATH_DENSE) return 2;
     if (o.force_path == SKNN_PATH_SPARSE) return 1;
-    // tensor cores pay once a distance costs more than the screen (dp >= 16)
-    return (dp >= 16 && dense_supported(dp)) ? 0 : 1;
+    // Measured per-pair cost ratio dense/sparse: ~0.3 at d = 16,
+    // ~0.1 at d = 28, ~0.01 at d = 128. With the per-query bounds the sparse
+    // scan wins at d <= 16, so the switch is armed only above.
+    if (o.dense_threshold > 0.f) return dense_supported(dp) ? 0 : 1;
+    return (dp > 16 && dense_supported(dp)) ? 0 : 1;
+}
+
+// default window-share threshold of the elastic switch (dp > 16)
+static float dense_tau_for(const sknn_options& o, int dp) {
+    if (o.dense_threshold > 0.f) return o.dense_threshold;
+    return dp >= 64 ? 0.5f : 0.95f;
 }
 
 // The query half of Fig. 4 (lines 3-6) given both clustered sides:
@@ -211,7 +220,7 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     lp.shard_rank = o.shard_count > 1 ? o.shard_rank : 0;
     lp.shard_count = o.shard_count > 1 ? o.shard_count : 1;
     lp.dense_mode = dense_mode_for(o, ts.dp);
-    lp.dense_tau = o.dense_threshold > 0.f ? o.dense_threshold : 0.5f;
+    lp.dense_tau = dense_tau_for(o, ts.dp);
     if (lp.dense_mode == 2 && !dense_supported(ts.dp)) {
         set_last_error("force_path = DENSE needs d <= 256");
         return SKNN_ERR_UNSUPPORTED;

@@ -278,11 +278,12 @@ def test_dense_tiles_ties_and_dims(sknn):
 def test_auto_switch_mixes_paths(sknn):
     """The elastic switch (auto) on a dp >= 16 workload sends some pairs to
     dense tiles and the rest to the sparse scan; results stay exact."""
-    Q, T, k, sj = datagen.workload("C5", 0.0025)
+    Q, T, k, sj = datagen.workload("C4", 0.01)
     idx, dist, st = run(sknn, Q, T, k, sj)
     ridx, rdist = oracle.knn_join(Q, T, k)
     assert_knn_bitexact(idx, dist, ridx, rdist)
-    assert st["dense_pairs"] > 0
+    assert st["dense_pairs"] > 0 and st["dist_evals_sparse"] > 0
+    assert st["dense_pairs"] < st["cand_pairs"]
 
 
 # ------------------------------------------------------------ multi-GPU --
