@@ -125,6 +125,14 @@ __global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
                 int L = R - 1;
                 float dtL = L >= lo ? __ldg(a.tdist + L) : 0.f;
                 float dtR = R < hi ? __ldg(a.tdist + R) : 0.f;
+                // DP == 4: both frontier rows are kept in registers, the consumed
+                // side is refilled while its distance is computed
+                constexpr bool kPre = DP == 4;
+                float4 rowL = make_float4(0.f, 0.f, 0.f, 0.f), rowR = rowL;
+                if constexpr (kPre) {
+                    if (L >= lo) rowL = __ldg(reinterpret_cast<const float4*>(a.trows) + L);
+                    if (R < hi) rowR = __ldg(reinterpret_cast<const float4*>(a.trows) + R);
+                }
                 for (;;) {
                     const float bL = L >= lo ? dtL - dq : INF;       // -l on the left (dt > dq)
                     const float bR = R < hi ? dq - dtR : INF;        // l on the right (dt <= dq)
@@ -133,14 +141,33 @@ __global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
                     const float dtc = takeL ? dtL : dtR;
                     if (!ti_keep(bmin, theta, dq + dtc, a.eta)) break;  // both sides beyond theta
                     const int jc = takeL ? L : R;
-                    if (takeL) {
-                        --L;
-                        if (L >= lo) dtL = __ldg(a.tdist + L);
+                    float d2;                                                   // line 15
+                    if constexpr (kPre) {
+                        const float4 row = takeL ? rowL : rowR;
+                        if (takeL) {
+                            --L;
+                            if (L >= lo) {
+                                dtL = __ldg(a.tdist + L);
+                                rowL = __ldg(reinterpret_cast<const float4*>(a.trows) + L);
+                            }
+                        } else {
+                            ++R;
+                            if (R < hi) {
+                                dtR = __ldg(a.tdist + R);
+                                rowR = __ldg(reinterpret_cast<const float4*>(a.trows) + R);
+                            }
+                        }
+                        d2 = d2_acc4(0.f, q[0], row);
                     } else {
-                        ++R;
-                        if (R < hi) dtR = __ldg(a.tdist + R);
+                        if (takeL) {
+                            --L;
+                            if (L >= lo) dtL = __ldg(a.tdist + L);
+                        } else {
+                            ++R;
+                            if (R < hi) dtR = __ldg(a.tdist + R);
+                        }
+                        d2 = d2_reg<DP>(q, a.trows + (int64_t)jc * DP);
                     }
-                    const float d2 = d2_reg<DP>(q, a.trows + (int64_t)jc * DP);  // line 15
                     ++evals;
                     if (d2 <= kth_d2) {                                         // line 16 (distance part)
                         const key_t key = make_key(d2, __ldg(a.torig + jc));
