@@ -67,13 +67,19 @@ __host__ __device__ constexpr uint32_t idesc_bf16_m128(int n) {
     return (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(n >> 3) << 17) | (uint32_t(kTcM >> 4) << 24);
 }
 
-// o = mean of the m centers (one CTA, fixed order per column)
+// o = mean of the m centers: one CTA per column, fixed-order tree (deterministic)
 __global__ void k_center_mean(const float* __restrict__ centers, int m, int dp, float* __restrict__ o) {
-    for (int c = threadIdx.x; c < dp; c += blockDim.x) {
-        double s = 0.0;
-        for (int j = 0; j < m; ++j) s += centers[(int64_t)j * dp + c];
-        o[c] = (float)(s / m);
+    __shared__ double red[256];
+    const int c = blockIdx.x;
+    double s = 0.0;
+    for (int j = threadIdx.x; j < m; j += blockDim.x) s += centers[(int64_t)j * dp + c];
+    red[threadIdx.x] = s;
+    __syncthreads();
+    for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+        if (threadIdx.x < w) red[threadIdx.x] += red[threadIdx.x + w];
+        __syncthreads();
     }
+    if (threadIdx.x == 0) o[c] = (float)(red[0] / m);
 }
 
 // centers -> bf16 (c - o) in chunked core-matrix layout + ||b||^2 of the rounded values
@@ -260,7 +266,7 @@ sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
     SKNN_TRY(cx.alloc_scratch((void**)&o, sizeof(float) * dp));
     SKNN_TRY(cx.alloc_scratch((void**)&cbf, (size_t)mpad * kp * 2));
     SKNN_TRY(cx.alloc_scratch((void**)&bn, sizeof(float) * mpad));
-    k_center_mean<<<1, 128, 0, cx.stream>>>(centers, m, dp, o);
+    k_center_mean<<<dp, 256, 0, cx.stream>>>(centers, m, dp, o);
     cx.launched();
     const int64_t work = (int64_t)mpad * (kp / 8);
     k_centers_to_tc<<<(int)std::min<int64_t>((work + 255) / 256, 148 * 8), 256, 0, cx.stream>>>(centers, m, mpad, dp, kp,
@@ -269,6 +275,7 @@ sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
     // >= 90 KB keeps at most two CTAs per SM: each holds 256 of the 512 TMEM columns
     const size_t smem = std::max<size_t>((size_t)kTcM * kp * 2 + 2 * (size_t)kTcN * kp * 2 + 2 * kTcN * 4, 90 * 1024);
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     const int64_t grid = (n + kTcM - 1) / kTcM;
     k_assign_tc<<<(unsigned)grid, kTcM, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, bn, m, nchunks, centers, cid, dist,
                                                           sums, fx, counts);

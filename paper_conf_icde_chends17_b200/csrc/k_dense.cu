@@ -1,76 +1,51 @@
 // k_dense.cu -- the elastic switch's dense-tile branch (
-// the paper's partial level-2 filter idea: when a cluster pair is
-// dense, regularity beats per-point TI checks).
+// the paper's "regular" partial level-2 filter idea: when a
+// cluster pair is dense, regularity beats per-point TI checks).
 //
 // For a tile of up to 128 queries of one query cluster and each of its dense
-// candidate target clusters, the whole target cluster (no per-point TI checks:
-// the regular path of the elastic switch) is streamed through shared memory in
-// chunks of NCH targets and the 128 x NCH dot products run on the
-// 5th-generation tensor cores:
+// candidate target clusters, the whole target cluster (no per-point TI checks)
+// is streamed in chunks of NCH targets and the 128 x NCH dot products run on
+// the 5th-generation tensor cores:
 //
-//   a = q - c_r, b = t - c_r            (c_r = query-cluster center rounded to
-//                                        integers: re-centring avoids the
-//                                        ||q||^2 + ||t||^2 - 2 q.t cancellation)
+//   a = q - o, b = t - o        o = mean target center rounded to integers
+//                               (re-centring against ||q||^2 + ||t||^2 - 2 q.t
+//                               cancellation; integer data stays integer)
 //   a = a_hi + a_lo (bf16 split), same for b
-//   D = a_hi.b_hi + a_hi.b_lo + a_lo.b_hi   tcgen05.mma kind::f16, fp32 accumulator in TMEM
-//   d2~ = ||a||^2 + ||b||^2 - 2 D            (lo terms skipped when every lo is 0)
+//   D = a_hi.b_hi [+ a_hi.b_lo + a_lo.b_hi]   tcgen05.mma kind::f16, fp32 in TMEM
+//   d2~ = ||a||^2 + ||b||^2 - 2 D             (lo terms only when some lo != 0)
 //
-// The epilogue (one thread per TMEM lane = query row, tcgen05.ld) is a SCREEN:
-// d2~ has a rigorous error bound E = eps (||a||^2 + ||b||^2) + (K+2) 2^-23 d2_k,
-// eps = 2^-12 max(1, K/128) (bf16 split truncation 3*2^-16 + fp32 accumulation
-// of 3K terms, doubled). A target survives iff d2~ - E <= the row's k-th
-// squared distance; survivors are recomputed with the exact fp32 formula every
-// path shares (d2_rows) and inserted into the row's register top-k, so the
-// result keys are bit-identical to the sparse path's. The per-row top-k is
-// handed to the sparse scan, which continues over the remaining (sparse)
-// candidate clusters.
+// B200 data path: both point sets are converted ONCE per join into the UMMA
+// canonical K-major SWIZZLE_NONE layout (8-row x 16-byte core matrices; LBO =
+// 128 B, SBO = KP*16 B), every cluster starting on an 8-row boundary, so a
+// 128-query A tile and every NCH-target B chunk are contiguous byte ranges.
+// They move with 1-D bulk async copies (cp.async.bulk, the TMA engine) through
+// a 2-deep shared-memory ring, while the MMA of chunk g+1 runs into the second
+// TMEM accumulator and the four warps reduce chunk g (tcgen05.ld).
 //
-// Operands use the UMMA canonical K-major SWIZZLE_NONE layout: 8-row x 16-byte
-// core matrices; LBO = 128 B (next 8 K-elements), SBO = KP*16 B (next 8 rows).
+// The epilogue (one thread per TMEM lane = query row) is a SCREEN: d2~ has the
+// rigorous error bound E = eps (||a||^2 + ||b||^2) + (K+2) 2^-23 d2_k with
+// eps = 2^-12 max(1, K/128) (bf16 split truncation + fp32 accumulation of 3K
+// terms, doubled). A target survives iff d2~ - E <= the row's k-th squared
+// distance; survivors are recomputed with the exact fp32 formula every path
+// shares (d2_rows) and inserted into the row's register top-k, so the keys are
+// bit-identical to the sparse path's. The sparse scan continues from the
+// per-row top-k over the remaining (sparse) candidate clusters.
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
+#include <math.h>
 #include <stdint.h>
 
 #include "k_scan_common.cuh"
 
 namespace sknn {
 
-struct DenseArgs {
-    const float* qrows;
-    const int32_t* qoff;
-    const float* qcent;
-    const float* trows;
-    const float* tdist;
-    const int32_t* torig;
-    const int32_t* toff;
-    const float* tcent;
-    const float* ub;
-    const int32_t* dcand;
-    const int32_t* dcount;
-    const int2* tiles;
-    const int* ntiles;
-    int* counter;
-    int mt;
-    int dp;
-    int kp;       // K padded to a multiple of 16 (bf16 MMA K)
-    int k;
-    float eta;
-    float eps_tc;
-    key_t* topk_out;  // [n_q x k] in permuted query order
-    Counters* counters;
-};
-
 constexpr int kDenseM = 128;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
-__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
-    uint64_t d = 0;
-    d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
-    d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
-    d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
-    d |= (uint64_t)1 << 46;  // descriptor version 1 (sm_100); base offset 0; SWIZZLE_NONE
-    return d;
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t sbo) {
+    return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)(128u >> 4) << 16) | ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) |
+           ((uint64_t)1 << 46);  // LBO 128 B, descriptor version 1 (sm_100), SWIZZLE_NONE
 }
 
 // kind::f16 instruction descriptor: BF16 x BF16 -> F32, both K-major, M = 128
@@ -80,25 +55,32 @@ __host__ __device__ constexpr uint32_t umma_idesc_bf16(int n) {
 
 __device__ __forceinline__ void umma_bf16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
     asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "setp.ne.b32 p, %4, 0;\n\t"
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(tmem_d),
         "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
 
-__device__ __forceinline__ void umma_commit(uint64_t* bar) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+__device__ __forceinline__ void umma_commit(uint32_t bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t phase) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\tWAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@!P1 bra WAIT_%=;\n\t}\n" ::"r"(bar),
+        "r"(phase)
+        : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+                 "l"(src), "r"(bytes), "r"(bar)
                  : "memory");
 }
 
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
-    asm volatile(
-        "{\n\t.reg .pred P1;\n\t"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-        "@!P1 bra WAIT_%=;\n\t}\n" ::"r"(smem_u32(bar)),
-        "r"(phase)
-        : "memory");
+__device__ __forceinline__ void expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
 }
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
@@ -113,52 +95,171 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
-__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
-// 8 fp32 -> (hi, lo) bf16 pairs packed as two 16-byte core-matrix rows
-__device__ __forceinline__ bool split8(const float (&v)[8], uint4& hi, uint4& lo) {
-    uint32_t h[4], l[4];
-    bool nz = false;
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-        __nv_bfloat16 h0 = __float2bfloat16_rn(v[2 * i]), h1 = __float2bfloat16_rn(v[2 * i + 1]);
-        __nv_bfloat16 l0 = __float2bfloat16_rn(v[2 * i] - __bfloat162float(h0));
-        __nv_bfloat16 l1 = __float2bfloat16_rn(v[2 * i + 1] - __bfloat162float(h1));
-        h[i] = (uint32_t)__bfloat16_as_ushort(h0) | ((uint32_t)__bfloat16_as_ushort(h1) << 16);
-        l[i] = (uint32_t)__bfloat16_as_ushort(l0) | ((uint32_t)__bfloat16_as_ushort(l1) << 16);
-        nz |= (l[i] & 0x7fff7fffu) != 0u;
+// ------------------------------------------------------ tile conversion --
+// rintf of the mean center: the common origin o of both point sets
+__global__ void k_dense_origin(const float* __restrict__ centers, int m, int dp, int kp, float* __restrict__ o) {
+    __shared__ double red[256];
+    const int c = blockIdx.x;
+    double s = 0.0;
+    if (c < dp)
+        for (int j = threadIdx.x; j < m; j += blockDim.x) s += centers[(int64_t)j * dp + c];
+    red[threadIdx.x] = s;
+    __syncthreads();
+    for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+        if (threadIdx.x < w) red[threadIdx.x] += red[threadIdx.x + w];
+        __syncthreads();
     }
-    hi = make_uint4(h[0], h[1], h[2], h[3]);
-    lo = make_uint4(l[0], l[1], l[2], l[3]);
-    return nz;
+    if (threadIdx.x == 0) o[c] = c < dp ? rintf((float)(red[0] / m)) : 0.f;
 }
+
+// cluster sizes rounded up to 8 rows (padded CSR for 8-row-aligned tiles)
+__global__ void k_pad8(const int32_t* __restrict__ off, int m, int32_t* __restrict__ cnt8) {
+    for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < m; c += gridDim.x * blockDim.x)
+        cnt8[c] = ((off[c + 1] - off[c]) + 7) & ~7;
+}
+
+// rows (cluster order) -> bf16 hi/lo (x - o) tiles + ||x - o||^2 * nscale, at padded positions
+__global__ void __launch_bounds__(256) k_to_tiles(const float* __restrict__ rows, const int32_t* __restrict__ off,
+                                                  const int32_t* __restrict__ offp, int dp, int kp,
+                                                  const float* __restrict__ o, float nscale,
+                                                  __nv_bfloat16* __restrict__ hi, __nv_bfloat16* __restrict__ lo,
+                                                  float* __restrict__ norm, float* __restrict__ norm_raw,
+                                                  int* __restrict__ lo_flag) {
+    const int c = blockIdx.x;
+    const int lo0 = off[c], size = off[c + 1] - lo0, p0 = offp[c];
+    const int c8n = kp / 8;
+    const size_t sbo = (size_t)kp * 16;
+    bool nz = false;
+    for (int w = threadIdx.x; w < size * c8n; w += blockDim.x) {
+        const int r = w / c8n, c8 = w % c8n;
+        const float* src = rows + (int64_t)(lo0 + r) * dp;
+        uint32_t h[4], l[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            float v[2];
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+                const int kk = c8 * 8 + 2 * i + e;
+                v[e] = kk < dp ? src[kk] - o[kk] : 0.f;
+            }
+            const __nv_bfloat16 h0 = __float2bfloat16_rn(v[0]), h1 = __float2bfloat16_rn(v[1]);
+            const __nv_bfloat16 l0 = __float2bfloat16_rn(v[0] - __bfloat162float(h0));
+            const __nv_bfloat16 l1 = __float2bfloat16_rn(v[1] - __bfloat162float(h1));
+            h[i] = (uint32_t)__bfloat16_as_ushort(h0) | ((uint32_t)__bfloat16_as_ushort(h1) << 16);
+            l[i] = (uint32_t)__bfloat16_as_ushort(l0) | ((uint32_t)__bfloat16_as_ushort(l1) << 16);
+            nz |= (l[i] & 0x7fff7fffu) != 0u;
+        }
+        const int p = p0 + r;
+        const size_t byte = (size_t)(p >> 3) * sbo + (size_t)c8 * 128 + (size_t)(p & 7) * 16;
+        *reinterpret_cast<uint4*>(reinterpret_cast<unsigned char*>(hi) + byte) = make_uint4(h[0], h[1], h[2], h[3]);
+        *reinterpret_cast<uint4*>(reinterpret_cast<unsigned char*>(lo) + byte) = make_uint4(l[0], l[1], l[2], l[3]);
+    }
+    for (int r = threadIdx.x; r < size; r += blockDim.x) {
+        const float* src = rows + (int64_t)(lo0 + r) * dp;
+        float s = 0.f;
+        for (int kk = 0; kk < dp; ++kk) {
+            const float v = src[kk] - o[kk];
+            s = __fmaf_rn(v, v, s);
+        }
+        norm[p0 + r] = s * nscale;
+        if (norm_raw) norm_raw[p0 + r] = s;
+    }
+    if (__syncthreads_or(nz) && threadIdx.x == 0) atomicOr(lo_flag, 1);
+}
+
+__global__ void k_fill_f(float* __restrict__ p, int64_t n, float v) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
+
+// ----------------------------------------------------------------- kernel --
+struct DenseArgs {
+    const float* qrows;
+    const int32_t* qoff;
+    const int32_t* qoffp;
+    const unsigned char* qhi;
+    const unsigned char* qlo;
+    const float* qn;
+    const float* trows;
+    const int32_t* torig;
+    const int32_t* toff;
+    const int32_t* toffp;
+    const unsigned char* thi;
+    const unsigned char* tlo;
+    const float* tn;       // ||b||^2 (1 - eps), +inf on padding rows
+    const int* lo_flag;    // [2]: query side, target side has a nonzero lo part
+    const float* ub;
+    const int32_t* dcand;
+    const int32_t* dcount;
+    const int2* tiles;
+    const int* ntiles;
+    int* counter;
+    int mt;
+    int dp;
+    int kp;
+    int k;
+    float eps_tc;
+    key_t* topk_out;
+    Counters* counters;
+};
+
+// per-tile chunk sequence: every dense candidate cluster in NCH-target chunks
+template <int NCH>
+struct ChunkIter {
+    const int32_t* dl;
+    int nd, ci, c, nch, tc, size;
+    __device__ __forceinline__ void start(const DenseArgs& a, int qc) {
+        dl = a.dcand + (int64_t)qc * a.mt;
+        nd = a.dcount[qc];
+        ci = -1;
+        c = 0;
+        nch = 0;
+        advance(a);
+    }
+    // moves to the next chunk; false when exhausted
+    __device__ __forceinline__ bool advance(const DenseArgs& a) {
+        ++c;
+        while (c >= nch) {
+            if (++ci >= nd) return false;
+            tc = __ldg(dl + ci);
+            size = __ldg(a.toff + tc + 1) - __ldg(a.toff + tc);
+            nch = (size + NCH - 1) / NCH;
+            c = 0;
+        }
+        return true;
+    }
+    __device__ __forceinline__ bool valid() const { return ci < nd; }
+};
 
 template <int KMAX, int NCH>
 __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
     extern __shared__ __align__(128) unsigned char smem[];
     const int KP = a.kp;
     const int dp = a.dp;
-    const uint32_t sbo = (uint32_t)KP * 16u;  // bytes between 8-row groups
-    unsigned char* sA_hi = smem;
-    unsigned char* sA_lo = sA_hi + (size_t)kDenseM * KP * 2;
-    unsigned char* sB_hi = sA_lo + (size_t)kDenseM * KP * 2;
-    unsigned char* sB_lo = sB_hi + (size_t)NCH * KP * 2;
-    float* s_tn = reinterpret_cast<float*>(sB_lo + (size_t)NCH * KP * 2);  // [NCH]
-    float* s_cr = s_tn + NCH;                                             // [KP]
-    __shared__ uint64_t s_bar;
+    const uint32_t sbo = (uint32_t)KP * 16u;
+    const uint32_t a_bytes = (uint32_t)kDenseM * KP * 2, b_bytes = (uint32_t)NCH * KP * 2;
+    // layout: A_hi | A_lo | B_hi[2] | B_lo[2] | tn[2][NCH]
+    unsigned char* sA = smem;
+    unsigned char* sB = smem + 2 * a_bytes;
+    float* s_tn = reinterpret_cast<float*>(sB + 4 * b_bytes);
+    __shared__ __align__(8) uint64_t bar_a, bar_full[2], bar_mma[2];
     __shared__ uint32_t s_tmem;
-    __shared__ int s_tile, s_loA, s_loB;
+    __shared__ int s_tile;
 
     const int tid = threadIdx.x, warp = tid >> 5;
     if (warp == 0) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&s_tmem)),
-                     "r"((uint32_t)NCH));
+                     "r"((uint32_t)(2 * NCH)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     if (tid == 0) {
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&s_bar)));
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&bar_a)));
+        for (int i = 0; i < 2; ++i) {
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&bar_full[i])));
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&bar_mma[i])));
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     tc_fence_before();
@@ -166,11 +267,37 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
     tc_fence_after();
     const uint32_t tmem = s_tmem;
     const uint32_t tmem_row = tmem + ((uint32_t)(warp * 32) << 16);
-    uint32_t phase = 0;
     const uint32_t idesc = umma_idesc_bf16(NCH);
+    const bool loA = a.lo_flag[0] != 0, loB = a.lo_flag[1] != 0;
+    const uint32_t bstage = loB ? 2 * b_bytes : b_bytes;  // bytes moved per B chunk
     const float INF = __int_as_float(0x7f800000);
     const float rel_k = 1.f + (float)(KP + 2) * 1.1920929e-7f;  // (K+2) 2^-23
+    const float qscale = 1.f - a.eps_tc;
+    uint32_t ph_a = 0, ph_full[2] = {0, 0}, ph_mma[2] = {0, 0};
     unsigned long long covered = 0, recomputed = 0;
+
+    auto issue_b = [&](const ChunkIter<NCH>& it, int buf) {
+        const uint32_t bar = smem_u32(&bar_full[buf]);
+        expect_tx(bar, bstage + NCH * 4);
+        const size_t p = (size_t)__ldg(a.toffp + it.tc) + (size_t)it.c * NCH;  // 8-aligned padded row
+        const size_t byte = (p >> 3) * sbo;
+        bulk_g2s(smem_u32(sB + buf * b_bytes), a.thi + byte, b_bytes, bar);
+        if (loB) bulk_g2s(smem_u32(sB + (2 + buf) * b_bytes), a.tlo + byte, b_bytes, bar);
+        bulk_g2s(smem_u32(s_tn + buf * NCH), a.tn + p, NCH * 4, bar);
+    };
+    auto issue_mma = [&](int buf) {
+        tc_fence_after();
+        const uint32_t aH = smem_u32(sA), aL = smem_u32(sA + a_bytes);
+        const uint32_t bH = smem_u32(sB + buf * b_bytes), bL = smem_u32(sB + (2 + buf) * b_bytes);
+        const uint32_t d = tmem + (uint32_t)(buf * NCH);
+        for (int s = 0; s < KP / 16; ++s) {
+            const uint32_t ko = (uint32_t)s * 256u;
+            umma_bf16(d, umma_desc(aH + ko, sbo), umma_desc(bH + ko, sbo), idesc, s > 0);
+            if (loB) umma_bf16(d, umma_desc(aH + ko, sbo), umma_desc(bL + ko, sbo), idesc, 1);
+            if (loA) umma_bf16(d, umma_desc(aL + ko, sbo), umma_desc(bH + ko, sbo), idesc, 1);
+        }
+        umma_commit(smem_u32(&bar_mma[buf]));
+    };
 
     for (;;) {
         if (tid == 0) s_tile = atomicAdd(a.counter, 1);
@@ -184,148 +311,91 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
         const bool active = tl.y + r < qsz;
         const int qpos = qlo + tl.y + (active ? r : 0);
         const float* qrow = a.qrows + (int64_t)qpos * dp;
-        // rounded query-cluster center (re-centring point)
-        for (int c = tid; c < KP; c += blockDim.x) s_cr[c] = c < dp ? rintf(a.qcent[(int64_t)qc * dp + c]) : 0.f;
-        if (tid == 0) s_loA = 0;
-        __syncthreads();
-        // stage A = q - c_r (hi/lo bf16) in core-matrix layout; ||a||^2 per row
-        {
-            const int c8n = KP / 8;
-            bool nz = false;
-            for (int w = tid; w < kDenseM * c8n; w += blockDim.x) {
-                const int row = w / c8n, c8 = w % c8n;
-                const bool rv = tl.y + row < qsz;
-                const float* src = a.qrows + (int64_t)(qlo + tl.y + (rv ? row : 0)) * dp;
-                float v[8];
-#pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    const int kk = c8 * 8 + i;
-                    v[i] = (rv && kk < dp) ? src[kk] - s_cr[kk] : 0.f;
-                }
-                uint4 hi, lo;
-                nz |= split8(v, hi, lo);
-                const uint32_t off = (uint32_t)(row >> 3) * sbo + (uint32_t)c8 * 128u + (uint32_t)(row & 7) * 16u;
-                *reinterpret_cast<uint4*>(sA_hi + off) = hi;
-                *reinterpret_cast<uint4*>(sA_lo + off) = lo;
+        const size_t qp = (size_t)a.qoffp[qc] + tl.y;  // padded row of the tile's first query
+        ChunkIter<NCH> prod, cons;
+        prod.start(a, qc);
+        cons.start(a, qc);
+        if (tid == 0) {
+            const uint32_t bar = smem_u32(&bar_a);
+            expect_tx(bar, loA ? 2 * a_bytes : a_bytes);
+            bulk_g2s(smem_u32(sA), a.qhi + (qp >> 3) * sbo, a_bytes, bar);
+            if (loA) bulk_g2s(smem_u32(sA + a_bytes), a.qlo + (qp >> 3) * sbo, a_bytes, bar);
+            if (prod.valid()) {
+                issue_b(prod, 0);
+                if (prod.advance(a)) issue_b(prod, 1);
+                prod.advance(a);  // now two chunks ahead of the consumer
             }
-            if (__syncthreads_or(nz) && tid == 0) s_loA = 1;
+            mbar_wait(smem_u32(&bar_a), ph_a);
+            if (cons.valid()) {
+                mbar_wait(smem_u32(&bar_full[0]), ph_full[0]);
+                issue_mma(0);
+            }
         }
-        float qn = 0.f;
-        for (int c = 0; c < dp; ++c) {
-            const float x = qrow[c] - s_cr[c];
-            qn = __fmaf_rn(x, x, qn);
-        }
+        ph_a ^= 1u;
+        if (cons.valid()) ph_full[0] ^= 1u;
+        const float qn = active ? __ldg(a.qn + qp + r) : 0.f;
         RegTopK<KMAX> top;
         top.init(a.k);
-        const float ub = a.ub[qc];
-        float theta = ub;
         key_t kth = top.kth();
+        const float ub = a.ub[qc];
         float kth2 = __fmul_ru(ub, ub);
-        float thr = kth2 * rel_k - qn * (1.f - a.eps_tc);
-        const int nd = a.dcount[qc];
-        const int32_t* dl = a.dcand + (int64_t)qc * a.mt;
-        for (int ci = 0; ci < nd; ++ci) {
-            const int tc = __ldg(dl + ci);
-            const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
-            // dense pair: the whole target cluster is screened (no per-point TI
-            // checks -- the regular tiled path of the elastic switch)
-            const int W0 = lo, W1 = hi;
-            for (int j0 = W0; j0 < W1; j0 += NCH) {
-                const int nb = min(NCH, W1 - j0);
-                // stage B = t - c_r and ||b||^2 (1 - eps)
-                if (tid == 0) s_loB = 0;
-                __syncthreads();
-                {
-                    // TPR threads per target row; each converts a contiguous K range
-                    constexpr int TPR = kDenseM / NCH;
-                    const int row = tid / TPR, part = tid % TPR;
-                    const int c8n = KP / 8, c8per = c8n / TPR;
-                    const bool rv = row < nb;
-                    const float4* src4 = reinterpret_cast<const float4*>(a.trows + (int64_t)(j0 + (rv ? row : 0)) * dp);
-                    const float4* cr4 = reinterpret_cast<const float4*>(s_cr);
-                    bool nz = false;
-                    float tn = 0.f;
-#pragma unroll 4
-                    for (int c8 = part * c8per; c8 < (part + 1) * c8per; ++c8) {
-                        float v[8];
-#pragma unroll
-                        for (int h = 0; h < 2; ++h) {
-                            const int k4 = c8 * 2 + h;
-                            float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-                            if (rv && k4 * 4 < dp) {
-                                const float4 t4 = __ldg(src4 + k4), c4 = cr4[k4];
-                                x = make_float4(t4.x - c4.x, t4.y - c4.y, t4.z - c4.z, t4.w - c4.w);
-                            }
-                            v[4 * h + 0] = x.x; v[4 * h + 1] = x.y; v[4 * h + 2] = x.z; v[4 * h + 3] = x.w;
-                            tn = __fmaf_rn(x.x, x.x, tn); tn = __fmaf_rn(x.y, x.y, tn);
-                            tn = __fmaf_rn(x.z, x.z, tn); tn = __fmaf_rn(x.w, x.w, tn);
-                        }
-                        uint4 hi4, lo4;
-                        nz |= split8(v, hi4, lo4);
-                        const uint32_t off = (uint32_t)(row >> 3) * sbo + (uint32_t)c8 * 128u + (uint32_t)(row & 7) * 16u;
-                        *reinterpret_cast<uint4*>(sB_hi + off) = hi4;
-                        *reinterpret_cast<uint4*>(sB_lo + off) = lo4;
-                    }
-#pragma unroll
-                    for (int o = 1; o < TPR; o <<= 1) tn += __shfl_xor_sync(0xffffffffu, tn, o);
-                    if (part == 0) s_tn[row] = rv ? tn * (1.f - a.eps_tc) : INF;
-                    if (__syncthreads_or(nz) && tid == 0) s_loB = 1;
-                }
-                fence_async_smem();
-                __syncthreads();
-                if (tid == 0) {
-                    tc_fence_after();
-                    const bool loA = s_loA != 0, loB = s_loB != 0;
-                    const uint32_t aH = smem_u32(sA_hi), aL = smem_u32(sA_lo);
-                    const uint32_t bH = smem_u32(sB_hi), bL = smem_u32(sB_lo);
-                    for (int s = 0; s < KP / 16; ++s) {
-                        const uint32_t ko = (uint32_t)s * 256u;
-                        umma_bf16(tmem, umma_desc(aH + ko, 128u, sbo), umma_desc(bH + ko, 128u, sbo), idesc, s > 0);
-                        if (loB) umma_bf16(tmem, umma_desc(aH + ko, 128u, sbo), umma_desc(bL + ko, 128u, sbo), idesc, 1);
-                        if (loA) umma_bf16(tmem, umma_desc(aL + ko, 128u, sbo), umma_desc(bH + ko, 128u, sbo), idesc, 1);
-                    }
-                    umma_commit(&s_bar);
-                }
-                mbar_wait(&s_bar, phase);
-                phase ^= 1u;
-                tc_fence_after();
-                // epilogue: screen d2~ - E against the row's k-th, exact recompute of survivors
-#pragma unroll 1
-                for (int cb = 0; cb < NCH / 32; ++cb) {
-                    uint32_t v[32];
-                    tmem_ld32(tmem_row + (uint32_t)(cb * 32), v);
-                    if (!active || cb * 32 >= nb) continue;
-                    uint32_t mask = 0;
-#pragma unroll
-                    for (int j = 0; j < 32; ++j) {
-                        const float sc = __fmaf_rn(-2.f, __uint_as_float(v[j]), s_tn[cb * 32 + j]);
-                        mask |= (sc <= thr ? 1u : 0u) << j;
-                    }
-                    while (mask) {
-                        const int j = __ffs(mask) - 1;
-                        mask &= mask - 1;
-                        const int jj = j0 + cb * 32 + j;
-                        const float d2 = d2_rows(qrow, a.trows + (int64_t)jj * dp, dp);
-                        ++recomputed;
-                        if (d2 <= key_d2(kth)) {
-                            const key_t key = make_key(d2, __ldg(a.torig + jj));
-                            if (key < kth) {
-                                top.insert(key);
-                                kth = top.kth();
-                                const float k2 = key_d2(kth);
-                                if (k2 < INF) {
-                                    theta = fminf(ub, __fsqrt_ru(k2));
-                                    kth2 = fminf(kth2, k2);
-                                    thr = kth2 * rel_k - qn * (1.f - a.eps_tc);
-                                }
-                            }
-                        }
-                    }
-                }
-                if (active) covered += (unsigned long long)nb;
-                tc_fence_before();
-                __syncthreads();
+        float thr = kth2 * rel_k - qn * qscale;
+        for (int g = 0; cons.valid(); ++g) {
+            const int buf = g & 1;
+            // next chunk's MMA goes into the other accumulator while this one is reduced
+            ChunkIter<NCH> nxt = cons;
+            const bool has_next = nxt.advance(a);
+            if (tid == 0 && has_next) {
+                mbar_wait(smem_u32(&bar_full[buf ^ 1]), ph_full[buf ^ 1]);
+                issue_mma(buf ^ 1);
             }
+            if (has_next) ph_full[buf ^ 1] ^= 1u;
+            mbar_wait(smem_u32(&bar_mma[buf]), ph_mma[buf]);
+            ph_mma[buf] ^= 1u;
+            tc_fence_after();
+            const int nb = min(NCH, cons.size - cons.c * NCH);
+            const int j0 = __ldg(a.toff + cons.tc) + cons.c * NCH;  // real (unpadded) first target
+            const float* tnv = s_tn + buf * NCH;
+#pragma unroll 1
+            for (int cb = 0; cb < NCH / 32; ++cb) {
+                uint32_t v[32];
+                tmem_ld32(tmem_row + (uint32_t)(buf * NCH + cb * 32), v);
+                if (!active || cb * 32 >= nb) continue;
+                uint32_t mask = 0;
+#pragma unroll
+                for (int j = 0; j < 32; ++j) {
+                    const float sc = __fmaf_rn(-2.f, __uint_as_float(v[j]), tnv[cb * 32 + j]);
+                    mask |= (sc <= thr ? 1u : 0u) << j;
+                }
+                if (cb * 32 + 32 > nb) mask &= (1u << (nb - cb * 32)) - 1u;
+                while (mask) {
+                    const int j = __ffs(mask) - 1;
+                    mask &= mask - 1;
+                    const int jj = j0 + cb * 32 + j;
+                    const float d2 = d2_rows(qrow, a.trows + (int64_t)jj * dp, dp);
+                    ++recomputed;
+                    if (d2 <= key_d2(kth)) {
+                        const key_t key = make_key(d2, __ldg(a.torig + jj));
+                        if (key < kth) {
+                            top.insert(key);
+                            kth = top.kth();
+                            const float k2 = key_d2(kth);
+                            if (k2 < kth2) {
+                                kth2 = k2;
+                                thr = kth2 * rel_k - qn * qscale;
+                            }
+                        }
+                    }
+                }
+            }
+            if (active) covered += (unsigned long long)nb;
+            tc_fence_before();
+            __syncthreads();  // stage `buf` (smem) and accumulator `buf` (TMEM) are free
+            if (tid == 0 && prod.valid()) {
+                issue_b(prod, buf);
+                prod.advance(a);
+            }
+            cons = nxt;
         }
         if (active) {
 #pragma unroll
@@ -340,16 +410,17 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
     add_counter(&a.counters->dist_recompute, recomputed);
     tc_fence_before();
     __syncthreads();
-    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)NCH));
+    if (warp == 0)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)(2 * NCH)));
 }
 
 template <int KMAX, int NCH>
 static sknn_status launch_dense_k(Ctx& cx, const DenseArgs& a) {
-    const size_t smem = (size_t)kDenseM * a.kp * 4 + (size_t)NCH * a.kp * 4 + sizeof(float) * (NCH + a.kp);
+    const size_t smem = 2 * (size_t)kDenseM * a.kp * 2 + 4 * (size_t)NCH * a.kp * 2 + 2 * NCH * 4;
     SKNN_CUDA(cudaFuncSetAttribute(k_dense<KMAX, NCH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_dense<KMAX, NCH>, kDenseM, smem);
-    per_sm = std::max(1, std::min(per_sm, 512 / NCH));  // TMEM: NCH columns per CTA, 512 per SM
+    per_sm = std::max(1, std::min(per_sm, 512 / (2 * NCH)));  // TMEM: 2*NCH columns per CTA
     k_dense<KMAX, NCH><<<per_sm * cx.num_sms, kDenseM, smem, cx.stream>>>(a);
     cx.launched();
     return cx.check_launch("dense tiles");
@@ -366,16 +437,79 @@ static sknn_status launch_dense_n(Ctx& cx, const DenseArgs& a) {
 int dense_kp(int dp) { return (dp + 15) & ~15; }
 bool dense_supported(int dp) { return dense_kp(dp) <= 256; }
 
+// Converted tile set of one side: padded CSR + bf16 hi/lo + norms
+// (scaled by 1 - eps for the target role, raw for the query role).
+struct DenseSide {
+    int32_t* offp = nullptr;
+    unsigned char* hi = nullptr;
+    unsigned char* lo = nullptr;
+    float* norm = nullptr;
+    float* norm_raw = nullptr;
+};
+
+static sknn_status convert_side(Ctx& cx, const Side& sd, int kp, const float* o, float nscale, bool want_raw,
+                                int* lo_flag, DenseSide& out) {
+    const int m = sd.m;
+    int32_t* cnt8;
+    SKNN_TRY(cx.alloc_scratch((void**)&out.offp, sizeof(int32_t) * (m + 1)));
+    SKNN_TRY(cx.alloc_scratch((void**)&cnt8, sizeof(int32_t) * 2 * m));
+    int32_t* dummy = cnt8 + m;
+    k_pad8<<<std::max(1, std::min((m + 255) / 256, 148 * 4)), 256, 0, cx.stream>>>(sd.off, m, cnt8);
+    cx.launched();
+    k_offsets<<<1, 1024, 0, cx.stream>>>(cnt8, m, out.offp, dummy);
+    cx.launched();
+    // upper bound of padded rows + a guard for the 128-row tile over-read
+    const int64_t npad = sd.n + 7LL * m + 256;
+    const size_t tile_bytes = (size_t)npad * kp * 2;
+    SKNN_TRY(cx.alloc_scratch((void**)&out.hi, tile_bytes));
+    SKNN_TRY(cx.alloc_scratch((void**)&out.lo, tile_bytes));
+    SKNN_TRY(cx.alloc_scratch((void**)&out.norm, sizeof(float) * npad));
+    if (want_raw) SKNN_TRY(cx.alloc_scratch((void**)&out.norm_raw, sizeof(float) * npad));
+    SKNN_CUDA(cudaMemsetAsync(out.hi, 0, tile_bytes, cx.stream));
+    SKNN_CUDA(cudaMemsetAsync(out.lo, 0, tile_bytes, cx.stream));
+    const int fb = (int)std::min<int64_t>((npad + 255) / 256, 148 * 8);
+    k_fill_f<<<fb, 256, 0, cx.stream>>>(out.norm, npad, INFINITY);
+    cx.launched();
+    if (want_raw) {
+        k_fill_f<<<fb, 256, 0, cx.stream>>>(out.norm_raw, npad, 0.f);
+        cx.launched();
+    }
+    k_to_tiles<<<m, 256, 0, cx.stream>>>(sd.rows, sd.off, out.offp, sd.dp, kp, o, nscale,
+                                        reinterpret_cast<__nv_bfloat16*>(out.hi),
+                                        reinterpret_cast<__nv_bfloat16*>(out.lo), out.norm, out.norm_raw, lo_flag);
+    cx.launched();
+    return cx.check_launch("dense tile conversion");
+}
+
 sknn_status run_dense(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const DenseParams& p) {
+    const int kp = dense_kp(ts.dp);
+    const float eps_tc = (float)ldexp(1.0, -12) * std::max(1.f, (float)kp / 128.f);
+    const bool self = &qs == &ts;
+    float* o;
+    int* lo_flag;
+    SKNN_TRY(cx.alloc_scratch((void**)&o, sizeof(float) * kp));
+    SKNN_TRY(cx.alloc_scratch((void**)&lo_flag, sizeof(int) * 2));
+    SKNN_CUDA(cudaMemsetAsync(lo_flag, 0, sizeof(int) * 2, cx.stream));
+    k_dense_origin<<<kp, 256, 0, cx.stream>>>(ts.centers, ts.m, ts.dp, kp, o);
+    cx.launched();
+    DenseSide tq, tt;
+    SKNN_TRY(convert_side(cx, ts, kp, o, 1.f - eps_tc, self, lo_flag + 1, tt));
+    if (self) {
+        tq = tt;
+        tq.norm = tt.norm_raw;
+        SKNN_CUDA(cudaMemcpyAsync(lo_flag, lo_flag + 1, sizeof(int), cudaMemcpyDeviceToDevice, cx.stream));
+    } else {
+        SKNN_TRY(convert_side(cx, qs, kp, o, 1.f, false, lo_flag, tq));
+    }
     DenseArgs a{};
-    a.qrows = qs.rows; a.qoff = qs.off; a.qcent = qs.centers;
-    a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
+    a.qrows = qs.rows; a.qoff = qs.off; a.qoffp = tq.offp; a.qhi = tq.hi; a.qlo = tq.lo; a.qn = tq.norm;
+    a.trows = ts.rows; a.torig = ts.orig; a.toff = ts.off; a.toffp = tt.offp; a.thi = tt.hi; a.tlo = tt.lo;
+    a.tn = tt.norm; a.lo_flag = lo_flag;
     a.ub = l1.ub; a.dcand = l1.dcand; a.dcount = l1.dcount;
     a.tiles = l1.dtiles; a.ntiles = l1.dntiles; a.counter = l1.dntiles + 1;
-    a.mt = ts.m; a.dp = ts.dp; a.kp = dense_kp(ts.dp); a.k = p.k; a.eta = p.eta;
-    a.eps_tc = (float)ldexp(1.0, -12) * std::max(1.f, (float)a.kp / 128.f);
+    a.mt = ts.m; a.dp = ts.dp; a.kp = kp; a.k = p.k; a.eps_tc = eps_tc;
     a.topk_out = p.topk_out; a.counters = p.counters;
-    if (a.kp <= 64) return launch_dense_n<128>(cx, a);
+    if (kp <= 64) return launch_dense_n<128>(cx, a);
     return launch_dense_n<64>(cx, a);
 }
 

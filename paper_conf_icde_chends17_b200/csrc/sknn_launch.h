@@ -81,6 +81,8 @@ struct Ctx {
 };
 
 // k_build.cu
+__global__ void k_offsets(const int32_t* __restrict__ counts, int m, int32_t* __restrict__ off,
+                          int32_t* __restrict__ cursor);
 sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int trials, int lloyd, uint64_t seed,
                        Side& out);
 
