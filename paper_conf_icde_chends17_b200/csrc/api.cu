@@ -225,6 +225,12 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
         set_last_error("force_path = DENSE needs d <= 256");
         return SKNN_ERR_UNSUPPORTED;
     }
+    DenseOrigin dorg;
+    if (lp.dense_mode != 1) {
+        SKNN_TRY(dense_prepare(cx, qs, ts, dorg));
+        lp.dorg = &dorg;
+    }
+    if (lp.dense_mode == 0 && !lp.dorg) lp.dense_mode = 1;
     SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
     SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp), lp.shard_rank, lp.shard_count, l1));
     mk.l1 = tm.mark();
@@ -233,6 +239,7 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
         SKNN_TRY(cx.alloc_scratch((void**)&init_topk, sizeof(key_t) * (size_t)qs.n * k));
         SKNN_TRY(run_dense_tiles(cx, qs, l1));
         DenseParams dpar;
+        dpar.origin = dorg.o;
         dpar.k = k;
         dpar.eta = eta;
         dpar.topk_out = init_topk;

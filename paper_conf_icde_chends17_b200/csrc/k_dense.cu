@@ -115,6 +115,19 @@ __global__ void k_dense_origin(const float* __restrict__ centers, int m, int dp,
     if (threadIdx.x == 0) o[c] = c < dp ? rintf((float)(red[0] / m)) : 0.f;
 }
 
+// ||c - o|| of every center: the magnitude the dense screen's error bound scales with
+__global__ void k_center_dist_o(const float* __restrict__ centers, int m, int dp, const float* __restrict__ o,
+                                float* __restrict__ out) {
+    for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < m; c += gridDim.x * blockDim.x) {
+        float s = 0.f;
+        for (int k = 0; k < dp; ++k) {
+            const float v = centers[(int64_t)c * dp + k] - o[k];
+            s = __fmaf_rn(v, v, s);
+        }
+        out[c] = sqrtf(s);
+    }
+}
+
 // cluster sizes rounded up to 8 rows (padded CSR for 8-row-aligned tiles)
 __global__ void k_pad8(const int32_t* __restrict__ off, int m, int32_t* __restrict__ cnt8) {
     for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < m; c += gridDim.x * blockDim.x)
@@ -481,17 +494,36 @@ static sknn_status convert_side(Ctx& cx, const Side& sd, int kp, const float* o,
     return cx.check_launch("dense tile conversion");
 }
 
+float dense_eps(int dp) { return (float)ldexp(1.0, -12) * std::max(1.f, (float)dense_kp(dp) / 128.f); }
+
+// common origin o (rounded mean target center) and ||c - o|| per cluster of both sides
+sknn_status dense_prepare(Ctx& cx, const Side& qs, const Side& ts, DenseOrigin& out) {
+    const int kp = dense_kp(ts.dp);
+    SKNN_TRY(cx.alloc_scratch((void**)&out.o, sizeof(float) * kp));
+    SKNN_TRY(cx.alloc_scratch((void**)&out.ct_o, sizeof(float) * ts.m));
+    k_dense_origin<<<kp, 256, 0, cx.stream>>>(ts.centers, ts.m, ts.dp, kp, out.o);
+    cx.launched();
+    k_center_dist_o<<<(ts.m + 255) / 256, 256, 0, cx.stream>>>(ts.centers, ts.m, ts.dp, out.o, out.ct_o);
+    cx.launched();
+    if (&qs == &ts) {
+        out.cq_o = out.ct_o;
+    } else {
+        SKNN_TRY(cx.alloc_scratch((void**)&out.cq_o, sizeof(float) * qs.m));
+        k_center_dist_o<<<(qs.m + 255) / 256, 256, 0, cx.stream>>>(qs.centers, qs.m, qs.dp, out.o, out.cq_o);
+        cx.launched();
+    }
+    out.eps = dense_eps(ts.dp);
+    return cx.check_launch("dense origin");
+}
+
 sknn_status run_dense(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const DenseParams& p) {
     const int kp = dense_kp(ts.dp);
-    const float eps_tc = (float)ldexp(1.0, -12) * std::max(1.f, (float)kp / 128.f);
+    const float eps_tc = dense_eps(ts.dp);
     const bool self = &qs == &ts;
-    float* o;
+    const float* o = p.origin;
     int* lo_flag;
-    SKNN_TRY(cx.alloc_scratch((void**)&o, sizeof(float) * kp));
     SKNN_TRY(cx.alloc_scratch((void**)&lo_flag, sizeof(int) * 2));
     SKNN_CUDA(cudaMemsetAsync(lo_flag, 0, sizeof(int) * 2, cx.stream));
-    k_dense_origin<<<kp, 256, 0, cx.stream>>>(ts.centers, ts.m, ts.dp, kp, o);
-    cx.launched();
     DenseSide tq, tt;
     SKNN_TRY(convert_side(cx, ts, kp, o, 1.f - eps_tc, self, lo_flag + 1, tt));
     if (self) {

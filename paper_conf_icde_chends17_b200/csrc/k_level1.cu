@@ -105,7 +105,8 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     const float* __restrict__ qcent, const float* __restrict__ qrad, const int32_t* __restrict__ qoff,
     const float* __restrict__ tcent, const float* __restrict__ trad, const int32_t* __restrict__ toff,
     const float* __restrict__ tdist, int mt, int dp, int k, float eta, int keys_cap, int shard_rank,
-    int shard_count, int dense_mode, float dense_tau, float* __restrict__ ub_out, int32_t* __restrict__ cand,
+    int shard_count, int dense_mode, float dense_tau, const float* __restrict__ cq_o,
+    const float* __restrict__ ct_o, float dense_eps, float* __restrict__ ub_out, int32_t* __restrict__ cand,
     int32_t* __restrict__ cand_count, float* __restrict__ cand_D, int32_t* __restrict__ dcand,
     int32_t* __restrict__ dcount,
     Counters* __restrict__ counters) {
@@ -233,7 +234,11 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
                 const float rt = __ldg(trad + tc);
                 const float Dp = s_D[tc];
                 const float ov = fminf(rt, Dp + Vk) - fmaxf(0.f, Dp - Vk);
-                dense = sz >= 32 && ov >= dense_tau * fmaxf(rt, 1e-30f);
+                // and the tensor-core screen must stay selective: its error bound
+                // eps (||a||^2 + ||b||^2) small against the k-th distance^2 ~ V_k^2
+                const float ma = cq_o[qc] + rq, mb = ct_o[tc] + rt;
+                const bool sharp = dense_eps * (ma * ma + mb * mb) <= 0.25f * Vk * Vk;
+                dense = sz >= 32 && sharp && ov >= dense_tau * fmaxf(rt, 1e-30f);
             }
         }
         const unsigned md = __ballot_sync(0xffffffffu, i < nc && dense);
@@ -292,7 +297,9 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
     SKNN_CUDA(cudaFuncSetAttribute(k_level1, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     k_level1<<<mq, kL1Threads, smem, cx.stream>>>(qs.centers, qs.radius, qs.off, ts.centers, ts.radius, ts.off,
                                                   ts.dist, mt, dp, p.k, p.eta, cap, p.shard_rank, p.shard_count,
-                                                  p.dense_mode, p.dense_tau, out.ub, out.cand, out.cand_count, out.cand_D,
+                                                  p.dense_mode, p.dense_tau, p.dorg ? p.dorg->cq_o : nullptr,
+                                                  p.dorg ? p.dorg->ct_o : nullptr, p.dorg ? p.dorg->eps : 0.f,
+                                                  out.ub, out.cand, out.cand_count, out.cand_D,
                                                   out.dcand, out.dcount, counters);
     cx.launched();
     return cx.check_launch("level1");

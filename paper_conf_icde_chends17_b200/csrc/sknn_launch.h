@@ -105,7 +105,14 @@ struct Level1 {
     int2* dtiles = nullptr;       // dense work tiles (128 queries of one cluster)
     int* dntiles = nullptr;       // [2]
 };
+struct DenseOrigin {          // common re-centring point of the dense tiles
+    float* o = nullptr;         // [kp] rounded mean target center
+    float* cq_o = nullptr;      // [mq] ||c_q - o||
+    float* ct_o = nullptr;      // [mt] ||c_t - o||
+    float eps = 0.f;            // screen error-bound factor
+};
 struct Level1Params {
+    const DenseOrigin* dorg = nullptr;  // dense screen magnitudes (elastic switch), NULL when unarmed
     int k = 0;
     float eta = 0.f;
     int shard_rank = 0, shard_count = 1;
@@ -116,6 +123,7 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
                        Counters* counters);
 // k_dense.cu
 struct DenseParams {
+    const float* origin = nullptr;
     int k = 0;
     float eta = 0.f;
     key_t* topk_out = nullptr;
@@ -123,6 +131,8 @@ struct DenseParams {
 };
 int dense_kp(int dp);
 bool dense_supported(int dp);
+float dense_eps(int dp);
+sknn_status dense_prepare(Ctx& cx, const Side& qs, const Side& ts, DenseOrigin& out);
 sknn_status run_dense_tiles(Ctx& cx, const Side& qs, Level1& l1);
 sknn_status run_dense(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const DenseParams& p);
 // k_scan.cu: tiles of `tile` queries of one query cluster (thread-data remapping)

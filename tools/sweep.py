@@ -27,6 +27,7 @@ VARIANTS = {
     "dense": {"force_path": "dense"},
     "tau4": {"dense_threshold": 4.0},
     "tau25": {"dense_threshold": 0.25},
+    "tau50": {"dense_threshold": 0.5},
     "tau75": {"dense_threshold": 0.75},
     "tau95": {"dense_threshold": 0.95},
     "warp": {"mapping": "warp"},
