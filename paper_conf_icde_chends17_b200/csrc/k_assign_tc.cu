@@ -124,7 +124,7 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
                                                        const float* __restrict__ centers,
                                                        int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
                                                        long long* __restrict__ sums, const double* __restrict__ fx,
-                                                       int32_t* __restrict__ counts) {
+                                                       int32_t* __restrict__ counts, int stride) {
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t a_bytes = (uint32_t)kTcM * kp * 2, b_bytes = (uint32_t)kTcN * kp * 2;
     unsigned char* sA = smem;
@@ -153,7 +153,7 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
         const int c8n = kp / 8;
         for (int w = tid; w < kTcM * c8n; w += blockDim.x) {
             const int r = w / c8n, c8 = w % c8n;
-            const int64_t i = row0 + r;
+            const int64_t i = (row0 + r) * stride;
             uint32_t h[4];
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
@@ -238,7 +238,7 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
         __syncthreads();  // buffer `buf` (smem + TMEM) is free again
         if (tid == 0 && c + 2 < nchunks) issue_copy(c + 2, buf);
     }
-    const int64_t i = row0 + tid;
+    const int64_t i = (row0 + tid) * stride;
     if (i < n) {
         bi = min(bi, m - 1);
         const float* xr = Xp + i * dp;
@@ -256,7 +256,7 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
 bool assign_tc_supported(int dp) { return dp >= 8 && ((dp + 15) & ~15) <= 256; }
 
 sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m, int32_t* cid,
-                          float* dist, long long* sums, const double* fx, int32_t* counts) {
+                          float* dist, long long* sums, const double* fx, int32_t* counts, int stride) {
     const int kp = (dp + 15) & ~15;
     const int nchunks = (m + kTcN - 1) / kTcN;
     const int mpad = nchunks * kTcN;
@@ -276,9 +276,9 @@ sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
     const size_t smem = std::max<size_t>((size_t)kTcM * kp * 2 + 2 * (size_t)kTcN * kp * 2 + 2 * kTcN * 4, 90 * 1024);
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-    const int64_t grid = (n + kTcM - 1) / kTcM;
+    const int64_t grid = ((n + stride - 1) / stride + kTcM - 1) / kTcM;
     k_assign_tc<<<(unsigned)grid, kTcM, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, bn, m, nchunks, centers, cid, dist,
-                                                          sums, fx, counts);
+                                                          sums, fx, counts, stride);
     cx.launched();
     return cx.check_launch("assign (tensor cores)");
 }

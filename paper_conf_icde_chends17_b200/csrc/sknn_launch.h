@@ -89,7 +89,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
 // k_assign_tc.cu: nearest-center screen on the tensor cores
 bool assign_tc_supported(int dp);
 sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m, int32_t* cid,
-                          float* dist, long long* sums, const double* fx, int32_t* counts);
+                          float* dist, long long* sums, const double* fx, int32_t* counts, int stride = 1);
 
 // k_level1.cu
 struct Level1 {
