@@ -260,21 +260,33 @@ def main():
         stage[key] /= args.steps
 
     # ---- roofline of the dominant kernel (the level-2 scan), timed live above ----
+    # Algorithmic bytes per launch: the query rows, every
+    # evaluated member (row + member distance), every candidate-center
+    # distance (center row + CSR bounds), the per-(query, candidate) bound
+    # inputs (D, r_t) and the result rows. Intensity ~0.6 flop/B, far below
+    # the B200 balance point (74 TF / 6.5 TB/s ~ 11 flop/B): the binding
+    # roofline is the memory one, reported against HBM bandwidth.
     scan_ms = stage["ms_sparse"]
-    flops = 3.0 * d * (last["dist_evals"] + last["center_evals"])
-    bytes_alg = (nq * 16 * ((d + 3) // 4)) / max(1, ws) + (16 * ((d + 3) // 4) + 8) * last["dist_evals"] + 8.0 * k * nq / max(1, ws)
+    dpad = 4 * ((d + 3) // 4)
+    E = float(last["dist_evals_sparse"])
+    C = float(last["center_evals"])
+    P = float(last["cand_pairs"]) * (nq / max(1, last["mq"]))  # (query, candidate cluster) bound checks
+    bytes_alg = (4.0 * dpad * nq / max(1, ws) + (4.0 * dpad + 4.0) * E + (4.0 * dpad + 8.0) * C + 8.0 * P +
+                 8.0 * k * nq / max(1, ws))
+    flops = 3.0 * d * (E + C)
     sm_mhz = peaks.get("sm_max_mhz", 1965.0)
     alu_peak_tflops = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
-    roofline = {"kernel": "k_scan_tpq/k_scan_wpq (level-2 filtered scan + top-k)", "bound": "alu",
-                "achieved": flops / (scan_ms / 1000.0) / 1e12 if scan_ms > 0 else None,
-                "peak": alu_peak_tflops, "unit": "TFLOP/s",
-                "frac": (flops / (scan_ms / 1000.0) / 1e12) / alu_peak_tflops if scan_ms > 0 else None,
-                "traffic": None, "launch_ms": scan_ms,
-                "algorithmic_flops": flops, "algorithmic_bytes": bytes_alg,
-                "achieved_gbs": bytes_alg / (scan_ms / 1000.0) / 1e9 if scan_ms > 0 else None,
-                "hbm_peak_gbs": peaks.get("hbm_gbs"),
-                "peak_source": "fp32 FMA pipe: 148 SMs x 128 lanes x 2 flop x %.0f MHz (derived); HBM %s" % (
-                    sm_mhz, peaks["_source"]),
+    hbm = peaks.get("hbm_gbs")
+    achieved_gbs = bytes_alg / (scan_ms / 1000.0) / 1e9 if scan_ms > 0 else None
+    roofline = {"kernel": "k_scan_tpq (level-2 filtered scan fused with top-k)", "bound": "hbm",
+                "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
+                "frac": achieved_gbs / hbm if achieved_gbs else None,
+                "traffic": None, "launch_ms": scan_ms, "algorithmic_bytes": bytes_alg,
+                "algorithmic_flops": flops, "intensity_flop_per_byte": flops / bytes_alg if bytes_alg else None,
+                "alu_achieved_tflops": flops / (scan_ms / 1000.0) / 1e12 if scan_ms > 0 else None,
+                "alu_peak_tflops": alu_peak_tflops,
+                "peak_source": "HBM %s; fp32 FMA pipe derived: 148 SMs x 128 lanes x 2 flop x %.0f MHz" % (
+                    peaks["_source"], sm_mhz),
                 "share_of_step": scan_ms / ms_step if ms_step else None}
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
