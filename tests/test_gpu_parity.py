@@ -343,3 +343,34 @@ def test_build_is_deterministic(sknn):
         _, _, s2 = run(sknn, Q, T, k, sj)
         for key in ("dist_evals", "cand_pairs", "center_evals", "dense_pairs"):
             assert s1[key] == s2[key], key
+
+
+def test_index_self_join_and_reuse(sknn):
+    """sknn_query with Q == the indexed T (self-join through the index) and
+    repeated queries against one resident index on another stream."""
+    X = datagen.c3_kegg(4000, integer=True)
+    dX = dev(X)
+    ix = sknn.build(dX)
+    ridx, rdist = oracle.knn_join(X, X, 16)
+    i1, d1 = ix.query(dX, 16)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        i2, d2 = ix.query(dX, 16, stream=s)
+    s.synchronize()
+    torch.cuda.synchronize()
+    assert_knn_bitexact(i1.cpu().numpy(), d1.cpu().numpy(), ridx, rdist)
+    assert_knn_bitexact(i2.cpu().numpy(), d2.cpu().numpy(), ridx, rdist)
+    Q = datagen.c3_kegg(700, integer=True, seed=8)
+    i3, d3 = ix.query(Q, 16)  # host buffers through the index
+    r3i, r3d = oracle.knn_join(Q, X, 16)
+    assert_knn_bitexact(i3, d3, r3i, r3d)
+    ix.close()
+
+
+def test_squared_output_and_index_base(sknn):
+    Q, T, k, sj = datagen.workload("C1")
+    dQ = dev(Q)
+    i, d2 = sknn.join(dQ, dQ, k, out_squared=1, index_base=1000)
+    ridx, rdist, rd2 = oracle.knn_join(Q, T, k, return_d2=True)
+    np.testing.assert_array_equal(i.cpu().numpy(), ridx + 1000)
+    np.testing.assert_array_equal(d2.cpu().numpy(), rd2.astype(np.float32))
