@@ -63,10 +63,12 @@ typedef enum {
     SKNN_ERR_WRONG_DEVICE = -6    /* index used on a device other than the one that built it */
 } sknn_status;
 
-/* Largest k the register / warp top-k supports in this version (P:L529-535,
- * Fig. 8 placement: on B200 k*4 <= th2 = 1020 B fits registers; the large-k
- * partial filter of §IV-B1 is future work). */
-#define SKNN_MAX_K 32
+/* Largest k supported (the paper's largest, Fig. 10 / Table V).
+ * kNearests placement follows Fig. 8: shared memory for
+ * k*4 <= th1, registers for k <= 32, shared memory with fewer threads per CTA
+ * beyond. k > 32 uses the thread-per-query scan only (no dense tiles, no
+ * brute-force path); sknn_merge_partials supports k > 32 with P <= 16. */
+#define SKNN_MAX_K 512
 
 /* Execution-path override (sknn_options.force_path). */
 enum {

@@ -27,7 +27,7 @@ STATUS = {0: "SKNN_OK", -1: "SKNN_ERR_INVALID_ARG", -2: "SKNN_ERR_NOT_DEVICE_PTR
           -4: "SKNN_ERR_CUDA", -5: "SKNN_ERR_UNSUPPORTED", -6: "SKNN_ERR_WRONG_DEVICE"}
 PATH = {"auto": 0, "sparse": 1, "dense": 2, "brute": 3}
 MAPPING = {"auto": 0, "thread": 1, "warp": 2}
-MAX_K = 32
+MAX_K = 512
 
 # every symbol include/sknn.h declares (tests check the library exports them)
 ABI_SYMBOLS = ["sknn_options_default", "sknn_join", "sknn_join_ex", "sknn_build", "sknn_query",

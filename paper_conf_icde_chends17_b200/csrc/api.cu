@@ -161,8 +161,9 @@ struct Timer {
     }
 };
 
-static int choose_mapping(const sknn_options& o, const DevInfo& di, int64_t nq, int dp) {
+static int choose_mapping(const sknn_options& o, const DevInfo& di, int64_t nq, int dp, int k) {
     if (o.mapping == SKNN_MAP_THREAD || o.mapping == SKNN_MAP_WARP) return o.mapping;
+    if (k > 32) return SKNN_MAP_THREAD;  // lane-distributed warp top-k holds at most 32
     // Fig. 8 bottom chooses query-level parallelism when
     // |Q| >= r*max_cur and several threads per query otherwise. Measured on
     // B200 (profiles/r01_sweep.md) the thread-per-query scan wins for every
@@ -183,7 +184,7 @@ static sknn_status validate(const float* Q, int64_t nq, const float* T, int64_t 
     if (d <= 0) return fail(SKNN_ERR_INVALID_ARG, "d <= 0");
     if (k <= 0) return fail(SKNN_ERR_INVALID_ARG, "k <= 0");
     if ((int64_t)k > nt) return fail(SKNN_ERR_INVALID_ARG, "k > nt");
-    if (k > SKNN_MAX_K) return fail(SKNN_ERR_UNSUPPORTED, "k > SKNN_MAX_K (large-k partial filter not built yet)");
+    if (k > SKNN_MAX_K) return fail(SKNN_ERR_UNSUPPORTED, "k > SKNN_MAX_K");
     return SKNN_OK;
 }
 
@@ -221,10 +222,11 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     lp.shard_count = o.shard_count > 1 ? o.shard_count : 1;
     lp.dense_mode = dense_mode_for(o, ts.dp);
     lp.dense_tau = dense_tau_for(o, ts.dp);
-    if (lp.dense_mode == 2 && !dense_supported(ts.dp)) {
-        set_last_error("force_path = DENSE needs d <= 256");
+    if (lp.dense_mode == 2 && (!dense_supported(ts.dp) || k > 32)) {
+        set_last_error("force_path = DENSE needs d <= 256 and k <= 32");
         return SKNN_ERR_UNSUPPORTED;
     }
+    if (k > 32) lp.dense_mode = 1;  // the dense tiles keep a register top-k (k <= 32)
     DenseOrigin dorg;
     if (lp.dense_mode != 1) {
         SKNN_TRY(dense_prepare(cx, qs, ts, dorg));
@@ -232,7 +234,7 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     }
     if (lp.dense_mode == 0 && !lp.dorg) lp.dense_mode = 1;
     SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
-    SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp), lp.shard_rank, lp.shard_count, l1));
+    SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp, k), lp.shard_rank, lp.shard_count, l1));
     mk.l1 = tm.mark();
     key_t* init_topk = nullptr;
     if (lp.dense_mode != 1) {
@@ -320,7 +322,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     sknn_status st = SKNN_OK;
     const int dp = (d + 3) & ~3;
     const bool self = index ? (Q == index->user_ptr && nq == index->t.n) : (Q == T && nq == nt);
-    int mapping = choose_mapping(o, di, nq, dp);
+    int mapping = choose_mapping(o, di, nq, dp, k);
     int path = o.force_path == SKNN_PATH_BRUTE ? SKNN_PATH_BRUTE : SKNN_PATH_SPARSE;
     Marks mk;
     int mq = 0, mt = 0;
@@ -367,6 +369,10 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
             sp.out_dist = d_odist;
             sp.counters = counters;
             mapping = SKNN_MAP_WARP;
+            if (k > 32) {
+                st = fail(SKNN_ERR_UNSUPPORTED, "force_path = BRUTE supports k <= 32");
+                break;
+            }
             st = run_brute(cx, dQ, nq, dT, nt, d, sp);
             mk.bt = tm.mark();
             mk.scan = mk.bt;
@@ -652,7 +658,7 @@ sknn_status sknn_config_decide(int64_t nq, int64_t nt, int32_t d, int32_t k, con
     if (out->tpq_raw > 1.0) tpq = 1 << (int)lround(log2(out->tpq_raw));       // reading R15
     out->threads_per_query = tpq;
     const int dp = (d + 3) & ~3;
-    out->mapping = dp <= 32 ? SKNN_MAP_THREAD : SKNN_MAP_WARP;  // B200 rule, see choose_mapping
+    out->mapping = (dp <= 32 || k > 32) ? SKNN_MAP_THREAD : SKNN_MAP_WARP;  // B200 rule, see choose_mapping
     out->mq = det_lm_num(std::max<int64_t>(nq, 1), 0);
     out->mt = det_lm_num(nt, 0);
     return SKNN_OK;

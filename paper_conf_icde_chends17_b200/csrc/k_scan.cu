@@ -167,7 +167,8 @@ static void launch_wpq(Ctx& cx, const ScanArgs& a) {
     k_scan_wpq<DP><<<grid, 256, smem, cx.stream>>>(a);
 }
 
-int scan_tile_size(int mapping, int dp) { return (mapping == SKNN_MAP_THREAD && dp <= 32) ? 32 : 8; }
+bool scan_uses_tpq(int mapping, int dp, int k) { return (mapping == SKNN_MAP_THREAD && dp <= 32) || k > 32; }
+int scan_tile_size(int mapping, int dp, int k) { return scan_uses_tpq(mapping, dp, k) ? 32 : 8; }
 
 sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int shard_rank, int shard_count, Level1& l1) {
     int64_t max_tiles = (qs.n + tile - 1) / tile + qs.m;
@@ -194,7 +195,7 @@ sknn_status run_dense_tiles(Ctx& cx, const Side& qs, Level1& l1) {
 
 sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
     const int dp = ts.dp;
-    const bool tpq = p.mapping == SKNN_MAP_THREAD && dp <= 32;
+    const bool tpq = scan_uses_tpq(p.mapping, dp, p.k);
     ScanArgs a{};
     a.qrows = qs.rows; a.qorig = qs.orig; a.qoff = qs.off;
     a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
@@ -214,7 +215,8 @@ sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, 
             case 20: launch_tpq_dp<20>(cx, a); break;
             case 24: launch_tpq_dp<24>(cx, a); break;
             case 28: launch_tpq_dp<28>(cx, a); break;
-            default: launch_tpq_dp<32>(cx, a); break;
+            case 32: launch_tpq_dp<32>(cx, a); break;
+            default: launch_tpq_dp<0>(cx, a); break;  // dp > 32 with k > 32
         }
     } else {
         switch (dp) {
@@ -324,8 +326,43 @@ __global__ void __launch_bounds__(256) k_merge(const int32_t* __restrict__ pidx,
     }
 }
 
+// k > 32: one thread per query, P-way merge of the sorted lists by repeated
+// selection of the smallest head (O(k P) per query).
+__global__ void k_merge_big(const int32_t* __restrict__ pidx, const float* __restrict__ pd2, int P, int64_t nq, int k,
+                            int32_t* __restrict__ out_idx, float* __restrict__ out_dist, int out_squared) {
+    int head[16];
+    for (int64_t qi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; qi < nq; qi += (int64_t)gridDim.x * blockDim.x) {
+        for (int p = 0; p < P; ++p) head[p] = 0;
+        for (int r = 0; r < k; ++r) {
+            key_t best = kInfKey;
+            int bp = 0;
+            for (int p = 0; p < P; ++p) {
+                if (head[p] >= k) continue;
+                const int64_t e = ((int64_t)p * nq + qi) * k + head[p];
+                const key_t key = make_key(pd2[e], pidx[e]);
+                if (key < best) { best = key; bp = p; }
+            }
+            head[bp] += 1;
+            const int64_t o = qi * k + r;
+            const float d2 = key_d2(best);
+            out_dist[o] = out_squared ? d2 : __fsqrt_rn(d2);
+            if (out_idx) out_idx[o] = key_idx(best);
+        }
+    }
+}
+
 sknn_status run_merge(Ctx& cx, const int32_t* part_idx, const float* part_d2, int P, int64_t nq, int k,
                       int32_t* out_idx, float* out_dist, int out_squared) {
+    if (k > 32) {
+        if (P > 16) {
+            set_last_error("sknn_merge_partials: k > 32 supports at most 16 partial lists");
+            return SKNN_ERR_UNSUPPORTED;
+        }
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nq + 255) / 256, (int64_t)cx.num_sms * 8));
+        k_merge_big<<<grid, 256, 0, cx.stream>>>(part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared);
+        cx.launched();
+        return cx.check_launch("merge");
+    }
     int64_t blocks = (nq + 7) / 8;
     int grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)cx.num_sms * 8));
     k_merge<<<grid, 256, 0, cx.stream>>>(part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared);

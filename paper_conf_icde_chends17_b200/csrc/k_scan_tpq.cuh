@@ -24,33 +24,34 @@ namespace sknn {
 // P:L629), laid out like the paper's Layout 2 (Fig. 6b): slot r of
 // thread t at [r][t], so a warp's accesses to one slot are contiguous. Sorted
 // ascending; an insertion shifts only the slots above the insertion point.
-constexpr int kTpqThreads = 256;
+template <int STRIDE>
 struct SmemTopK {
     key_t* s;
     int k;
     __device__ __forceinline__ void init(key_t* col, int k_) {
         s = col;
         k = k_;
-        for (int r = 0; r < k; ++r) s[r * kTpqThreads] = kInfKey;
+        for (int r = 0; r < k; ++r) s[r * STRIDE] = kInfKey;
     }
-    __device__ __forceinline__ key_t get(int r) const { return s[r * kTpqThreads]; }
-    __device__ __forceinline__ void set(int r, key_t v) { s[r * kTpqThreads] = v; }
+    __device__ __forceinline__ key_t get(int r) const { return s[r * STRIDE]; }
+    __device__ __forceinline__ void set(int r, key_t v) { s[r * STRIDE] = v; }
     // precondition: key < current k-th; returns the new k-th
     __device__ __forceinline__ key_t insert(key_t key) {
         int i = k - 1;
         while (i > 0) {
-            const key_t v = s[(i - 1) * kTpqThreads];
+            const key_t v = s[(i - 1) * STRIDE];
             if (!(key < v)) break;
-            s[i * kTpqThreads] = v;
+            s[i * STRIDE] = v;
             --i;
         }
-        s[i * kTpqThreads] = key;
-        return s[(k - 1) * kTpqThreads];
+        s[i * STRIDE] = key;
+        return s[(k - 1) * STRIDE];
     }
 };
 
-template <int DP, int KMAX, bool SMEM>
-__global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
+// DP == 0: runtime dp (> 32), the query row is re-read from L1/L2 (large k only)
+template <int DP, int KMAX, bool SMEM, int THREADS>
+__global__ void __launch_bounds__(THREADS) k_scan_tpq(ScanArgs a) {
     extern __shared__ __align__(16) key_t s_topk[];  // [k][256] when SMEM
     const float INF = __int_as_float(0x7f800000);
     const int lane = threadIdx.x & 31;
@@ -67,11 +68,19 @@ __global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
         const int i = tl.y + lane;
         const bool active = i < qsz;
         const int qpos = qlo + (active ? i : 0);
-        float4 q[DP / 4];
+        constexpr int QV = DP > 0 ? DP / 4 : 1;
+        float4 q[QV];
+        const float* qrow = a.qrows + (int64_t)qpos * a.dp;
+        if constexpr (DP > 0) {
 #pragma unroll
-        for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(a.qrows + (int64_t)qpos * DP) + c);
+            for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(qrow) + c);
+        }
+        auto d2q = [&](const float* t) -> float {
+            if constexpr (DP > 0) return d2_reg<DP>(q, t);
+            else return d2_rows(qrow, t, a.dp);
+        };
         RegTopK<SMEM ? 1 : KMAX> top;
-        SmemTopK stop;
+        SmemTopK<THREADS> stop;
         key_t kth;
         if constexpr (SMEM) {
             stop.init(s_topk + threadIdx.x, a.k);
@@ -109,7 +118,7 @@ __global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
                 const float D = __ldg(cD + c), rt = __ldg(a.trad + tc);
                 if (!ti_keep(D - rown - rt, theta, D + rown + rt, a.eta)) continue;
                 const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
-                const float dq = __fsqrt_rn(d2_reg<DP>(q, a.tcent + (int64_t)tc * DP));  // Alg. 2 line 6
+                const float dq = __fsqrt_rn(d2q(a.tcent + (int64_t)tc * a.dp));  // Alg. 2 line 6
                 ++cevals;
                 // empty window: every member distance lies in [dt_min, r_t]
                 if (!ti_keep(dq - rt, theta, dq + rt, a.eta)) continue;
@@ -139,6 +148,7 @@ __global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
                     const bool takeL = bL < bR;
                     const float bmin = takeL ? bL : bR;
                     const float dtc = takeL ? dtL : dtR;
+                    if (bmin == INF) break;                          // window exhausted (theta may be +inf)
                     if (!ti_keep(bmin, theta, dq + dtc, a.eta)) break;  // both sides beyond theta
                     const int jc = takeL ? L : R;
                     float d2;                                                   // line 15
@@ -166,7 +176,7 @@ __global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
                             ++R;
                             if (R < hi) dtR = __ldg(a.tdist + R);
                         }
-                        d2 = d2_reg<DP>(q, a.trows + (int64_t)jc * DP);
+                        d2 = d2q(a.trows + (int64_t)jc * a.dp);
                     }
                     ++evals;
                     if (d2 <= kth_d2) {                                         // line 16 (distance part)
@@ -200,36 +210,48 @@ __global__ void __launch_bounds__(kTpqThreads) k_scan_tpq(ScanArgs a) {
     add_counter(&a.counters->center_evals, cevals);
 }
 
-template <int DP, int KMAX, bool SMEM>
+template <int DP, int KMAX, bool SMEM, int THREADS>
 static void launch_tpq(Ctx& cx, const ScanArgs& a) {
-    const size_t smem = SMEM ? sizeof(key_t) * (size_t)a.k * kTpqThreads : 0;
+    const size_t smem = SMEM ? sizeof(key_t) * (size_t)a.k * THREADS : 0;
     if (smem > 48 * 1024)
-        cudaFuncSetAttribute(k_scan_tpq<DP, KMAX, SMEM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    int grid = occupancy_grid(cx, (const void*)k_scan_tpq<DP, KMAX, SMEM>, kTpqThreads, smem);
-    k_scan_tpq<DP, KMAX, SMEM><<<grid, kTpqThreads, smem, cx.stream>>>(a);
+        cudaFuncSetAttribute(k_scan_tpq<DP, KMAX, SMEM, THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int grid = occupancy_grid(cx, (const void*)k_scan_tpq<DP, KMAX, SMEM, THREADS>, THREADS, smem);
+    k_scan_tpq<DP, KMAX, SMEM, THREADS><<<grid, THREADS, smem, cx.stream>>>(a);
 }
 
 // kNearests placement (Fig. 8, P:L587-609 re-derived for B200 in DESIGN.md):
-// shared memory when k*4 <= th1 (k <= 28 on B200), registers otherwise;
-// SKNN_TOPK=reg|smem overrides for ablation.
+// shared memory when k*4 <= th1 (k <= 28 on B200), registers for k <= 32
+// otherwise; beyond the register budget (large k, NEXT-2) shared memory with
+// fewer threads per CTA so k * 8 B per thread still fits. SKNN_TOPK=reg|smem
+// overrides for ablation.
 template <int DP>
-void launch_tpq_dp(Ctx& cx, const ScanArgs& a) {
+static void launch_tpq_small_k(Ctx& cx, const ScanArgs& a) {
     const char* ov = getenv("SKNN_TOPK");
     const bool smem = ov ? (ov[0] == 's') : (a.k * 4 <= 114);
     if (smem) {
-        launch_tpq<DP, 1, true>(cx, a);
+        launch_tpq<DP, 1, true, 256>(cx, a);
         return;
     }
     switch ((a.k + 3) / 4) {
-        case 1: launch_tpq<DP, 4, false>(cx, a); break;
-        case 2: launch_tpq<DP, 8, false>(cx, a); break;
-        case 3: launch_tpq<DP, 12, false>(cx, a); break;
-        case 4: launch_tpq<DP, 16, false>(cx, a); break;
-        case 5: launch_tpq<DP, 20, false>(cx, a); break;
-        case 6: launch_tpq<DP, 24, false>(cx, a); break;
-        case 7: launch_tpq<DP, 28, false>(cx, a); break;
-        default: launch_tpq<DP, 32, false>(cx, a); break;
+        case 1: launch_tpq<DP, 4, false, 256>(cx, a); break;
+        case 2: launch_tpq<DP, 8, false, 256>(cx, a); break;
+        case 3: launch_tpq<DP, 12, false, 256>(cx, a); break;
+        case 4: launch_tpq<DP, 16, false, 256>(cx, a); break;
+        case 5: launch_tpq<DP, 20, false, 256>(cx, a); break;
+        case 6: launch_tpq<DP, 24, false, 256>(cx, a); break;
+        case 7: launch_tpq<DP, 28, false, 256>(cx, a); break;
+        default: launch_tpq<DP, 32, false, 256>(cx, a); break;
     }
 }
 
+template <int DP>
+void launch_tpq_dp(Ctx& cx, const ScanArgs& a) {
+    if (a.k > 32 || DP == 0) {
+        if (a.k <= 96) launch_tpq<DP, 1, true, 256>(cx, a);
+        else if (a.k <= 384) launch_tpq<DP, 1, true, 64>(cx, a);
+        else launch_tpq<DP, 1, true, 32>(cx, a);
+        return;
+    }
+    if constexpr (DP > 0) launch_tpq_small_k<DP>(cx, a);
+}
 }  // namespace sknn

@@ -137,7 +137,8 @@ sknn_status run_dense_tiles(Ctx& cx, const Side& qs, Level1& l1);
 sknn_status run_dense(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const DenseParams& p);
 // k_scan.cu: tiles of `tile` queries of one query cluster (thread-data remapping)
 sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int shard_rank, int shard_count, Level1& l1);
-int scan_tile_size(int mapping, int dp);
+int scan_tile_size(int mapping, int dp, int k);
+bool scan_uses_tpq(int mapping, int dp, int k);
 
 // k_scan.cu
 struct ScanParams {

@@ -70,10 +70,10 @@ def test_null_pointers_rejected(L):
     assert L.sknn_index_free(None) == 0
 
 
-def test_large_k_unsupported(L):
-    Q = np.zeros((64, 2), np.float32)
-    out = np.zeros((64, 33), np.float32)
-    assert L.sknn_join(Q.ctypes.data, 64, Q.ctypes.data, 64, 2, 33, None, out.ctypes.data, None) == -5
+def test_k_above_max_unsupported(L):
+    Q = np.zeros((1000, 2), np.float32)
+    out = np.zeros((1000, 513), np.float32)
+    assert L.sknn_join(Q.ctypes.data, 1000, Q.ctypes.data, 1000, 2, 513, None, out.ctypes.data, None) == -5
 
 
 def test_nq_zero_is_noop(L):

@@ -374,3 +374,38 @@ def test_squared_output_and_index_base(sknn):
     ridx, rdist, rd2 = oracle.knn_join(Q, T, k, return_d2=True)
     np.testing.assert_array_equal(i.cpu().numpy(), ridx + 1000)
     np.testing.assert_array_equal(d2.cpu().numpy(), rd2.astype(np.float32))
+
+
+# ----------------------------------------------------------- large k (NEXT-2) --
+@pytest.mark.parametrize("k", [33, 64, 100, 256, 512])
+def test_large_k(sknn, k):
+    """k beyond the register budget: shared-memory kNearests with fewer threads
+    per CTA (Fig. 8 placement); bit-exact on integer inputs, low and high d."""
+    rng = np.random.default_rng(k)
+    for d in (4, 28, 40):
+        T = rng.integers(0, 60, size=(4000, d)).astype(np.float32)
+        Q = rng.integers(0, 60, size=(500, d)).astype(np.float32)
+        idx, dist, _ = run(sknn, Q, T, k, False)
+        ridx, rdist = oracle.knn_join(Q, T, k)
+        assert_knn_bitexact(idx, dist, ridx, rdist)
+    X = datagen.c1_uniform_int(2048)
+    idx, dist, _ = run(sknn, X, X, k, True)
+    ridx, rdist = oracle.knn_join(X, X, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+def test_merge_partials_large_k(sknn):
+    T = datagen.c5_blobs(12000, which="T")
+    Q = datagen.c5_blobs(1500, which="Q")
+    k = 64
+    dQ = dev(Q)
+    parts_i, parts_d = [], []
+    bounds = np.linspace(0, T.shape[0], 4).astype(int)
+    for r in range(3):
+        i, d = sknn.join(dQ, dev(T[bounds[r]:bounds[r + 1]]), k, out_squared=1, index_base=int(bounds[r]))
+        parts_i.append(i)
+        parts_d.append(d)
+    idx, dist = sknn.merge_partials(torch.stack(parts_i), torch.stack(parts_d), k)
+    torch.cuda.synchronize()
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx.cpu().numpy(), dist.cpu().numpy(), ridx, rdist)
