@@ -159,6 +159,15 @@ def c5_blobs(n: int = 4_000_000, d: int = 16, which: str = "T") -> np.ndarray:
 def workload(name: str, scale: float = 1.0):
     """Return (Q, T, k, self_join) for a named config; ``scale`` < 1 shrinks n
     (parity tests at sizes the oracle finishes in seconds)."""
+    if name[0] in "GK" and name[1:].isdigit():
+        # ablation shapes (not bench configs): G<d> = 200,000-point integer blob
+        # self-join (C5 recipe, 1,000 blobs), K<d> = C3's KEGG recipe at dimension d
+        d = int(name[1:])
+        if name[0] == "G":
+            X = gaussian_blobs(max(16, int(round(200_000 * scale))), d, 1000, 0.0, 1023.0, 10.0, 40.0, 1023.0, 7, 70)
+        else:
+            X = c3_kegg(max(16, int(round(65_554 * scale))), d=d)
+        return X, X, 16, True
     cfg = CONFIGS[name.replace("int", "")]
     n = max(16, int(round(cfg["n"] * scale)))
     k = cfg["k"]

@@ -234,7 +234,8 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     }
     if (lp.dense_mode == 0 && !lp.dorg) lp.dense_mode = 1;
     SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
-    SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp, k), lp.shard_rank, lp.shard_count, l1));
+    SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp, k), k, scan_resident_warps(cx, mapping, ts.dp, k),
+                       lp.shard_rank, lp.shard_count, l1));
     mk.l1 = tm.mark();
     key_t* init_topk = nullptr;
     if (lp.dense_mode != 1) {

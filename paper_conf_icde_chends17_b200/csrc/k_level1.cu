@@ -108,7 +108,7 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     int shard_count, int dense_mode, float dense_tau, const float* __restrict__ cq_o,
     const float* __restrict__ ct_o, float dense_eps, float* __restrict__ ub_out, int32_t* __restrict__ cand,
     int32_t* __restrict__ cand_count, float* __restrict__ cand_D, int32_t* __restrict__ dcand,
-    int32_t* __restrict__ dcount,
+    int32_t* __restrict__ dcount, unsigned long long* __restrict__ work,
     Counters* __restrict__ counters) {
     extern __shared__ __align__(16) unsigned char smem[];
     u64* s_keys = reinterpret_cast<u64*>(smem);                               // keys_cap (>= mt) entries
@@ -123,7 +123,7 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     const int qc = blockIdx.x;
     const int qsize = qoff[qc + 1] - qoff[qc];
     if (qsize == 0 || (shard_count > 1 && qc % shard_count != shard_rank)) {
-        if (threadIdx.x == 0) { ub_out[qc] = 0.f; cand_count[qc] = 0; dcount[qc] = 0; }
+        if (threadIdx.x == 0) { ub_out[qc] = 0.f; cand_count[qc] = 0; dcount[qc] = 0; work[qc] = 0; }
         return;
     }
     for (int i = threadIdx.x; i < dp; i += blockDim.x) s_qc[i] = qcent[(int64_t)qc * dp + i];
@@ -216,31 +216,39 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     float* Drow = cand_D + (int64_t)qc * mt;
     __shared__ int s_wcnt[2][kL1Threads / 32];
     __shared__ int s_base[2];
-    if (threadIdx.x == 0) { s_base[0] = 0; s_base[1] = 0; }
+    __shared__ unsigned long long s_work;
+    if (threadIdx.x == 0) { s_base[0] = 0; s_base[1] = 0; s_work = 0; }
     __syncthreads();
     for (int base = 0; base < nc; base += blockDim.x) {
         const int i = base + threadIdx.x;
         int tc = -1;
         bool dense = false;
+        unsigned cost = 0;
         if (i < nc) {
             tc = int32_t(uint32_t(s_keys[i] & 0xffffffffu));
+            // expected share of tc's members inside a typical query's Alg. 2
+            // window [dq - th, dq + th] with dq ~ D and th ~ V_k (the k-th
+            // nearest target bound of the cluster center, without r_q)
+            const int sz = __ldg(toff + tc + 1) - __ldg(toff + tc);
+            const float rt = __ldg(trad + tc);
+            const float Dp = s_D[tc];
+            const float ov = fminf(rt, Dp + Vk) - fmaxf(0.f, Dp - Vk);
+            const float share = fminf(1.f, fmaxf(0.f, ov) / fmaxf(rt, 1e-30f));
             if (dense_mode == 2) {
                 dense = true;
             } else if (dense_mode == 0) {
-                // expected share of tc's members inside a typical query's Alg. 2
-                // window [dq - th, dq + th] with dq ~ D and th ~ V_k (the k-th
-                // nearest target bound of the cluster center, without r_q)
-                const int sz = __ldg(toff + tc + 1) - __ldg(toff + tc);
-                const float rt = __ldg(trad + tc);
-                const float Dp = s_D[tc];
-                const float ov = fminf(rt, Dp + Vk) - fmaxf(0.f, Dp - Vk);
                 // and the tensor-core screen must stay selective: its error bound
                 // eps (||a||^2 + ||b||^2) small against the k-th distance^2 ~ V_k^2
                 const float ma = cq_o[qc] + rq, mb = ct_o[tc] + rt;
                 const bool sharp = dense_eps * (ma * ma + mb * mb) <= 0.25f * Vk * Vk;
                 dense = sz >= 32 && sharp && ov >= dense_tau * fmaxf(rt, 1e-30f);
             }
+            // scan work estimate of a sparse pair (per query): the per-candidate
+            // tests plus the expected member visits (load balancing only)
+            if (!dense) cost = 4u + (unsigned)(share * (float)sz);
         }
+        for (int o = 16; o > 0; o >>= 1) cost += __shfl_xor_sync(0xffffffffu, cost, o);
+        if ((threadIdx.x & 31) == 0 && cost) atomicAdd(&s_work, (unsigned long long)cost);
         const unsigned md = __ballot_sync(0xffffffffu, i < nc && dense);
         const unsigned ms = __ballot_sync(0xffffffffu, i < nc && !dense);
         const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -269,6 +277,7 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     if (threadIdx.x == 0) {
         cand_count[qc] = s_base[0];
         dcount[qc] = s_base[1];
+        work[qc] = s_work;
         if (counters) {
             atomicAdd(&counters->cand_pairs, (unsigned long long)nc);
             if (s_base[1]) atomicAdd(&counters->dense_pairs, (unsigned long long)s_base[1]);
@@ -285,6 +294,7 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
     SKNN_TRY(cx.alloc_scratch((void**)&out.cand_D, sizeof(float) * (size_t)mq * mt));
     SKNN_TRY(cx.alloc_scratch((void**)&out.dcand, sizeof(int32_t) * (size_t)mq * mt));
     SKNN_TRY(cx.alloc_scratch((void**)&out.dcount, sizeof(int32_t) * mq));
+    SKNN_TRY(cx.alloc_scratch((void**)&out.work, sizeof(unsigned long long) * mq));
     int cap = 1;
     while (cap < mt) cap <<= 1;
     cap = std::max(cap, kL1Vals);
@@ -300,7 +310,7 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
                                                   p.dense_mode, p.dense_tau, p.dorg ? p.dorg->cq_o : nullptr,
                                                   p.dorg ? p.dorg->ct_o : nullptr, p.dorg ? p.dorg->eps : 0.f,
                                                   out.ub, out.cand, out.cand_count, out.cand_D,
-                                                  out.dcand, out.dcount, counters);
+                                                  out.dcand, out.dcount, out.work, counters);
     cx.launched();
     return cx.check_launch("level1");
 }

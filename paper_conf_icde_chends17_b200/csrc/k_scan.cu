@@ -1,3 +1,4 @@
+#include <stdlib.h>
 // k_scan.cu -- Step 3 of the method: level-2 (point-level) filtering fused
 // with exact distance evaluation and per-query top-k (Alg. 2, P:L355-375;
 // Fig. 4 pointFilter), plus the brute-force anchor and the partial
@@ -17,6 +18,10 @@
 // member with l > theta (line 10, `break`) -- re-tested as theta shrinks.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdio.h>
+
+#include <algorithm>
+#include <vector>
 
 #include "k_scan_common.cuh"
 
@@ -43,7 +48,7 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
         if (lane == 0) tile = atomicAdd(a.tile_counter, 1);
         tile = __shfl_sync(0xffffffffu, tile, 0);
         if (tile >= ntiles) break;
-        const int2 tl = a.tiles[tile];
+        const int4 tl = a.tiles[tile];
         const int qc = tl.x;
         const int qlo = a.qoff[qc], qsz = a.qoff[qc + 1] - qlo;
         const int nq_tile = min(a.tile, qsz - tl.y);
@@ -152,6 +157,136 @@ __global__ void __launch_bounds__(1024) k_make_tiles(const int32_t* __restrict__
     if (threadIdx.x == 0) { *ntiles = s_carry; *counter = 0; }
 }
 
+// exclusive scan over a 1024-thread block (warp shuffles + one smem row)
+__device__ __forceinline__ int block_exscan(int v, int* s_warp, int& total) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int x = v;
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) s_warp[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        int t = s_warp[lane];
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, t, o);
+            if (lane >= o) t += y;
+        }
+        s_warp[lane] = t;
+    }
+    __syncthreads();
+    const int r = (w ? s_warp[w - 1] : 0) + x - v;
+    total = s_warp[31];
+    __syncthreads();
+    return r;
+}
+
+__device__ __forceinline__ unsigned long long block_sum_u64(unsigned long long v, unsigned long long* s_red) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if (lane == 0) s_red[w] = v;
+    __syncthreads();
+    unsigned long long t = 0;
+    for (int i = 0; i < 32; ++i) t += s_red[i];
+    __syncthreads();
+    return t;
+}
+
+// Level-2 task list (single CTA), load-balanced on the level-1 work estimate:
+//  * a tile (`tile` queries of one cluster) whose estimated work exceeds both
+//    total / resident warps (it alone would outlast the average warp) and 4x
+//    the mean tile (measured: splitting moderate tiles costs more than the
+//    balance gains) is SPLIT into S <= 32 tasks of about half the per-warp
+//    average that take every S-th candidate cluster (interleaved, so each task sees near and far
+//    clusters); the S tasks of a tile share the queries' k-th distance bound
+//    through `theta2` and their partial lists are merged by k_merge_split;
+//  * order: split tasks first, then unsplit tiles heavier than W0 / 4, then
+//    the rest (longest work first, so no straggler starts last).
+// Split tasks are capped at `cap_split` (W0 doubles until they fit); their
+// part index equals their task index. split == false (warp-per-query scan)
+// keeps S = 1 and only orders.
+__global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__ qoff, int mq, int tile,
+                                                     int shard_rank, int shard_count,
+                                                     const unsigned long long* __restrict__ work,
+                                                     const int32_t* __restrict__ ccount, int slots, int cap_split,
+                                                     int split, int order, float wfac, float hfac, int4* __restrict__ tasks, int* __restrict__ ntasks,
+                                                     int4* __restrict__ merges, int* __restrict__ nmerges) {
+    __shared__ int s_warp[32];
+    __shared__ unsigned long long s_red[32];
+    auto nt_of = [&](int c) -> int {
+        if (c >= mq) return 0;
+        if (shard_count > 1 && c % shard_count != shard_rank) return 0;
+        return (qoff[c + 1] - qoff[c] + tile - 1) / tile;
+    };
+    unsigned long long tot = 0, ntl = 0;
+    for (int c = threadIdx.x; c < mq; c += 1024) {
+        tot += (unsigned long long)nt_of(c) * work[c];
+        ntl += (unsigned long long)nt_of(c);
+    }
+    tot = block_sum_u64(tot, s_red);
+    ntl = block_sum_u64(ntl, s_red);
+    // a tile is a straggler when its work exceeds both the average per
+    // resident warp and hfac x the mean tile; it is cut into pieces of
+    // wfac x the average per resident warp
+    const double per_slot = (double)tot / (double)slots;
+    const double mean = (double)tot / (double)(ntl ? ntl : 1);
+    const unsigned long long H = (unsigned long long)fmax(per_slot, hfac * mean);
+    unsigned long long W0 = (unsigned long long)(per_slot * wfac);
+    if (W0 < 64) W0 = 64;
+    auto s_of = [&](int c, unsigned long long w0) -> int {
+        if (!split || c >= mq || work[c] <= H) return 1;
+        unsigned long long s = (work[c] + w0 - 1) / w0;
+        s = s < 32 ? (s > 2 ? s : 2) : 32;
+        const unsigned long long nc = (unsigned long long)(ccount[c] > 1 ? ccount[c] : 1);
+        return (int)(s < nc ? s : nc);
+    };
+    for (int it = 0; it < 40; ++it) {
+        unsigned long long n = 0;
+        for (int c = threadIdx.x; c < mq; c += 1024) {
+            const int S = s_of(c, W0);
+            if (S > 1) n += (unsigned long long)nt_of(c) * S;
+        }
+        n = block_sum_u64(n, s_red);
+        if (n <= (unsigned long long)cap_split) break;
+        W0 *= 2;
+    }
+    int carry = 0, mcarry = 0;
+    for (int pass = 0; pass < 3; ++pass) {
+        if (!order && pass == 2) break;
+        for (int base = 0; base < mq; base += 1024) {
+            const int c = base + threadIdx.x;
+            const int nt = nt_of(c);
+            const int S = s_of(c, W0);
+            bool mine;
+            if (pass == 0) mine = S > 1;
+            else if (!order) mine = S == 1 && c < mq;
+            else if (pass == 1) mine = S == 1 && c < mq && work[c] * 4 >= W0;
+            else mine = S == 1 && c < mq && work[c] * 4 < W0;
+            const int n = mine ? nt * S : 0;
+            int total, mtotal;
+            const int start = carry + block_exscan(n, s_warp, total);
+            const int mstart = mcarry + block_exscan(pass == 0 && mine ? nt : 0, s_warp, mtotal);
+            if (mine) {
+                for (int t = 0; t < nt; ++t) {
+                    for (int sp = 0; sp < S; ++sp) {
+                        const int id = start + t * S + sp;
+                        tasks[id] = make_int4(c, t * tile, sp | (S << 8), S > 1 ? id : -1);
+                    }
+                    if (pass == 0) merges[mstart + t] = make_int4(c, t * tile, S, start + t * S);
+                }
+            }
+            carry += total;
+            mcarry += mtotal;
+        }
+    }
+    if (threadIdx.x == 0) {
+        ntasks[0] = carry;
+        ntasks[1] = 0;
+        *nmerges = mcarry;
+    }
+}
+
 int occupancy_grid(Ctx& cx, const void* fn, int threads, size_t smem) {
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem);
@@ -164,21 +299,70 @@ static void launch_wpq(Ctx& cx, const ScanArgs& a) {
     size_t smem = DP > 0 ? 0 : sizeof(float) * 8 * a.dp;
     if (smem > 48 * 1024) cudaFuncSetAttribute(k_scan_wpq<DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int grid = occupancy_grid(cx, (const void*)k_scan_wpq<DP>, 256, smem);
+    if (a.probe_warps) {  // dry run: report resident warps for the task planner
+        *a.probe_warps = grid * (256 / 32);
+        return;
+    }
     k_scan_wpq<DP><<<grid, 256, smem, cx.stream>>>(a);
 }
 
 bool scan_uses_tpq(int mapping, int dp, int k) { return (mapping == SKNN_MAP_THREAD && dp <= 32) || k > 32; }
 int scan_tile_size(int mapping, int dp, int k) { return scan_uses_tpq(mapping, dp, k) ? 32 : 8; }
 
-sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int shard_rank, int shard_count, Level1& l1) {
-    int64_t max_tiles = (qs.n + tile - 1) / tile + qs.m;
-    SKNN_TRY(cx.alloc_scratch((void**)&l1.tiles, sizeof(int2) * max_tiles));
+sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int shard_rank, int shard_count,
+                      Level1& l1) {
+    const char* ev = getenv("SKNN_SPLIT");  // ablation: SKNN_SPLIT=0 disables tile splitting
+    const bool split = tile == 32 && !(ev && ev[0] == '0');  // thread-per-query scan only
+    const char* eo = getenv("SKNN_TASKORDER");  // ablation: SKNN_TASKORDER=0 keeps cluster order
+    const int order = (eo && eo[0] == '0') ? 0 : 1;
+    const char* ew = getenv("SKNN_SPLITW");  // piece size, x total work / resident warps
+    const float wfac = ew ? (float)atof(ew) : 0.5f;
+    const char* eh = getenv("SKNN_SPLITH");  // straggler threshold, x mean tile work
+    const float hfac = eh ? (float)atof(eh) : 4.0f;
+    // partial lists of split tasks: at most 2 x resident warps of them, <= 256 MB
+    int cap = 0;
+    if (split) {
+        const int64_t per_task = (int64_t)32 * k * sizeof(key_t);
+        cap = (int)std::min<int64_t>(2 * (int64_t)slots, ((int64_t)256 << 20) / per_task);
+    }
+    int64_t max_tiles = (qs.n + tile - 1) / tile + qs.m + cap;
+    SKNN_TRY(cx.alloc_scratch((void**)&l1.tiles, sizeof(int4) * max_tiles));
     SKNN_TRY(cx.alloc_scratch((void**)&l1.ntiles, sizeof(int) * 2));
+    SKNN_TRY(cx.alloc_scratch((void**)&l1.nmerges, sizeof(int)));
+    if (split && cap > 0) {
+        SKNN_TRY(cx.alloc_scratch((void**)&l1.merges, sizeof(int4) * cap));
+        SKNN_TRY(cx.alloc_scratch((void**)&l1.part, sizeof(key_t) * (size_t)cap * 32 * k));
+        SKNN_TRY(cx.alloc_scratch((void**)&l1.theta2, sizeof(unsigned) * (size_t)std::max<int64_t>(1, qs.n)));
+        // 0x7f7f7f7f = 3.4e38f: "no bound yet" for the float-bits atomicMin
+        SKNN_CUDA(cudaMemsetAsync(l1.theta2, 0x7f, sizeof(unsigned) * (size_t)qs.n, cx.stream));
+    }
     l1.tile = tile;
-    k_make_tiles<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, nullptr, l1.tiles,
-                                             l1.ntiles, l1.ntiles + 1);
+    k_make_tasks<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, l1.work, l1.cand_count,
+                                             slots, cap, split && cap > 0 ? 1 : 0, order, wfac, hfac, l1.tiles, l1.ntiles, l1.merges,
+                                             l1.nmerges);
     cx.launched();
-    return cx.check_launch("tiles");
+    if (getenv("SKNN_PLANDBG")) {  // diagnostics: the plan on stderr (synchronises)
+        cudaStreamSynchronize(cx.stream);
+        std::vector<unsigned long long> w(qs.m);
+        std::vector<int32_t> off(qs.m + 1), cc(qs.m);
+        int nt[2] = {0, 0}, nm = 0;
+        cudaMemcpy(w.data(), l1.work, sizeof(unsigned long long) * qs.m, cudaMemcpyDeviceToHost);
+        cudaMemcpy(off.data(), qs.off, sizeof(int32_t) * (qs.m + 1), cudaMemcpyDeviceToHost);
+        cudaMemcpy(cc.data(), l1.cand_count, sizeof(int32_t) * qs.m, cudaMemcpyDeviceToHost);
+        cudaMemcpy(nt, l1.ntiles, sizeof(int) * 2, cudaMemcpyDeviceToHost);
+        if (l1.nmerges) cudaMemcpy(&nm, l1.nmerges, sizeof(int), cudaMemcpyDeviceToHost);
+        double tot = 0, mx = 0;
+        long tiles = 0;
+        for (int c = 0; c < qs.m; ++c) {
+            const int t = (off[c + 1] - off[c] + tile - 1) / tile;
+            tiles += t;
+            tot += (double)t * (double)w[c];
+            mx = std::max(mx, (double)w[c]);
+        }
+        fprintf(stderr, "[plan] slots=%d tiles=%ld tasks=%d split_tiles=%d tot=%.3g mean/tile=%.3g max/tile=%.3g "
+                "tot/slots=%.3g\n", slots, tiles, nt[0], nm, tot, tot / std::max(1L, tiles), mx, tot / slots);
+    }
+    return cx.check_launch("tasks");
 }
 
 // dense-tile work list: tiles of 128 queries of the clusters with dense pairs
@@ -193,19 +377,9 @@ sknn_status run_dense_tiles(Ctx& cx, const Side& qs, Level1& l1) {
     return cx.check_launch("dense tiles list");
 }
 
-sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
-    const int dp = ts.dp;
-    const bool tpq = scan_uses_tpq(p.mapping, dp, p.k);
-    ScanArgs a{};
-    a.qrows = qs.rows; a.qorig = qs.orig; a.qoff = qs.off;
-    a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
-    a.ub = l1.ub; a.cand = l1.cand; a.cand_count = l1.cand_count; a.cand_D = l1.cand_D;
-    a.qdist = qs.dist; a.trad = ts.radius;
-    a.tiles = l1.tiles; a.ntiles = l1.ntiles; a.tile_counter = l1.ntiles + 1;
-    a.init_topk = p.init_topk; a.dcount = l1.dcount;
-    a.mt = ts.m; a.dp = dp; a.k = p.k; a.tile = l1.tile; a.eta = p.eta;
-    a.out_squared = p.out_squared; a.index_base = p.index_base; a.out_idx = p.out_idx; a.out_dist = p.out_dist;
-    a.counters = p.counters;
+__global__ void k_merge_split(ScanArgs a, const int4* __restrict__ merges, const int* __restrict__ nmerges);
+
+static void dispatch_scan(Ctx& cx, const ScanArgs& a, bool tpq, int dp) {
     if (tpq) {
         switch (dp) {
             case 4: launch_tpq_dp<4>(cx, a); break;
@@ -231,8 +405,42 @@ sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, 
             default: launch_wpq<0>(cx, a); break;
         }
     }
+}
+
+// resident warps of the scan kernel the dispatch would launch (task planner)
+int scan_resident_warps(Ctx& cx, int mapping, int dp, int k) {
+    ScanArgs a{};
+    a.dp = dp;
+    a.k = k;
+    int w = 0;
+    a.probe_warps = &w;
+    dispatch_scan(cx, a, scan_uses_tpq(mapping, dp, k), dp);
+    return w > 0 ? w : cx.num_sms * 32;
+}
+
+sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
+    const int dp = ts.dp;
+    const bool tpq = scan_uses_tpq(p.mapping, dp, p.k);
+    ScanArgs a{};
+    a.qrows = qs.rows; a.qorig = qs.orig; a.qoff = qs.off;
+    a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
+    a.ub = l1.ub; a.cand = l1.cand; a.cand_count = l1.cand_count; a.cand_D = l1.cand_D;
+    a.qdist = qs.dist; a.trad = ts.radius;
+    a.tiles = l1.tiles; a.ntiles = l1.ntiles; a.tile_counter = l1.ntiles + 1;
+    a.part = l1.part; a.theta2 = l1.theta2;
+    a.init_topk = p.init_topk; a.dcount = l1.dcount;
+    a.mt = ts.m; a.dp = dp; a.k = p.k; a.tile = l1.tile; a.eta = p.eta;
+    a.out_squared = p.out_squared; a.index_base = p.index_base; a.out_idx = p.out_idx; a.out_dist = p.out_dist;
+    a.counters = p.counters;
+    dispatch_scan(cx, a, tpq, dp);
     cx.launched();
-    return cx.check_launch("level2 scan");
+    SKNN_TRY(cx.check_launch("level2 scan"));
+    if (tpq && l1.merges) {
+        k_merge_split<<<cx.num_sms * 4, 256, 0, cx.stream>>>(a, l1.merges, l1.nmerges);
+        cx.launched();
+        SKNN_TRY(cx.check_launch("merge split tasks"));
+    }
+    return SKNN_OK;
 }
 
 // ------------------------------------------------------------ brute force --
@@ -290,6 +498,39 @@ sknn_status run_brute(Ctx& cx, const float* Q, int64_t nq, const float* T, int64
     k_brute<<<grid, 256, smem, cx.stream>>>(Q, nq, T, nt, d, a);
     cx.launched();
     return cx.check_launch("brute");
+}
+
+// ------------------------------------------------------ merge split tasks --
+// One thread per query of a split tile: S-way merge of the tasks' sorted
+// partial lists (disjoint member sets, so the keys are distinct) into the
+// final k (the paper's final merge of partial heaps).
+__global__ void __launch_bounds__(256) k_merge_split(ScanArgs a, const int4* __restrict__ merges,
+                                                     const int* __restrict__ nmerges) {
+    __shared__ unsigned short s_head[256][33];  // k <= 512
+    unsigned short* head = s_head[threadIdx.x];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int n = *nmerges;
+    for (int e = blockIdx.x * 8 + warp; e < n; e += gridDim.x * 8) {
+        const int4 m = merges[e];
+        const int qlo = a.qoff[m.x], qsz = a.qoff[m.x + 1] - qlo;
+        const int i = m.y + lane;
+        if (i >= qsz) continue;
+        const int S = m.z;
+        for (int s = 0; s < S; ++s) head[s] = 0;
+        const int qo = __ldg(a.qorig + qlo + i);
+        for (int r = 0; r < a.k; ++r) {
+            key_t best = kInfKey;
+            int bs = 0;
+            for (int s = 0; s < S; ++s) {
+                const int h = head[s];
+                if (h >= a.k) continue;
+                const key_t key = a.part[((int64_t)(m.w + s) * a.k + h) * 32 + lane];
+                if (key < best) { best = key; bs = s; }
+            }
+            head[bs] += 1;
+            write_result(a, qo, r, best);
+        }
+    }
 }
 
 // --------------------------------------------------------- merge partials --

@@ -26,8 +26,10 @@ struct ScanArgs {
     const float* cand_D;
     const float* qdist;   // query's own member distance d(q, c_q)
     const float* trad;    // target cluster radius
-    const int2* tiles;
+    const int4* tiles;       // tasks {query cluster, first member, split | nsplit << 8, part}
     const int* ntiles;
+    key_t* part;             // partial lists of split tasks [part][k][32]
+    unsigned* theta2;        // [nq] shared k-th distance^2 bound of split queries (float bits)
     int* tile_counter;     // dynamic tile scheduler (zeroed by k_make_tiles)
     const key_t* init_topk;  // optional [nq_perm x k] keys from the dense-tile pass (NULL = none)
     const int32_t* dcount;   // optional [mq] dense pairs per query cluster (init_topk valid iff > 0)
@@ -41,6 +43,7 @@ struct ScanArgs {
     int32_t* out_idx;
     float* out_dist;
     Counters* counters;
+    int* probe_warps;  // non-NULL: launchers only report resident warps (no launch)
 };
 
 // First member position in [lo, hi) that is NOT in Alg. 2's `continue`

@@ -58,9 +58,13 @@ __device__ __forceinline__ float d2_rows(const float* __restrict__ a, const floa
 template <int DP>
 __device__ __forceinline__ float d2_reg(const float4 (&q)[DP / 4], const float* __restrict__ t) {
     const float4* t4 = reinterpret_cast<const float4*>(t);
+    // all row loads first (memory-level parallelism), then the fixed-order sum
+    float4 r[DP / 4];
+#pragma unroll
+    for (int c = 0; c < DP / 4; ++c) r[c] = __ldg(t4 + c);
     float s = 0.f;
 #pragma unroll
-    for (int c = 0; c < DP / 4; ++c) s = d2_acc4(s, q[c], __ldg(t4 + c));
+    for (int c = 0; c < DP / 4; ++c) s = d2_acc4(s, q[c], r[c]);
     return s;
 }
 

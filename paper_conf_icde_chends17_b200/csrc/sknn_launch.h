@@ -97,9 +97,14 @@ struct Level1 {
     int32_t* cand = nullptr;      // [mq x mt] candidate target clusters, ascending center distance
     int32_t* cand_count = nullptr;  // [mq]
     float* cand_D = nullptr;      // [mq x mt] center distance D(qc, tc) of each sparse candidate
-    int2* tiles = nullptr;        // level-2 work tiles (query cluster, first member)
-    int* ntiles = nullptr;        // [2]: tile count, scheduler counter
+    unsigned long long* work = nullptr;  // [mq] scan work estimate per query (load balancing)
+    int4* tiles = nullptr;        // level-2 tasks {query cluster, first member, split | nsplit << 8, part}
+    int* ntiles = nullptr;        // [2]: task count, scheduler counter
     int tile = 0;
+    int4* merges = nullptr;       // split tiles {query cluster, first member, nsplit, first part}
+    int* nmerges = nullptr;       // [1]
+    key_t* part = nullptr;        // [split tasks x k x 32] partial lists of split tasks
+    unsigned* theta2 = nullptr;   // [nq] shared k-th distance^2 bound of split queries (float bits)
     int32_t* dcand = nullptr;     // [mq x mt] dense-tile candidates (elastic switch), ascending D
     int32_t* dcount = nullptr;    // [mq]
     int2* dtiles = nullptr;       // dense work tiles (128 queries of one cluster)
@@ -136,7 +141,10 @@ sknn_status dense_prepare(Ctx& cx, const Side& qs, const Side& ts, DenseOrigin& 
 sknn_status run_dense_tiles(Ctx& cx, const Side& qs, Level1& l1);
 sknn_status run_dense(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const DenseParams& p);
 // k_scan.cu: tiles of `tile` queries of one query cluster (thread-data remapping)
-sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int shard_rank, int shard_count, Level1& l1);
+// level-2 task list; slots = resident warps of the scan kernel (scan_resident_warps)
+sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int shard_rank, int shard_count,
+                      Level1& l1);
+int scan_resident_warps(Ctx& cx, int mapping, int dp, int k);
 int scan_tile_size(int mapping, int dp, int k);
 bool scan_uses_tpq(int mapping, int dp, int k);
 

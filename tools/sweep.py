@@ -60,7 +60,11 @@ def main():
         nq, nt = Q.shape[0], T.shape[0]
         flush = torch.empty(128 * 1024 * 1024, dtype=torch.float32, device="cuda")
         for vname in args.variants.split(","):
-            v = dict(VARIANTS[vname])
+            if vname.startswith("env:"):  # ad-hoc variant: env:NAME=VALUE
+                n_, v_ = vname[4:].split("=")
+                v = {"_env": (n_, v_)}
+            else:
+                v = dict(VARIANTS[vname])
             env = v.pop("_env", None)
             cl = v.pop("_cl", None)
             if cl:
