@@ -101,29 +101,67 @@ __global__ void __launch_bounds__(256) k_landmark_sums(const float* __restrict__
         __syncthreads();
     }
     double s = 0.0;
-    for (int p = threadIdx.x; p < kLmTile * kLmTile; p += blockDim.x) {
-        int i = p / kLmTile, j = p % kLmTile;
-        int gi = bi * kLmTile + i, gj = bj * kLmTile + j;
-        if (gi >= gj || gj >= m) continue;
-        const float* ra = smem ? A + i * dp : Xp + (int64_t)idx[t * m + gi] * dp;
-        const float* rb = smem ? B + j * dp : Xp + (int64_t)idx[t * m + gj] * dp;
-        float d2 = 0.f;
-        for (int c = 0; c < dp / 4; ++c)
-            d2 = d2_acc4(d2, reinterpret_cast<const float4*>(ra)[c], reinterpret_cast<const float4*>(rb)[c]);
-        s += (double)__fsqrt_rn(d2);
+    if (smem) {
+        // 16 x 16 threads, each a 4 x 4 block of pairs with its rows in registers
+        const int ti = threadIdx.x >> 4, tj = threadIdx.x & 15;
+        const float4* A4 = reinterpret_cast<const float4*>(A);
+        const float4* B4 = reinterpret_cast<const float4*>(B);
+        const int dq = dp / 4;
+        float acc[4][4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+#pragma unroll
+            for (int v = 0; v < 4; ++v) acc[u][v] = 0.f;
+        for (int c = 0; c < dq; ++c) {
+            float4 ra[4], rb[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                ra[u] = A4[(ti * 4 + u) * dq + c];
+                rb[u] = B4[(tj * 4 + u) * dq + c];
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+#pragma unroll
+                for (int v = 0; v < 4; ++v) acc[u][v] = d2_acc4(acc[u][v], ra[u], rb[v]);
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+#pragma unroll
+            for (int v = 0; v < 4; ++v) {
+                const int gi = bi * kLmTile + ti * 4 + u, gj = bj * kLmTile + tj * 4 + v;
+                if (gi < gj && gj < m) s += (double)__fsqrt_rn(acc[u][v]);
+            }
+    } else {
+        for (int p = threadIdx.x; p < kLmTile * kLmTile; p += blockDim.x) {
+            int i = p / kLmTile, j = p % kLmTile;
+            int gi = bi * kLmTile + i, gj = bj * kLmTile + j;
+            if (gi >= gj || gj >= m) continue;
+            const float* ra = Xp + (int64_t)idx[t * m + gi] * dp;
+            const float* rb = Xp + (int64_t)idx[t * m + gj] * dp;
+            float d2 = 0.f;
+            for (int c = 0; c < dp / 4; ++c)
+                d2 = d2_acc4(d2, reinterpret_cast<const float4*>(ra)[c], reinterpret_cast<const float4*>(rb)[c]);
+            s += (double)__fsqrt_rn(d2);
+        }
     }
-    __shared__ double red[256];
-    red[threadIdx.x] = s;
+    // fixed-shape reduction (deterministic)
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    __shared__ double red[8];
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
     __syncthreads();
-    for (int w = blockDim.x / 2; w > 0; w >>= 1) {
-        if (threadIdx.x < w) red[threadIdx.x] += red[threadIdx.x + w];
-        __syncthreads();
+    if (threadIdx.x == 0) {
+        double t8 = 0.0;
+        for (int w = 0; w < 8; ++w) t8 += red[w];
+        partial[t * gridDim.x + blockIdx.x] = t8;
     }
-    if (threadIdx.x == 0) partial[t * gridDim.x + blockIdx.x] = red[0];
 }
 
-__global__ void k_landmark_pick(const double* __restrict__ partial, int nblk, int trials, const int32_t* __restrict__ idx,
-                                int m, const float* __restrict__ Xp, int dp, float* __restrict__ centers) {
+// Every block recomputes the winning trial (same fixed-order sums, so all
+// agree) and gathers its slice of the winning candidates' rows.
+__global__ void __launch_bounds__(512) k_landmark_pick(const double* __restrict__ partial, int nblk, int trials,
+                                                      const int32_t* __restrict__ idx, int m,
+                                                      const float* __restrict__ Xp, int dp,
+                                                      float* __restrict__ centers) {
     __shared__ double s_tr[64];
     __shared__ int best;
     // warp w sums trial w's partials: fixed lane strides + a fixed shuffle tree (deterministic)
@@ -144,8 +182,9 @@ __global__ void k_landmark_pick(const double* __restrict__ partial, int nblk, in
     }
     __syncthreads();
     const int32_t* w = idx + best * m;
-    for (int e = threadIdx.x; e < m * dp; e += blockDim.x) {
-        int c = e / dp, col = e - c * dp;
+    const int e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e < m * dp) {
+        const int c = e / dp, col = e - c * dp;
         centers[e] = Xp[(int64_t)w[c] * dp + col];
     }
 }
@@ -233,6 +272,25 @@ __global__ void __launch_bounds__(256) k_assign(const float* __restrict__ Xp, in
 // cost n*m*d per pass). nbr[c] = the kNbr nearest centers of c (itself first).
 constexpr int kNbr = 32;
 
+// ascending bitonic sort of one key per lane across the warp
+__device__ __forceinline__ key_t warp_sort32(key_t v, int lane) {
+#pragma unroll
+    for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            const key_t o = __shfl_xor_sync(0xffffffffu, v, j);
+            const bool up = (lane & k) == 0 || k == 32;
+            const bool lower = (lane & j) == 0;
+            v = (lower == up) ? (o < v ? o : v) : (o > v ? o : v);
+        }
+    }
+    return v;
+}
+
+// 32-NN graph of the centers, warp per center: a batch of 32 candidate keys
+// with many keys below the current 32nd (the first batches) is sorted
+// (bitonic) and merged with the sorted top-32 by a bitonic half-cleaner;
+// batches with few such keys insert them one by one.
 __global__ void __launch_bounds__(256) k_center_knn(const float* __restrict__ centers, int m, int dp,
                                                     int32_t* __restrict__ nbr) {
     const int lane = threadIdx.x & 31;
@@ -240,21 +298,34 @@ __global__ void __launch_bounds__(256) k_center_knn(const float* __restrict__ ce
     if (c >= m) return;
     const float* rc = centers + (int64_t)c * dp;
     const int L = min(kNbr, m);
-    key_t mine = (lane < 32 - L) ? kNegKey : kInfKey;
+    key_t mine = (lane < 32 - L) ? kNegKey : kInfKey;  // sorted ascending across lanes
     key_t kth = kInfKey;
     for (int base = 0; base < m; base += 32) {
         const int j = base + lane;
         key_t key = kInfKey;
         if (j < m) key = make_key(d2_rows(rc, centers + (int64_t)j * dp, dp), j);
         unsigned cm = __ballot_sync(0xffffffffu, key < kth);
-        while (cm) {
-            const int src = __ffs(cm) - 1;
-            const key_t kk = __shfl_sync(0xffffffffu, key, src);
-            mine = warp_insert(mine, kk, lane);
-            kth = __shfl_sync(0xffffffffu, mine, 31);
-            cm &= ~(1u << src);
-            cm &= __ballot_sync(0xffffffffu, key < kth);
+        if (__popc(cm) <= 6) {  // few accepted keys: serial insertion
+            while (cm) {
+                const int src = __ffs(cm) - 1;
+                const key_t kk = __shfl_sync(0xffffffffu, key, src);
+                mine = warp_insert(mine, kk, lane);
+                kth = __shfl_sync(0xffffffffu, mine, 31);
+                cm &= ~(1u << src);
+                cm &= __ballot_sync(0xffffffffu, key < kth);
+            }
+            continue;
         }
+        key = warp_sort32(key, lane);
+        const key_t r = __shfl_sync(0xffffffffu, key, 31 - lane);  // descending
+        key_t v = r < mine ? r : mine;                               // bitonic: the 32 smallest
+#pragma unroll
+        for (int jj = 16; jj > 0; jj >>= 1) {
+            const key_t o = __shfl_xor_sync(0xffffffffu, v, jj);
+            v = ((lane & jj) == 0) ? (o < v ? o : v) : (o > v ? o : v);
+        }
+        mine = v;
+        kth = __shfl_sync(0xffffffffu, mine, 31);
     }
     if (lane >= 32 - L) nbr[(int64_t)c * kNbr + lane - (32 - L)] = key_idx(mine);
     if (lane < kNbr - L) nbr[(int64_t)c * kNbr + L + lane] = c;  // pad short lists with self
@@ -698,7 +769,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         SKNN_CUDA(cudaFuncSetAttribute(k_landmark_sums, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lsm));
     k_landmark_sums<<<dim3(ntile, trials), 256, lsm, s>>>(Xp, dp, m0, lidx, nb, partial);
     cx.launched();
-    k_landmark_pick<<<1, 512, 0, s>>>(partial, ntile, trials, lidx, m0, Xp, dp, out.centers);
+    k_landmark_pick<<<(m0 * dp + 511) / 512, 512, 0, s>>>(partial, ntile, trials, lidx, m0, Xp, dp, out.centers);
     cx.launched();
 
     int32_t* cid;

@@ -187,42 +187,87 @@ __device__ __forceinline__ unsigned long long block_sum_u64(unsigned long long v
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
     if (lane == 0) s_red[w] = v;
     __syncthreads();
-    unsigned long long t = 0;
-    for (int i = 0; i < 32; ++i) t += s_red[i];
+    if (w == 0) {
+        unsigned long long t = lane < (int)(blockDim.x >> 5) ? s_red[lane] : 0ull;
+        for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+        if (lane == 0) s_red[32] = t;
+    }
+    __syncthreads();
+    const unsigned long long t = s_red[32];
     __syncthreads();
     return t;
 }
 
-// Level-2 task list (single CTA), load-balanced on the level-1 work estimate:
+// componentwise exclusive scan of an int4 over a 1024-thread block
+__device__ __forceinline__ int4 block_exscan4(int4 v, int4* s_warp, int4& total) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int4 x = v;
+    for (int o = 1; o < 32; o <<= 1) {
+        const int yx = __shfl_up_sync(0xffffffffu, x.x, o), yy = __shfl_up_sync(0xffffffffu, x.y, o);
+        const int yz = __shfl_up_sync(0xffffffffu, x.z, o), yw = __shfl_up_sync(0xffffffffu, x.w, o);
+        if (lane >= o) { x.x += yx; x.y += yy; x.z += yz; x.w += yw; }
+    }
+    if (lane == 31) s_warp[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        int4 t = s_warp[lane];
+        for (int o = 1; o < 32; o <<= 1) {
+            const int yx = __shfl_up_sync(0xffffffffu, t.x, o), yy = __shfl_up_sync(0xffffffffu, t.y, o);
+            const int yz = __shfl_up_sync(0xffffffffu, t.z, o), yw = __shfl_up_sync(0xffffffffu, t.w, o);
+            if (lane >= o) { t.x += yx; t.y += yy; t.z += yz; t.w += yw; }
+        }
+        s_warp[lane] = t;
+    }
+    __syncthreads();
+    const int4 base = w ? s_warp[w - 1] : make_int4(0, 0, 0, 0);
+    total = s_warp[31];
+    return make_int4(base.x + x.x - v.x, base.y + x.y - v.y, base.z + x.z - v.z, base.w + x.w - v.w);
+}
+
+// Level-2 task list (single CTA, each thread owns <= kTaskPer consecutive
+// clusters), load-balanced on the level-1 work estimate:
 //  * a tile (`tile` queries of one cluster) whose estimated work exceeds both
 //    total / resident warps (it alone would outlast the average warp) and 4x
 //    the mean tile (measured: splitting moderate tiles costs more than the
 //    balance gains) is SPLIT into S <= 32 tasks of about half the per-warp
-//    average that take every S-th candidate cluster (interleaved, so each task sees near and far
-//    clusters); the S tasks of a tile share the queries' k-th distance bound
-//    through `theta2` and their partial lists are merged by k_merge_split;
+//    average that take every S-th candidate cluster (interleaved, so each
+//    task sees near and far clusters); the S tasks of a tile share the
+//    queries' k-th distance bound through `theta2` and their partial lists
+//    are merged by k_merge_split;
 //  * order: split tasks first, then unsplit tiles heavier than W0 / 4, then
 //    the rest (longest work first, so no straggler starts last).
 // Split tasks are capped at `cap_split` (W0 doubles until they fit); their
 // part index equals their task index. split == false (warp-per-query scan)
 // keeps S = 1 and only orders.
+constexpr int kTaskPer = kMaxClusters / 1024;
 __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__ qoff, int mq, int tile,
                                                      int shard_rank, int shard_count,
                                                      const unsigned long long* __restrict__ work,
                                                      const int32_t* __restrict__ ccount, int slots, int cap_split,
-                                                     int split, int order, float wfac, float hfac, int4* __restrict__ tasks, int* __restrict__ ntasks,
+                                                     int split, int order, float wfac, float hfac,
+                                                     int4* __restrict__ tasks, int* __restrict__ ntasks,
                                                      int4* __restrict__ merges, int* __restrict__ nmerges) {
-    __shared__ int s_warp[32];
-    __shared__ unsigned long long s_red[32];
-    auto nt_of = [&](int c) -> int {
-        if (c >= mq) return 0;
-        if (shard_count > 1 && c % shard_count != shard_rank) return 0;
-        return (qoff[c + 1] - qoff[c] + tile - 1) / tile;
-    };
+    __shared__ unsigned long long s_red[33];
+    __shared__ int4 s_warp4[32];
+    const int per = (mq + 1023) / 1024;
+    const int c0 = threadIdx.x * per;
+    int nt[kTaskPer];
+    unsigned long long wk[kTaskPer];
+    int ncc[kTaskPer];
     unsigned long long tot = 0, ntl = 0;
-    for (int c = threadIdx.x; c < mq; c += 1024) {
-        tot += (unsigned long long)nt_of(c) * work[c];
-        ntl += (unsigned long long)nt_of(c);
+#pragma unroll
+    for (int u = 0; u < kTaskPer; ++u) {
+        const int c = c0 + u;
+        nt[u] = 0;
+        wk[u] = 0;
+        ncc[u] = 1;
+        if (u < per && c < mq && !(shard_count > 1 && c % shard_count != shard_rank)) {
+            nt[u] = (qoff[c + 1] - qoff[c] + tile - 1) / tile;
+            wk[u] = work[c];
+            ncc[u] = ccount[c] > 1 ? ccount[c] : 1;
+        }
+        tot += (unsigned long long)nt[u] * wk[u];
+        ntl += (unsigned long long)nt[u];
     }
     tot = block_sum_u64(tot, s_red);
     ntl = block_sum_u64(ntl, s_red);
@@ -234,56 +279,63 @@ __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__
     const unsigned long long H = (unsigned long long)fmax(per_slot, hfac * mean);
     unsigned long long W0 = (unsigned long long)(per_slot * wfac);
     if (W0 < 64) W0 = 64;
-    auto s_of = [&](int c, unsigned long long w0) -> int {
-        if (!split || c >= mq || work[c] <= H) return 1;
-        unsigned long long s = (work[c] + w0 - 1) / w0;
+    auto s_of = [&](int u, unsigned long long w0) -> int {
+        if (!split || nt[u] == 0 || wk[u] <= H) return 1;
+        unsigned long long s = (wk[u] + w0 - 1) / w0;
         s = s < 32 ? (s > 2 ? s : 2) : 32;
-        const unsigned long long nc = (unsigned long long)(ccount[c] > 1 ? ccount[c] : 1);
-        return (int)(s < nc ? s : nc);
+        return (int)(s < (unsigned long long)ncc[u] ? s : (unsigned long long)ncc[u]);
     };
-    for (int it = 0; it < 40; ++it) {
-        unsigned long long n = 0;
-        for (int c = threadIdx.x; c < mq; c += 1024) {
-            const int S = s_of(c, W0);
-            if (S > 1) n += (unsigned long long)nt_of(c) * S;
-        }
-        n = block_sum_u64(n, s_red);
-        if (n <= (unsigned long long)cap_split) break;
-        W0 *= 2;
-    }
-    int carry = 0, mcarry = 0;
-    for (int pass = 0; pass < 3; ++pass) {
-        if (!order && pass == 2) break;
-        for (int base = 0; base < mq; base += 1024) {
-            const int c = base + threadIdx.x;
-            const int nt = nt_of(c);
-            const int S = s_of(c, W0);
-            bool mine;
-            if (pass == 0) mine = S > 1;
-            else if (!order) mine = S == 1 && c < mq;
-            else if (pass == 1) mine = S == 1 && c < mq && work[c] * 4 >= W0;
-            else mine = S == 1 && c < mq && work[c] * 4 < W0;
-            const int n = mine ? nt * S : 0;
-            int total, mtotal;
-            const int start = carry + block_exscan(n, s_warp, total);
-            const int mstart = mcarry + block_exscan(pass == 0 && mine ? nt : 0, s_warp, mtotal);
-            if (mine) {
-                for (int t = 0; t < nt; ++t) {
-                    for (int sp = 0; sp < S; ++sp) {
-                        const int id = start + t * S + sp;
-                        tasks[id] = make_int4(c, t * tile, sp | (S << 8), S > 1 ? id : -1);
-                    }
-                    if (pass == 0) merges[mstart + t] = make_int4(c, t * tile, S, start + t * S);
-                }
+    if (split) {
+        for (int it = 0; it < 40; ++it) {
+            unsigned long long n = 0;
+#pragma unroll
+            for (int u = 0; u < kTaskPer; ++u) {
+                const int S = s_of(u, W0);
+                if (S > 1) n += (unsigned long long)nt[u] * S;
             }
-            carry += total;
-            mcarry += mtotal;
+            n = block_sum_u64(n, s_red);
+            if (n <= (unsigned long long)cap_split) break;
+            W0 *= 2;
+        }
+    }
+    // bucket sizes: x = split tasks, y = heavy unsplit tiles, z = the rest, w = merge entries
+    int4 cnt = make_int4(0, 0, 0, 0);
+#pragma unroll
+    for (int u = 0; u < kTaskPer; ++u) {
+        const int S = s_of(u, W0);
+        if (S > 1) { cnt.x += nt[u] * S; cnt.w += nt[u]; }
+        else if (!order || wk[u] * 4 >= W0) cnt.y += nt[u];
+        else cnt.z += nt[u];
+    }
+    int4 total;
+    int4 off = block_exscan4(cnt, s_warp4, total);
+    off.y += total.x;
+    off.z += total.x + total.y;
+#pragma unroll
+    for (int u = 0; u < kTaskPer; ++u) {
+        if (nt[u] == 0) continue;
+        const int c = c0 + u;
+        const int S = s_of(u, W0);
+        if (S > 1) {
+            for (int t = 0; t < nt[u]; ++t) {
+                for (int sp = 0; sp < S; ++sp) {
+                    const int id = off.x + t * S + sp;
+                    tasks[id] = make_int4(c, t * tile, sp | (S << 8), id);
+                }
+                merges[off.w + t] = make_int4(c, t * tile, S, off.x + t * S);
+            }
+            off.x += nt[u] * S;
+            off.w += nt[u];
+        } else {
+            int& o = (!order || wk[u] * 4 >= W0) ? off.y : off.z;
+            for (int t = 0; t < nt[u]; ++t) tasks[o + t] = make_int4(c, t * tile, 1 << 8, -1);
+            o += nt[u];
         }
     }
     if (threadIdx.x == 0) {
-        ntasks[0] = carry;
+        ntasks[0] = total.x + total.y + total.z;
         ntasks[1] = 0;
-        *nmerges = mcarry;
+        *nmerges = total.w;
     }
 }
 

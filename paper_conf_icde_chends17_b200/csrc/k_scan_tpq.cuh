@@ -157,6 +157,25 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
                 if (L >= lo) rowL = __ldg(reinterpret_cast<const float4*>(a.trows) + L);
                 if (R < hi) rowR = __ldg(reinterpret_cast<const float4*>(a.trows) + R);
             }
+            auto consider = [&](float d2, int jc) {
+                if (d2 <= kth_d2) {                                         // line 16 (distance part)
+                    const key_t key = make_key(d2, __ldg(a.torig + jc));
+                    if (key < kth) {
+                        if constexpr (SMEM) {
+                            kth = stop.insert_from(key, min(nfill, a.k - 1));
+                            ++nfill;
+                        } else {
+                            top.insert(key);
+                            kth = top.kth();
+                        }
+                        if (key_d2(kth) < kth_d2) {
+                            kth_d2 = key_d2(kth);
+                            theta = fminf(ub, __fsqrt_ru(kth_d2));          // line 17 (R8)
+                            if (SPLIT) atomicMin(th2, __float_as_uint(kth_d2));
+                        }
+                    }
+                }
+            };
             for (;;) {
                 const float bL = L >= lo ? dtL - dq : INF;       // -l on the left (dt > dq)
                 const float bR = R < hi ? dq - dtR : INF;        // l on the right (dt <= dq)
@@ -194,23 +213,7 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
                     d2 = d2q(a.trows + (int64_t)jc * a.dp);
                 }
                 ++evals;
-                if (d2 <= kth_d2) {                                         // line 16 (distance part)
-                    const key_t key = make_key(d2, __ldg(a.torig + jc));
-                    if (key < kth) {
-                        if constexpr (SMEM) {
-                            kth = stop.insert_from(key, min(nfill, a.k - 1));
-                            ++nfill;
-                        } else {
-                            top.insert(key);
-                            kth = top.kth();
-                        }
-                        if (key_d2(kth) < kth_d2) {
-                            kth_d2 = key_d2(kth);
-                            theta = fminf(ub, __fsqrt_ru(kth_d2));          // line 17 (R8)
-                            if (SPLIT) atomicMin(th2, __float_as_uint(kth_d2));
-                        }
-                    }
-                }
+                consider(d2, jc);
             }
         }
         if (SPLIT) {  // partial list of this task -> k_merge_split
