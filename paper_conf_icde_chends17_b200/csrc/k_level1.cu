@@ -56,11 +56,45 @@ __device__ void block_sort_u64(u64* s, int S) {
     }
 }
 
+constexpr int kSmallSel = 64;  // a radix bin this small finishes with a warp rank-select
+
+// k-th smallest (1-based) of n <= kSmallSel floats in shared memory, by one
+// warp: the value whose stable rank is k-1 (exact, no rounding involved).
+__device__ __forceinline__ float warp_rank_select(const float* v, int n, int k) {
+    const int lane = threadIdx.x & 31;
+    float ans = 0.f;
+    bool found = false;
+    for (int i = lane; i < n; i += 32) {
+        const float x = v[i];
+        int r = 0;
+        for (int j = 0; j < n; ++j) {
+            const float y = v[j];
+            r += (y < x || (y == x && j < i)) ? 1 : 0;
+        }
+        if (r == k - 1) { ans = x; found = true; }
+    }
+    const unsigned m = __ballot_sync(0xffffffffu, found);
+    return __shfl_sync(0xffffffffu, ans, __ffs(m) - 1);
+}
+
 // k-th smallest (1-based) of n non-negative floats in shared memory: MSB-first
-// radix select on the IEEE bits (monotone for x >= 0), 8 bits per round.
-// Returns +inf when n < k. All threads of the block must call it.
-__device__ float block_kth_smallest(const float* vals, int n, int k, int* s_hist, int* s_sel) {
+// radix select on the IEEE bits (monotone for x >= 0), 8 bits per round;
+// once the bin that holds rank k has at most kSmallSel values they are
+// compacted into `small` and warp 0 finishes with a rank-select. Returns +inf
+// when n < k. All threads of the block must call it.
+__device__ float block_kth_smallest(const float* vals, int n, int k, int* s_hist, int* s_sel, float* small) {
     if (n < k) return __int_as_float(0x7f800000);
+    if (n <= kSmallSel) {
+        float r = 0.f;
+        if (threadIdx.x < 32) {
+            r = warp_rank_select(vals, n, k);
+            if (threadIdx.x == 0) small[kSmallSel] = r;
+        }
+        __syncthreads();
+        r = small[kSmallSel];
+        __syncthreads();
+        return r;
+    }
     uint32_t prefix = 0;
     int kk = k;
     for (int shift = 24; shift >= 0; shift -= 8) {
@@ -83,22 +117,58 @@ __device__ float block_kth_smallest(const float* vals, int n, int k, int* s_hist
             }
             const int excl = incl - tot;
             if (excl < kk && kk <= incl) {
-                int run = excl, bin = threadIdx.x * 8;
+                int run = excl, bin = threadIdx.x * 8, cnt = c[0];
 #pragma unroll
                 for (int j = 0; j < 8; ++j) {
-                    if (run + c[j] >= kk) { bin = threadIdx.x * 8 + j; break; }
+                    if (run + c[j] >= kk) { bin = threadIdx.x * 8 + j; cnt = c[j]; break; }
                     run += c[j];
                 }
                 s_sel[0] = bin;
                 s_sel[1] = kk - run;
+                s_sel[2] = cnt;
+                s_sel[3] = 0;
             }
         }
         __syncthreads();
         prefix |= uint32_t(s_sel[0]) << shift;
         kk = s_sel[1];
+        const int cnt = s_sel[2];
+        if (shift > 0 && cnt <= kSmallSel) {
+            const uint32_t m2 = 0xffffffffu << shift;
+            __syncthreads();
+            for (int i = threadIdx.x; i < n; i += blockDim.x) {
+                const float x = vals[i];
+                if ((__float_as_uint(x) & m2) == prefix) small[atomicAdd(&s_sel[3], 1)] = x;
+            }
+            __syncthreads();
+            float r = 0.f;
+            if (threadIdx.x < 32) {
+                r = warp_rank_select(small, cnt, kk);
+                if (threadIdx.x == 0) small[kSmallSel] = r;
+            }
+            __syncthreads();
+            r = small[kSmallSel];
+            __syncthreads();
+            return r;
+        }
         __syncthreads();
     }
     return __uint_as_float(prefix);
+}
+
+// ascending bitonic sort of one key per lane across the warp
+__device__ __forceinline__ u64 warp_sort_u64(u64 v, int lane) {
+#pragma unroll
+    for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            const u64 o = __shfl_xor_sync(0xffffffffu, v, j);
+            const bool up = (lane & k) == 0 || k == 32;
+            const bool lower = (lane & j) == 0;
+            v = (lower == up) ? (o < v ? o : v) : (o > v ? o : v);
+        }
+    }
+    return v;
 }
 
 __global__ void __launch_bounds__(kL1Threads) k_level1(
@@ -118,7 +188,8 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     float* s_qc = s_v + max(mt4, kL1Vals);                                    // [dp], float4-aligned
     __shared__ int s_cnt;
     __shared__ int s_hist[256];
-    __shared__ int s_sel[2];
+    __shared__ int s_sel[4];
+    __shared__ float s_small[kSmallSel + 1];
 
     const int qc = blockIdx.x;
     const int qsize = qoff[qc + 1] - qoff[qc];
@@ -141,7 +212,7 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
         s_v[tc] = (lo == hi) ? INF : D + __ldg(tdist + hi - 1);
     }
     __syncthreads();
-    const float Mk = block_kth_smallest(s_v, mt, k, s_hist, s_sel);
+    const float Mk = block_kth_smallest(s_v, mt, k, s_hist, s_sel, s_small);
     // gather every bound <= M_k of the clusters with v0 <= M_k
     for (int tc = threadIdx.x; tc < mt; tc += blockDim.x) {
         if (!(s_v[tc] <= Mk)) continue;
@@ -169,7 +240,7 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     // stage the gathered values as floats (alias-free copy into s_v)
     for (int i = threadIdx.x; i < min(nv, kL1Vals); i += blockDim.x) s_v[i] = __uint_as_float(uint32_t(s_keys[i]));
     __syncthreads();
-    float Vk = (nv <= kL1Vals) ? block_kth_smallest(s_v, nv, k, s_hist, s_sel) : Mk;  // overflow: M_k is a valid bound
+    float Vk = (nv <= kL1Vals) ? block_kth_smallest(s_v, nv, k, s_hist, s_sel, s_small) : Mk;  // overflow: M_k is a valid bound
     if (!(Vk <= Mk)) Vk = Mk;
     // UB = r_q + V_k, inflated to cover the rounding of the three summed distances (R7)
     const float UB = __fmul_ru(rq + Vk, 1.f + 2.f * eta);
@@ -201,11 +272,20 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     }
     __syncthreads();
     const int nc = s_cnt;
-    int S = 1;
-    while (S < nc) S <<= 1;
-    for (int i = nc + threadIdx.x; i < S; i += blockDim.x) s_keys[i] = ~0ull;
-    __syncthreads();
-    block_sort_u64(s_keys, S);
+    if (nc <= 32) {  // one warp sorts in registers (the common case)
+        if (threadIdx.x < 32) {
+            u64 v = (int)threadIdx.x < nc ? s_keys[threadIdx.x] : ~0ull;
+            v = warp_sort_u64(v, threadIdx.x);
+            if ((int)threadIdx.x < nc) s_keys[threadIdx.x] = v;
+        }
+        __syncthreads();
+    } else {
+        int S = 1;
+        while (S < nc) S <<= 1;
+        for (int i = nc + threadIdx.x; i < S; i += blockDim.x) s_keys[i] = ~0ull;
+        __syncthreads();
+        block_sort_u64(s_keys, S);
+    }
     // elastic switch (S8): split the sorted candidates into the sparse list
     // (point-level scan, Alg. 2) and the dense-tile list (tensor cores),
     // stable in ascending D. auto: a pair is dense when a typical query's
