@@ -238,6 +238,29 @@ def test_c2_full_size_sampled(sknn):
     assert st["pruned_pct"] > 99.0
 
 
+@pytest.mark.slow
+@pytest.mark.parametrize("name,nsample", [("C3", 3000), ("C3int", 3000), ("C4", 400), ("C5", 400)])
+def test_full_size_sampled(sknn, name, nsample):
+    """C3 / C4 / C5 at BASELINE.json's full sizes in the launch configuration
+    `bench.py --config` times (auto path: elastic switch, dense tiles, split
+    tasks); the oracle checks a seeded sample of query rows one by one.
+    Integer-valued workloads bit-exact, real-valued within 1e-5 (c.2)."""
+    Q, T, k, sj = datagen.workload(name)
+    idx, dist, st = run(sknn, Q, T, k, sj)
+    rng = np.random.default_rng(7)
+    s = np.sort(rng.choice(Q.shape[0], nsample, replace=False))
+    ridx, rdist = oracle.knn_join(Q[s], T, k)
+    if name == "C3":
+        assert_knn_tolerant(Q[s], T, idx[s], dist[s], rdist)
+    else:
+        assert_knn_bitexact(idx[s], dist[s], ridx, rdist)
+    # every row is a sorted, duplicate-free list of in-range indices
+    assert np.all(np.diff(dist, axis=1) >= 0)
+    assert np.all((idx >= 0) & (idx < T.shape[0]))
+    nq, nt = Q.shape[0], T.shape[0]
+    assert nq * k <= st["dist_evals"] <= nq * nt
+
+
 # ------------------------------------------------------------ dense tiles --
 @pytest.mark.parametrize("name,scale", [("C1", 1.0), ("C3int", 0.05), ("C4", 0.004), ("C5", 0.0025)])
 @pytest.mark.parametrize("mapping", ["thread", "warp"])
