@@ -124,6 +124,7 @@ typedef struct {
     int32_t mq, mt;                /* cluster counts used                                             */
     int32_t kernel_launches;       /* kernels this call launched                                      */
     int32_t pad0;
+    uint64_t topk_inserts;         /* kNearests updates by the level-2 scan (P:L453 update overhead)   */
 } sknn_stats;
 
 /* Opaque resident target index (sknn_build / sknn_query). Owns device memory:

@@ -20,25 +20,73 @@
 
 namespace sknn {
 
-// kNearests in shared memory (Fig. 8: k*4 <= th1 = smem/SM / threads/SM,
-// P:L629), laid out like the paper's Layout 2 (Fig. 6b): slot r of
-// thread t at [r][t], so a warp's accesses to one slot are contiguous. Sorted
-// ascending; an insertion shifts only the slots above the insertion point.
-template <int STRIDE>
-struct SmemTopK {
+// kNearests of one query (Alg. 2 line 4), three placements (Fig. 8,
+// P:L587-609, re-derived for B200 in DESIGN.md):
+//  LIST_REG    sorted keys in registers (k*4 B <= th2); branch-free insertion
+//  LIST_SORTED sorted keys in shared memory (k*4 B <= th1 = 114 B), laid out
+//              like the paper's Layout 2 (Fig. 6b): slot r of thread t
+//              at [r][t], so a warp's accesses to one slot are contiguous; an
+//              insertion shifts only the slots above the insertion point
+//  LIST_HEAP   max-heap in shared memory, same layout: the root is the k-th
+//              key, an insertion is one sift-down (log2 k levels instead of
+//              up to k shifts); heap-sorted once at the end
+// All three keep the k smallest (d2, index) keys seen; insert() requires
+// key < kth() and returns the new k-th key.
+enum { LIST_REG = 0, LIST_SORTED = 1, LIST_HEAP = 2 };
+
+template <int LIST, int KMAX, int STRIDE>
+struct TopList;
+
+template <int KMAX, int STRIDE>
+struct TopList<LIST_REG, KMAX, STRIDE> {
+    RegTopK<KMAX> r;
+    int k;
+    __device__ __forceinline__ void init(key_t*, int k_) {
+        k = k_;
+        r.init(k_);
+    }
+    __device__ __forceinline__ key_t kth() const { return r.kth(); }
+    __device__ __forceinline__ void load_sorted(const key_t* src) {
+#pragma unroll
+        for (int s = 0; s < KMAX; ++s) {
+            const int i = s - (KMAX - k);
+            if (i >= 0) r.a[s] = src[i];
+        }
+    }
+    __device__ __forceinline__ key_t insert(key_t key) {
+        r.insert(key);
+        return r.kth();
+    }
+    __device__ __forceinline__ void finalize() {}
+    template <class F>
+    __device__ __forceinline__ void emit(F f) const {
+#pragma unroll
+        for (int s = 0; s < KMAX; ++s) {
+            const int i = s - (KMAX - k);
+            if (i >= 0) f(i, r.a[s]);
+        }
+    }
+};
+
+template <int KMAX, int STRIDE>
+struct TopList<LIST_SORTED, KMAX, STRIDE> {
     key_t* s;
     int k;
+    int nfill;  // slots >= nfill still hold +inf keys: the shift starts at min(nfill, k - 1)
     __device__ __forceinline__ void init(key_t* col, int k_) {
         s = col;
         k = k_;
+        nfill = 0;
         for (int r = 0; r < k; ++r) s[r * STRIDE] = kInfKey;
     }
-    __device__ __forceinline__ key_t get(int r) const { return s[r * STRIDE]; }
-    __device__ __forceinline__ void set(int r, key_t v) { s[r * STRIDE] = v; }
-    // precondition: key < current k-th; returns the new k-th
-    __device__ __forceinline__ key_t insert(key_t key) { return insert_from(key, k - 1); }
-    // slots >= n are still +inf: start the shift at min(n, k - 1)
-    __device__ __forceinline__ key_t insert_from(key_t key, int i) {
+    __device__ __forceinline__ key_t kth() const { return s[(k - 1) * STRIDE]; }
+    __device__ __forceinline__ void load_sorted(const key_t* src) {
+        for (int r = 0; r < k; ++r) s[r * STRIDE] = src[r];
+        nfill = k;
+    }
+    __device__ __forceinline__ key_t insert(key_t key) {
+        int i = min(nfill, k - 1);
+        ++nfill;
         while (i > 0) {
             const key_t v = s[(i - 1) * STRIDE];
             if (!(key < v)) break;
@@ -48,12 +96,71 @@ struct SmemTopK {
         s[i * STRIDE] = key;
         return s[(k - 1) * STRIDE];
     }
+    __device__ __forceinline__ void finalize() {}
+    template <class F>
+    __device__ __forceinline__ void emit(F f) const {
+        for (int r = 0; r < k; ++r) f(r, s[r * STRIDE]);
+    }
+};
+
+template <int KMAX, int STRIDE>
+struct TopList<LIST_HEAP, KMAX, STRIDE> {
+    key_t* s;
+    int k;
+    __device__ __forceinline__ void init(key_t* col, int k_) {
+        s = col;
+        k = k_;
+        for (int r = 0; r < k; ++r) s[r * STRIDE] = kInfKey;
+    }
+    __device__ __forceinline__ key_t kth() const { return s[0]; }
+    // an ascending list read backwards is a max-heap
+    __device__ __forceinline__ void load_sorted(const key_t* src) {
+        for (int r = 0; r < k; ++r) s[r * STRIDE] = src[k - 1 - r];
+    }
+    // place `key` at the root of the heap s[0, n) and sift it down
+    __device__ __forceinline__ void sift(key_t key, int n) {
+        int i = 0;
+        for (;;) {
+            const int l = 2 * i + 1;
+            if (l >= n) break;
+            key_t c = s[l * STRIDE];
+            int ci = l;
+            if (l + 1 < n) {
+                const key_t c2 = s[(l + 1) * STRIDE];
+                if (c < c2) {
+                    c = c2;
+                    ci = l + 1;
+                }
+            }
+            if (!(key < c)) break;
+            s[i * STRIDE] = c;
+            i = ci;
+        }
+        s[i * STRIDE] = key;
+    }
+    __device__ __forceinline__ key_t insert(key_t key) {
+        sift(key, k);  // the old root (the k-th key) is dropped
+        return s[0];
+    }
+    // in-place heapsort: ascending order in s[0, k)
+    __device__ __forceinline__ void finalize() {
+        for (int end = k - 1; end > 0; --end) {
+            const key_t top = s[0];
+            const key_t last = s[end * STRIDE];
+            s[end * STRIDE] = top;
+            sift(last, end);
+        }
+    }
+    template <class F>
+    __device__ __forceinline__ void emit(F f) const {
+        for (int r = 0; r < k; ++r) f(r, s[r * STRIDE]);
+    }
 };
 
 // One warp tile of the thread-per-query scan (Alg. 2 for 32 queries).
-template <int DP, int KMAX, bool SMEM, int THREADS, bool SPLIT>
+template <int DP, int KMAX, int LIST, int THREADS, bool SPLIT>
 __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t* s_topk, unsigned long long& evals,
-                                         unsigned long long& cevals) {
+                                         unsigned long long& cevals, unsigned long long& ins) {
     const float INF = __int_as_float(0x7f800000);
     const int lane = threadIdx.x & 31;
     const int qc = tl.x;
@@ -76,37 +183,18 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
         if constexpr (DP > 0) return d2_reg<DP>(q, t);
         else return d2_rows(qrow, t, a.dp);
     };
-    RegTopK<SMEM ? 1 : KMAX> top;
-    SmemTopK<THREADS> stop;
-    key_t kth;
-    if constexpr (SMEM) {
-        stop.init(s_topk + threadIdx.x, a.k);
-        kth = kInfKey;
-    } else {
-        top.init(a.k);
-        kth = top.kth();
-    }
+    TopList<LIST, KMAX, THREADS> top;
+    top.init(s_topk + threadIdx.x, a.k);
+    key_t kth = top.kth();
     const float ub = a.ub[qc];
     float theta = ub;
-    // slots >= nfill still hold +inf keys (the shift starts at nfill); no
-    // member beyond UB can enter the list (UB bounds every query's k-th
+    // no member beyond UB can enter the list (UB bounds every query's k-th
     // distance, R7), so inserts are gated by ub^2 until the list is full
-    int nfill = 0;
     float kth_d2 = __fmul_ru(ub, ub);
     if (a.init_topk && a.dcount[qc] > 0) {  // continue from the dense-tile pass
         if (split == 0) {  // (the other tasks of a split tile only take its bound)
-            if constexpr (SMEM) {
-                for (int r = 0; r < a.k; ++r) stop.set(r, a.init_topk[(int64_t)qpos * a.k + r]);
-                kth = stop.get(a.k - 1);
-            } else {
-#pragma unroll
-                for (int s = 0; s < KMAX; ++s) {
-                    const int r = s - (KMAX - a.k);
-                    if (r >= 0) top.a[s] = a.init_topk[(int64_t)qpos * a.k + r];
-                }
-                kth = top.kth();
-            }
-            nfill = a.k;
+            top.load_sorted(a.init_topk + (int64_t)qpos * a.k);
+            kth = top.kth();
             kth_d2 = fminf(kth_d2, key_d2(kth));
         } else {
             kth_d2 = fminf(kth_d2, key_d2(a.init_topk[(int64_t)qpos * a.k + a.k - 1]));
@@ -161,13 +249,8 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
                 if (d2 <= kth_d2) {                                         // line 16 (distance part)
                     const key_t key = make_key(d2, __ldg(a.torig + jc));
                     if (key < kth) {
-                        if constexpr (SMEM) {
-                            kth = stop.insert_from(key, min(nfill, a.k - 1));
-                            ++nfill;
-                        } else {
-                            top.insert(key);
-                            kth = top.kth();
-                        }
+                        ++ins;
+                        kth = top.insert(key);
                         if (key_d2(kth) < kth_d2) {
                             kth_d2 = key_d2(kth);
                             theta = fminf(ub, __fsqrt_ru(kth_d2));          // line 17 (R8)
@@ -218,103 +301,312 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
         }
         if (SPLIT) {  // partial list of this task -> k_merge_split
             key_t* pl = a.part + (int64_t)tl.w * a.k * 32 + lane;
-            if constexpr (SMEM) {
-                for (int r = 0; r < a.k; ++r) pl[r * 32] = stop.get(r);
-            } else {
+            top.finalize();
+            top.emit([&](int r, key_t v) { pl[r * 32] = v; });
+        } else {
+            const int qo = __ldg(a.qorig + qpos);
+            top.finalize();
+            top.emit([&](int r, key_t v) { write_result(a, qo, r, v); });
+        }
+    }
+}
+
+// Members evaluated per block of the warp-union walk (rows held in registers
+// while their distances are computed): ~32 floats of row data per block.
+template <int DP>
+constexpr int union_block() {
+    return DP == 0 ? 1 : (DP <= 4 ? 8 : (DP <= 8 ? 4 : (DP <= 16 ? 2 : 1)));
+}
+
+// One warp tile of the thread-per-query scan with a WARP-UNION member walk
+// (the regularity side of Sweet KNN's reconciliation, §IV, on B200): for a
+// candidate cluster the 32 lanes walk the union of their Alg. 2 windows
+// together, every lane computing the distance of the same member, so each row
+// is one broadcast load for the whole warp and the loop has no per-lane
+// control flow except the kNearests insert. The walk starts at the split
+// point of a middle lane's dq and grows both sides in blocks of
+// union_block<DP>() members; a side stops when no lane's window (Alg. 2
+// lines 10-13 with its own running theta) reaches its next member. Lanes
+// evaluate members outside their own window (harmless: every evaluated
+// distance is a real (query, target) distance and the list keeps the k
+// smallest keys), so every member of every lane's window is evaluated
+// (monotone break tests, DESIGN.md §2 exactness argument).
+template <int DP, int KMAX, int LIST, int THREADS, bool SPLIT>
+__device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key_t* s_topk, unsigned long long& evals,
+                                           unsigned long long& cevals, unsigned long long& ins) {
+    constexpr unsigned FULL = 0xffffffffu;
+    const int lane = threadIdx.x & 31;
+    const int qc = tl.x;
+    const int qlo = a.qoff[qc], qsz = a.qoff[qc + 1] - qlo;
+    const int i = tl.y + lane;
+    const bool active = i < qsz;
+    const int qpos = qlo + (active ? i : 0);  // an idle lane shadows the tile's first query
+    const int split = SPLIT ? (tl.z & 0xff) : 0;
+    const int nsplit = SPLIT ? (tl.z >> 8) : 1;
+    constexpr int QV = DP > 0 ? DP / 4 : 1;
+    constexpr int U = union_block<DP>();
+    float4 q[QV];
+    const float* qrow = a.qrows + (int64_t)qpos * a.dp;
+    if constexpr (DP > 0) {
 #pragma unroll
-                for (int s = 0; s < KMAX; ++s) {
-                    const int r = s - (KMAX - a.k);
-                    if (r >= 0) pl[r * 32] = top.a[s];
+        for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(qrow) + c);
+    }
+    auto d2q = [&](const float* t) -> float {
+        if constexpr (DP > 0) return d2_reg<DP>(q, t);
+        else return d2_rows(qrow, t, a.dp);
+    };
+    TopList<LIST, KMAX, THREADS> top;
+    top.init(s_topk + threadIdx.x, a.k);
+    key_t kth = top.kth();
+    const float ub = a.ub[qc];
+    float theta = ub;
+    float kth_d2 = __fmul_ru(ub, ub);
+    if (a.init_topk && a.dcount[qc] > 0) {  // continue from the dense-tile pass
+        if (split == 0) {
+            top.load_sorted(a.init_topk + (int64_t)qpos * a.k);
+            kth = top.kth();
+            kth_d2 = fminf(kth_d2, key_d2(kth));
+        } else {
+            kth_d2 = fminf(kth_d2, key_d2(a.init_topk[(int64_t)qpos * a.k + a.k - 1]));
+        }
+        theta = fminf(ub, __fsqrt_ru(kth_d2));
+    }
+    const int ncand = a.cand_count[qc];
+    const int32_t* cl = a.cand + (int64_t)qc * a.mt;
+    const float* cD = a.cand_D + (int64_t)qc * a.mt;
+    const float rown = __ldg(a.qdist + qpos);  // d(q, c_q)
+    unsigned* th2 = a.theta2 + qpos;
+    const float4* trow4 = reinterpret_cast<const float4*>(a.trows);
+    bool dirty = false;
+    auto consider = [&](float d2, int jc) {
+        if (d2 <= kth_d2) {                                          // Alg. 2 line 16 (distance part)
+            const key_t key = make_key(d2, __ldg(a.torig + jc));
+            if (key < kth) {
+                ++ins;
+                kth = top.insert(key);
+                if (key_d2(kth) < kth_d2) {
+                    kth_d2 = key_d2(kth);
+                    dirty = true;  // theta follows once per block
+                }
+            }
+        }
+    };
+    // line 17 (R8): theta = min(UB, sqrt(k-th d2) rounded up), refreshed once
+    // per block of members (a stale, larger theta only evaluates more)
+    auto refresh = [&]() {
+        if (dirty) {
+            dirty = false;
+            theta = fminf(ub, __fsqrt_ru(kth_d2));
+            if (SPLIT && active) atomicMin(th2, __float_as_uint(kth_d2));
+        }
+    };
+    // distances of members j0, j0 + step, ... (n of them, n <= U): all row
+    // loads first (one broadcast transaction each), then the fixed-order sums
+    auto eval_block = [&](int j0, int step, int n) {
+        if constexpr (DP > 0) {
+            float4 r[U][DP / 4];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int j = j0 + step * min(u, n - 1);
+#pragma unroll
+                for (int c = 0; c < DP / 4; ++c) r[u][c] = __ldg(trow4 + (int64_t)j * (DP / 4) + c);
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                if (u < n) {
+                    float s = 0.f;
+#pragma unroll
+                    for (int c = 0; c < DP / 4; ++c) s = d2_acc4(s, q[c], r[u][c]);
+                    consider(s, j0 + step * u);
                 }
             }
         } else {
-            const int qo = __ldg(a.qorig + qpos);
-            if constexpr (SMEM) {
-                for (int r = 0; r < a.k; ++r) write_result(a, qo, r, stop.get(r));
-            } else {
-#pragma unroll
-                for (int s = 0; s < KMAX; ++s) {
-                    const int r = s - (KMAX - a.k);
-                    if (r >= 0) write_result(a, qo, r, top.a[s]);
-                }
+            for (int u = 0; u < n; ++u) consider(d2_rows(qrow, a.trows + (int64_t)(j0 + step * u) * a.dp, a.dp),
+                                                 j0 + step * u);
+        }
+    };
+    for (int c = split; c < ncand; c += nsplit) {  // warp-uniform: the tile's lanes share qc
+        if (SPLIT) {  // the bound the tile's other tasks have reached
+            const float g = __uint_as_float(*(volatile unsigned*)th2);
+            if (g < kth_d2) {
+                kth_d2 = g;
+                theta = fminf(ub, __fsqrt_ru(g));
             }
+        }
+        const int tc = __ldg(cl + c);
+        // per-query 2-landmark bound (Eq. 3 with the query in place of the
+        // query cluster's farthest member): D - d(q,c_q) - r_t <= d(q,t)
+        const float D = __ldg(cD + c), rt = __ldg(a.trad + tc);
+        bool ok = active && ti_keep(D - rown - rt, theta, D + rown + rt, a.eta);
+        if (!__any_sync(FULL, ok)) continue;
+        const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
+        const float dq = __fsqrt_rn(d2q(a.tcent + (int64_t)tc * a.dp));  // Alg. 2 line 6
+        cevals += active;
+        // empty window: every member distance lies in [dt_min, r_t]
+        const float dtmin = __ldg(a.tdist + hi - 1);
+        ok = ok && ti_keep(dq - rt, theta, dq + rt, a.eta) && ti_keep(dtmin - dq, theta, dq + dtmin, a.eta);
+        const unsigned okm = __ballot_sync(FULL, ok);
+        if (!okm) continue;
+        // split point at the dq of the lane midway between the first and last
+        // lane with a window (any split point is correct; lanes of a tile are
+        // in member-distance order, so this is near their median)
+        const int mid = ((__ffs(okm) - 1) + (31 - __clz(okm))) >> 1;
+        const float dsplit = __shfl_sync(FULL, dq, mid);
+        const int p = window_start_geq(a.tdist, lo, hi, dsplit);  // first member with dt <= dsplit
+        int R = p, L = p - 1;
+        // right side (dt <= dsplit, l = dq - dt growing): lane needs member R
+        // unless Alg. 2 breaks there (line 10); left side (dt > dsplit): lane
+        // needs member L unless it is in the `continue` region (line 12)
+        bool aliveR = R < hi && __any_sync(FULL, ok && ti_keep(dq - __ldg(a.tdist + R), theta,
+                                                                dq + __ldg(a.tdist + R), a.eta));
+        bool aliveL = L >= lo && __any_sync(FULL, ok && ti_keep(__ldg(a.tdist + L) - dq, theta,
+                                                                 dq + __ldg(a.tdist + L), a.eta));
+        unsigned walked = 0;
+        while (aliveR || aliveL) {
+            if (aliveR) {
+                const int n = min(U, hi - R);
+                eval_block(R, 1, n);
+                refresh();
+                R += n;
+                walked += n;
+                float dtn = 0.f;
+                if (R < hi) dtn = __ldg(a.tdist + R);
+                aliveR = R < hi && __any_sync(FULL, ok && ti_keep(dq - dtn, theta, dq + dtn, a.eta));
+            }
+            if (aliveL) {
+                const int n = min(U, L - lo + 1);
+                eval_block(L, -1, n);
+                refresh();
+                L -= n;
+                walked += n;
+                float dtn = 0.f;
+                if (L >= lo) dtn = __ldg(a.tdist + L);
+                aliveL = L >= lo && __any_sync(FULL, ok && ti_keep(dtn - dq, theta, dq + dtn, a.eta));
+            }
+        }
+        if (active) evals += walked;
+    }
+    if (active) {
+        if (SPLIT) {  // partial list of this task -> k_merge_split
+            key_t* pl = a.part + (int64_t)tl.w * a.k * 32 + lane;
+            top.finalize();
+            top.emit([&](int r, key_t v) { pl[r * 32] = v; });
+        } else {
+            const int qo = __ldg(a.qorig + qpos);
+            top.finalize();
+            top.emit([&](int r, key_t v) { write_result(a, qo, r, v); });
         }
     }
 }
 
 // DP == 0: runtime dp (> 32), the query row is re-read from L1/L2 (large k only)
-// register caps (measured): DP == 4 with the shared-memory list at 64 (4 CTAs
+// register caps (measured): DP == 4 with a shared-memory list at 64 (4 CTAs
 // / SM; C2 0.62 vs 0.68 ms at the compiler's 80), register lists at 128
 // (2 CTAs / SM; the two inlined task bodies otherwise take ~190)
-template <int DP, bool SMEM, int THREADS>
+template <int DP, int LIST, int THREADS>
 constexpr int tpq_min_blocks() {
-    return THREADS != 256 ? 1 : (!SMEM ? 2 : (DP == 4 ? 4 : 1));
+    return THREADS != 256 ? 1 : (LIST == LIST_REG ? 2 : (DP == 4 ? 4 : 1));
 }
-template <int DP, int KMAX, bool SMEM, int THREADS>
-__global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, SMEM, THREADS>())) k_scan_tpq(ScanArgs a) {
-    extern __shared__ __align__(16) key_t s_topk[];  // [k][256] when SMEM
+template <int DP, int KMAX, int LIST, int THREADS, bool UNI>
+__global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, LIST, THREADS>())) k_scan_tpq(ScanArgs a) {
+    extern __shared__ __align__(16) key_t s_topk[];  // [k][THREADS] for the shared-memory lists
     const int lane = threadIdx.x & 31;
     const int ntiles = *a.ntiles;
-    unsigned long long evals = 0, cevals = 0;
+    unsigned long long evals = 0, cevals = 0, ins = 0;
     for (;;) {
         int tile = 0;
         if (lane == 0) tile = atomicAdd(a.tile_counter, 1);
         tile = __shfl_sync(0xffffffffu, tile, 0);
         if (tile >= ntiles) break;
         const int4 tl = a.tiles[tile];
-        if ((tl.z >> 8) > 1) tpq_tile<DP, KMAX, SMEM, THREADS, true>(a, tl, s_topk, evals, cevals);
-        else tpq_tile<DP, KMAX, SMEM, THREADS, false>(a, tl, s_topk, evals, cevals);
+        if constexpr (UNI) {
+            if ((tl.z >> 8) > 1) union_tile<DP, KMAX, LIST, THREADS, true>(a, tl, s_topk, evals, cevals, ins);
+            else union_tile<DP, KMAX, LIST, THREADS, false>(a, tl, s_topk, evals, cevals, ins);
+        } else {
+            if ((tl.z >> 8) > 1) tpq_tile<DP, KMAX, LIST, THREADS, true>(a, tl, s_topk, evals, cevals, ins);
+            else tpq_tile<DP, KMAX, LIST, THREADS, false>(a, tl, s_topk, evals, cevals, ins);
+        }
     }
     add_counter(&a.counters->evals_sparse, evals);
     add_counter(&a.counters->center_evals, cevals);
+    add_counter(&a.counters->topk_inserts, ins);
 }
 
-template <int DP, int KMAX, bool SMEM, int THREADS>
-static void launch_tpq(Ctx& cx, const ScanArgs& a) {
-    const size_t smem = SMEM ? sizeof(key_t) * (size_t)a.k * THREADS : 0;
-    if (smem > 48 * 1024)
-        cudaFuncSetAttribute(k_scan_tpq<DP, KMAX, SMEM, THREADS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    int grid = occupancy_grid(cx, (const void*)k_scan_tpq<DP, KMAX, SMEM, THREADS>, THREADS, smem);
+template <int DP, int KMAX, int LIST, int THREADS, bool UNI>
+static void launch_tpq_walk(Ctx& cx, const ScanArgs& a) {
+    const size_t smem = LIST != LIST_REG ? sizeof(key_t) * (size_t)a.k * THREADS : 0;
+    auto fn = k_scan_tpq<DP, KMAX, LIST, THREADS, UNI>;
+    if (smem > 48 * 1024) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int grid = occupancy_grid(cx, (const void*)fn, THREADS, smem);
     if (a.probe_warps) {  // dry run: report resident warps for the task planner
         *a.probe_warps = grid * (THREADS / 32);
         return;
     }
-    k_scan_tpq<DP, KMAX, SMEM, THREADS><<<grid, THREADS, smem, cx.stream>>>(a);
+    fn<<<grid, THREADS, smem, cx.stream>>>(a);
 }
 
-
+// member walk: warp-union (default) or per-lane LB-ordered (SKNN_WALK=lane)
+template <int DP, int KMAX, int LIST, int THREADS>
+static void launch_tpq(Ctx& cx, const ScanArgs& a) {
+    const char* w = getenv("SKNN_WALK");
+    if (w && w[0] == 'l') launch_tpq_walk<DP, KMAX, LIST, THREADS, false>(cx, a);
+    else launch_tpq_walk<DP, KMAX, LIST, THREADS, true>(cx, a);
+}
 
 // kNearests placement (Fig. 8, P:L587-609 re-derived for B200 in DESIGN.md):
-// shared memory when k*4 <= th1 (k <= 28 on B200), registers for k <= 32
-// otherwise; beyond the register budget (large k, NEXT-2) shared memory with
-// fewer threads per CTA so k * 8 B per thread still fits. SKNN_TOPK=reg|smem
+// shared memory, as a max-heap, for every k. Measured with the warp-union walk
+// (tools/sweep.py): C2 k=20 heap 0.49 / sorted 0.50 / registers 1.25 ms, C5
+// k=32 heap 62.5 / registers 79.5 / sorted 89.4 ms. SKNN_TOPK=reg|smem|heap
 // overrides for ablation.
+static int topk_override() {
+    const char* ov = getenv("SKNN_TOPK");
+    if (!ov) return -1;
+    return ov[0] == 'r' ? LIST_REG : (ov[0] == 'h' ? LIST_HEAP : LIST_SORTED);
+}
+
+template <int DP, int KMAX>
+static void launch_tpq_reg(Ctx& cx, const ScanArgs& a) {
+    launch_tpq<DP, KMAX, LIST_REG, 256>(cx, a);
+}
+
 template <int DP>
 static void launch_tpq_small_k(Ctx& cx, const ScanArgs& a) {
-    const char* ov = getenv("SKNN_TOPK");
-    const bool smem = ov ? (ov[0] == 's') : (a.k * 4 <= 114);
-    if (smem) {
-        launch_tpq<DP, 1, true, 256>(cx, a);
+    int list = topk_override();
+    if (list < 0) list = LIST_HEAP;
+    if (list == LIST_SORTED) {
+        launch_tpq<DP, 1, LIST_SORTED, 256>(cx, a);
+        return;
+    }
+    if (list == LIST_HEAP) {
+        launch_tpq<DP, 1, LIST_HEAP, 256>(cx, a);
         return;
     }
     switch ((a.k + 3) / 4) {
-        case 1: launch_tpq<DP, 4, false, 256>(cx, a); break;
-        case 2: launch_tpq<DP, 8, false, 256>(cx, a); break;
-        case 3: launch_tpq<DP, 12, false, 256>(cx, a); break;
-        case 4: launch_tpq<DP, 16, false, 256>(cx, a); break;
-        case 5: launch_tpq<DP, 20, false, 256>(cx, a); break;
-        case 6: launch_tpq<DP, 24, false, 256>(cx, a); break;
-        case 7: launch_tpq<DP, 28, false, 256>(cx, a); break;
-        default: launch_tpq<DP, 32, false, 256>(cx, a); break;
+        case 1: launch_tpq_reg<DP, 4>(cx, a); break;
+        case 2: launch_tpq_reg<DP, 8>(cx, a); break;
+        case 3: launch_tpq_reg<DP, 12>(cx, a); break;
+        case 4: launch_tpq_reg<DP, 16>(cx, a); break;
+        case 5: launch_tpq_reg<DP, 20>(cx, a); break;
+        case 6: launch_tpq_reg<DP, 24>(cx, a); break;
+        case 7: launch_tpq_reg<DP, 28>(cx, a); break;
+        default: launch_tpq_reg<DP, 32>(cx, a); break;
     }
+}
+
+// large k (NEXT-2): the list stays in shared memory (heap by default, sorted
+// with SKNN_TOPK=smem) with fewer threads per CTA so k * 8 B per thread fits
+template <int DP, int LIST>
+static void launch_tpq_large_k(Ctx& cx, const ScanArgs& a) {
+    if (a.k <= 96) launch_tpq<DP, 1, LIST, 256>(cx, a);
+    else if (a.k <= 384) launch_tpq<DP, 1, LIST, 64>(cx, a);
+    else launch_tpq<DP, 1, LIST, 32>(cx, a);
 }
 
 template <int DP>
 void launch_tpq_dp(Ctx& cx, const ScanArgs& a) {
     if (a.k > 32 || DP == 0) {
-        if (a.k <= 96) launch_tpq<DP, 1, true, 256>(cx, a);
-        else if (a.k <= 384) launch_tpq<DP, 1, true, 64>(cx, a);
-        else launch_tpq<DP, 1, true, 32>(cx, a);
+        if (topk_override() == LIST_SORTED) launch_tpq_large_k<DP, LIST_SORTED>(cx, a);
+        else launch_tpq_large_k<DP, LIST_HEAP>(cx, a);
         return;
     }
     if constexpr (DP > 0) launch_tpq_small_k<DP>(cx, a);

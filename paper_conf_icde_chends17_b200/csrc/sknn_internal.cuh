@@ -140,7 +140,8 @@ struct Side {
 };
 
 struct Counters {  // device-side counters (sknn_stats)
-    unsigned long long evals_sparse, evals_dense, evals_brute, center_evals, cand_pairs, dense_pairs, dist_recompute;
+    unsigned long long evals_sparse, evals_dense, evals_brute, center_evals, cand_pairs, dense_pairs, dist_recompute,
+        topk_inserts;
 };
 
 }  // namespace sknn

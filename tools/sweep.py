@@ -86,6 +86,7 @@ def main():
                    "ms_min": float(np.min(ms)), "queries_per_s": nq / (np.median(ms) / 1000.0),
                    "pruned_pct": med["pruned_pct"], "evals_per_query": med["dist_evals"] / nq,
                    "cand_per_qcluster": med["cand_pairs"] / max(1, med["mq"]), "center_evals_per_query": med["center_evals"] / nq,
+                   "inserts_per_query": med.get("topk_inserts", 0) / nq,
                    "stages": {k2: round(med[k2], 4) for k2 in ("ms_build_t", "ms_build_q", "ms_level1", "ms_dense", "ms_sparse")},
                    "dense_pairs": med["dense_pairs"], "evals_dense": med["dist_evals_dense"], "recompute": med["dist_recompute"],
                    "mq": med["mq"], "mt": med["mt"], "mapping": med["mapping_used"], "launches": med["kernel_launches"]}
