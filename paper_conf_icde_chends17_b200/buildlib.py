@@ -34,13 +34,17 @@ def _stale():
     return any(os.path.getmtime(p) > t for p in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, out: str = None) -> str:
+    """Build the library (to `out`, default in-tree). NVCC_EXTRA adds compiler
+    flags, e.g. -D tuning macros for an A/B variant built into abl/."""
+    extra = os.environ.get("NVCC_EXTRA", "").split()
+    lib = out or LIB
+    if not force and not extra and lib == LIB and not _stale():
         return LIB
-    objdir = os.path.join(HERE, "build")
+    objdir = os.path.join(HERE, "build" + ("_" + str(abs(hash(" ".join(extra))) % 10**8) if extra else ""))
     os.makedirs(objdir, exist_ok=True)
     common = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I", INCLUDE,
-                     "--expt-relaxed-constexpr"]
+                     "--expt-relaxed-constexpr"] + extra
     if verbose:
         common += ["-Xptxas", "-v"]
     objs = []
@@ -60,12 +64,15 @@ def build(force: bool = False, verbose: bool = False) -> str:
             failed = True
     if failed:
         raise RuntimeError("nvcc failed building libsweetknn.so")
-    tmp = LIB + ".tmp.%d" % os.getpid()
+    tmp = lib + ".tmp.%d" % os.getpid()
     subprocess.check_call([NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-lcudart_static"])
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose="--verbose" in sys.argv)
-    print(LIB)
+    out = None
+    if "--out" in sys.argv:
+        out = os.path.abspath(sys.argv[sys.argv.index("--out") + 1])
+        os.makedirs(os.path.dirname(out), exist_ok=True)
+    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv, out=out))

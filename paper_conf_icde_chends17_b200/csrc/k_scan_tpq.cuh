@@ -313,9 +313,15 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
 
 // Members evaluated per block of the warp-union walk (rows held in registers
 // while their distances are computed): ~32 floats of row data per block.
+#ifndef SKNN_U4
+#define SKNN_U4 8
+#endif
+#ifndef SKNN_UNION_MINB4
+#define SKNN_UNION_MINB4 3
+#endif
 template <int DP>
 constexpr int union_block() {
-    return DP == 0 ? 1 : (DP <= 4 ? 8 : (DP <= 8 ? 4 : (DP <= 16 ? 2 : 1)));
+    return DP == 0 ? 1 : (DP <= 4 ? SKNN_U4 : (DP <= 8 ? 4 : (DP <= 16 ? 2 : 1)));
 }
 
 // One warp tile of the thread-per-query scan with a WARP-UNION member walk
@@ -331,7 +337,7 @@ constexpr int union_block() {
 // distance is a real (query, target) distance and the list keeps the k
 // smallest keys), so every member of every lane's window is evaluated
 // (monotone break tests, DESIGN.md §2 exactness argument).
-template <int DP, int KMAX, int LIST, int THREADS, bool SPLIT>
+template <int DP, int KMAX, int LIST, int THREADS, bool SPLIT, int BUF>
 __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key_t* s_topk, unsigned long long& evals,
                                            unsigned long long& cevals, unsigned long long& ins) {
     constexpr unsigned FULL = 0xffffffffu;
@@ -378,17 +384,47 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
     unsigned* th2 = a.theta2 + qpos;
     const float4* trow4 = reinterpret_cast<const float4*>(a.trows);
     bool dirty = false;
-    auto consider = [&](float d2, int jc) {
+    // BUF > 0: keys that pass the (possibly stale) k-th bound wait in a
+    // per-lane register buffer; the warp flushes all buffers into the lists
+    // together once some lane's buffer is full, so the insert code runs with
+    // many lanes active instead of once per member with a few
+    key_t buf[BUF > 0 ? BUF : 1];
+    int nb = 0;
+    auto flush = [&]() {
+#pragma unroll
+        for (int b = 0; b < BUF; ++b) {
+            if (b < nb && buf[b] < kth) {
+                ++ins;
+                kth = top.insert(buf[b]);
+            }
+        }
+        nb = 0;
+        if (key_d2(kth) < kth_d2) {
+            kth_d2 = key_d2(kth);
+            dirty = true;
+        }
+    };
+    auto consider = [&](float d2, int jc) {  // called by all 32 lanes
         if (d2 <= kth_d2) {                                          // Alg. 2 line 16 (distance part)
             const key_t key = make_key(d2, __ldg(a.torig + jc));
             if (key < kth) {
-                ++ins;
-                kth = top.insert(key);
-                if (key_d2(kth) < kth_d2) {
-                    kth_d2 = key_d2(kth);
-                    dirty = true;  // theta follows once per block
+                if constexpr (BUF > 0) {
+#pragma unroll
+                    for (int b = 0; b < BUF; ++b)
+                        if (b == nb) buf[b] = key;
+                    ++nb;
+                } else {
+                    ++ins;
+                    kth = top.insert(key);
+                    if (key_d2(kth) < kth_d2) {
+                        kth_d2 = key_d2(kth);
+                        dirty = true;  // theta follows once per block
+                    }
                 }
             }
+        }
+        if constexpr (BUF > 0) {
+            if (__any_sync(FULL, nb == BUF)) flush();
         }
     };
     // line 17 (R8): theta = min(UB, sqrt(k-th d2) rounded up), refreshed once
@@ -486,6 +522,7 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
         }
         if (active) evals += walked;
     }
+    if constexpr (BUF > 0) flush();
     if (active) {
         if (SPLIT) {  // partial list of this task -> k_merge_split
             key_t* pl = a.part + (int64_t)tl.w * a.k * 32 + lane;
@@ -503,12 +540,12 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
 // register caps (measured): DP == 4 with a shared-memory list at 64 (4 CTAs
 // / SM; C2 0.62 vs 0.68 ms at the compiler's 80), register lists at 128
 // (2 CTAs / SM; the two inlined task bodies otherwise take ~190)
-template <int DP, int LIST, int THREADS>
+template <int DP, int LIST, int THREADS, int WALK>
 constexpr int tpq_min_blocks() {
-    return THREADS != 256 ? 1 : (LIST == LIST_REG ? 2 : (DP == 4 ? 4 : 1));
+    return THREADS != 256 ? 1 : (LIST == LIST_REG ? 2 : (DP == 4 ? (WALK ? SKNN_UNION_MINB4 : 4) : 1));
 }
-template <int DP, int KMAX, int LIST, int THREADS, bool UNI>
-__global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, LIST, THREADS>())) k_scan_tpq(ScanArgs a) {
+template <int DP, int KMAX, int LIST, int THREADS, int WALK>
+__global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, LIST, THREADS, WALK>())) k_scan_tpq(ScanArgs a) {
     extern __shared__ __align__(16) key_t s_topk[];  // [k][THREADS] for the shared-memory lists
     const int lane = threadIdx.x & 31;
     const int ntiles = *a.ntiles;
@@ -519,9 +556,10 @@ __global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, LIST, THREADS>())
         tile = __shfl_sync(0xffffffffu, tile, 0);
         if (tile >= ntiles) break;
         const int4 tl = a.tiles[tile];
-        if constexpr (UNI) {
-            if ((tl.z >> 8) > 1) union_tile<DP, KMAX, LIST, THREADS, true>(a, tl, s_topk, evals, cevals, ins);
-            else union_tile<DP, KMAX, LIST, THREADS, false>(a, tl, s_topk, evals, cevals, ins);
+        if constexpr (WALK > 0) {
+            constexpr int BUF = WALK == 2 ? 4 : 0;
+            if ((tl.z >> 8) > 1) union_tile<DP, KMAX, LIST, THREADS, true, BUF>(a, tl, s_topk, evals, cevals, ins);
+            else union_tile<DP, KMAX, LIST, THREADS, false, BUF>(a, tl, s_topk, evals, cevals, ins);
         } else {
             if ((tl.z >> 8) > 1) tpq_tile<DP, KMAX, LIST, THREADS, true>(a, tl, s_topk, evals, cevals, ins);
             else tpq_tile<DP, KMAX, LIST, THREADS, false>(a, tl, s_topk, evals, cevals, ins);
@@ -532,10 +570,10 @@ __global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, LIST, THREADS>())
     add_counter(&a.counters->topk_inserts, ins);
 }
 
-template <int DP, int KMAX, int LIST, int THREADS, bool UNI>
+template <int DP, int KMAX, int LIST, int THREADS, int WALK>
 static void launch_tpq_walk(Ctx& cx, const ScanArgs& a) {
     const size_t smem = LIST != LIST_REG ? sizeof(key_t) * (size_t)a.k * THREADS : 0;
-    auto fn = k_scan_tpq<DP, KMAX, LIST, THREADS, UNI>;
+    auto fn = k_scan_tpq<DP, KMAX, LIST, THREADS, WALK>;
     if (smem > 48 * 1024) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int grid = occupancy_grid(cx, (const void*)fn, THREADS, smem);
     if (a.probe_warps) {  // dry run: report resident warps for the task planner
@@ -545,12 +583,19 @@ static void launch_tpq_walk(Ctx& cx, const ScanArgs& a) {
     fn<<<grid, THREADS, smem, cx.stream>>>(a);
 }
 
-// member walk: warp-union (default) or per-lane LB-ordered (SKNN_WALK=lane)
+// member walk: warp-union with immediate inserts (k <= 24) or with buffered
+// inserts (k > 24, where a heap insert is deep enough that running it for many
+// lanes at once pays: C5 k=32 93.6 -> 84.5 ms; C2 k=20 0.94 -> 1.54 ms,
+// C3 k=16 4.13 -> 4.24 ms the other way). SKNN_WALK=union|ubuf|lane
+// (per-lane LB-ordered walk) overrides for ablation.
 template <int DP, int KMAX, int LIST, int THREADS>
 static void launch_tpq(Ctx& cx, const ScanArgs& a) {
     const char* w = getenv("SKNN_WALK");
-    if (w && w[0] == 'l') launch_tpq_walk<DP, KMAX, LIST, THREADS, false>(cx, a);
-    else launch_tpq_walk<DP, KMAX, LIST, THREADS, true>(cx, a);
+    int walk = a.k > 24 ? 2 : 1;
+    if (w) walk = w[0] == 'l' ? 0 : (w[1] == 'b' ? 2 : 1);
+    if (walk == 0) launch_tpq_walk<DP, KMAX, LIST, THREADS, 0>(cx, a);
+    else if (walk == 1) launch_tpq_walk<DP, KMAX, LIST, THREADS, 1>(cx, a);
+    else launch_tpq_walk<DP, KMAX, LIST, THREADS, 2>(cx, a);
 }
 
 // kNearests placement (Fig. 8, P:L587-609 re-derived for B200 in DESIGN.md):

@@ -60,9 +60,8 @@ def main():
         nq, nt = Q.shape[0], T.shape[0]
         flush = torch.empty(128 * 1024 * 1024, dtype=torch.float32, device="cuda")
         for vname in args.variants.split(","):
-            if vname.startswith("env:"):  # ad-hoc variant: env:NAME=VALUE
-                n_, v_ = vname[4:].split("=")
-                v = {"_env": (n_, v_)}
+            if vname.startswith("env:"):  # ad-hoc variant: env:NAME=VALUE[+NAME2=VALUE2...]
+                v = {"_env": [tuple(kv.split("=")) for kv in vname[4:].split("+")]}
             else:
                 v = dict(VARIANTS[vname])
             env = v.pop("_env", None)
@@ -70,16 +69,18 @@ def main():
             if cl:
                 v["n_clusters_t"] = int(3 * np.sqrt(nt) * cl)
                 v["n_clusters_q"] = int(3 * np.sqrt(nq) * cl)
-            if env:
-                os.environ[env[0]] = env[1]
+            if env and isinstance(env, tuple):
+                env = [env]
+            for n_, v_ in env or []:
+                os.environ[n_] = v_
             res = []
             for r in range(args.reps + 2):
                 flush.zero_()
                 _, _, st = sknn.join(dQ, dT, k, stats=True, **v)
                 if r >= 2:
                     res.append(st)
-            if env:
-                del os.environ[env[0]]
+            for n_, _ in env or []:
+                del os.environ[n_]
             ms = [x["ms_total"] for x in res]
             med = res[int(np.argsort(ms)[len(ms) // 2])]
             out = {"config": name, "variant": vname, "nq": nq, "nt": nt, "k": k, "ms_total": float(np.median(ms)),
