@@ -266,35 +266,47 @@ def main():
     for key in stage:
         stage[key] /= n_stats
 
-    # ---- roofline of the dominant kernel (the level-2 scan), timed live above ----
-    # Algorithmic bytes per launch: the query rows, every
-    # evaluated member (row + member distance), every candidate-center
-    # distance (center row + CSR bounds), the per-(query, candidate) bound
-    # inputs (D, r_t) and the result rows. Intensity ~0.6 flop/B, far below
-    # the B200 balance point (74 TF / 6.5 TB/s ~ 11 flop/B): the binding
-    # roofline is the memory one, reported against HBM bandwidth.
+    # ---- roofline of the dominant kernel (the level-2 scan), its duration
+    # from CUDA events on the launching stream (stats pass above) ----
+    # Algorithmic work per launch, SURVEY.md §8(d) "Sparse (S9-S10)":
+    #  bytes = query rows once + target rows (row + member distance) as the
+    #          method's reuse unit fetches them -- once per warp tile and member
+    #          for the warp-union walk (counter rows_loaded) -- + result rows;
+    #          per-(tile, candidate) center rows and bound inputs, 4*dp + 16 B
+    #  flops = 3d per evaluated distance and per candidate-center distance
+    #          + log2 |tc| per (query, candidate) window search
+    # The binding roofline is the one with the larger fraction.
     scan_ms = stage["ms_sparse"]
     dpad = 4 * ((d + 3) // 4)
     E = float(last["dist_evals_sparse"])
     C = float(last["center_evals"])
-    P = float(last["cand_pairs"]) * (nq / max(1, last["mq"]))  # (query, candidate cluster) bound checks
-    bytes_alg = (4.0 * dpad * nq / max(1, ws) + (4.0 * dpad + 4.0) * E + (4.0 * dpad + 8.0) * C + 8.0 * P +
-                 8.0 * k * nq / max(1, ws))
-    flops = 3.0 * d * (E + C)
+    Rl = float(last.get("rows_loaded", E))
+    nq_r = nq / max(1, ws)
+    P = float(last["cand_pairs"]) * (nq_r / max(1, last["mq"] / max(1, ws)))  # (query, candidate) pairs
+    bytes_alg = 4.0 * dpad * nq_r + (4.0 * dpad + 4.0) * Rl + 8.0 * k * nq_r + (4.0 * dpad + 16.0) * P / 32.0
+    tc_mean = nt / max(1, last["mt"])
+    flops = 3.0 * d * (E + C) + P * float(np.log2(max(2.0, tc_mean)))
     sm_mhz = peaks.get("sm_max_mhz", 1965.0)
     alu_peak_tflops = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
     hbm = peaks.get("hbm_gbs")
-    achieved_gbs = bytes_alg / (scan_ms / 1000.0) / 1e9 if scan_ms > 0 else None
-    roofline = {"kernel": "k_scan_tpq (level-2 filtered scan fused with top-k)", "bound": "hbm",
-                "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
-                "frac": achieved_gbs / hbm if achieved_gbs else None,
+    achieved_gbs = bytes_alg / (scan_ms / 1000.0) / 1e9 if scan_ms > 0 else 0.0
+    achieved_tf = flops / (scan_ms / 1000.0) / 1e12 if scan_ms > 0 else 0.0
+    f_hbm = achieved_gbs / hbm if hbm else 0.0
+    f_alu = achieved_tf / alu_peak_tflops
+    if f_hbm >= f_alu:
+        bound, achieved, peak, unit, frac = "hbm", achieved_gbs, hbm, "GB/s", f_hbm
+    else:
+        bound, achieved, peak, unit, frac = "alu", achieved_tf, alu_peak_tflops, "TFLOP/s", f_alu
+    roofline = {"kernel": "k_scan_tpq (level-2 warp-union scan fused with top-k)", "bound": bound,
+                "achieved": achieved, "peak": peak, "unit": unit, "frac": frac,
                 "traffic": None, "launch_ms": scan_ms, "algorithmic_bytes": bytes_alg,
                 "algorithmic_flops": flops, "intensity_flop_per_byte": flops / bytes_alg if bytes_alg else None,
-                "alu_achieved_tflops": flops / (scan_ms / 1000.0) / 1e12 if scan_ms > 0 else None,
-                "alu_peak_tflops": alu_peak_tflops,
+                "hbm": {"achieved_gbs": achieved_gbs, "peak_gbs": hbm, "frac": f_hbm},
+                "alu": {"achieved_tflops": achieved_tf, "peak_tflops": alu_peak_tflops, "frac": f_alu},
                 "peak_source": "HBM %s; fp32 FMA pipe derived: 148 SMs x 128 lanes x 2 flop x %.0f MHz" % (
                     peaks["_source"], sm_mhz),
-                "share_of_step": scan_ms / ms_step if ms_step else None}
+                "share_of_step": scan_ms / ms_step if ms_step else None,
+                "note": "issue-bound (control flow and kNearests updates), not DRAM- or FMA-bound; see DESIGN.md §6"}
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         try:

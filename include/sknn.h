@@ -125,6 +125,8 @@ typedef struct {
     int32_t kernel_launches;       /* kernels this call launched                                      */
     int32_t pad0;
     uint64_t topk_inserts;         /* kNearests updates by the level-2 scan (P:L453 update overhead)   */
+    uint64_t rows_loaded;          /* target rows fetched by the level-2 scan: once per warp for the  */
+                                   /*   warp-union walk, once per evaluation otherwise (§8(d) bytes)  */
 } sknn_stats;
 
 /* Opaque resident target index (sknn_build / sknn_query). Owns device memory:

@@ -61,7 +61,8 @@ class Stats(ctypes.Structure):
                 ("ms_level1", ctypes.c_float), ("ms_sparse", ctypes.c_float), ("ms_dense", ctypes.c_float),
                 ("ms_final", ctypes.c_float), ("mapping_used", ctypes.c_int32), ("path_used", ctypes.c_int32),
                 ("mq", ctypes.c_int32), ("mt", ctypes.c_int32), ("kernel_launches", ctypes.c_int32),
-                ("pad0", ctypes.c_int32), ("topk_inserts", ctypes.c_uint64)]
+                ("pad0", ctypes.c_int32), ("topk_inserts", ctypes.c_uint64),
+                ("rows_loaded", ctypes.c_uint64)]
 
     def to_dict(self):
         d = {name: getattr(self, name) for name, _ in self._fields_ if name not in ("struct_size", "pad0")}

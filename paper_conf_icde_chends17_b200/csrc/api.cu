@@ -280,6 +280,7 @@ static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt
     s.dense_pairs = c.dense_pairs;
     s.dist_recompute = c.dist_recompute;
     s.topk_inserts = c.topk_inserts;
+    s.rows_loaded = c.rows_loaded;
     s.ms_total = tm.ms(0, mk.end);
     s.ms_build_t = tm.ms(0, mk.bt);
     s.ms_build_q = mk.bq >= 0 ? tm.ms(mk.bt, mk.bq) : 0.f;

@@ -121,6 +121,7 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
         }
     }
     add_counter(&a.counters->evals_sparse, evals);
+    add_counter(&a.counters->rows_loaded, evals);
     add_counter(&a.counters->center_evals, cevals);
 }
 

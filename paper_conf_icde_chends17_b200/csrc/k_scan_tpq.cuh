@@ -160,7 +160,8 @@ struct TopList<LIST_HEAP, KMAX, STRIDE> {
 // One warp tile of the thread-per-query scan (Alg. 2 for 32 queries).
 template <int DP, int KMAX, int LIST, int THREADS, bool SPLIT>
 __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t* s_topk, unsigned long long& evals,
-                                         unsigned long long& cevals, unsigned long long& ins) {
+                                         unsigned long long& cevals, unsigned long long& ins,
+                                         unsigned long long& rows) {
     const float INF = __int_as_float(0x7f800000);
     const int lane = threadIdx.x & 31;
     const int qc = tl.x;
@@ -296,6 +297,7 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
                     d2 = d2q(a.trows + (int64_t)jc * a.dp);
                 }
                 ++evals;
+                ++rows;
                 consider(d2, jc);
             }
         }
@@ -339,7 +341,8 @@ constexpr int union_block() {
 // (monotone break tests, DESIGN.md §2 exactness argument).
 template <int DP, int KMAX, int LIST, int THREADS, bool SPLIT, int BUF>
 __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key_t* s_topk, unsigned long long& evals,
-                                           unsigned long long& cevals, unsigned long long& ins) {
+                                           unsigned long long& cevals, unsigned long long& ins,
+                                         unsigned long long& rows) {
     constexpr unsigned FULL = 0xffffffffu;
     const int lane = threadIdx.x & 31;
     const int qc = tl.x;
@@ -521,6 +524,7 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
             }
         }
         if (active) evals += walked;
+        if (lane == 0) rows += walked;  // one broadcast row load per member for the warp
     }
     if constexpr (BUF > 0) flush();
     if (active) {
@@ -549,7 +553,7 @@ __global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, LIST, THREADS, WA
     extern __shared__ __align__(16) key_t s_topk[];  // [k][THREADS] for the shared-memory lists
     const int lane = threadIdx.x & 31;
     const int ntiles = *a.ntiles;
-    unsigned long long evals = 0, cevals = 0, ins = 0;
+    unsigned long long evals = 0, cevals = 0, ins = 0, rows = 0;
     for (;;) {
         int tile = 0;
         if (lane == 0) tile = atomicAdd(a.tile_counter, 1);
@@ -558,16 +562,17 @@ __global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, LIST, THREADS, WA
         const int4 tl = a.tiles[tile];
         if constexpr (WALK > 0) {
             constexpr int BUF = WALK == 2 ? 4 : 0;
-            if ((tl.z >> 8) > 1) union_tile<DP, KMAX, LIST, THREADS, true, BUF>(a, tl, s_topk, evals, cevals, ins);
-            else union_tile<DP, KMAX, LIST, THREADS, false, BUF>(a, tl, s_topk, evals, cevals, ins);
+            if ((tl.z >> 8) > 1) union_tile<DP, KMAX, LIST, THREADS, true, BUF>(a, tl, s_topk, evals, cevals, ins, rows);
+            else union_tile<DP, KMAX, LIST, THREADS, false, BUF>(a, tl, s_topk, evals, cevals, ins, rows);
         } else {
-            if ((tl.z >> 8) > 1) tpq_tile<DP, KMAX, LIST, THREADS, true>(a, tl, s_topk, evals, cevals, ins);
-            else tpq_tile<DP, KMAX, LIST, THREADS, false>(a, tl, s_topk, evals, cevals, ins);
+            if ((tl.z >> 8) > 1) tpq_tile<DP, KMAX, LIST, THREADS, true>(a, tl, s_topk, evals, cevals, ins, rows);
+            else tpq_tile<DP, KMAX, LIST, THREADS, false>(a, tl, s_topk, evals, cevals, ins, rows);
         }
     }
     add_counter(&a.counters->evals_sparse, evals);
     add_counter(&a.counters->center_evals, cevals);
     add_counter(&a.counters->topk_inserts, ins);
+    add_counter(&a.counters->rows_loaded, rows);
 }
 
 template <int DP, int KMAX, int LIST, int THREADS, int WALK>

@@ -141,7 +141,7 @@ struct Side {
 
 struct Counters {  // device-side counters (sknn_stats)
     unsigned long long evals_sparse, evals_dense, evals_brute, center_evals, cand_pairs, dense_pairs, dist_recompute,
-        topk_inserts;
+        topk_inserts, rows_loaded;
 };
 
 }  // namespace sknn
