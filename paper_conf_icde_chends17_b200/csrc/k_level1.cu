@@ -9,9 +9,13 @@
 //           D + d(c_tc, u_0) be each cluster's smallest bound and M_k the k-th
 //           smallest v0. k distinct bounds are <= M_k, so the pooled k-th
 //           smallest V_k <= M_k, and every bound <= V_k belongs to a cluster
-//           with v0 <= M_k. So: radix-select M_k over the mt values v0, gather
-//           the bounds <= M_k of those (about k) clusters -- the footnote's
-//           early termination -- and radix-select their k-th smallest.
+//           with v0 <= M_k. Cheaper and usually tighter: a cluster with >= k
+//           members holds k distinct bounds <= D + (its k-th smallest member
+//           distance), so the minimum of that over clusters (one block
+//           reduction) bounds V_k too; M_k is selected only when no cluster
+//           has k members. Gather the bounds <= M of the clusters with
+//           v0 <= M -- the footnote's early termination -- and select
+//           their k-th smallest.
 //   groupFilter (Alg. 1; Fig. 4 getLB/groupFilter P:L273-277;
 //           GPU version P:L339): keep tc iff lb = D - r_q - r_t <= UB
 //           (reading R6, plus the R7 rounding slack). Survivors are compacted
@@ -205,14 +209,26 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
 
     // ---- calUB (Step 2.1) ----
     // v0(tc) = D + smallest member distance (the member closest to c_tc)
+    // m1(tc) = D + k-th smallest member distance: one cluster with >= k
+    // members alone holds k distinct bounds <= m1, so min m1 >= V_k as well
+    __shared__ unsigned s_m1;
+    if (threadIdx.x == 0) s_m1 = __float_as_uint(INF);
+    __syncthreads();
+    float m1 = INF;
     for (int tc = threadIdx.x; tc < mt; tc += blockDim.x) {
         const int lo = __ldg(toff + tc), hi = __ldg(toff + tc + 1);
         const float D = __fsqrt_rn(d2_rows(s_qc, tcent + (int64_t)tc * dp, dp));
         s_D[tc] = D;
         s_v[tc] = (lo == hi) ? INF : D + __ldg(tdist + hi - 1);
+        if (hi - lo >= k) m1 = fminf(m1, D + __ldg(tdist + hi - k));
     }
+    for (int o = 16; o > 0; o >>= 1) m1 = fminf(m1, __shfl_xor_sync(0xffffffffu, m1, o));
+    if ((threadIdx.x & 31) == 0) atomicMin(&s_m1, __float_as_uint(m1));  // m1 >= 0: bits order like values
     __syncthreads();
-    const float Mk = block_kth_smallest(s_v, mt, k, s_hist, s_sel, s_small);
+    // gather threshold: the tighter of min m1 (no selection needed) and, only
+    // when no cluster has k members, the k-th smallest v0 (radix select)
+    float Mk = __uint_as_float(s_m1);
+    if (Mk == INF) Mk = block_kth_smallest(s_v, mt, k, s_hist, s_sel, s_small);
     // gather every bound <= M_k of the clusters with v0 <= M_k
     for (int tc = threadIdx.x; tc < mt; tc += blockDim.x) {
         if (!(s_v[tc] <= Mk)) continue;
