@@ -116,8 +116,11 @@ __global__ void k_centers_to_tc(const float* __restrict__ centers, int m, int mp
     }
 }
 
-// One CTA = 128 points; streams every center chunk through a 2-deep bulk-copy ring.
-__global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__ Xp, int64_t n, int dp, int kp,
+// One CTA = 128 points, 8 warps: warps w and w + 4 read the same 32 TMEM lanes
+// (points) and split each chunk's 128 columns in halves. Streams every center
+// chunk through a 2-deep bulk-copy ring.
+constexpr int kTcThreads = 256;
+__global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __restrict__ Xp, int64_t n, int dp, int kp,
                                                        const float* __restrict__ o,
                                                        const __nv_bfloat16* __restrict__ cbf,
                                                        const float* __restrict__ bn, int m, int nchunks,
@@ -210,7 +213,8 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
     ph_full[0] = 1;
     float best = __int_as_float(0x7f800000);
     int bi = 0;
-    const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
+    const int half = warp >> 2;  // columns [64 * half, 64 * half + 64) of every chunk
+    const uint32_t trow = tmem + ((uint32_t)((warp & 3) * 32) << 16);
     for (int c = 0; c < nchunks; ++c) {
         const int buf = c & 1;
         // issue the next chunk's MMA as soon as its copy landed (overlaps this epilogue)
@@ -224,24 +228,58 @@ __global__ void __launch_bounds__(kTcM, 1) k_assign_tc(const float* __restrict__
         ph_mma[buf] ^= 1u;
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const float* bnv = sBn(buf);
+        // per 32 columns: the scores, their minimum by a min tree (one FMNMX
+        // per score) and, only when it beats the running best, the lowest
+        // column holding it (a strict running argmin over increasing columns)
 #pragma unroll 1
-        for (int cb = 0; cb < kTcN / 32; ++cb) {
+        for (int cb = 0; cb < 2; ++cb) {
+            const int col = half * 64 + cb * 32;
             uint32_t v[32];
-            ld32(trow + (uint32_t)(buf * kTcN + cb * 32), v);
+            ld32(trow + (uint32_t)(buf * kTcN + col), v);
+            float sc[32];
+            const float4* bn4 = reinterpret_cast<const float4*>(bnv + col);
 #pragma unroll
-            for (int j = 0; j < 32; ++j) {
-                const float sc = __fmaf_rn(-2.f, __uint_as_float(v[j]), bnv[cb * 32 + j]);
-                if (sc < best) { best = sc; bi = c * kTcN + cb * 32 + j; }
+            for (int j4 = 0; j4 < 8; ++j4) {
+                const float4 b4 = bn4[j4];
+                sc[4 * j4 + 0] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 0]), b4.x);
+                sc[4 * j4 + 1] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 1]), b4.y);
+                sc[4 * j4 + 2] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 2]), b4.z);
+                sc[4 * j4 + 3] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 3]), b4.w);
+            }
+            float t[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) t[j] = fminf(sc[j], sc[j + 16]);
+#pragma unroll
+            for (int w = 8; w > 0; w >>= 1)
+#pragma unroll
+                for (int j = 0; j < w; ++j) t[j] = fminf(t[j], t[j + w]);
+            if (t[0] < best) {  // the lowest column holding the new best
+                int jm = 31;
+#pragma unroll
+                for (int j = 31; j >= 0; --j) jm = (sc[j] == t[0]) ? j : jm;
+                best = t[0];
+                bi = c * kTcN + col + jm;
             }
         }
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         __syncthreads();  // buffer `buf` (smem + TMEM) is free again
         if (tid == 0 && c + 2 < nchunks) issue_copy(c + 2, buf);
     }
+    // merge the two column halves (the lower column wins ties)
+    __shared__ float s_best[kTcM];
+    __shared__ int s_bi[kTcM];
+    if (half == 1) {
+        s_best[tid - kTcM] = best;
+        s_bi[tid - kTcM] = bi;
+    }
+    __syncthreads();
     const int64_t i = (row0 + tid) * stride;
-    if (i < n) {
-        bi = min(bi, m - 1);
+    if (half == 0 && i < n) {
+        const float ob = s_best[tid];
+        const int obi = s_bi[tid];
+        if (ob < best || (ob == best && obi < bi)) bi = obi;
         const float* xr = Xp + i * dp;
+        bi = min(bi, m - 1);
         const float d2 = d2_rows(xr, centers + (int64_t)bi * dp, dp);  // exact fp32, shared formula
         if (cid_out) cid_out[i] = bi;
         if (dist_out) dist_out[i] = __fsqrt_rn(d2);
@@ -277,7 +315,7 @@ sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     const int64_t grid = ((n + stride - 1) / stride + kTcM - 1) / kTcM;
-    k_assign_tc<<<(unsigned)grid, kTcM, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, bn, m, nchunks, centers, cid, dist,
+    k_assign_tc<<<(unsigned)grid, kTcThreads, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, bn, m, nchunks, centers, cid, dist,
                                                           sums, fx, counts, stride);
     cx.launched();
     return cx.check_launch("assign (tensor cores)");

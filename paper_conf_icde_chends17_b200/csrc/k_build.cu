@@ -495,13 +495,19 @@ __global__ void k_d2_fill(const float* __restrict__ Xp, int64_t n, int dp, int m
 }
 
 // Lloyd update from the fixed-point sums (deterministic: integer adds commute)
-__global__ void k_lloyd_update(float* __restrict__ centers, const long long* __restrict__ sums,
-                               const double* __restrict__ fx, const int32_t* __restrict__ counts, int m, int dp) {
+// one thread per center; the sums and counts are zeroed after use, ready for
+// the next pass (no memsets between passes)
+__global__ void k_lloyd_update(float* __restrict__ centers, long long* __restrict__ sums,
+                               const double* __restrict__ fx, int32_t* __restrict__ counts, int m, int dp) {
     const double inv = 1.0 / *fx;
-    for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < m * dp; e += gridDim.x * blockDim.x) {
-        const int c = e / dp;
+    for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < m; c += gridDim.x * blockDim.x) {
         const int cnt = counts[c];
-        if (cnt > 0) centers[e] = (float)((double)sums[e] * inv / (double)cnt);
+        for (int j = 0; j < dp; ++j) {
+            const int64_t e = (int64_t)c * dp + j;
+            if (cnt > 0) centers[e] = (float)((double)sums[e] * inv / (double)cnt);
+            sums[e] = 0;
+        }
+        counts[c] = 0;
     }
 }
 
@@ -877,19 +883,18 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     if (lloyd > 0) {
         long long* sums;
         SKNN_TRY(cx.alloc_scratch((void**)&sums, sizeof(long long) * m * dp));
-        for (int it = 0; it < lloyd; ++it) {
-            SKNN_CUDA(cudaMemsetAsync(sums, 0, sizeof(long long) * m * dp, s));
-            SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
+        SKNN_CUDA(cudaMemsetAsync(sums, 0, sizeof(long long) * m * dp, s));
+        SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
+        for (int it = 0; it < lloyd; ++it) {  // k_lloyd_update re-zeroes sums and counts
             SKNN_TRY(assign(prev, cid, nullptr, sums, m, lstride, prev ? prev_stride : 1));
             prev = cid;
             prev_stride = lstride;
-            int blocks = std::max(1, std::min((m * dp + 255) / 256, 148 * 8));
-            k_lloyd_update<<<blocks, 256, 0, s>>>(out.centers, sums, fx, counts, m, dp);
+            k_lloyd_update<<<(m + 127) / 128, 128, 0, s>>>(out.centers, sums, fx, counts, m, dp);
             cx.launched();
         }
     }
     // final assignment with exact member distances + histogram
-    SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
+    if (lloyd <= 0) SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
     SKNN_TRY(assign(prev, cid, pdist, nullptr, m, 1, prev_stride));
     k_offsets<<<1, 1024, 0, s>>>(counts, m, out.off, cursor);
     cx.launched();
