@@ -34,6 +34,7 @@ namespace sknn {
 // key < kth() and returns the new k-th key.
 enum { LIST_REG = 0, LIST_SORTED = 1, LIST_HEAP = 2 };
 
+
 template <int LIST, int KMAX, int STRIDE>
 struct TopList;
 
@@ -118,6 +119,9 @@ struct TopList<LIST_HEAP, KMAX, STRIDE> {
         for (int r = 0; r < k; ++r) s[r * STRIDE] = src[k - 1 - r];
     }
     // place `key` at the root of the heap s[0, n) and sift it down
+    // (measured: pushing with a sift-up, or appending + one Floyd heapify,
+    // while the list fills is no faster on C2/C3 than this full-depth
+    // sift-down from the +inf root)
     __device__ __forceinline__ void sift(key_t key, int n) {
         int i = 0;
         for (;;) {
@@ -318,6 +322,9 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
 #ifndef SKNN_U4
 #define SKNN_U4 8
 #endif
+#ifndef SKNN_COLLECT
+#define SKNN_COLLECT 1
+#endif
 #ifndef SKNN_UNION_MINB4
 #define SKNN_UNION_MINB4 3
 #endif
@@ -450,6 +457,45 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
 #pragma unroll
                 for (int c = 0; c < DP / 4; ++c) r[u][c] = __ldg(trow4 + (int64_t)j * (DP / 4) + c);
             }
+#if SKNN_COLLECT
+            if constexpr (BUF == 0) {
+                // all U distances first; the members that pass the lane's
+                // current k-th bound are collected in a bit mask and inserted
+                // by a per-lane loop, so the insert code runs once per
+                // max-over-lanes pending count with every pending lane active
+                // (instead of once per member that any lane inserts)
+                float dd[U];
+                unsigned pass = 0;
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    float s = 0.f;
+#pragma unroll
+                    for (int c = 0; c < DP / 4; ++c) s = d2_acc4(s, q[c], r[u][c]);
+                    dd[u] = s;
+                    if (u < n && s <= kth_d2) pass |= 1u << u;  // Alg. 2 line 16 (distance part)
+                }
+                while (pass) {
+                    const int u = __ffs(pass) - 1;
+                    pass &= pass - 1;
+                    float d2 = dd[0];
+#pragma unroll
+                    for (int v = 1; v < U; ++v)
+                        if (u == v) d2 = dd[v];
+                    if (d2 <= kth_d2) {  // re-checked: an earlier insert may have lowered the bound
+                        const key_t key = make_key(d2, __ldg(a.torig + j0 + step * u));
+                        if (key < kth) {
+                            ++ins;
+                            kth = top.insert(key);
+                            if (key_d2(kth) < kth_d2) {
+                                kth_d2 = key_d2(kth);
+                                dirty = true;
+                            }
+                        }
+                    }
+                }
+                return;
+            }
+#endif
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 if (u < n) {

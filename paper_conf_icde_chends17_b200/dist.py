@@ -15,7 +15,12 @@ SURVEY.md §8(e). Two modes:
   NVLink and merged exactly by ``sknn_merge_partials`` (the paper's merge of
   sorted per-thread heaps, across ranks). The (d2, index) keys are
   global and the merge is a selection on their total order, so the result is
-  bit-identical to the single-GPU join.
+  bit-identical to the single-GPU join. ``exchange="all_to_all"`` (SURVEY
+  §8(f) NEXT-1) instead sends each rank only the partial lists of ITS query
+  rows [r*nq/P, (r+1)*nq/P) (one all-to-all, (P-1)/P x nq*k*8 B received per
+  rank instead of (P-1) x), merges them there and returns that slice -- or
+  the assembled result when ``gather=True`` (one all-gather of the final
+  8*k*nq/P bytes per rank).
 
 The local join and merge default to the CUDA library; tests may inject other
 callables to exercise the orchestration on CPU with the gloo backend.
@@ -71,9 +76,13 @@ def join_query_sharded(Q, T, k: int, *, group=None, self_join: bool | None = Non
 
 
 def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, local_join=None, merge=None,
-                        out_squared: bool = False, **opts):
+                        out_squared: bool = False, exchange: str = "all_gather", gather: bool = True, **opts):
     """Target-sharded join: local partial lists of every query against this
-    rank's T_shard (global indices), all-gathered and merged exactly."""
+    rank's T_shard (global indices), exchanged and merged exactly.
+    exchange="all_gather": every rank merges all nq rows (returns the full
+    result). exchange="all_to_all": rank r merges only its rows
+    shard_bounds(nq, P, r); gather=False returns that slice, gather=True the
+    full result assembled by one all-gather of the merged slices."""
     world, rank = _world(group)
     local_join = local_join or _cuda_join
     merge = merge or _cuda_merge
@@ -85,8 +94,41 @@ def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, lo
         pad_d = torch.full((nq, k - kk), float("inf"), dtype=torch.float32, device=Q.device)
         pidx = torch.cat([pidx, pad_i], 1)
         pd2 = torch.cat([pd2, pad_d], 1)
-    all_i = torch.empty((world * nq, k), dtype=torch.int32, device=Q.device)
-    all_d = torch.empty((world * nq, k), dtype=torch.float32, device=Q.device)
-    dist.all_gather_into_tensor(all_i, pidx.contiguous(), group=group)
-    dist.all_gather_into_tensor(all_d, pd2.contiguous(), group=group)
-    return merge(all_i.view(world, nq, k), all_d.view(world, nq, k), k, out_squared=out_squared)
+    if exchange == "all_gather":
+        all_i = torch.empty((world * nq, k), dtype=torch.int32, device=Q.device)
+        all_d = torch.empty((world * nq, k), dtype=torch.float32, device=Q.device)
+        dist.all_gather_into_tensor(all_i, pidx.contiguous(), group=group)
+        dist.all_gather_into_tensor(all_d, pd2.contiguous(), group=group)
+        return merge(all_i.view(world, nq, k), all_d.view(world, nq, k), k, out_squared=out_squared)
+    if exchange != "all_to_all":
+        raise ValueError("exchange must be 'all_gather' or 'all_to_all'")
+    # rank r receives the partial lists of its query rows from every rank: the
+    # rows are contiguous per destination, so one all_to_all_single per array
+    splits = [shard_bounds(nq, world, r) for r in range(world)]
+    send = [(hi - lo) * k for lo, hi in splits]
+    lo, hi = splits[rank]
+    mine = hi - lo
+    recv_i = torch.empty((world, mine, k), dtype=torch.int32, device=Q.device)
+    recv_d = torch.empty((world, mine, k), dtype=torch.float32, device=Q.device)
+    dist.all_to_all_single(recv_i.view(-1), pidx.contiguous().view(-1), [mine * k] * world, send, group=group)
+    dist.all_to_all_single(recv_d.view(-1), pd2.contiguous().view(-1), [mine * k] * world, send, group=group)
+    if mine > 0:
+        ri, rd = merge(recv_i, recv_d, k, out_squared=out_squared)
+    else:
+        ri = torch.empty((0, k), dtype=torch.int32, device=Q.device)
+        rd = torch.empty((0, k), dtype=torch.float32, device=Q.device)
+    if not gather:
+        return ri, rd
+    # assemble the merged slices (ragged when P does not divide nq: pad to the largest)
+    cap = max(h - l for l, h in splits)
+    pad_i = torch.full((cap, k), -1, dtype=torch.int32, device=Q.device)
+    pad_d = torch.zeros((cap, k), dtype=torch.float32, device=Q.device)
+    pad_i[:mine] = ri
+    pad_d[:mine] = rd
+    all_i = torch.empty((world * cap, k), dtype=torch.int32, device=Q.device)
+    all_d = torch.empty((world * cap, k), dtype=torch.float32, device=Q.device)
+    dist.all_gather_into_tensor(all_i, pad_i, group=group)
+    dist.all_gather_into_tensor(all_d, pad_d, group=group)
+    out_i = torch.cat([all_i[r * cap:r * cap + (h - l)] for r, (l, h) in enumerate(splits)])
+    out_d = torch.cat([all_d[r * cap:r * cap + (h - l)] for r, (l, h) in enumerate(splits)])
+    return out_i, out_d

@@ -67,13 +67,21 @@ def _worker(rank, world, port, results):
         lo, hi = sdist.shard_bounds(X.shape[0], world, rank)
         i, d = sdist.join_target_sharded(torch.from_numpy(Q), torch.from_numpy(X[lo:hi]).contiguous(), k, lo,
                                          local_join=oracle_local_join, merge=host_merge)
+        # target sharding, all-to-all exchange (NEXT-1): a ragged query count
+        Q2 = datagen.c1_uniform_int(151, seed=10)
+        ai, ad = sdist.join_target_sharded(torch.from_numpy(Q2), torch.from_numpy(X[lo:hi]).contiguous(), k, lo,
+                                           local_join=oracle_local_join, merge=host_merge, exchange="all_to_all")
+        si_, sd_ = sdist.join_target_sharded(torch.from_numpy(Q2), torch.from_numpy(X[lo:hi]).contiguous(), k, lo,
+                                             local_join=oracle_local_join, merge=host_merge, exchange="all_to_all",
+                                             gather=False)
         # query sharding, non-self join (contiguous rows)
         qi, qd = sdist.join_query_sharded(torch.from_numpy(Q), torch.from_numpy(X), k, self_join=False,
                                           local_join=oracle_local_join)
         # query sharding, self join (cluster-interleaved rows, assembled by all-reduce)
         Xt = torch.from_numpy(X)
         si, sd = sdist.join_query_sharded(Xt, Xt, k, local_join=oracle_local_join)
-        results[rank] = (i.numpy(), d.numpy(), qi.numpy(), qd.numpy(), si.numpy(), sd.numpy())
+        results[rank] = (i.numpy(), d.numpy(), qi.numpy(), qd.numpy(), si.numpy(), sd.numpy(),
+                         ai.numpy(), ad.numpy(), si_.numpy(), sd_.numpy())
     finally:
         dist.destroy_process_group()
 
@@ -100,8 +108,16 @@ def test_two_rank_gloo_matches_single_join():
     k = 8
     ridx, rdist = oracle.knn_join(Q, X, k)
     sidx, sdist_ = oracle.knn_join(X, X, k)
+    Q2 = datagen.c1_uniform_int(151, seed=10)
+    aidx, adist = oracle.knn_join(Q2, X, k)
+    from paper_conf_icde_chends17_b200.dist import shard_bounds
     for r in range(world):
-        i, d, qi, qd, si, sd = results[r]
+        i, d, qi, qd, si, sd, ai, ad, ri, rd = results[r]
+        np.testing.assert_array_equal(ai, aidx)      # all-to-all exchange, assembled
+        np.testing.assert_array_equal(ad, adist)
+        lo, hi = shard_bounds(Q2.shape[0], world, r)
+        np.testing.assert_array_equal(ri, aidx[lo:hi])  # all-to-all, this rank's merged slice
+        np.testing.assert_array_equal(rd, adist[lo:hi])
         np.testing.assert_array_equal(i, ridx)       # target-sharded == single join (bit-exact)
         np.testing.assert_array_equal(d, rdist)
         np.testing.assert_array_equal(qi, ridx)      # query-sharded, assembled

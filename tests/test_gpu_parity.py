@@ -348,6 +348,8 @@ def test_dist_nccl_world1(sknn):
         ridx, rdist = oracle.knn_join(Q, T, k)
         i, d = sdist.join_target_sharded(dev(Q), dev(T), k, 0)
         assert_knn_bitexact(i.cpu().numpy(), d.cpu().numpy(), ridx, rdist)
+        i, d = sdist.join_target_sharded(dev(Q), dev(T), k, 0, exchange="all_to_all")
+        assert_knn_bitexact(i.cpu().numpy(), d.cpu().numpy(), ridx, rdist)
         i, d = sdist.join_query_sharded(dev(Q), dev(T), k, self_join=False)
         assert_knn_bitexact(i.cpu().numpy(), d.cpu().numpy(), ridx, rdist)
     finally:
