@@ -531,7 +531,7 @@ sknn_status sknn_index_free(sknn_index* ix) {
     int cur = 0;
     cudaGetDevice(&cur);
     if (ix->device != cur) cudaSetDevice(ix->device);
-    void* ptrs[] = {ix->t.rows, ix->t.dist, ix->t.orig, ix->t.off, ix->t.centers, ix->t.radius};
+    void* ptrs[] = {ix->t.rows, ix->t.dist, ix->t.orig, ix->t.off, ix->t.centers, ix->t.radius, ix->t.tinfo};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     if (ix->device != cur) cudaSetDevice(cur);

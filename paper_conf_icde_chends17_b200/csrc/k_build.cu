@@ -300,10 +300,16 @@ __global__ void __launch_bounds__(256) k_center_knn(const float* __restrict__ ce
     const int L = min(kNbr, m);
     key_t mine = (lane < 32 - L) ? kNegKey : kInfKey;  // sorted ascending across lanes
     key_t kth = kInfKey;
+    // software-pipelined: the next batch's distance (its row load) is issued
+    // before the current batch is merged, so the warp's 62 batches (C2) do
+    // not serialise one L2 round trip each
+    auto batch_key = [&](int j) -> key_t {
+        return j < m ? make_key(d2_rows(rc, centers + (int64_t)j * dp, dp), j) : kInfKey;
+    };
+    key_t next = batch_key(lane);
     for (int base = 0; base < m; base += 32) {
-        const int j = base + lane;
-        key_t key = kInfKey;
-        if (j < m) key = make_key(d2_rows(rc, centers + (int64_t)j * dp, dp), j);
+        key_t key = next;
+        next = batch_key(base + 32 + lane);
         unsigned cm = __ballot_sync(0xffffffffu, key < kth);
         if (__popc(cm) <= 6) {  // few accepted keys: serial insertion
             while (cm) {
@@ -592,16 +598,16 @@ __global__ void __launch_bounds__(128) k_segsort_small(u64* __restrict__ keys, c
     while (S < size) S <<= 1;
     for (int i = threadIdx.x; i < S; i += blockDim.x) s[i] = (i < size) ? keys[lo + i] : ~0ull;
     __syncthreads();
-    for (int k = 2; k <= S; k <<= 1) {
+    for (int k = 2, lk = 1; k <= S; k <<= 1, ++lk) {
         for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {  // flip
-            int blk = t / (k / 2), r = t % (k / 2);
-            int i = blk * k + r, p = blk * k + k - 1 - r;
+            const int blk = t >> (lk - 1), r = t & (k / 2 - 1);  // powers of two: shifts, not divisions
+            const int i = (blk << lk) + r, p = (blk << lk) + k - 1 - r;
             cmpx(s, i, p);
         }
         __syncthreads();
-        for (int j = k / 4; j > 0; j >>= 1) {  // half-cleaners
+        for (int j = k / 4, lj = lk - 2; j > 0; j >>= 1, --lj) {  // half-cleaners
             for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
-                int i = (t / j) * 2 * j + (t % j);
+                const int i = ((t >> lj) << (lj + 1)) + (t & (j - 1));
                 cmpx(s, i, i + j);
             }
             __syncthreads();
@@ -632,15 +638,15 @@ __global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, co
     for (int base = 0; base < size; base += kSmallSeg) {
         for (int i = threadIdx.x; i < kSmallSeg; i += blockDim.x) s[i] = (base + i < size) ? g[base + i] : ~0ull;
         __syncthreads();
-        for (int k = 2; k <= kSmallSeg; k <<= 1) {
+        for (int k = 2, lk = 1; k <= kSmallSeg; k <<= 1, ++lk) {
             for (int t = threadIdx.x; t < kSmallSeg / 2; t += blockDim.x) {
-                int blk = t / (k / 2), r = t % (k / 2);
-                cmpx(s, blk * k + r, blk * k + k - 1 - r);
+                const int blk = t >> (lk - 1), r = t & (k / 2 - 1);
+                cmpx(s, (blk << lk) + r, (blk << lk) + k - 1 - r);
             }
             __syncthreads();
-            for (int j = k / 4; j > 0; j >>= 1) {
+            for (int j = k / 4, lj = lk - 2; j > 0; j >>= 1, --lj) {
                 for (int t = threadIdx.x; t < kSmallSeg / 2; t += blockDim.x) {
-                    int i = (t / j) * 2 * j + (t % j);
+                    const int i = ((t >> lj) << (lj + 1)) + (t & (j - 1));
                     cmpx(s, i, i + j);
                 }
                 __syncthreads();
@@ -650,17 +656,16 @@ __global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, co
         __syncthreads();
     }
     // phase B: merges of size > kSmallSeg
-    for (int k = 2 * kSmallSeg; k <= S; k <<= 1) {
+    for (int k = 2 * kSmallSeg, lk = __ffs(2 * kSmallSeg) - 1; k <= S; k <<= 1, ++lk) {
         for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
-            int blk = t / (k / 2), r = t % (k / 2);
-            int i = blk * k + r, p = blk * k + k - 1 - r;
+            const int blk = t >> (lk - 1), r = t & (k / 2 - 1);  // powers of two: shifts, not divisions
+            const int i = (blk << lk) + r, p = (blk << lk) + k - 1 - r;
             if (i < size) gx(i, p);
         }
         __syncthreads();
-        int j = k / 4;
-        for (; j >= kSmallSeg; j >>= 1) {
+        for (int j = k / 4, lj = lk - 2; j >= kSmallSeg; j >>= 1, --lj) {
             for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
-                int i = (t / j) * 2 * j + (t % j);
+                const int i = ((t >> lj) << (lj + 1)) + (t & (j - 1));
                 if (i < size) gx(i, i + j);
             }
             __syncthreads();
@@ -669,9 +674,9 @@ __global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, co
         for (int base = 0; base < size; base += kSmallSeg) {
             for (int i = threadIdx.x; i < kSmallSeg; i += blockDim.x) s[i] = (base + i < size) ? g[base + i] : ~0ull;
             __syncthreads();
-            for (int jj = kSmallSeg / 2; jj > 0; jj >>= 1) {
+            for (int jj = kSmallSeg / 2, ljj = __ffs(kSmallSeg / 2) - 1; jj > 0; jj >>= 1, --ljj) {
                 for (int t = threadIdx.x; t < kSmallSeg / 2; t += blockDim.x) {
-                    int i = (t / jj) * 2 * jj + (t % jj);
+                    const int i = ((t >> ljj) << (ljj + 1)) + (t & (jj - 1));
                     cmpx(s, i, i + jj);
                 }
                 __syncthreads();
@@ -681,6 +686,17 @@ __global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, co
         }
     }
     if (threadIdx.x == 0) radius[c] = key_member_dist(g[0]);
+}
+
+// per-cluster summary read by level-1 and the scan with one 16-byte load:
+// {lo, hi, radius, smallest member distance} (the last member: R11 order)
+__global__ void k_side_info(const int32_t* __restrict__ off, const float* __restrict__ radius,
+                            const float* __restrict__ dist, int m, int4* __restrict__ tinfo) {
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= m) return;
+    const int lo = off[c], hi = off[c + 1];
+    const float dmin = hi > lo ? dist[hi - 1] : __int_as_float(0x7f800000);
+    tinfo[c] = make_int4(lo, hi, __float_as_int(radius[c]), __float_as_int(dmin));
 }
 
 // rows_out[p] = Xp[idx(p)], dist_out[p], orig_out[p]; one thread per float4
@@ -739,6 +755,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     SKNN_TRY(cx.alloc_persistent((void**)&out.off, sizeof(int32_t) * (m + 1)));
     SKNN_TRY(cx.alloc_persistent((void**)&out.centers, sizeof(float) * m * dp));
     SKNN_TRY(cx.alloc_persistent((void**)&out.radius, sizeof(float) * m));
+    SKNN_TRY(cx.alloc_persistent((void**)&out.tinfo, sizeof(int4) * m));
     out.owned = true;
 
     // padded copy of X (skipped when X already has 16-byte rows)
@@ -910,6 +927,8 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     int64_t tot = n * (dp / 4);
     int gblocks = (int)std::min<int64_t>((tot + 255) / 256, 148 * 16);
     k_gather_side<<<gblocks, 256, 0, s>>>(keys, Xp, n, dp, out.rows, out.dist, out.orig);
+    cx.launched();
+    k_side_info<<<(m + 255) / 256, 256, 0, s>>>(out.off, out.radius, out.dist, m, out.tinfo);
     cx.launched();
     return cx.check_launch("build_side");
 }

@@ -44,15 +44,15 @@ __device__ __forceinline__ void cmpx64(u64* s, int i, int p) {
 
 // ascending bitonic (flip + half-cleaner form) over S (power of two) entries
 __device__ void block_sort_u64(u64* s, int S) {
-    for (int k = 2; k <= S; k <<= 1) {
+    for (int k = 2, lk = 1; k <= S; k <<= 1, ++lk) {
         for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
-            int blk = t / (k / 2), r = t % (k / 2);
-            cmpx64(s, blk * k + r, blk * k + k - 1 - r);
+            const int blk = t >> (lk - 1), r = t & (k / 2 - 1);  // powers of two: shifts, not divisions
+            cmpx64(s, (blk << lk) + r, (blk << lk) + k - 1 - r);
         }
         __syncthreads();
-        for (int j = k / 4; j > 0; j >>= 1) {
+        for (int j = k / 4, lj = lk - 2; j > 0; j >>= 1, --lj) {
             for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {
-                int i = (t / j) * 2 * j + (t % j);
+                const int i = ((t >> lj) << (lj + 1)) + (t & (j - 1));
                 cmpx64(s, i, i + j);
             }
             __syncthreads();
@@ -175,9 +175,19 @@ __device__ __forceinline__ u64 warp_sort_u64(u64 v, int lane) {
     return v;
 }
 
+// d(c_tc, u_k): the k-th smallest member distance of every target cluster
+// (+inf with fewer than k members) -- the single-cluster bound of calUB
+__global__ void k_kth_member(const int4* __restrict__ tinfo, const float* __restrict__ tdist, int mt, int k,
+                             float* __restrict__ tdk) {
+    const int tc = blockIdx.x * blockDim.x + threadIdx.x;
+    if (tc >= mt) return;
+    const int4 ti = tinfo[tc];
+    tdk[tc] = ti.y - ti.x >= k ? tdist[ti.y - k] : __int_as_float(0x7f800000);
+}
+
 __global__ void __launch_bounds__(kL1Threads) k_level1(
     const float* __restrict__ qcent, const float* __restrict__ qrad, const int32_t* __restrict__ qoff,
-    const float* __restrict__ tcent, const float* __restrict__ trad, const int32_t* __restrict__ toff,
+    const float* __restrict__ tcent, const int4* __restrict__ tinfo, const float* __restrict__ tdk,
     const float* __restrict__ tdist, int mt, int dp, int k, float eta, int keys_cap, int shard_rank,
     int shard_count, int dense_mode, float dense_tau, const float* __restrict__ cq_o,
     const float* __restrict__ ct_o, float dense_eps, float* __restrict__ ub_out, int32_t* __restrict__ cand,
@@ -215,12 +225,16 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     if (threadIdx.x == 0) s_m1 = __float_as_uint(INF);
     __syncthreads();
     float m1 = INF;
+    // independent loads only (cluster summary, k-th member distance, center
+    // row), unrolled so several clusters' loads are in flight per thread
+#pragma unroll 4
     for (int tc = threadIdx.x; tc < mt; tc += blockDim.x) {
-        const int lo = __ldg(toff + tc), hi = __ldg(toff + tc + 1);
+        const float dmin = __int_as_float(__ldg(&tinfo[tc].w));  // +inf if empty
+        const float dk = __ldg(tdk + tc);                        // +inf if fewer than k members
         const float D = __fsqrt_rn(d2_rows(s_qc, tcent + (int64_t)tc * dp, dp));
         s_D[tc] = D;
-        s_v[tc] = (lo == hi) ? INF : D + __ldg(tdist + hi - 1);
-        if (hi - lo >= k) m1 = fminf(m1, D + __ldg(tdist + hi - k));
+        s_v[tc] = D + dmin;
+        m1 = fminf(m1, D + dk);
     }
     for (int o = 16; o > 0; o >>= 1) m1 = fminf(m1, __shfl_xor_sync(0xffffffffu, m1, o));
     if ((threadIdx.x & 31) == 0) atomicMin(&s_m1, __float_as_uint(m1));  // m1 >= 0: bits order like values
@@ -232,7 +246,8 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     // gather every bound <= M_k of the clusters with v0 <= M_k
     for (int tc = threadIdx.x; tc < mt; tc += blockDim.x) {
         if (!(s_v[tc] <= Mk)) continue;
-        const int lo = __ldg(toff + tc), hi = __ldg(toff + tc + 1);
+        const int4 ti = __ldg(tinfo + tc);
+        const int lo = ti.x, hi = ti.y;
         const float D = s_D[tc];
         const int cnt = min(k, hi - lo);
         // members closest to the center first; batches of 8 independent loads
@@ -271,9 +286,10 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
         const int tc = base + threadIdx.x;
         bool keep = false;
         float D = 0.f;
-        if (tc < mt && __ldg(toff + tc) != __ldg(toff + tc + 1)) {
+        const int4 ti = tc < mt ? __ldg(tinfo + tc) : make_int4(0, 0, 0, 0);
+        if (ti.x != ti.y) {
             D = s_D[tc];
-            const float rt = __ldg(trad + tc);
+            const float rt = __int_as_float(ti.z);
             const float lb = D - rq - rt;                        // getLB (Eq. 3)
             keep = ti_keep(lb, UB, D + rq + rt, eta);             // Alg. 1 line 4 (R6, R7)
         }
@@ -325,8 +341,9 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
             // expected share of tc's members inside a typical query's Alg. 2
             // window [dq - th, dq + th] with dq ~ D and th ~ V_k (the k-th
             // nearest target bound of the cluster center, without r_q)
-            const int sz = __ldg(toff + tc + 1) - __ldg(toff + tc);
-            const float rt = __ldg(trad + tc);
+            const int4 ti = __ldg(tinfo + tc);
+            const int sz = ti.y - ti.x;
+            const float rt = __int_as_float(ti.z);
             const float Dp = s_D[tc];
             const float ov = fminf(rt, Dp + Vk) - fmaxf(0.f, Dp - Vk);
             const float share = fminf(1.f, fmaxf(0.f, ov) / fmaxf(rt, 1e-30f));
@@ -401,7 +418,11 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
         return SKNN_ERR_UNSUPPORTED;
     }
     SKNN_CUDA(cudaFuncSetAttribute(k_level1, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    k_level1<<<mq, kL1Threads, smem, cx.stream>>>(qs.centers, qs.radius, qs.off, ts.centers, ts.radius, ts.off,
+    float* tdk;
+    SKNN_TRY(cx.alloc_scratch((void**)&tdk, sizeof(float) * mt));
+    k_kth_member<<<(mt + 255) / 256, 256, 0, cx.stream>>>(ts.tinfo, ts.dist, mt, p.k, tdk);
+    cx.launched();
+    k_level1<<<mq, kL1Threads, smem, cx.stream>>>(qs.centers, qs.radius, qs.off, ts.centers, ts.tinfo, tdk,
                                                   ts.dist, mt, dp, p.k, p.eta, cap, p.shard_rank, p.shard_count,
                                                   p.dense_mode, p.dense_tau, p.dorg ? p.dorg->cq_o : nullptr,
                                                   p.dorg ? p.dorg->ct_o : nullptr, p.dorg ? p.dorg->eps : 0.f,

@@ -75,16 +75,17 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
             for (int c = 0; c < ncand; ++c) {
                 const int tc = __ldg(cl + c);
                 // per-query 2-landmark bound (Eq. 3), then the empty-window checks
-                const float D = __ldg(cD + c), rt = __ldg(a.trad + tc);
+                const int4 ti = __ldg(a.tinfo + tc);  // {lo, hi, r_t, smallest member distance}
+                const float D = __ldg(cD + c), rt = __int_as_float(ti.z);
                 if (!ti_keep(D - rown - rt, theta, D + rown + rt, a.eta)) continue;
-                const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
+                const int lo = ti.x, hi = ti.y;
                 float dq2;
                 if constexpr (DP > 0) dq2 = d2_reg<DP>(q, a.tcent + (int64_t)tc * DP);
                 else dq2 = d2_rows(sq, a.tcent + (int64_t)tc * dp, dp);
                 const float dq = __fsqrt_rn(dq2);
                 if (lane == 0) ++cevals;
                 if (!ti_keep(dq - rt, theta, dq + rt, a.eta)) continue;
-                const float dtmin = __ldg(a.tdist + hi - 1);
+                const float dtmin = __int_as_float(ti.w);
                 if (!ti_keep(dtmin - dq, theta, dq + dtmin, a.eta)) continue;
                 const int j0 = window_start(a.tdist, lo, hi, dq, theta, a.eta);
                 for (int base = j0; base < hi; base += 32) {
@@ -478,7 +479,7 @@ sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, 
     a.qrows = qs.rows; a.qorig = qs.orig; a.qoff = qs.off;
     a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
     a.ub = l1.ub; a.cand = l1.cand; a.cand_count = l1.cand_count; a.cand_D = l1.cand_D;
-    a.qdist = qs.dist; a.trad = ts.radius;
+    a.qdist = qs.dist; a.trad = ts.radius; a.tinfo = ts.tinfo;
     a.tiles = l1.tiles; a.ntiles = l1.ntiles; a.tile_counter = l1.ntiles + 1;
     a.part = l1.part; a.theta2 = l1.theta2;
     a.init_topk = p.init_topk; a.dcount = l1.dcount;

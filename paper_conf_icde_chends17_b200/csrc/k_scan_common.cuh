@@ -26,6 +26,7 @@ struct ScanArgs {
     const float* cand_D;
     const float* qdist;   // query's own member distance d(q, c_q)
     const float* trad;    // target cluster radius
+    const int4* tinfo;    // target cluster summary {lo, hi, radius bits, smallest member distance bits}
     const int4* tiles;       // tasks {query cluster, first member, split | nsplit << 8, part}
     const int* ntiles;
     key_t* part;             // partial lists of split tasks [part][k][32]

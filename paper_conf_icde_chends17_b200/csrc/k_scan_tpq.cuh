@@ -223,14 +223,15 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
             const int tc = __ldg(cl + c);
             // per-query 2-landmark bound (Eq. 3 with the query itself in place of
             // the query cluster's farthest member): D - d(q,c_q) - r_t <= d(q,t)
-            const float D = __ldg(cD + c), rt = __ldg(a.trad + tc);
+            const int4 ti = __ldg(a.tinfo + tc);  // {lo, hi, r_t, smallest member distance}
+            const float D = __ldg(cD + c), rt = __int_as_float(ti.z);
             if (!ti_keep(D - rown - rt, theta, D + rown + rt, a.eta)) continue;
-            const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
+            const int lo = ti.x, hi = ti.y;
             const float dq = __fsqrt_rn(d2q(a.tcent + (int64_t)tc * a.dp));  // Alg. 2 line 6
             ++cevals;
             // empty window: every member distance lies in [dt_min, r_t]
             if (!ti_keep(dq - rt, theta, dq + rt, a.eta)) continue;
-            const float dtmin = __ldg(a.tdist + hi - 1);
+            const float dtmin = __int_as_float(ti.w);
             if (!ti_keep(dtmin - dq, theta, dq + dtmin, a.eta)) continue;
             // Alg. 2 lines 7-17, visited in order of the 1-landmark lower bound
             // |l| = |dq - dt| (Eq. 1): start where dt ~ dq and walk outward on
@@ -521,14 +522,15 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
         const int tc = __ldg(cl + c);
         // per-query 2-landmark bound (Eq. 3 with the query in place of the
         // query cluster's farthest member): D - d(q,c_q) - r_t <= d(q,t)
-        const float D = __ldg(cD + c), rt = __ldg(a.trad + tc);
+        const int4 ti = __ldg(a.tinfo + tc);  // {lo, hi, r_t, smallest member distance}
+        const float D = __ldg(cD + c), rt = __int_as_float(ti.z);
         bool ok = active && ti_keep(D - rown - rt, theta, D + rown + rt, a.eta);
         if (!__any_sync(FULL, ok)) continue;
-        const int lo = __ldg(a.toff + tc), hi = __ldg(a.toff + tc + 1);
+        const int lo = ti.x, hi = ti.y;
         const float dq = __fsqrt_rn(d2q(a.tcent + (int64_t)tc * a.dp));  // Alg. 2 line 6
         cevals += active;
         // empty window: every member distance lies in [dt_min, r_t]
-        const float dtmin = __ldg(a.tdist + hi - 1);
+        const float dtmin = __int_as_float(ti.w);
         ok = ok && ti_keep(dq - rt, theta, dq + rt, a.eta) && ti_keep(dtmin - dq, theta, dq + dtmin, a.eta);
         const unsigned okm = __ballot_sync(FULL, ok);
         if (!okm) continue;

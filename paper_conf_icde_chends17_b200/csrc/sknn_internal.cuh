@@ -136,6 +136,8 @@ struct Side {
     int32_t* off = nullptr;    // [m+1] cluster offsets
     float* centers = nullptr;  // [m x dp]
     float* radius = nullptr;   // [m] max member distance (0 if empty)
+    int4* tinfo = nullptr;     // [m] {lo, hi, radius bits, smallest member distance bits (+inf if empty)}:
+                               // one 16-byte load per candidate cluster in level-1 and the scan
     bool owned = false;
 };
 
