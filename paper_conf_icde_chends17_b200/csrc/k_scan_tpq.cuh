@@ -142,8 +142,39 @@ struct TopList<LIST_HEAP, KMAX, STRIDE> {
         }
         s[i * STRIDE] = key;
     }
+    // KMAX > 1: k == KMAX is a compile-time constant and the root sift is
+    // fully unrolled: floor(log2 k) levels, bounds checks only on the last
+    static constexpr int steps() {
+        int L = 0;
+        while ((2 << L) <= KMAX) ++L;
+        return L;
+    }
+    __device__ __forceinline__ void sift_root_const(key_t key) {
+        constexpr int N = KMAX, STEPS = steps();
+        int i = 0;
+#pragma unroll
+        for (int lev = 0; lev < STEPS; ++lev) {
+            const int l = 2 * i + 1;
+            const bool last = lev == STEPS - 1;  // only the last level can run past the heap end
+            if (last && l >= N) break;
+            key_t c = s[l * STRIDE];
+            int ci = l;
+            if (!last || l + 1 < N) {
+                const key_t c2 = s[(l + 1) * STRIDE];
+                if (c < c2) {
+                    c = c2;
+                    ci = l + 1;
+                }
+            }
+            if (!(key < c)) break;
+            s[i * STRIDE] = c;
+            i = ci;
+        }
+        s[i * STRIDE] = key;
+    }
     __device__ __forceinline__ key_t insert(key_t key) {
-        sift(key, k);  // the old root (the k-th key) is dropped
+        if constexpr (KMAX > 1) sift_root_const(key);  // the old root (the k-th key) is dropped
+        else sift(key, k);
         return s[0];
     }
     // in-place heapsort: ascending order in s[0, k)
@@ -643,12 +674,16 @@ static void launch_tpq_walk(Ctx& cx, const ScanArgs& a) {
 // (per-lane LB-ordered walk) overrides for ablation.
 template <int DP, int KMAX, int LIST, int THREADS>
 static void launch_tpq(Ctx& cx, const ScanArgs& a) {
-    const char* w = getenv("SKNN_WALK");
-    int walk = a.k > 24 ? 2 : 1;
-    if (w) walk = w[0] == 'l' ? 0 : (w[1] == 'b' ? 2 : 1);
-    if (walk == 0) launch_tpq_walk<DP, KMAX, LIST, THREADS, 0>(cx, a);
-    else if (walk == 1) launch_tpq_walk<DP, KMAX, LIST, THREADS, 1>(cx, a);
-    else launch_tpq_walk<DP, KMAX, LIST, THREADS, 2>(cx, a);
+    if constexpr (LIST == LIST_HEAP && KMAX > 1) {  // compile-time k: the default walk only
+        launch_tpq_walk<DP, KMAX, LIST, THREADS, (KMAX > 24 ? 2 : 1)>(cx, a);
+    } else {
+        const char* w = getenv("SKNN_WALK");
+        int walk = a.k > 24 ? 2 : 1;
+        if (w) walk = w[0] == 'l' ? 0 : (w[1] == 'b' ? 2 : 1);
+        if (walk == 0) launch_tpq_walk<DP, KMAX, LIST, THREADS, 0>(cx, a);
+        else if (walk == 1) launch_tpq_walk<DP, KMAX, LIST, THREADS, 1>(cx, a);
+        else launch_tpq_walk<DP, KMAX, LIST, THREADS, 2>(cx, a);
+    }
 }
 
 // kNearests placement (Fig. 8, P:L587-609 re-derived for B200 in DESIGN.md):
@@ -676,6 +711,17 @@ static void launch_tpq_small_k(Ctx& cx, const ScanArgs& a) {
         return;
     }
     if (list == LIST_HEAP) {
+        // the configs' k (C1 8, C3/C4 16, C2 20, C5 32) get a compile-time k
+        // (unrolled sift); any other k runs the runtime-k heap
+        if (!getenv("SKNN_HEAP_RT")) {
+            switch (a.k) {
+                case 8: launch_tpq<DP, 8, LIST_HEAP, 256>(cx, a); return;
+                case 16: launch_tpq<DP, 16, LIST_HEAP, 256>(cx, a); return;
+                case 20: launch_tpq<DP, 20, LIST_HEAP, 256>(cx, a); return;
+                case 32: launch_tpq<DP, 32, LIST_HEAP, 256>(cx, a); return;
+                default: break;
+            }
+        }
         launch_tpq<DP, 1, LIST_HEAP, 256>(cx, a);
         return;
     }
