@@ -33,6 +33,8 @@ VARIANTS = {
     "warp": {"mapping": "warp"},
     "cl_half": {"_cl": 0.5},
     "cl_double": {"_cl": 2.0},
+    "cl_0.7": {"_cl": 0.7},
+    "cl_1.4": {"_cl": 1.4},
     "fullassign": {"_env": ("SKNN_ASSIGN", "full")},
     "walkassign": {"_env": ("SKNN_ASSIGN", "walk")},
     "tcassign": {"_env": ("SKNN_ASSIGN", "tc")},
