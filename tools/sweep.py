@@ -24,6 +24,7 @@ VARIANTS = {
     "lloyd4": {"lloyd_iters": 4},
     "thread": {"mapping": "thread"},
     "sparse": {"force_path": "sparse"},
+    "partial": {"force_path": "partial"},
     "dense": {"force_path": "dense"},
     "tau4": {"dense_threshold": 4.0},
     "tau25": {"dense_threshold": 0.25},
@@ -52,11 +53,13 @@ def main():
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--variants", default="default")
+    ap.add_argument("--k", type=int, default=0, help="override the config's k (k sweep, Fig. 10 / Table V)")
     args = ap.parse_args()
     import torch
     import paper_conf_icde_chends17_b200 as sknn
     for name in args.configs.split(","):
         Q, T, k, sj = datagen.workload(name, args.scale)
+        k = args.k or k
         dQ = torch.from_numpy(Q).cuda()
         dT = dQ if sj else torch.from_numpy(T).cuda()
         nq, nt = Q.shape[0], T.shape[0]
