@@ -75,7 +75,12 @@ enum {
     SKNN_PATH_AUTO = 0,   /* adaptive scheme (Fig. 8 re-derived for B200)                 */
     SKNN_PATH_SPARSE = 1, /* TI filters + point-level scan only (Alg. 1 + Alg. 2)          */
     SKNN_PATH_DENSE = 2,  /* TI filters; every surviving cluster pair on the dense tile path */
-    SKNN_PATH_BRUTE = 3   /* no filtering: every query against every target (the anchor)    */
+    SKNN_PATH_BRUTE = 3,  /* no filtering: every query against every target (the anchor)    */
+    SKNN_PATH_PARTIAL = 4 /* TI filters; PARTIAL level-2 filter (§IV-B1): theta   */
+                          /* fixed at the level-1 UB, every window member's distance stored  */
+                          /* in a global survivor buffer, then a k-selection kernel; k <= 512 */
+                          /* (falls back to the full filter when the buffer would not fit in */
+                          /* half of the free device memory)                                 */
 };
 
 /* Level-2 thread mapping override (sknn_options.mapping), §IV-B2 / §IV-D3. */

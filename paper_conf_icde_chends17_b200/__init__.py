@@ -25,7 +25,7 @@ LIB_PATH = os.environ.get("SKNN_LIB") or os.path.join(_HERE, "libsweetknn.so")
 SKNN_OK = 0
 STATUS = {0: "SKNN_OK", -1: "SKNN_ERR_INVALID_ARG", -2: "SKNN_ERR_NOT_DEVICE_PTR", -3: "SKNN_ERR_OOM",
           -4: "SKNN_ERR_CUDA", -5: "SKNN_ERR_UNSUPPORTED", -6: "SKNN_ERR_WRONG_DEVICE"}
-PATH = {"auto": 0, "sparse": 1, "dense": 2, "brute": 3}
+PATH = {"auto": 0, "sparse": 1, "dense": 2, "brute": 3, "partial": 4}
 MAPPING = {"auto": 0, "thread": 1, "warp": 2}
 MAX_K = 512
 

@@ -195,7 +195,7 @@ struct Marks {
 // Elastic switch mode for level-1 (S8): 2 = every pair dense, 1 = none, 0 = cost model.
 static int dense_mode_for(const sknn_options& o, int dp) {
     if (o.force_path == SKNN_PATH_DENSE) return 2;
-    if (o.force_path == SKNN_PATH_SPARSE) return 1;
+    if (o.force_path == SKNN_PATH_SPARSE || o.force_path == SKNN_PATH_PARTIAL) return 1;
     // Measured per-pair cost ratio dense/sparse: ~0.3 at d = 16,
     // ~0.1 at d = 28, ~0.01 at d = 128. With the per-query bounds the sparse
     // scan wins at d <= 16, so the switch is armed only above.
@@ -212,7 +212,8 @@ static float dense_tau_for(const sknn_options& o, int dp) {
 // The query half of Fig. 4 (lines 3-6) given both clustered sides:
 // calUB + groupFilter (+ the elastic switch) -> dense tiles -> pointFilter.
 static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, const sknn_options& o, int mapping,
-                              int32_t* out_idx, float* out_dist, Counters* counters, Timer& tm, Marks& mk) {
+                              int32_t* out_idx, float* out_dist, Counters* counters, Timer& tm, Marks& mk,
+                              int* path_used) {
     const float eta = rounding_eta(ts.d);
     Level1 l1;
     Level1Params lp;
@@ -234,7 +235,9 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     }
     if (lp.dense_mode == 0 && !lp.dorg) lp.dense_mode = 1;
     SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
-    SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp, k), k, scan_resident_warps(cx, mapping, ts.dp, k),
+    // the partial filter's passes take 32 queries per warp task (thread per query)
+    const int tile = o.force_path == SKNN_PATH_PARTIAL ? 32 : scan_tile_size(mapping, ts.dp, k);
+    SKNN_TRY(run_tiles(cx, qs, tile, k, scan_resident_warps(cx, mapping, ts.dp, k),
                        lp.shard_rank, lp.shard_count, l1));
     mk.l1 = tm.mark();
     key_t* init_topk = nullptr;
@@ -260,7 +263,14 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     sp.out_dist = out_dist;
     sp.counters = counters;
     sp.init_topk = init_topk;
-    SKNN_TRY(run_scan(cx, qs, ts, l1, sp));
+    bool full = true;
+    if (o.force_path == SKNN_PATH_PARTIAL) {  // §IV-B1 partial level-2 filter
+        bool fell_back = false;
+        SKNN_TRY(run_partial(cx, qs, ts, l1, sp, &fell_back));
+        full = fell_back;
+        if (!fell_back) *path_used = SKNN_PATH_PARTIAL;
+    }
+    if (full) SKNN_TRY(run_scan(cx, qs, ts, l1, sp));
     mk.scan = tm.mark();
     return SKNN_OK;
 }
@@ -290,7 +300,8 @@ static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt
     s.ms_sparse = mk.scan >= 0 ? tm.ms(mk.dense >= 0 ? mk.dense : mk.l1, mk.scan) : 0.f;
     s.ms_final = 0.f;
     s.mapping_used = mapping;
-    s.path_used = (path == SKNN_PATH_BRUTE) ? path : (c.dense_pairs ? SKNN_PATH_DENSE : SKNN_PATH_SPARSE);
+    s.path_used = (path == SKNN_PATH_BRUTE || path == SKNN_PATH_PARTIAL) ? path
+                                                                         : (c.dense_pairs ? SKNN_PATH_DENSE : SKNN_PATH_SPARSE);
     s.mq = mq;
     s.mt = mt;
     s.kernel_launches = launches;
@@ -405,7 +416,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
         }
         mq = qs->m;
         mt = ts->m;
-        st = query_core(cx, *qs, *ts, k, o, mapping, d_oidx, d_odist, counters, tm, mk);
+        st = query_core(cx, *qs, *ts, k, o, mapping, d_oidx, d_odist, counters, tm, mk, &path);
     } while (0);
     if (st == SKNN_OK) {
         if (oi_host) {

@@ -472,9 +472,8 @@ int scan_resident_warps(Ctx& cx, int mapping, int dp, int k) {
     return w > 0 ? w : cx.num_sms * 32;
 }
 
-sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
+ScanArgs make_scan_args(const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
     const int dp = ts.dp;
-    const bool tpq = scan_uses_tpq(p.mapping, dp, p.k);
     ScanArgs a{};
     a.qrows = qs.rows; a.qorig = qs.orig; a.qoff = qs.off;
     a.trows = ts.rows; a.tdist = ts.dist; a.torig = ts.orig; a.toff = ts.off; a.tcent = ts.centers;
@@ -486,6 +485,13 @@ sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, 
     a.mt = ts.m; a.dp = dp; a.k = p.k; a.tile = l1.tile; a.eta = p.eta;
     a.out_squared = p.out_squared; a.index_base = p.index_base; a.out_idx = p.out_idx; a.out_dist = p.out_dist;
     a.counters = p.counters;
+    return a;
+}
+
+sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
+    const int dp = ts.dp;
+    const bool tpq = scan_uses_tpq(p.mapping, dp, p.k);
+    ScanArgs a = make_scan_args(qs, ts, l1, p);
     dispatch_scan(cx, a, tpq, dp);
     cx.launched();
     SKNN_TRY(cx.check_launch("level2 scan"));

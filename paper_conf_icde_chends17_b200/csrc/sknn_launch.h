@@ -161,6 +161,12 @@ struct ScanParams {
     const key_t* init_topk = nullptr;    // dense-tile pass results to continue from
 };
 sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p);
+struct ScanArgs;
+ScanArgs make_scan_args(const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p);
+// k_partial.cu: the paper's partial level-2 filter (SKNN_PATH_PARTIAL); *fell_back
+// = true when it did not run (k > 512 or the survivor buffer does not fit)
+sknn_status run_partial(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p,
+                        bool* fell_back);
 sknn_status run_brute(Ctx& cx, const float* Q, int64_t nq, const float* T, int64_t nt, int d, const ScanParams& p);
 sknn_status run_merge(Ctx& cx, const int32_t* part_idx, const float* part_d2, int P, int64_t nq, int k,
                       int32_t* out_idx, float* out_dist, int out_squared);

@@ -470,3 +470,53 @@ def test_split_tasks_match_unsplit(sknn, name, scale):
     else:
         assert_knn_bitexact(i1, d1, ridx, rdist)
         assert_knn_bitexact(i0, d0, ridx, rdist)
+
+
+# ------------------------------------------- partial level-2 filter (§IV-B1) --
+@pytest.mark.parametrize("k", [1, 8, 20, 64, 512])
+def test_partial_filter_bitexact(sknn, k):
+    """SKNN_PATH_PARTIAL (fixed-UB level-2 filter, survivor buffer, k-select):
+    bit-exact on integer inputs at the paper's k sweep {1, 8, 20, 64, 512}
+    (Fig. 10 / Table V), self-join and non-self join, low and mid d."""
+    rng = np.random.default_rng(100 + k)
+    for d in (4, 28):
+        T = rng.integers(0, 60, size=(3000, d)).astype(np.float32)
+        Q = rng.integers(0, 60, size=(700, d)).astype(np.float32)
+        idx, dist, st = run(sknn, Q, T, k, False, force_path="partial")
+        assert st["path_used"] == 4
+        ridx, rdist = oracle.knn_join(Q, T, k)
+        assert_knn_bitexact(idx, dist, ridx, rdist)
+    X = datagen.c1_uniform_int(1024)
+    idx, dist, st = run(sknn, X, X, k, True, force_path="partial")
+    ridx, rdist = oracle.knn_join(X, X, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    assert X.shape[0] * k <= st["dist_evals"] <= X.shape[0] ** 2
+
+
+@pytest.mark.parametrize("name,scale", [("C3int", 0.05), ("C5", 0.0025), ("C4", 0.002)])
+def test_partial_filter_workloads(sknn, name, scale):
+    Q, T, k, sj = datagen.workload(name, scale)
+    idx, dist, st = run(sknn, Q, T, k, sj, force_path="partial")
+    assert st["path_used"] == 4
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+def test_partial_filter_real_and_ties(sknn):
+    """Real-valued C2/C3 shapes within the tolerance; the equal-norm sphere
+    (P10) keeps the lowest indices among exact ties; duplicates everywhere."""
+    for name, scale in (("C2", 0.02), ("C3", 0.05)):
+        Q, T, k, sj = datagen.workload(name, scale)
+        idx, dist, _ = run(sknn, Q, T, k, sj, force_path="partial")
+        _, rdist = oracle.knn_join(Q, T, k)
+        assert_knn_tolerant(Q, T, idx, dist, rdist)
+    S = datagen.sphere_ties()
+    Q0 = S[:1].copy()
+    for k in (1, 7, 100, 384):
+        idx, dist, _ = run(sknn, Q0, S, k, False, force_path="partial")
+        ridx, rdist = oracle.knn_join(Q0, S, k)
+        assert_knn_bitexact(idx, dist, ridx, rdist)
+    D = np.zeros((300, 4), np.float32)
+    idx, dist, _ = run(sknn, D, D, 16, True, force_path="partial")
+    ridx, rdist = oracle.knn_join(D, D, 16)
+    assert_knn_bitexact(idx, dist, ridx, rdist)

@@ -1,4 +1,4 @@
-"""Run a few joins of one workload (for ncu captures): python tools/run_one.py C4 [scale] [reps] [k=v ...]"""
+"""Run a few joins of one workload (for ncu captures): python tools/run_one.py C4 [scale] [reps] [opt=v ...] [knn_k=k]"""
 import os
 import sys
 
@@ -19,6 +19,7 @@ def main():
     import torch
     import paper_conf_icde_chends17_b200 as sknn
     Q, T, k, sj = datagen.workload(name, scale)
+    k = int(opts.pop("knn_k", k))  # knn_k=<k> overrides the config's k
     dQ = torch.from_numpy(Q).cuda()
     dT = dQ if sj else torch.from_numpy(T).cuda()
     for _ in range(reps):
