@@ -235,8 +235,15 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     }
     if (lp.dense_mode == 0 && !lp.dorg) lp.dense_mode = 1;
     SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
+    // Filter strength (§IV-D1, reading R13): the paper switches to the
+    // partial level-2 filter when k/d > 8. Measured on B200: it
+    // wins only with large lists (C3 k = 512: 60.6 vs 78.4 ms) and loses at
+    // k = 64 (C2, k/d = 16: 12.3 vs 4.6 ms), so auto takes it iff k/d > 8 and
+    // k > 128 (the survivor buffer falling back to the full filter if too big).
+    const bool partial = o.force_path == SKNN_PATH_PARTIAL ||
+                         (o.force_path == SKNN_PATH_AUTO && k > 128 && (int64_t)k > 8LL * ts.d);
     // the partial filter's passes take 32 queries per warp task (thread per query)
-    const int tile = o.force_path == SKNN_PATH_PARTIAL ? 32 : scan_tile_size(mapping, ts.dp, k);
+    const int tile = partial ? 32 : scan_tile_size(mapping, ts.dp, k);
     SKNN_TRY(run_tiles(cx, qs, tile, k, scan_resident_warps(cx, mapping, ts.dp, k),
                        lp.shard_rank, lp.shard_count, l1));
     mk.l1 = tm.mark();
@@ -264,7 +271,7 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     sp.counters = counters;
     sp.init_topk = init_topk;
     bool full = true;
-    if (o.force_path == SKNN_PATH_PARTIAL) {  // §IV-B1 partial level-2 filter
+    if (partial) {  // §IV-B1 partial level-2 filter
         bool fell_back = false;
         SKNN_TRY(run_partial(cx, qs, ts, l1, sp, &fell_back));
         full = fell_back;
