@@ -197,10 +197,12 @@ static int dense_mode_for(const sknn_options& o, int dp) {
     if (o.force_path == SKNN_PATH_DENSE) return 2;
     if (o.force_path == SKNN_PATH_SPARSE || o.force_path == SKNN_PATH_PARTIAL) return 1;
     // Measured per-pair cost ratio dense/sparse: ~0.3 at d = 16,
-    // ~0.1 at d = 28, ~0.01 at d = 128. With the per-query bounds the sparse
-    // scan wins at d <= 16, so the switch is armed only above.
+    // ~0.1 at d = 28, ~0.01 at d = 128. With the per-query bounds, the union
+    // walk and the compile-time-k heap the sparse scan wins at every d <= 32
+    // measured (C3 3.78 vs 3.95 ms, C3-int 6.74 vs 7.08 ms with the switch
+    // armed), so the switch is armed only above dp = 32.
     if (o.dense_threshold > 0.f) return dense_supported(dp) ? 0 : 1;
-    return (dp > 16 && dense_supported(dp)) ? 0 : 1;
+    return (dp > 32 && dense_supported(dp)) ? 0 : 1;
 }
 
 // default window-share threshold of the elastic switch (dp > 16)

@@ -31,6 +31,7 @@ VARIANTS = {
     "tau50": {"dense_threshold": 0.5},
     "tau75": {"dense_threshold": 0.75},
     "tau95": {"dense_threshold": 0.95},
+    "tau99": {"dense_threshold": 0.99},
     "warp": {"mapping": "warp"},
     "cl_half": {"_cl": 0.5},
     "cl_double": {"_cl": 2.0},
