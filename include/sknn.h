@@ -108,6 +108,9 @@ typedef struct {
     int64_t index_base;       /* added to every output index (target-sharded global indices)      */
     int32_t shard_rank;       /* query sharding: only query clusters c with c % shard_count ==    */
     int32_t shard_count;      /*   shard_rank are processed (0/1 = all); other output rows untouched */
+    int64_t query_batch;      /* sknn_query with HOST queries and outputs (out-of-core, the paper's */
+                              /*   query partitions P:L575): queries per device batch; 0 = auto   */
+                              /*   (all at once when they fit in 40% of the free device memory)   */
 } sknn_options;
 
 /* Counters and per-stage times of one call (filled only when a non-NULL
@@ -189,7 +192,12 @@ sknn_status sknn_build(const float* T, int64_t nt, int32_t d,
 
 /* Query a resident index: Step 1 for Q, then Steps 2-3 (Fig. 4 lines 3-6).
  * The index is read-only: concurrent queries on different streams are safe.
- * Must run on the device that built the index (else SKNN_ERR_WRONG_DEVICE). */
+ * Must run on the device that built the index (else SKNN_ERR_WRONG_DEVICE).
+ * Out-of-core (the paper's query partitions): when Q, out_dist and
+ * out_idx (if given) are all HOST memory, the queries stream through the
+ * device in batches of opt->query_batch rows (0 = auto from the free device
+ * memory), each batch an independent exact query, so results equal one call;
+ * stats are summed over the batches. The call synchronises `stream`. */
 sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq,
                        int32_t k, int32_t* out_idx, float* out_dist,
                        const sknn_options* opt, sknn_stats* stats,

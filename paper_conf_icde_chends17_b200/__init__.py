@@ -48,7 +48,7 @@ class Options(ctypes.Structure):
                 ("lloyd_iters", ctypes.c_int32), ("seed", ctypes.c_uint64), ("force_path", ctypes.c_int32),
                 ("mapping", ctypes.c_int32), ("dense_threshold", ctypes.c_float), ("r_factor", ctypes.c_float),
                 ("out_squared", ctypes.c_int32), ("pad0", ctypes.c_int32), ("index_base", ctypes.c_int64),
-                ("shard_rank", ctypes.c_int32), ("shard_count", ctypes.c_int32)]
+                ("shard_rank", ctypes.c_int32), ("shard_count", ctypes.c_int32), ("query_batch", ctypes.c_int64)]
 
 
 class Stats(ctypes.Structure):

@@ -524,8 +524,55 @@ sknn_status sknn_build(const float* T, int64_t nt, int32_t d, const sknn_options
 sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq, int32_t k, int32_t* out_idx,
                        float* out_dist, const sknn_options* opt, sknn_stats* stats, sknn_stream_t stream) {
     if (!index) return fail(SKNN_ERR_INVALID_ARG, "index is NULL");
-    return run_join(Q, nq, nullptr, index->t.n, index->t.d, k, out_idx, out_dist, opt, stats, (cudaStream_t)stream,
-                    index);
+    // Out-of-core queries (the paper partitions Q when it
+    // does not fit, "Q in Figure 8 represents one of the partitions"):
+    // with host queries and host outputs the queries stream through the device
+    // in batches against the resident index; every batch is an independent
+    // (exact) query, so the rows are identical to one call.
+    const int d = index->t.d;
+    if (nq > 0 && Q && out_dist && index->device >= 0 && classify(Q, index->device) == PTR_HOST &&
+        classify(out_dist, index->device) == PTR_HOST && (!out_idx || classify(out_idx, index->device) == PTR_HOST)) {
+        const sknn_options o = merge_options(opt ? opt : &index->opt);
+        int64_t B = o.query_batch;
+        if (B <= 0) {
+            size_t free_b = 0, tot_b = 0;
+            if (cudaMemGetInfo(&free_b, &tot_b) != cudaSuccess) return fail(SKNN_ERR_CUDA, "cudaMemGetInfo failed");
+            // per query: input row + output row + clustered copy, center distances and scan state (generous)
+            const double per_q = 4.0 * d + 8.0 * k + 2.0 * (4.0 * ((d + 3) & ~3) + 16.0) + 8.0 * k;
+            B = (int64_t)(0.4 * (double)free_b / per_q);
+        }
+        if (B >= (int64_t)k && B < nq) {
+            sknn_stats acc;
+            memset(&acc, 0, sizeof(acc));
+            for (int64_t b0 = 0; b0 < nq; b0 += B) {
+                const int64_t nb = std::min(B, nq - b0);
+                sknn_stats sb;
+                memset(&sb, 0, sizeof(sb));
+                sb.struct_size = sizeof(sb);
+                SKNN_TRY(run_join(Q + b0 * d, nb, nullptr, index->t.n, d, k, out_idx ? out_idx + b0 * k : nullptr,
+                                  out_dist + b0 * k, opt, stats ? &sb : nullptr, (cudaStream_t)stream, index));
+                if (stats) {  // batch sums (sizes and times add up over the batches)
+                    acc.pairs_total += sb.pairs_total; acc.dist_evals_sparse += sb.dist_evals_sparse;
+                    acc.dist_evals_dense += sb.dist_evals_dense; acc.dist_evals_brute += sb.dist_evals_brute;
+                    acc.center_evals += sb.center_evals; acc.cand_pairs += sb.cand_pairs;
+                    acc.dense_pairs += sb.dense_pairs; acc.dist_recompute += sb.dist_recompute;
+                    acc.topk_inserts += sb.topk_inserts; acc.rows_loaded += sb.rows_loaded;
+                    acc.ms_total += sb.ms_total; acc.ms_build_t += sb.ms_build_t; acc.ms_build_q += sb.ms_build_q;
+                    acc.ms_level1 += sb.ms_level1; acc.ms_sparse += sb.ms_sparse; acc.ms_dense += sb.ms_dense;
+                    acc.ms_final += sb.ms_final; acc.kernel_launches += sb.kernel_launches;
+                    acc.mapping_used = sb.mapping_used; acc.path_used = sb.path_used;
+                    acc.mq += sb.mq; acc.mt = sb.mt;
+                }
+            }
+            if (stats) {
+                acc.struct_size = sizeof(acc);
+                const size_t sz = stats->struct_size ? std::min(stats->struct_size, sizeof(sknn_stats)) : sizeof(sknn_stats);
+                memcpy(stats, &acc, sz);
+            }
+            return SKNN_OK;
+        }
+    }
+    return run_join(Q, nq, nullptr, index->t.n, d, k, out_idx, out_dist, opt, stats, (cudaStream_t)stream, index);
 }
 
 sknn_status sknn_merge_partials(const int32_t* part_idx, const float* part_d2, int32_t P, int64_t nq, int32_t k,

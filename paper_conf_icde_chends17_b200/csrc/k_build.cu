@@ -519,12 +519,23 @@ __global__ void k_lloyd_update(float* __restrict__ centers, long long* __restric
 }
 
 // fixed-point scale for the Lloyd sums: 2^s with max|x| * n * 2^s < 2^61
-__global__ void k_absmax(const float* __restrict__ Xp, int64_t total, unsigned int* __restrict__ out) {
+// max |x| over the padded rows (total = n * dp, a multiple of 4): float4
+// loads, one shared-memory and one global atomic per CTA
+__global__ void __launch_bounds__(256) k_absmax(const float* __restrict__ Xp, int64_t total,
+                                                unsigned int* __restrict__ out) {
+    __shared__ unsigned s_mx;
+    if (threadIdx.x == 0) s_mx = 0u;
+    __syncthreads();
     float mx = 0.f;
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x)
-        mx = fmaxf(mx, fabsf(Xp[e]));
+    const float4* X4 = reinterpret_cast<const float4*>(Xp);
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total / 4; e += (int64_t)gridDim.x * blockDim.x) {
+        const float4 v = __ldg(X4 + e);
+        mx = fmaxf(mx, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+    }
     for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-    if ((threadIdx.x & 31) == 0) atomicMax(out, __float_as_uint(mx));
+    if ((threadIdx.x & 31) == 0) atomicMax(&s_mx, __float_as_uint(mx));
+    __syncthreads();
+    if (threadIdx.x == 0) atomicMax(out, s_mx);
 }
 
 __global__ void k_fx_scale(const unsigned int* __restrict__ amax, int64_t n, double* __restrict__ fx) {
@@ -826,7 +837,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     amax = reinterpret_cast<unsigned int*>(fx + 1);
     if (lloyd > 0) {
         SKNN_CUDA(cudaMemsetAsync(amax, 0, sizeof(unsigned int), s));
-        k_absmax<<<(int)std::min<int64_t>((n * dp + 255) / 256, 148 * 8), 256, 0, s>>>(Xp, n * dp, amax);
+        k_absmax<<<(int)std::min<int64_t>((n * dp / 4 + 255) / 256, 148 * 2), 256, 0, s>>>(Xp, n * dp, amax);
         k_fx_scale<<<1, 1, 0, s>>>(amax, n, fx);
         cx.launched();
         cx.launched();

@@ -520,3 +520,21 @@ def test_partial_filter_real_and_ties(sknn):
     idx, dist, _ = run(sknn, D, D, 16, True, force_path="partial")
     ridx, rdist = oracle.knn_join(D, D, 16)
     assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+# ------------------------------------------------- out-of-core queries (NEXT-4) --
+@pytest.mark.parametrize("batch", [0, 333, 1000, 5000])
+def test_query_batches_host_memory(sknn, batch):
+    """sknn_query with host queries and outputs streams the queries through the
+    device in batches (the paper's query partitions): results equal the
+    oracle bit-exactly for every batch size (ragged last batch included) and
+    the per-batch stats add up."""
+    T = datagen.c5_blobs(20000, which="T")
+    Q = datagen.c5_blobs(3100, which="Q")
+    k = 32
+    ix = sknn.build(dev(T))
+    idx, dist, st = ix.query(Q, k, stats=True, query_batch=batch)   # numpy: host pointers
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(np.asarray(idx), np.asarray(dist), ridx, rdist)
+    assert st["pairs_total"] == Q.shape[0] * T.shape[0]
+    ix.close()
