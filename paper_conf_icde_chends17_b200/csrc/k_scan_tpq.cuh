@@ -447,7 +447,7 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
         }
     };
     auto consider = [&](float d2, int jc) {  // called by all 32 lanes
-        if (d2 <= kth_d2) {                                          // Alg. 2 line 16 (distance part)
+        if (active && d2 <= kth_d2) {                                // Alg. 2 line 16 (distance part)
             const key_t key = make_key(d2, __ldg(a.torig + jc));
             if (key < kth) {
                 if constexpr (BUF > 0) {
@@ -504,7 +504,9 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
 #pragma unroll
                     for (int c = 0; c < DP / 4; ++c) s = d2_acc4(s, q[c], r[u][c]);
                     dd[u] = s;
-                    if (u < n && s <= kth_d2) pass |= 1u << u;  // Alg. 2 line 16 (distance part)
+                    // Alg. 2 line 16 (distance part); a lane past the tile's last
+                    // query only shadows the walk and never inserts
+                    if (active && u < n && s <= kth_d2) pass |= 1u << u;
                 }
                 while (pass) {
                     const int u = __ffs(pass) - 1;
