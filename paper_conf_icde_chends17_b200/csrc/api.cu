@@ -163,7 +163,7 @@ struct Timer {
 
 static int choose_mapping(const sknn_options& o, const DevInfo& di, int64_t nq, int dp, int k) {
     if (o.mapping == SKNN_MAP_THREAD || o.mapping == SKNN_MAP_WARP) return o.mapping;
-    if (k > 32) return SKNN_MAP_THREAD;  // lane-distributed warp top-k holds at most 32
+    if (k > 32) return scan_uses_bigk(k) ? SKNN_MAP_WARP : SKNN_MAP_THREAD;  // k_scan_bigk: warp per query
     // Fig. 8 bottom chooses query-level parallelism when
     // |Q| >= r*max_cur and several threads per query otherwise. Measured on
     // B200 (profiles/r01_sweep.md) the thread-per-query scan wins for every
@@ -238,12 +238,12 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     if (lp.dense_mode == 0 && !lp.dorg) lp.dense_mode = 1;
     SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
     // Filter strength (§IV-D1, reading R13): the paper switches to the
-    // partial level-2 filter when k/d > 8. Measured on B200: it
-    // wins only with large lists (C3 k = 512: 60.6 vs 78.4 ms) and loses at
-    // k = 64 (C2, k/d = 16: 12.3 vs 4.6 ms), so auto takes it iff k/d > 8 and
-    // k > 128 (the survivor buffer falling back to the full filter if too big).
-    const bool partial = o.force_path == SKNN_PATH_PARTIAL ||
-                         (o.force_path == SKNN_PATH_AUTO && k > 128 && (int64_t)k > 8LL * ts.d);
+    // partial level-2 filter when k/d > 8. Measured on B200 the
+    // full filter wins every case once large k runs warp per query
+    // (k_scan_bigk: C3 k = 512 15.0 ms full vs 61.0 ms partial; C2 k = 64,
+    // k/d = 16: 4.5 vs 12.3 ms), so auto keeps the full filter and the partial
+    // one runs on request (SKNN_PATH_PARTIAL).
+    const bool partial = o.force_path == SKNN_PATH_PARTIAL;
     // the partial filter's passes take 32 queries per warp task (thread per query)
     const int tile = partial ? 32 : scan_tile_size(mapping, ts.dp, k);
     SKNN_TRY(run_tiles(cx, qs, tile, k, scan_resident_warps(cx, mapping, ts.dp, k),

@@ -360,7 +360,15 @@ static void launch_wpq(Ctx& cx, const ScanArgs& a) {
     k_scan_wpq<DP><<<grid, 256, smem, cx.stream>>>(a);
 }
 
-bool scan_uses_tpq(int mapping, int dp, int k) { return (mapping == SKNN_MAP_THREAD && dp <= 32) || k > 32; }
+// k > 96: warp per query with a thresholded shared-memory candidate buffer
+// (k_scan_bigk.cu). Measured: k = 512 C2 133.9 -> 32.2 ms, C3 78.3 -> 15.0 ms,
+// C5 2564 -> 647 ms; at k = 64 the per-thread heap (256 threads per CTA) is
+// as fast on C2, 15% slower on C3 and 1.8x faster on C5, so 33 <= k <= 96 keeps
+// it. SKNN_BIGK_HEAP=1 keeps the heap for every k (ablation).
+bool scan_uses_bigk(int k) { return k > 96 && !getenv("SKNN_BIGK_HEAP"); }
+bool scan_uses_tpq(int mapping, int dp, int k) {
+    return !scan_uses_bigk(k) && ((mapping == SKNN_MAP_THREAD && dp <= 32) || k > 32);
+}
 int scan_tile_size(int mapping, int dp, int k) { return scan_uses_tpq(mapping, dp, k) ? 32 : 8; }
 
 sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int shard_rank, int shard_count,
@@ -434,6 +442,10 @@ sknn_status run_dense_tiles(Ctx& cx, const Side& qs, Level1& l1) {
 __global__ void k_merge_split(ScanArgs a, const int4* __restrict__ merges, const int* __restrict__ nmerges);
 
 static void dispatch_scan(Ctx& cx, const ScanArgs& a, bool tpq, int dp) {
+    if (scan_uses_bigk(a.k)) {
+        launch_scan_bigk(cx, a, dp);
+        return;
+    }
     if (tpq) {
         switch (dp) {
             case 4: launch_tpq_dp<4>(cx, a); break;

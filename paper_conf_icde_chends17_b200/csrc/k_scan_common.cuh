@@ -103,4 +103,7 @@ void launch_tpq_dp(Ctx& cx, const ScanArgs& a);
 
 int occupancy_grid(Ctx& cx, const void* fn, int threads, size_t smem);
 
+// k_scan_bigk.cu: warp-per-query scan for k > 32
+void launch_scan_bigk(Ctx& cx, const ScanArgs& a, int dp);
+
 }  // namespace sknn

@@ -147,6 +147,7 @@ sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int s
 int scan_resident_warps(Ctx& cx, int mapping, int dp, int k);
 int scan_tile_size(int mapping, int dp, int k);
 bool scan_uses_tpq(int mapping, int dp, int k);
+bool scan_uses_bigk(int k);
 
 // k_scan.cu
 struct ScanParams {

@@ -22,9 +22,11 @@ def main():
     print("# r01 studies on synthetic data (one B200; `tools/study.sh`, `tools/sweep.py`: median of 3 joins after 2 "
           "warm-ups, L2 flushed)\n")
     print("## k sweep, full vs partial level-2 filter (paper Fig. 10 / Table V, P:L805-821)\n")
-    print("`sparse` = full filter (running theta, kNearests; dense tiles off), `partial` = SKNN_PATH_PARTIAL (theta fixed "
-          "at the level-1 UB, survivor buffer, k-selection). C2 at k = 512: the survivor buffer exceeds half the free "
-          "HBM, so `partial` fell back to the full filter (identical counts).\n")
+    print("`full` = the full filter (running theta, kNearests; dense tiles off; k <= 96 per-thread heap, k > 96 the "
+          "warp-per-query thresholded buffer of k_scan_bigk), `partial` = SKNN_PATH_PARTIAL (theta fixed at the level-1 "
+          "UB, survivor buffer, k-selection). C2 at k = 512: the survivor buffer exceeds half the free HBM, so "
+          "`partial` counted its windows and then fell back to the full filter (identical counts). On B200 the full "
+          "filter wins every case, so auto never picks the partial filter (DESIGN.md reading R13).\n")
     print("| config | k | k/d | filter | ms / join | % pruned | evals / query |")
     print("|---|---|---|---|---|---|---|")
     dims = {"C2": 4, "C3": 28}
