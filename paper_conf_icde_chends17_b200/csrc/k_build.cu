@@ -102,7 +102,9 @@ __global__ void __launch_bounds__(256) k_landmark_sums(const float* __restrict__
     }
     double s = 0.0;
     if (smem) {
-        // 16 x 16 threads, each a 4 x 4 block of pairs with its rows in registers
+        // 16 x 16 threads, each a 4 x 4 block of pairs with its rows in registers;
+        // the 16 distances sum in fp32 (MUFU sqrt) before one double add: S only
+        // ranks the trials, and the fixed order keeps it deterministic
         const int ti = threadIdx.x >> 4, tj = threadIdx.x & 15;
         const float4* A4 = reinterpret_cast<const float4*>(A);
         const float4* B4 = reinterpret_cast<const float4*>(B);
@@ -124,13 +126,17 @@ __global__ void __launch_bounds__(256) k_landmark_sums(const float* __restrict__
 #pragma unroll
                 for (int v = 0; v < 4; ++v) acc[u][v] = d2_acc4(acc[u][v], ra[u], rb[v]);
         }
+        float fs = 0.f;
 #pragma unroll
         for (int u = 0; u < 4; ++u)
 #pragma unroll
             for (int v = 0; v < 4; ++v) {
                 const int gi = bi * kLmTile + ti * 4 + u, gj = bj * kLmTile + tj * 4 + v;
-                if (gi < gj && gj < m) s += (double)__fsqrt_rn(acc[u][v]);
+                float r;
+                asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(acc[u][v]));
+                fs += (gi < gj && gj < m) ? r : 0.f;
             }
+        s = (double)fs;
     } else {
         for (int p = threadIdx.x; p < kLmTile * kLmTile; p += blockDim.x) {
             int i = p / kLmTile, j = p % kLmTile;
@@ -350,7 +356,7 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
                                                      int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
                                                      long long* __restrict__ sums, const double* __restrict__ fx,
                                                      int32_t* __restrict__ counts, int stride, int prev_stride,
-                                                     int nwalk) {
+                                                     int nwalk, int32_t* __restrict__ rank_out) {
     const int dp = DP > 0 ? DP : dp_rt;
     const int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * stride;  // Lloyd passes subsample
     if (i >= n) return;
@@ -389,7 +395,10 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
     }
     if (cid_out) cid_out[i] = best;
     if (dist_out) dist_out[i] = __fsqrt_rn(bd);
-    if (counts) atomicAdd(counts + best, 1);
+    if (counts) {  // rank_out: the member's slot in its cluster (k_scatter_keys needs no atomics)
+        const int r = atomicAdd(counts + best, 1);
+        if (rank_out) rank_out[i] = r;
+    }
     if (sums) {
         fx_accumulate(sums + (int64_t)best * dp, xr, dp, *fx);
     }
@@ -575,11 +584,13 @@ __global__ void __launch_bounds__(1024) k_offsets(const int32_t* __restrict__ co
 }
 
 // key: (~dist_bits) << 32 | index -> ascending key = descending distance, ascending index
+// rank (optional): slots already taken by the assignment's histogram atomics
 __global__ void k_scatter_keys(const int32_t* __restrict__ cid, const float* __restrict__ dist, int64_t n,
-                               const int32_t* __restrict__ off, int32_t* __restrict__ cursor, u64* __restrict__ keys) {
+                               const int32_t* __restrict__ off, int32_t* __restrict__ cursor,
+                               const int32_t* __restrict__ rank, u64* __restrict__ keys) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         int c = cid[i];
-        int pos = off[c] + atomicAdd(cursor + c, 1);
+        int pos = off[c] + (rank ? rank[i] : atomicAdd(cursor + c, 1));
         keys[pos] = (u64(~__float_as_uint(dist[i])) << 32) | u64(uint32_t(i));
     }
 }
@@ -594,14 +605,16 @@ __device__ __forceinline__ void cmpx(u64* s, int i, int p) {
     if (b < a) { s[i] = b; s[p] = a; }
 }
 
-constexpr int kSmallSeg = 4096;
+constexpr int kSmallSeg = 4096;  // smem chunk of k_segsort_big
+constexpr int kTinySeg = 1024;   // k_segsort_small capacity: 8 KB of smem, 16 CTAs per SM
+                                 // (one wave over C2's 1978 clusters; 4096 keys left 7 per SM)
 
 __global__ void __launch_bounds__(128) k_segsort_small(u64* __restrict__ keys, const int32_t* __restrict__ off,
                                                        float* __restrict__ radius) {
-    __shared__ u64 s[kSmallSeg];
+    __shared__ u64 s[kTinySeg];
     int c = blockIdx.x;
     int lo = off[c], size = off[c + 1] - lo;
-    if (size > kSmallSeg) return;
+    if (size > kTinySeg) return;
     if (size <= 1) {
         if (threadIdx.x == 0) radius[c] = size ? key_member_dist(keys[lo]) : 0.f;
         return;
@@ -629,7 +642,8 @@ __global__ void __launch_bounds__(128) k_segsort_small(u64* __restrict__ keys, c
     if (threadIdx.x == 0) radius[c] = key_member_dist(s[0]);
 }
 
-// Clusters larger than kSmallSeg: one CTA per cluster; stages whose partner
+// Clusters larger than kTinySeg: one CTA per cluster (up to kSmallSeg the
+// whole segment sorts in smem in phase A); stages whose partner
 // distance is < kSmallSeg run in shared memory chunk by chunk, the others
 // directly on global memory (virtual +inf padding beyond the segment).
 __global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, const int32_t* __restrict__ off,
@@ -637,7 +651,7 @@ __global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, co
     __shared__ u64 s[kSmallSeg];
     int c = blockIdx.x;
     int lo = off[c], size = off[c + 1] - lo;
-    if (size <= kSmallSeg) return;
+    if (size <= kTinySeg) return;
     u64* g = keys + lo;
     int S = 2;
     while (S < size) S <<= 1;
@@ -843,6 +857,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         cx.launched();
     }
     int graph_m = -1;
+    int32_t* rank_o = nullptr;  // set for the final walk pass only
     auto assign = [&](const int32_t* prev, int32_t* cid_o, float* dist_o, long long* sums_o, int mc, int stride,
                       int prev_stride) -> sknn_status {
         if (use_tc) return run_assign_tc(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, fx, counts, stride);
@@ -866,14 +881,14 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
 #define SKNN_WALK_CASE(D)                                                                                      \
     case D:                                                                                                    \
         k_assign_walk<D><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, mc, nbr, nentry, prev, cid_o, dist_o, sums_o, \
-                                              fx, counts, stride, prev_stride, nwalk);                         \
+                                              fx, counts, stride, prev_stride, nwalk, rank_o);                 \
         break;
             SKNN_WALK_CASE(4) SKNN_WALK_CASE(8) SKNN_WALK_CASE(12) SKNN_WALK_CASE(16)
             SKNN_WALK_CASE(20) SKNN_WALK_CASE(24) SKNN_WALK_CASE(28) SKNN_WALK_CASE(32)
 #undef SKNN_WALK_CASE
             default:
                 k_assign_walk<0><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, mc, nbr, nentry, prev, cid_o, dist_o,
-                                                      sums_o, fx, counts, stride, prev_stride, nwalk);
+                                                      sums_o, fx, counts, stride, prev_stride, nwalk, rank_o);
                 break;
         }
         cx.launched();
@@ -928,13 +943,14 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     }
     // final assignment with exact member distances + histogram
     if (lloyd <= 0) SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
+    if (walk) SKNN_TRY(cx.alloc_scratch((void**)&rank_o, sizeof(int32_t) * n));
     SKNN_TRY(assign(prev, cid, pdist, nullptr, m, 1, prev_stride));
     k_offsets<<<1, 1024, 0, s>>>(counts, m, out.off, cursor);
     cx.launched();
     unsigned long long* keys;
     SKNN_TRY(cx.alloc_scratch((void**)&keys, sizeof(unsigned long long) * n));
     int sblocks = (int)std::min<int64_t>((n + 255) / 256, 148 * 16);
-    k_scatter_keys<<<sblocks, 256, 0, s>>>(cid, pdist, n, out.off, cursor, keys);
+    k_scatter_keys<<<sblocks, 256, 0, s>>>(cid, pdist, n, out.off, cursor, rank_o, keys);
     cx.launched();
     k_segsort_small<<<m, 128, 0, s>>>(keys, out.off, out.radius);
     cx.launched();
