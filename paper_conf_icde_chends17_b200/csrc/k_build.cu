@@ -386,10 +386,25 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
     for (int step = 0; step < 64; ++step) {
         const int cur = best;
         const int32_t* nb = nbr + (int64_t)cur * kNbr;
-        for (int e = 1; e < nwalk; ++e) {  // the nwalk - 1 nearest graph neighbours
-            const int c = __ldg(nb + e);
-            const float v = dist2(c);
-            if (v < bd || (v == bd && c < best)) { bd = v; best = c; }
+        if (nwalk == kNbr) {  // default: the whole 128-byte row in 8 vector loads, then
+                              // 31 independent distances (one dependent round trip per step)
+            int cs[kNbr];
+#pragma unroll
+            for (int j = 0; j < kNbr / 4; ++j) {
+                const int4 v = __ldg(reinterpret_cast<const int4*>(nb) + j);
+                cs[4 * j] = v.x; cs[4 * j + 1] = v.y; cs[4 * j + 2] = v.z; cs[4 * j + 3] = v.w;
+            }
+#pragma unroll
+            for (int e = 1; e < kNbr; ++e) {
+                const float v = dist2(cs[e]);
+                if (v < bd || (v == bd && cs[e] < best)) { bd = v; best = cs[e]; }
+            }
+        } else {
+            for (int e = 1; e < nwalk; ++e) {  // the nwalk - 1 nearest graph neighbours
+                const int c = __ldg(nb + e);
+                const float v = dist2(c);
+                if (v < bd || (v == bd && c < best)) { bd = v; best = c; }
+            }
         }
         if (best == cur) break;
     }
@@ -606,17 +621,71 @@ __device__ __forceinline__ void cmpx(u64* s, int i, int p) {
 }
 
 constexpr int kSmallSeg = 4096;  // smem chunk of k_segsort_big
-constexpr int kTinySeg = 1024;   // k_segsort_small capacity: 8 KB of smem, 16 CTAs per SM
-                                 // (one wave over C2's 1978 clusters; 4096 keys left 7 per SM)
+constexpr int kTinySeg = 256;    // register sort in k_segsort_small (one warp, 8 keys per lane)
 
-__global__ void __launch_bounds__(128) k_segsort_small(u64* __restrict__ keys, const int32_t* __restrict__ off,
+// Segments of up to 32*R keys: one warp, R keys per lane in registers
+// (element e = r*32 + lane), the same ascending bitonic network with
+// partners e ^ j: shuffles for j < 32, in-thread exchanges for j >= 32.
+// No shared memory, no barriers (ncu, C2: the 128-thread smem network
+// issued 12.4M warp instructions for 1978 clusters of ~220 keys).
+template <int R>
+__device__ __forceinline__ void warp_segsort(u64* __restrict__ g, int size, float* __restrict__ radius_out) {
+    const int lane = threadIdx.x & 31;
+    u64 v[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) v[r] = (r * 32 + lane < size) ? g[r * 32 + lane] : ~0ull;
+#pragma unroll
+    for (int k = 2; k <= 32 * R; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            if (j >= 32) {  // k >= 64: the direction depends on the register index only
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    if (r & (j >> 5)) continue;
+                    const int p = r | (j >> 5);
+                    const bool asc = ((r * 32) & k) == 0;
+                    const u64 a = v[r], b = v[p];
+                    const bool sw = asc ? (b < a) : (a < b);
+                    v[r] = sw ? b : a;
+                    v[p] = sw ? a : b;
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    const u64 o = __shfl_xor_sync(0xffffffffu, v[r], j);
+                    const bool asc = ((r * 32 + lane) & k) == 0;
+                    const bool lower = (lane & j) == 0;
+                    v[r] = (lower == asc) ? (o < v[r] ? o : v[r]) : (o > v[r] ? o : v[r]);
+                }
+            }
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+        if (r * 32 + lane < size) g[r * 32 + lane] = v[r];
+    if (lane == 0) *radius_out = key_member_dist(v[0]);
+}
+
+// one 256-thread CTA per cluster of at most kMidSeg members: up to kTinySeg
+// members warp 0 sorts in registers (the other warps leave), larger clusters
+// run the bitonic network in 8 KB of shared memory
+constexpr int kMidSeg = 1024;
+__global__ void __launch_bounds__(256) k_segsort_small(u64* __restrict__ keys, const int32_t* __restrict__ off,
                                                        float* __restrict__ radius) {
-    __shared__ u64 s[kTinySeg];
-    int c = blockIdx.x;
-    int lo = off[c], size = off[c + 1] - lo;
-    if (size > kTinySeg) return;
+    __shared__ u64 s[kMidSeg];
+    const int c = blockIdx.x;
+    const int lo = off[c], size = off[c + 1] - lo;
+    if (size > kMidSeg) return;
     if (size <= 1) {
         if (threadIdx.x == 0) radius[c] = size ? key_member_dist(keys[lo]) : 0.f;
+        return;
+    }
+    if (size <= kTinySeg) {  // uniform per CTA
+        if (threadIdx.x >= 32) return;
+        if (size <= 32) warp_segsort<1>(keys + lo, size, radius + c);
+        else if (size <= 64) warp_segsort<2>(keys + lo, size, radius + c);
+        else if (size <= 128) warp_segsort<4>(keys + lo, size, radius + c);
+        else warp_segsort<8>(keys + lo, size, radius + c);
         return;
     }
     int S = 2;
@@ -625,7 +694,7 @@ __global__ void __launch_bounds__(128) k_segsort_small(u64* __restrict__ keys, c
     __syncthreads();
     for (int k = 2, lk = 1; k <= S; k <<= 1, ++lk) {
         for (int t = threadIdx.x; t < S / 2; t += blockDim.x) {  // flip
-            const int blk = t >> (lk - 1), r = t & (k / 2 - 1);  // powers of two: shifts, not divisions
+            const int blk = t >> (lk - 1), r = t & (k / 2 - 1);
             const int i = (blk << lk) + r, p = (blk << lk) + k - 1 - r;
             cmpx(s, i, p);
         }
@@ -642,7 +711,7 @@ __global__ void __launch_bounds__(128) k_segsort_small(u64* __restrict__ keys, c
     if (threadIdx.x == 0) radius[c] = key_member_dist(s[0]);
 }
 
-// Clusters larger than kTinySeg: one CTA per cluster (up to kSmallSeg the
+// Clusters larger than kMidSeg: one CTA per cluster (up to kSmallSeg the
 // whole segment sorts in smem in phase A); stages whose partner
 // distance is < kSmallSeg run in shared memory chunk by chunk, the others
 // directly on global memory (virtual +inf padding beyond the segment).
@@ -651,7 +720,7 @@ __global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, co
     __shared__ u64 s[kSmallSeg];
     int c = blockIdx.x;
     int lo = off[c], size = off[c + 1] - lo;
-    if (size <= kTinySeg) return;
+    if (size <= kMidSeg) return;
     u64* g = keys + lo;
     int S = 2;
     while (S < size) S <<= 1;
@@ -660,25 +729,26 @@ __global__ void __launch_bounds__(1024) k_segsort_big(u64* __restrict__ keys, co
         u64 a = g[i], b = g[p];
         if (b < a) { g[i] = b; g[p] = a; }
     };
-    // phase A: fully sort every aligned chunk of kSmallSeg in smem
-    for (int base = 0; base < size; base += kSmallSeg) {
-        for (int i = threadIdx.x; i < kSmallSeg; i += blockDim.x) s[i] = (base + i < size) ? g[base + i] : ~0ull;
+    // phase A: fully sort every aligned chunk of CL = min(kSmallSeg, S) keys in smem
+    const int CL = S < kSmallSeg ? S : kSmallSeg;
+    for (int base = 0; base < size; base += CL) {
+        for (int i = threadIdx.x; i < CL; i += blockDim.x) s[i] = (base + i < size) ? g[base + i] : ~0ull;
         __syncthreads();
-        for (int k = 2, lk = 1; k <= kSmallSeg; k <<= 1, ++lk) {
-            for (int t = threadIdx.x; t < kSmallSeg / 2; t += blockDim.x) {
+        for (int k = 2, lk = 1; k <= CL; k <<= 1, ++lk) {
+            for (int t = threadIdx.x; t < CL / 2; t += blockDim.x) {
                 const int blk = t >> (lk - 1), r = t & (k / 2 - 1);
                 cmpx(s, (blk << lk) + r, (blk << lk) + k - 1 - r);
             }
             __syncthreads();
             for (int j = k / 4, lj = lk - 2; j > 0; j >>= 1, --lj) {
-                for (int t = threadIdx.x; t < kSmallSeg / 2; t += blockDim.x) {
+                for (int t = threadIdx.x; t < CL / 2; t += blockDim.x) {
                     const int i = ((t >> lj) << (lj + 1)) + (t & (j - 1));
                     cmpx(s, i, i + j);
                 }
                 __syncthreads();
             }
         }
-        for (int i = threadIdx.x; i < kSmallSeg && base + i < size; i += blockDim.x) g[base + i] = s[i];
+        for (int i = threadIdx.x; i < CL && base + i < size; i += blockDim.x) g[base + i] = s[i];
         __syncthreads();
     }
     // phase B: merges of size > kSmallSeg
@@ -952,7 +1022,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     int sblocks = (int)std::min<int64_t>((n + 255) / 256, 148 * 16);
     k_scatter_keys<<<sblocks, 256, 0, s>>>(cid, pdist, n, out.off, cursor, rank_o, keys);
     cx.launched();
-    k_segsort_small<<<m, 128, 0, s>>>(keys, out.off, out.radius);
+    k_segsort_small<<<m, 256, 0, s>>>(keys, out.off, out.radius);
     cx.launched();
     k_segsort_big<<<m, 1024, 0, s>>>(keys, out.off, out.radius);
     cx.launched();
