@@ -538,3 +538,31 @@ def test_query_batches_host_memory(sknn, batch):
     assert_knn_bitexact(np.asarray(idx), np.asarray(dist), ridx, rdist)
     assert st["pairs_total"] == Q.shape[0] * T.shape[0]
     ix.close()
+
+
+SEGSORT_SIZES = [2, 31, 32, 33, 64, 65, 128, 129, 255, 256, 257, 1023, 1024, 1025, 4096, 4097]
+
+
+@pytest.mark.parametrize("n", SEGSORT_SIZES)
+def test_member_sort_bucket_boundaries(sknn, n):
+    """One cluster of exactly n members (n_clusters_t = 1) at every k_segsort_small/_big bucket edge
+    (register sort <= 32/64/128/256, smem network <= 1024, hybrid above): members ordered by distance
+    descending, index ascending (reading R11), radius = first member, then the join bit-exact."""
+    rng = np.random.default_rng(1000 + n)
+    X = rng.integers(0, 4, size=(n, 4)).astype(np.float32)   # many equal distances: tie order matters
+    ix = sknn.build(dev(X), n_clusters_t=1)
+    e = ix.export()
+    assert len(e["off"]) == 2 and e["off"][0] == 0 and e["off"][-1] == n   # det_lm_num: m = 1
+    assert np.array_equal(np.sort(e["orig"]), np.arange(n))
+    for c in range(len(e["off"]) - 1):
+        lo, hi = e["off"][c], e["off"][c + 1]
+        dd, oo = e["dist"][lo:hi], e["orig"][lo:hi]
+        ok = (dd[:-1] > dd[1:]) | ((dd[:-1] == dd[1:]) & (oo[:-1] < oo[1:]))
+        assert ok.all()
+        if hi > lo:
+            assert e["radius"][c] == dd[0]
+    ix.close()
+    k = min(8, n)
+    idx, dist, _ = run(sknn, X, X, k, True, n_clusters_t=1)
+    ridx, rdist = oracle.knn_join(X, X, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
