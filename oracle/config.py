@@ -1,8 +1,10 @@
 """The paper's adaptive-scheme arithmetic (Fig. 8, §IV-D), written out.
 
 TEST INFRASTRUCTURE ONLY (see oracle/__init__.py). The product computes the
-same decisions in C++ (csrc/config.cpp, exported through ``sknn_config_decide``);
-tests compare the two on the paper's K20c fixture and on the B200 fixture.
+same decisions in C++ (``sknn_config_decide`` in
+paper_conf_icde_chends17_b200/csrc/api.cu); tests pin this module to the
+numbers the paper prints for the K20c and to the B200
+fixture, and compare the product with it on both.
 
 Citations: P:L<n> = PAPER.md line n.
 """
@@ -58,9 +60,3 @@ def threads_per_query(nq: int, r: float, maxcur: int, cap: int | None = None) ->
     t = round_pow2_log(threads_per_query_raw(nq, r, maxcur))
     return min(t, cap) if cap else t
 
-
-def loop_split(tpq: int, nt: int, mt: int):
-    """Inner loop (Alg. 2 line 7) parallelised by |T|/|CT|, outer (line 5) by tpq/(|T|/|CT|) (reading R16)."""
-    inner = nt / mt
-    outer = tpq / inner
-    return inner, outer
