@@ -1,25 +1,46 @@
 #!/usr/bin/env python
 """Benchmark of the B200-native Sweet KNN join (one JSON line on rank 0).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2]
+                    [--mode query|target] [--exchange all_to_all|all_gather]
+                    [--impl reference]
 
-A step is one whole sknn_join (all §8(a) rows: clustering both sides, level-1
-calUB + groupFilter, level-2 filtered scan fused with top-k, result write) on
-the BASELINE.json metric's workload: C2, the 3D-road-network-shaped self-join
-(434,874 x 4, k = 20), inputs resident in HBM. Between timed steps L2 is
-flushed by writing a 512 MB buffer (untimed). N > 1 (torchrun, one process per
-GPU, NCCL process group): query sharding -- every rank clusters the replicated
-target set and processes the query clusters c with c % N == rank; no
-data-path collective; the step time is the max over ranks (strong scaling).
+A step is one whole exact KNN join (all SURVEY §8(a) rows: clustering both
+sides, level-1 calUB + groupFilter + elastic switch, dense tiles, level-2
+filtered scan fused with top-k, result write; multi-GPU: the exchange and the
+merge) on one workload, inputs resident in HBM. The default workload is
+BASELINE.json configs[1] = C2, the 3D-road-network-shaped self-join (434,874 x
+4, k = 20); --config picks C1..C5 (C4 and C5 are the configurations BASELINE
+quotes at 2/4/8 GPUs). Between timed steps L2 is flushed by writing a 512 MB
+buffer (untimed).
 
---impl reference: the CPU oracle (oracle/, brute force, all host cores) on a
-bounded sample of the same workload, timed as it stands (rank 0 only).
+N > 1: one process per GPU. Launched by torchrun (RANK/WORLD_SIZE/LOCAL_RANK
+in the environment) or, when --gpus N > 1 and WORLD_SIZE is unset, bench.py
+re-executes itself under `python -m torch.distributed.run --nproc-per-node N
+--master-addr 127.0.0.1`. Modes:
+  query   (default) query sharding, target index replicated, no data-path
+          collective: a self-join's ranks cluster the points identically and
+          take the query clusters c with c % N == rank; a Q != T join splits
+          the query rows. Strong scaling.
+  target  target sharding: rank r owns T[r*nt/N, (r+1)*nt/N), joins ALL
+          queries against it (partial k-lists, global indices), the partial
+          lists are exchanged over NCCL (all-to-all by default) and merged
+          exactly by sknn_merge_partials on the device; the step includes the
+          exchange and the merge. Strong scaling.
+The step time is the max over ranks of the per-rank CUDA-event time.
+
+--impl reference: the CPU oracle (oracle/, brute force, all host cores) timed
+as it stands on a bounded sample of the same workload (rank 0 only).
+--launcher-selftest: exercises only the launcher / process group / max-over-
+ranks reduction / JSON line (no KNN work at all; used by the CPU gloo test).
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
+import subprocess
 import sys
 import time
 
@@ -31,7 +52,12 @@ if ROOT not in sys.path:
 
 import datagen  # noqa: E402
 
-PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0}
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1590.0}
+
+
+def baseline_metric():
+    with open(os.path.join(ROOT, "BASELINE.json")) as f:
+        return json.load(f)["metric"]
 
 
 def load_peaks():
@@ -40,10 +66,20 @@ def load_peaks():
         with open(p) as f:
             d = json.load(f)
         d["_source"] = "measured (MEASURED_PEAKS.json)"
-        return d
-    d = dict(PEAKS_FALLBACK)
-    d["sm_max_mhz"] = 1965.0
-    d["_source"] = "fallback (B200_PROFILING.md)"
+    else:
+        d = dict(PEAKS_FALLBACK)
+        d["sm_max_mhz"] = 1965.0
+        d["_source"] = "fallback (B200_PROFILING.md)"
+    # fp32 FMA pipe: measured by tools/fma_peak.cu on a B200 of this pool
+    f = os.path.join(ROOT, "profiles", "r02_fma_peak.json")
+    if os.path.exists(f):
+        with open(f) as fh:
+            m = json.load(fh)
+        d["fp32_tflops"] = m["fp32_fma_tflops"]
+        d["_fp32_source"] = "measured (profiles/r02_fma_peak.json, tools/fma_peak.cu)"
+    else:
+        d["fp32_tflops"] = 148 * 128 * 2 * d.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+        d["_fp32_source"] = "derived: 148 SMs x 128 lanes x 2 flop x max SM clock"
     return d
 
 
@@ -52,6 +88,22 @@ def dist_env():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     return ws, rank, local
+
+
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def relaunch(ngpus):
+    """--gpus N > 1 without a torchrun environment: re-execute under torchrun
+    (one process per GPU, rendezvous on 127.0.0.1). Returns the exit code."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=%d" % ngpus,
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 class ClockSampler:
@@ -68,7 +120,6 @@ class ClockSampler:
         self.smax = None
         self._stop = False
         self._thr = None
-        self._nvml = None
 
     def _handle(self):
         import pynvml
@@ -86,8 +137,7 @@ class ClockSampler:
         try:
             nv, h = self._handle()
             self.smax = float(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM))
-        except Exception as e:  # pragma: no cover - no NVML
-            self._nvml_error = str(e)
+        except Exception:  # pragma: no cover - no NVML
             return
 
         def loop():
@@ -113,64 +163,157 @@ class ClockSampler:
                 "samples": len(self.samples), "reasons": sorted(self.reasons), "source": "nvml, 2 ms"}
 
 
-def cpu_baseline(cfg_name, target_s=12.0, max_queries=None):
-    """The oracle as it stands (brute force, fp64, all host threads) on a bounded
-    sample of the workload's queries against ALL its targets."""
+# ------------------------------------------------------------ CPU oracle --
+_WORKLOADS = {}
+
+
+def workload_cached(cfg_name):
+    if cfg_name not in _WORKLOADS:
+        _WORKLOADS[cfg_name] = datagen.workload(cfg_name)
+    return _WORKLOADS[cfg_name]
+
+
+def oracle_sample(cfg_name, n_queries, seed=99):
+    """The oracle as it stands (brute force, fp64, all host threads) on a
+    seeded sample of n_queries of the workload against ALL its targets."""
     import oracle
-    Q, T, k, _ = datagen.workload(cfg_name)
-    rng = np.random.default_rng(99)
-    n = 64
-    t_per = None
-    while True:
-        s = rng.choice(Q.shape[0], size=min(n, Q.shape[0]), replace=False)
-        t0 = time.perf_counter()
-        oracle.knn_join(Q[s], T, k)
-        dt = time.perf_counter() - t0
-        t_per = dt / len(s)
-        if dt >= 0.5 or n >= Q.shape[0]:
-            break
-        n *= 4
-    n_final = int(min(Q.shape[0], max(len(s), target_s / t_per)))
-    if max_queries:
-        n_final = min(n_final, max_queries)
-    s = rng.choice(Q.shape[0], size=n_final, replace=False)
+    Q, T, k, _ = workload_cached(cfg_name)
+    rng = np.random.default_rng(seed)
+    s = rng.choice(Q.shape[0], size=min(n_queries, Q.shape[0]), replace=False)
     t0 = time.perf_counter()
     oracle.knn_join(Q[s], T, k)
-    dt = time.perf_counter() - t0
-    return {"value": n_final / dt, "unit": "queries/s", "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": "%d seeded queries of %s against all %d targets (k=%d), %.1f s" % (n_final, cfg_name,
-                                                                                     T.shape[0], k, dt),
-            "seconds": dt}
+    return len(s), time.perf_counter() - t0, T.shape[0], k, oracle.num_threads()
+
+
+def calibrate_oracle(cfg_name, target_s):
+    """Number of sampled queries the oracle finishes in about target_s seconds."""
+    n = 64
+    while True:
+        ns, dt, _, _, _ = oracle_sample(cfg_name, n, seed=98)
+        if dt >= 0.5 or ns >= datagen.CONFIGS[cfg_name]["n"]:
+            break
+        n *= 4
+    return int(max(1, min(datagen.CONFIGS[cfg_name]["n"], target_s * ns / dt)))
+
+
+def cpu_baseline(cfg_name, target_s=12.0):
+    n = calibrate_oracle(cfg_name, target_s)
+    ns, dt, nt, k, cores = oracle_sample(cfg_name, n)
+    return {"value": ns / dt, "unit": "queries/s", "cores": cores, "kind": "oracle",
+            "sample": "%d seeded queries of %s against all %d targets (k=%d), %.1f s" % (ns, cfg_name, nt, k, dt)}
 
 
 def run_reference(args):
-    ws, rank, _ = dist_env()
+    """The reference arm: the CPU oracle as it stands. Each step is a bounded
+    seeded sample of the workload's queries against all targets; value =
+    sampled queries / measured seconds; ms_per_step = the measured step."""
+    _, rank, _ = dist_env()
     if rank != 0:
         return
     cfgd = datagen.CONFIGS[args.config]
-    # each step: a bounded sample (~target seconds) of the workload on the host cores
-    steps_total = args.steps + args.warmup
-    per_step = max(2.0, min(20.0, 150.0 / max(1, steps_total)))
-    times, vals = [], []
-    base = None
-    for i in range(steps_total):
-        b = cpu_baseline(args.config, target_s=per_step)
-        if i >= args.warmup:
-            vals.append(b["value"])
-            times.append(b["seconds"])
-            base = b
-    value = float(np.mean(vals))
-    nq = cfgd["n"]
-    line = {"impl": "reference", "metric": "KNN-join queries/sec (%s)" % args.config, "value": value,
-            "unit": "queries/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": 1000.0 * nq / value, "higher_is_better": True, "scaling": "strong",
+    per_step = max(1.0, min(8.0, 120.0 / max(1, args.steps)))
+    n = calibrate_oracle(args.config, per_step)
+    for i in range(args.warmup):
+        oracle_sample(args.config, max(1, n // 8), seed=1000 + i)
+    qs, secs = 0, 0.0
+    last = None
+    for i in range(args.steps):
+        ns, dt, nt, k, cores = oracle_sample(args.config, n, seed=2000 + i)
+        qs += ns
+        secs += dt
+        last = (ns, dt, nt, k, cores)
+    value = qs / secs
+    ns, dt, nt, k, cores = last
+    line = {"impl": "reference", "metric": baseline_metric(), "value": value, "unit": "queries/s",
+            "n_gpus": int(args.gpus), "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1000.0 * secs / args.steps, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": "%s: %s" % (args.config, cfgd["desc"]), "nq": nq, "nt": nq, "d": cfgd["d"],
-                       "k": cfgd["k"], "note": "ms_per_step extrapolated to the full join from the sample rate"},
-            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": base["cores"], "kind": "oracle",
-                             "sample": base["sample"]},
+            "config": {"workload": "%s: %s" % (args.config, cfgd["desc"]), "nq": cfgd["n"], "nt": cfgd["n"],
+                       "d": cfgd["d"], "k": cfgd["k"],
+                       "step": "a seeded sample of %d queries against all %d targets (brute force)" % (n, nt)},
+            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
+                             "sample": "%d steps x %d seeded queries of %s against all %d targets (k=%d), %.1f s" % (
+                                 args.steps, n, args.config, nt, k, secs)},
             "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+# -------------------------------------------------------------- roofline --
+def roofline_of(st, stage, peaks, nq_r, nt, d, k, ws):
+    """Roofline of the dominant kernel, the
+    duration from CUDA events on the launching stream (stats pass).
+
+    scan (S9-S10): bytes = query rows once + target rows as the method's reuse
+    unit fetches them (rows_loaded: once per warp tile and member for the
+    warp-union walk; once per query tile and member for the warp-per-query
+    scan) + result rows + center row and bound inputs per (tile, candidate);
+    flops = 3d per evaluated distance and per candidate-center distance +
+    log2 |tc| per (query, candidate) window search. Binding = larger fraction.
+    dense (S11): tensor flops = 2 KP per (query, target) pair covered by a
+    dense tile and MMA term, against the dense bf16 tensor peak."""
+    dpad = 4 * ((d + 3) // 4)
+    out = {}
+    scan_ms = stage["ms_sparse"]
+    if scan_ms > 0:
+        E = float(st["dist_evals_sparse"])
+        C = float(st["center_evals"])
+        Rl = float(st.get("rows_loaded", E))
+        P = float(st["cand_pairs"]) * (nq_r / max(1.0, st["mq"] / max(1, ws)))
+        tile = 32.0 if st["mapping_used"] == 1 else 8.0
+        bytes_alg = 4.0 * dpad * nq_r + (4.0 * dpad + 4.0) * Rl + 8.0 * k * nq_r + (4.0 * dpad + 16.0) * P / tile
+        flops = 3.0 * d * (E + C) + P * float(np.log2(max(2.0, nt / max(1, st["mt"]))))
+        gbs = bytes_alg / (scan_ms / 1e3) / 1e9
+        tfs = flops / (scan_ms / 1e3) / 1e12
+        f_hbm, f_alu = gbs / peaks["hbm_gbs"], tfs / peaks["fp32_tflops"]
+        if f_hbm >= f_alu:
+            b = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": f_hbm}
+        else:
+            b = {"bound": "alu", "achieved": tfs, "peak": peaks["fp32_tflops"], "unit": "TFLOP/s", "frac": f_alu}
+        b.update({"kernel": "k_scan_%s (level-2 scan fused with top-k)" % ("tpq" if st["mapping_used"] == 1 else "wpq"),
+                  "launch_ms": scan_ms, "algorithmic_bytes": bytes_alg, "algorithmic_flops": flops,
+                  "intensity_flop_per_byte": flops / bytes_alg if bytes_alg else None,
+                  "hbm": {"achieved_gbs": gbs, "peak_gbs": peaks["hbm_gbs"], "frac": f_hbm},
+                  "alu": {"achieved_tflops": tfs, "peak_tflops": peaks["fp32_tflops"], "frac": f_alu}})
+        out["scan"] = b
+    dense_ms = stage.get("ms_dense", 0.0)
+    if dense_ms > 0 and st["dist_evals_dense"]:
+        kp = 16 * ((dpad + 15) // 16)
+        terms = float(st.get("dense_terms", 1) or 1)
+        flops = 2.0 * kp * float(st["dist_evals_dense"]) * terms
+        tfs = flops / (dense_ms / 1e3) / 1e12
+        pk = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+        out["dense"] = {"bound": "tensor", "achieved": tfs, "peak": pk, "unit": "TFLOP/s", "frac": tfs / pk,
+                        "kernel": "k_dense (tcgen05 bf16 screen + exact fp32 recompute)", "launch_ms": dense_ms,
+                        "algorithmic_flops": flops, "mma_terms": terms}
+    if not out:
+        return None
+    dom = max(out, key=lambda s: out[s]["launch_ms"])
+    r = dict(out[dom])
+    r["others"] = {s: {kk: v for kk, v in out[s].items() if kk in ("kernel", "bound", "frac", "launch_ms")}
+                   for s in out if s != dom}
+    return r
+
+
+# ------------------------------------------------------------------ main --
+def launcher_selftest(args):
+    """No KNN work: process group + max-over-ranks timing + the JSON line."""
+    import torch
+    import torch.distributed as dist
+    ws, rank, _ = dist_env()
+    if ws > 1:
+        dist.init_process_group("gloo")
+    t0 = time.perf_counter()
+    time.sleep(0.01 * (rank + 1))
+    ms = (time.perf_counter() - t0) * 1e3
+    if ws > 1:
+        t = torch.tensor([ms])
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    if rank == 0:
+        print(json.dumps({"selftest": True, "metric": baseline_metric(), "n_gpus": ws, "ms_per_step": ms,
+                          "ranks_seen": ws}), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
 
 
 def main():
@@ -179,20 +322,30 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C2")
+    ap.add_argument("--mode", default="query", choices=["query", "target"])
+    ap.add_argument("--exchange", default="all_to_all", choices=["all_to_all", "all_gather"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--mapping", default="auto")
+    ap.add_argument("--launcher-selftest", action="store_true")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
     if args.impl == "reference":
         run_reference(args)
         return
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch(args.gpus))
+    if args.launcher_selftest:
+        launcher_selftest(args)
+        return
 
     import torch
     import torch.distributed as dist
 
     import paper_conf_icde_chends17_b200 as sknn
+    from paper_conf_icde_chends17_b200 import dist as sdist
 
     ws, rank, local = dist_env()
     torch.cuda.set_device(local)
@@ -203,37 +356,72 @@ def main():
     peaks = load_peaks()
 
     cfgd = datagen.CONFIGS[args.config]
-    Qh, Th, k, self_join = datagen.workload(args.config)
+    Qh, Th, k, self_join = workload_cached(args.config)
     nq, nt, d = Qh.shape[0], Th.shape[0], Qh.shape[1]
     Q = torch.from_numpy(Qh).to(dev)
     T = Q if self_join else torch.from_numpy(Th).to(dev)
-    out_idx = torch.empty((nq, k), dtype=torch.int32, device=dev)
-    out_dist = torch.empty((nq, k), dtype=torch.float32, device=dev)
     flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     opts = dict(mapping=args.mapping)
-    if ws > 1:
-        opts.update(shard_rank=rank, shard_count=ws)
 
-    def step(stats=False):
-        return sknn.join(Q, T, k, out=(out_idx, out_dist), stats=stats, stream=stream, **opts)
+    # ---- the per-rank step (and the stats call of its local join) ----
+    if args.mode == "query":
+        out_idx = torch.empty((nq, k), dtype=torch.int32, device=dev)
+        out_dist = torch.empty((nq, k), dtype=torch.float32, device=dev)
+        if self_join:
+            if ws > 1:
+                opts.update(shard_rank=rank, shard_count=ws)
+            lo, hi = 0, nq
+            Qr, Tr, oi, od = Q, Q, out_idx, out_dist
+        else:
+            lo, hi = sdist.shard_bounds(nq, ws, rank)
+            Qr, Tr, oi, od = Q[lo:hi], T, out_idx[lo:hi], out_dist[lo:hi]
+
+        def local_join(stats=False):
+            return sknn.join(Qr, Tr, k, out=(oi, od), stats=stats, stream=stream, **opts)
+
+        def step():
+            local_join()
+        parallelism = "query-sharded x%d (target index replicated, no data-path collective)" % ws
+        nq_rank = (nq / ws) if self_join else (hi - lo)
+    else:
+        tlo, thi = sdist.shard_bounds(nt, ws, rank)
+        Tshard = T[tlo:thi].contiguous()
+        group = None
+
+        def local_join(stats=False):
+            return sknn.join(Q, Tshard, min(k, thi - tlo), stats=stats, stream=stream, out_squared=1,
+                             index_base=int(tlo), **opts)
+
+        def step():
+            if ws == 1:
+                local_join()
+            else:
+                sdist.join_target_sharded(Q, Tshard, k, tlo, group=group, exchange=args.exchange, gather=False,
+                                          **opts)
+        parallelism = "target-sharded x%d (%s exchange of partial k-lists + exact merge)" % (
+            ws, args.exchange if ws > 1 else "no")
+        nq_rank = nq
 
     for _ in range(args.warmup):
         flush.zero_()
         step()
     torch.cuda.synchronize()
 
-    # stats pass (untimed): per-stage CUDA events, counters and the launch count
-    # of one join; the stage split is the mean over a few such joins
-    stage = {"ms_build_t": 0.0, "ms_level1": 0.0, "ms_sparse": 0.0, "ms_total": 0.0}
+    # stats pass (untimed): per-stage CUDA events, counters and the launch
+    # count of the local join; the stage split is the mean over a few joins
+    stage = {"ms_build_t": 0.0, "ms_build_q": 0.0, "ms_level1": 0.0, "ms_dense": 0.0, "ms_sparse": 0.0,
+             "ms_total": 0.0}
     n_stats = 3
     last = None
     for _ in range(n_stats):
         flush.zero_()
-        _, _, st = step(stats=True)
+        st = local_join(stats=True)[2]
         for key in stage:
             stage[key] += st[key]
         last = st
-    launches_per_step = last["kernel_launches"]
+    for key in stage:
+        stage[key] /= n_stats
+    launches_per_step = last["kernel_launches"] + (1 if (args.mode == "target" and ws > 1) else 0)  # + k_merge
 
     clocks = ClockSampler(local)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
@@ -249,113 +437,125 @@ def main():
     torch.cuda.synchronize()
     if ws > 1:
         dist.barrier()
-    launches = launches_per_step * args.steps
     clk = clocks.stop()
     ms = [a.elapsed_time(b) for a, b in ev]
     ms_step = float(np.mean(ms))
+    evals_all = float(last["dist_evals"])
+    launches = launches_per_step * args.steps
     if ws > 1:
         t = torch.tensor([ms_step], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms_step = float(t.item())
-        ev_t = torch.tensor([last["dist_evals"], last["pairs_total"]], dtype=torch.float64, device=dev)
-        dist.all_reduce(ev_t)
-        evals_all = float(ev_t[0].item())
-    else:
-        evals_all = float(last["dist_evals"])
+        sums = torch.tensor([evals_all, float(launches)], dtype=torch.float64, device=dev)
+        dist.all_reduce(sums)
+        evals_all, launches = float(sums[0].item()), int(sums[1].item())
     value = nq / (ms_step / 1000.0)
-    for key in stage:
-        stage[key] /= n_stats
 
-    # ---- roofline of the dominant kernel (the level-2 scan), its duration
-    # from CUDA events on the launching stream (stats pass above) ----
-    # Algorithmic work per launch, SURVEY.md §8(d) "Sparse (S9-S10)":
-    #  bytes = query rows once + target rows (row + member distance) as the
-    #          method's reuse unit fetches them -- once per warp tile and member
-    #          for the warp-union walk (counter rows_loaded) -- + result rows;
-    #          per-(tile, candidate) center rows and bound inputs, 4*dp + 16 B
-    #  flops = 3d per evaluated distance and per candidate-center distance
-    #          + log2 |tc| per (query, candidate) window search
-    # The binding roofline is the one with the larger fraction.
-    scan_ms = stage["ms_sparse"]
-    dpad = 4 * ((d + 3) // 4)
-    E = float(last["dist_evals_sparse"])
-    C = float(last["center_evals"])
-    Rl = float(last.get("rows_loaded", E))
-    nq_r = nq / max(1, ws)
-    P = float(last["cand_pairs"]) * (nq_r / max(1, last["mq"] / max(1, ws)))  # (query, candidate) pairs
-    bytes_alg = 4.0 * dpad * nq_r + (4.0 * dpad + 4.0) * Rl + 8.0 * k * nq_r + (4.0 * dpad + 16.0) * P / 32.0
-    tc_mean = nt / max(1, last["mt"])
-    flops = 3.0 * d * (E + C) + P * float(np.log2(max(2.0, tc_mean)))
-    sm_mhz = peaks.get("sm_max_mhz", 1965.0)
-    alu_peak_tflops = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
-    hbm = peaks.get("hbm_gbs")
-    achieved_gbs = bytes_alg / (scan_ms / 1000.0) / 1e9 if scan_ms > 0 else 0.0
-    achieved_tf = flops / (scan_ms / 1000.0) / 1e12 if scan_ms > 0 else 0.0
-    f_hbm = achieved_gbs / hbm if hbm else 0.0
-    f_alu = achieved_tf / alu_peak_tflops
-    if f_hbm >= f_alu:
-        bound, achieved, peak, unit, frac = "hbm", achieved_gbs, hbm, "GB/s", f_hbm
-    else:
-        bound, achieved, peak, unit, frac = "alu", achieved_tf, alu_peak_tflops, "TFLOP/s", f_alu
-    roofline = {"kernel": "k_scan_tpq (level-2 warp-union scan fused with top-k)", "bound": bound,
-                "achieved": achieved, "peak": peak, "unit": unit, "frac": frac,
-                "traffic": None, "launch_ms": scan_ms, "algorithmic_bytes": bytes_alg,
-                "algorithmic_flops": flops, "intensity_flop_per_byte": flops / bytes_alg if bytes_alg else None,
-                "hbm": {"achieved_gbs": achieved_gbs, "peak_gbs": hbm, "frac": f_hbm},
-                "alu": {"achieved_tflops": achieved_tf, "peak_tflops": alu_peak_tflops, "frac": f_alu},
-                "peak_source": "HBM %s; fp32 FMA pipe derived: 148 SMs x 128 lanes x 2 flop x %.0f MHz" % (
-                    peaks["_source"], sm_mhz),
-                "share_of_step": scan_ms / ms_step if ms_step else None,
-                "note": "issue-bound (control flow and kNearests updates), not DRAM- or FMA-bound; see DESIGN.md §6"}
-    tf = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tf):
-        try:
-            with open(tf) as f:
-                roofline["traffic"] = json.load(f).get(args.config)
-        except Exception:
-            pass
+    roof = roofline_of(last, stage, peaks, nq_rank, nt if args.mode == "query" else (thi - tlo), d, k, ws)
+    if roof is not None:
+        roof["peak_source"] = "HBM/bf16 %s; fp32 FMA %s" % (peaks["_source"], peaks["_fp32_source"])
+        roof["share_of_step"] = roof["launch_ms"] / ms_step if ms_step else None
+        roof["traffic"] = None
+        tf = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tf):
+            try:
+                with open(tf) as f:
+                    tr = json.load(f).get(args.config)
+                if isinstance(tr, dict):
+                    tr = tr.get(roof["kernel"].split()[0])
+                roof["traffic"] = tr
+            except Exception:
+                pass
 
-    # ---- end-to-end through the C ABI with host (pinned) buffers ----
+    # ---- end to end through the public API with host (pinned) buffers ----
     e2e = None
-    if ws == 1:
-        Qp = torch.from_numpy(Qh).pin_memory()
-        Tp = Qp if self_join else torch.from_numpy(Th).pin_memory()
-        oi = torch.empty((nq, k), dtype=torch.int32).pin_memory()
-        od = torch.empty((nq, k), dtype=torch.float32).pin_memory()
-        host_args = (Qp, Tp)
-        for _ in range(2):
-            sknn.join(host_args[0], host_args[1], k, out=(oi, od))
-        t0 = time.perf_counter()
-        reps = max(3, args.steps // 2)
-        for _ in range(reps):
-            sknn.join(host_args[0], host_args[1], k, out=(oi, od))   # H2D + join + D2H + sync inside
-        e2e_s = (time.perf_counter() - t0) / reps
-        h2d = nq * d * 4 + (0 if self_join else nt * d * 4)
-        e2e = {"value": nq / e2e_s, "unit": "queries/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": nq * k * 8,
-               "ms_per_step": e2e_s * 1000.0, "timer": "host wall clock around the blocking C-ABI call"}
+    if not args.no_e2e:
+        e2e = measure_e2e(args, sknn, sdist, Qh, Th, k, self_join, ws, rank, dev, opts)
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(args.config)
-        cpu.pop("seconds", None)
 
     if rank == 0:
-        pruned = 100.0 * (1.0 - evals_all / (float(nq) * nt))
-        line = {"metric": "KNN-join queries/sec (%s); %% distance computations pruned" % args.config,
-                "value": value, "unit": "queries/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
-                "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
+        pairs = float(nq) * nt
+        line = {"metric": baseline_metric(), "value": value, "unit": "queries/s", "n_gpus": ws, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": {"workload": "%s: %s" % (args.config, cfgd["desc"]), "nq": nq, "nt": nt, "d": d, "k": k,
-                           "self_join": self_join, "parallelism": "query-sharded x%d (target index replicated)" % ws,
+                           "self_join": self_join, "mode": args.mode, "parallelism": parallelism,
                            "l2": "flushed between steps (512 MB write, untimed)", "mapping": last["mapping_used"],
                            "mq": last["mq"], "mt": last["mt"]},
-                "pruned_pct": pruned, "dist_evals": evals_all, "joins_per_s": 1000.0 / ms_step,
-                "stage_ms": stage, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
-                "gpu_launches": launches, "clocks": clk}
+                "pruned_pct": 100.0 * (1.0 - evals_all / pairs), "dist_evals": evals_all,
+                "joins_per_s": 1000.0 / ms_step, "stage_ms": stage, "roofline": roof, "cpu_baseline": cpu,
+                "e2e": e2e, "gpu_launches": launches, "clocks": clk}
         print(json.dumps(line), flush=True)
     if ws > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def measure_e2e(args, sknn, sdist, Qh, Th, k, self_join, ws, rank, dev, opts):
+    """The same metric through the public API with HOST buffers: every step
+    copies that step's inputs from pinned host memory to the device and reads
+    the step's result back (inside the timed region), then synchronises; the
+    step time is the max over ranks of the host clock around it."""
+    import torch
+    import torch.distributed as dist
+    nq, nt, d = Qh.shape[0], Th.shape[0], Qh.shape[1]
+    Qp = torch.from_numpy(Qh).pin_memory()
+    Tp = Qp if self_join else torch.from_numpy(Th).pin_memory()
+    if args.mode == "query":
+        if self_join:
+            oi = torch.empty((nq, k), dtype=torch.int32).pin_memory()
+            od = torch.empty((nq, k), dtype=torch.float32).pin_memory()
+
+            def e2e_step():  # the C ABI stages the host arrays (H2D, join, D2H, sync inside)
+                sknn.join(Qp, Qp, k, out=(oi, od), **opts)
+            h2d, d2h = nq * d * 4, nq * k * 8
+        else:
+            lo, hi = sdist.shard_bounds(nq, ws, rank)
+            Qs = Qp[lo:hi]
+            oi = torch.empty((hi - lo, k), dtype=torch.int32).pin_memory()
+            od = torch.empty((hi - lo, k), dtype=torch.float32).pin_memory()
+
+            def e2e_step():
+                sknn.join(Qs, Tp, k, out=(oi, od), **opts)
+            h2d, d2h = (hi - lo) * d * 4 + nt * d * 4, (hi - lo) * k * 8
+    else:
+        tlo, thi = sdist.shard_bounds(nt, ws, rank)
+        Ts = Tp[tlo:thi]
+        lo, hi = sdist.shard_bounds(nq, ws, rank)
+        oi = torch.empty((hi - lo, k), dtype=torch.int32).pin_memory()
+        od = torch.empty((hi - lo, k), dtype=torch.float32).pin_memory()
+        stream = torch.cuda.current_stream()
+
+        def e2e_step():
+            dQ = Qp.to(dev, non_blocking=True)
+            dT = Ts.to(dev, non_blocking=True)
+            if ws == 1:
+                ri, rd = sknn.join(dQ, dT, k, stream=stream, **opts)
+            else:
+                ri, rd = sdist.join_target_sharded(dQ, dT, k, tlo, exchange=args.exchange, gather=False, **opts)
+            oi.copy_(ri, non_blocking=True)
+            od.copy_(rd, non_blocking=True)
+            torch.cuda.synchronize()
+        h2d, d2h = nq * d * 4 + (thi - tlo) * d * 4, (hi - lo) * k * 8
+    for _ in range(2):
+        e2e_step()
+    reps = max(3, args.steps // 2)
+    if ws > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        e2e_step()
+    s = (time.perf_counter() - t0) / reps
+    if ws > 1:
+        t = torch.tensor([s], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        s = float(t.item())
+    return {"value": nq / s, "unit": "queries/s", "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+            "ms_per_step": s * 1000.0, "per_rank_bytes": ws > 1,
+            "timer": "host wall clock around the blocking call, max over ranks"}
 
 
 if __name__ == "__main__":

@@ -67,7 +67,7 @@ typedef enum {
  * kNearests placement follows Fig. 8: shared memory for
  * k*4 <= th1, registers for k <= 32, shared memory with fewer threads per CTA
  * beyond. k > 32 uses the thread-per-query scan only (no dense tiles, no
- * brute-force path); sknn_merge_partials supports k > 32 with P <= 16. */
+ * brute-force path). */
 #define SKNN_MAX_K 512
 
 /* Execution-path override (sknn_options.force_path). */
@@ -111,6 +111,15 @@ typedef struct {
     int64_t query_batch;      /* sknn_query with HOST queries and outputs (out-of-core, the paper's */
                               /*   query partitions P:L575): queries per device batch; 0 = auto   */
                               /*   (all at once when they fit in 40% of the free device memory)   */
+    int32_t self_query;       /* sknn_query / sknn_debug_level1: is Q the index's build set (reuse */
+                              /*   its clustering for the query side, a self-join)?        */
+                              /*   1 = yes (caller asserts Q holds the build rows), -1 = never,     */
+                              /*   0 = auto: yes iff Q is the SAME POINTER and size as the build    */
+                              /*   input -- the build buffer must then still be alive and unchanged */
+                              /*   (a freed-and-reused address would silently answer for old rows) */
+    int32_t use_graph;        /* sknn_join_ex on device pointers without stats: 0 = auto (replay a */
+                              /*   captured CUDA graph of the whole join when the same shapes,     */
+                              /*   pointers and options repeat), -1 = never                         */
 } sknn_options;
 
 /* Counters and per-stage times of one call (filled only when a non-NULL
@@ -135,6 +144,9 @@ typedef struct {
     uint64_t topk_inserts;         /* kNearests updates by the level-2 scan (P:L453 update overhead)   */
     uint64_t rows_loaded;          /* target rows fetched by the level-2 scan: once per warp for the  */
                                    /*   warp-union walk, once per evaluation otherwise (§8(d) bytes)  */
+    uint32_t dense_terms;          /* bf16 MMA terms per K-step of the dense tiles: 1 = exact integer */
+                                   /*   tiles (hi parts only), 2-3 = split-precision screen; 0 = none */
+    uint32_t pad1;
 } sknn_stats;
 
 /* Opaque resident target index (sknn_build / sknn_query). Owns device memory:
@@ -209,7 +221,8 @@ sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq,
  * fp32 SQUARED distances, each row sorted ascending by (d2, idx) (as written
  * by sknn_query with out_squared = 1). Output: the k smallest (d2, idx) keys
  * of each query over all P lists; out_dist gets sqrt(d2) unless
- * out_squared != 0. Device pointers only. */
+ * out_squared != 0. Any P >= 1 and k <= SKNN_MAX_K (one warp per query,
+ * bitonic merge of sorted lists). Device pointers only. */
 sknn_status sknn_merge_partials(const int32_t* part_idx, const float* part_d2,
                                 int32_t P, int64_t nq, int32_t k,
                                 int32_t* out_idx, float* out_dist,
@@ -229,6 +242,32 @@ sknn_status sknn_index_info(const sknn_index* index, int64_t* nt, int32_t* d,
  * [mt x dp], radius [mt] (max member distance, 0 for an empty cluster). */
 sknn_status sknn_index_export(const sknn_index* index, int32_t* off, int32_t* orig,
                               float* dist, float* centers, float* radius);
+
+/* Device arrays of an index (no copy): the build-once-and-share path of the
+ * multi-GPU query-sharded mode ("rank 0 builds and broadcasts
+ * it", e.g. ncclBroadcast over NVLink). ptr[i] / bytes[i] for i in
+ * SKNN_INDEX_ARRAY_*; the arrays stay owned by the index. Writing into them is
+ * allowed only for an index made by sknn_index_create and before any query. */
+enum {
+    SKNN_INDEX_ARRAY_ROWS = 0,    /* [nt x dp] fp32 points in cluster order        */
+    SKNN_INDEX_ARRAY_DIST = 1,    /* [nt] fp32 member-to-center distance          */
+    SKNN_INDEX_ARRAY_ORIG = 2,    /* [nt] int32 original row index                 */
+    SKNN_INDEX_ARRAY_OFF = 3,     /* [mt+1] int32 cluster offsets                  */
+    SKNN_INDEX_ARRAY_CENTERS = 4, /* [mt x dp] fp32                                */
+    SKNN_INDEX_ARRAY_RADIUS = 5,  /* [mt] fp32                                     */
+    SKNN_INDEX_ARRAY_TINFO = 6,   /* [mt] int4 {lo, hi, radius bits, min dist bits} */
+    SKNN_INDEX_ARRAYS = 7
+};
+sknn_status sknn_index_arrays(const sknn_index* index, void** ptr, size_t* bytes);
+
+/* An index of the given geometry with allocated but UNINITIALISED arrays on
+ * the current device, to be filled through sknn_index_arrays with the arrays
+ * of an index built elsewhere (same nt, d, mt; e.g. broadcast from rank 0).
+ * opt is stored as the index's default options (NULL = defaults). The index
+ * has no build input pointer: self-joins through it need
+ * sknn_options.self_query = 1. */
+sknn_status sknn_index_create(int64_t nt, int32_t d, int32_t mt, const sknn_options* opt,
+                              sknn_index** out);
 
 /* Level-1 products of a query against an index, to HOST buffers (testing):
  * q_cluster [nq] cluster of each query, ub [mq] the inflated upper bound of

@@ -33,7 +33,8 @@ MAX_K = 512
 ABI_SYMBOLS = ["sknn_options_default", "sknn_join", "sknn_join_ex", "sknn_build", "sknn_query",
                "sknn_merge_partials", "sknn_index_free", "sknn_index_info", "sknn_index_export",
                "sknn_debug_level1", "sknn_config_decide", "sknn_error_string", "sknn_last_error",
-               "sknn_version"]
+               "sknn_version", "sknn_index_arrays", "sknn_index_create"]
+INDEX_ARRAYS = ("rows", "dist", "orig", "off", "centers", "radius", "tinfo")
 
 
 class SknnError(RuntimeError):
@@ -48,7 +49,8 @@ class Options(ctypes.Structure):
                 ("lloyd_iters", ctypes.c_int32), ("seed", ctypes.c_uint64), ("force_path", ctypes.c_int32),
                 ("mapping", ctypes.c_int32), ("dense_threshold", ctypes.c_float), ("r_factor", ctypes.c_float),
                 ("out_squared", ctypes.c_int32), ("pad0", ctypes.c_int32), ("index_base", ctypes.c_int64),
-                ("shard_rank", ctypes.c_int32), ("shard_count", ctypes.c_int32), ("query_batch", ctypes.c_int64)]
+                ("shard_rank", ctypes.c_int32), ("shard_count", ctypes.c_int32), ("query_batch", ctypes.c_int64),
+                ("self_query", ctypes.c_int32), ("use_graph", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -62,10 +64,10 @@ class Stats(ctypes.Structure):
                 ("ms_final", ctypes.c_float), ("mapping_used", ctypes.c_int32), ("path_used", ctypes.c_int32),
                 ("mq", ctypes.c_int32), ("mt", ctypes.c_int32), ("kernel_launches", ctypes.c_int32),
                 ("pad0", ctypes.c_int32), ("topk_inserts", ctypes.c_uint64),
-                ("rows_loaded", ctypes.c_uint64)]
+                ("rows_loaded", ctypes.c_uint64), ("dense_terms", ctypes.c_uint32), ("pad1", ctypes.c_uint32)]
 
     def to_dict(self):
-        d = {name: getattr(self, name) for name, _ in self._fields_ if name not in ("struct_size", "pad0")}
+        d = {name: getattr(self, name) for name, _ in self._fields_ if name not in ("struct_size", "pad0", "pad1")}
         evals = self.dist_evals_sparse + self.dist_evals_dense + self.dist_evals_brute
         d["dist_evals"] = evals
         d["pruned_pct"] = 100.0 * (self.pairs_total - evals) / self.pairs_total if self.pairs_total else 0.0
@@ -123,9 +125,11 @@ def lib():
             L.sknn_error_string.restype = ctypes.c_char_p
             L.sknn_last_error.restype = ctypes.c_char_p
             L.sknn_version.restype = _i32
+            L.sknn_index_arrays.argtypes = [_vp, ctypes.POINTER(_vp), ctypes.POINTER(ctypes.c_size_t)]
+            L.sknn_index_create.argtypes = [_i64, _i32, _i32, ctypes.POINTER(Options), ctypes.POINTER(_vp)]
             for fn in ("sknn_join", "sknn_join_ex", "sknn_build", "sknn_query", "sknn_merge_partials",
                        "sknn_index_free", "sknn_index_info", "sknn_index_export", "sknn_debug_level1",
-                       "sknn_config_decide"):
+                       "sknn_config_decide", "sknn_index_arrays", "sknn_index_create"):
                 getattr(L, fn).restype = _i32
             _lib = L
     return _lib
@@ -152,13 +156,36 @@ def make_options(**kw) -> Options:
     return o
 
 
-def _stream_ptr(stream):
+def _stream_ptr(stream, device=None):
+    """The stream to enqueue on: `stream`, else torch's current stream of the
+    tensors' device (not of the current device: ADVICE r1)."""
     if stream is None:
         import torch
         if torch.cuda.is_available():
-            return torch.cuda.current_stream().cuda_stream
+            return torch.cuda.current_stream(device).cuda_stream
         return None
     return getattr(stream, "cuda_stream", stream)
+
+
+class _on_device:
+    """Make the tensors' CUDA device current for the C call (the library checks
+    pointers against cudaGetDevice()); a no-op for host arrays."""
+
+    def __init__(self, device):
+        self.device = device
+        self._ctx = None
+
+    def __enter__(self):
+        if self.device is not None and getattr(self.device, "type", None) == "cuda":
+            import torch
+            self._ctx = torch.cuda.device(self.device)
+            self._ctx.__enter__()
+        return self
+
+    def __exit__(self, *exc):
+        if self._ctx is not None:
+            self._ctx.__exit__(*exc)
+        return False
 
 
 def _as_points(X):
@@ -212,8 +239,10 @@ def join(Q, T, k: int, *, stream=None, stats: bool = False, with_index: bool = T
     o = make_options(**opts)
     st = Stats()
     st.struct_size = ctypes.sizeof(Stats)
-    _check(lib().sknn_join_ex(qp, nq, tp, nt, d, k, ip, dp_, ctypes.byref(o),
-                              ctypes.byref(st) if stats else None, _stream_ptr(stream) if qcuda else None))
+    qdev = qkeep.device if qcuda else None
+    with _on_device(qdev):
+        _check(lib().sknn_join_ex(qp, nq, tp, nt, d, k, ip, dp_, ctypes.byref(o),
+                                  ctypes.byref(st) if stats else None, _stream_ptr(stream, qdev) if qcuda else None))
     if stats:
         return idx, dist, st.to_dict()
     return idx, dist
@@ -227,9 +256,36 @@ class Index:
         self._keep = keep  # the index remembers T's pointer for self-join detection
         self._handle = ctypes.c_void_p()
         o = make_options(**opts)
-        _check(lib().sknn_build(tp, nt, d, ctypes.byref(o), ctypes.byref(self._handle),
-                                _stream_ptr(stream) if cuda else None))
+        tdev = keep.device if cuda else None
+        with _on_device(tdev):
+            _check(lib().sknn_build(tp, nt, d, ctypes.byref(o), ctypes.byref(self._handle),
+                                    _stream_ptr(stream, tdev) if cuda else None))
         self.nt, self.d = nt, d
+
+    @classmethod
+    def create(cls, nt: int, d: int, mt: int, **opts):
+        """An index of this geometry with uninitialised device arrays (to be
+        filled, e.g. by a broadcast of another rank's index: dist.py)."""
+        self = cls.__new__(cls)
+        self._keep = None
+        self._handle = ctypes.c_void_p()
+        o = make_options(**opts)
+        _check(lib().sknn_index_create(nt, d, mt, ctypes.byref(o), ctypes.byref(self._handle)))
+        self.nt, self.d = nt, d
+        return self
+
+    def arrays(self):
+        """The index's device arrays as torch uint8 tensors (views, no copy),
+        in INDEX_ARRAYS order."""
+        import torch
+        ptr = (_vp * len(INDEX_ARRAYS))()
+        nb = (ctypes.c_size_t * len(INDEX_ARRAYS))()
+        _check(lib().sknn_index_arrays(self._handle, ptr, nb))
+        dev = torch.cuda.current_device()
+        out = []
+        for i in range(len(INDEX_ARRAYS)):
+            out.append(_device_bytes(ptr[i], nb[i], dev, owner=self))
+        return out
 
     def info(self):
         nt, d, dp, mt, dev = _i64(), _i32(), _i32(), _i32(), _i32()
@@ -263,8 +319,10 @@ class Index:
         o = make_options(**opts) if opts else None
         st = Stats()
         st.struct_size = ctypes.sizeof(Stats)
-        _check(lib().sknn_query(self._handle, qp, nq, k, ip, dp_, ctypes.byref(o) if o is not None else None,
-                                ctypes.byref(st) if stats else None, _stream_ptr(stream) if qcuda else None))
+        qdev = qkeep.device if qcuda else None
+        with _on_device(qdev):
+            _check(lib().sknn_query(self._handle, qp, nq, k, ip, dp_, ctypes.byref(o) if o is not None else None,
+                                    ctypes.byref(st) if stats else None, _stream_ptr(stream, qdev) if qcuda else None))
         if stats:
             return idx, dist, st.to_dict()
         return idx, dist
@@ -297,11 +355,25 @@ class Index:
             pass
 
 
+class _DevBuf:
+    """__cuda_array_interface__ view of library-owned device bytes."""
+
+    def __init__(self, ptr, nbytes, owner):
+        self.__cuda_array_interface__ = {"shape": (int(nbytes),), "typestr": "|u1", "data": (int(ptr), False),
+                                         "version": 3, "strides": None, "stream": None}
+        self._owner = owner
+
+
+def _device_bytes(ptr, nbytes, device, owner):
+    import torch
+    return torch.as_tensor(_DevBuf(ptr, nbytes, owner), device=torch.device("cuda", device))
+
+
 def build(T, **opts) -> Index:
     return Index(T, **opts)
 
 
-def merge_partials(part_idx, part_d2, k: int, *, out_squared: bool = False, stream=None):
+def merge_partials(part_idx, part_d2, k: int, *, out_squared: bool = False, stream=None, out=None):
     """Merge [P, nq, k] sorted partial lists (torch CUDA int32 / fp32 squared
     distances, global indices) into the k nearest per query (sknn_merge_partials)."""
     import torch
@@ -309,10 +381,15 @@ def merge_partials(part_idx, part_d2, k: int, *, out_squared: bool = False, stre
     assert kk == k and part_idx.shape == part_d2.shape
     part_idx = part_idx.contiguous()
     part_d2 = part_d2.contiguous()
-    idx = torch.empty((nq, k), dtype=torch.int32, device=part_d2.device)
-    dist = torch.empty((nq, k), dtype=torch.float32, device=part_d2.device)
-    _check(lib().sknn_merge_partials(part_idx.data_ptr(), part_d2.data_ptr(), P, nq, k, idx.data_ptr(),
-                                     dist.data_ptr(), int(out_squared), _stream_ptr(stream)))
+    if out is not None:
+        idx, dist = out
+    else:
+        idx = torch.empty((nq, k), dtype=torch.int32, device=part_d2.device)
+        dist = torch.empty((nq, k), dtype=torch.float32, device=part_d2.device)
+    with _on_device(part_d2.device):
+        _check(lib().sknn_merge_partials(part_idx.data_ptr(), part_d2.data_ptr(), P, nq, k,
+                                         idx.data_ptr() if idx is not None else None, dist.data_ptr(),
+                                         int(out_squared), _stream_ptr(stream, part_d2.device)))
     return idx, dist
 
 

@@ -60,14 +60,51 @@ static sknn_status device_info(DevInfo& di) {
     if (di.major != 10 || di.minor != 0)
         return fail(SKNN_ERR_UNSUPPORTED, "device " + std::to_string(dev) + " is sm_" + std::to_string(p.major) +
                                               std::to_string(p.minor) + "; this library is built for sm_100a (B200)");
-    // keep freed scratch in the pool between calls
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-        uint64_t thr = UINT64_MAX;
-        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
+    if (!scratch_pool(dev)) return fail(SKNN_ERR_CUDA, "cudaMemPoolCreate failed");
     if (dev >= 0 && dev < 64) cache[dev] = di;
     return SKNN_OK;
+}
+
+// Private stream-ordered pool per device. Freed scratch stays reserved up to
+// kPoolRetainBytes between calls (repeated joins reuse it without new
+// cudaMalloc work); above that the driver releases it at synchronisation.
+constexpr uint64_t kPoolRetainBytes = uint64_t(2) << 30;
+
+cudaMemPool_t scratch_pool(int device) {
+    static std::mutex mu;
+    static cudaMemPool_t pools[64] = {};
+    if (device < 0 || device >= 64) return nullptr;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!pools[device]) {
+        cudaMemPoolProps props;
+        memset(&props, 0, sizeof(props));
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = device;
+        cudaMemPool_t p = nullptr;
+        if (cudaMemPoolCreate(&p, &props) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        uint64_t thr = kPoolRetainBytes;
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[device] = p;
+    }
+    return pools[device];
+}
+
+size_t usable_free_bytes(int device) {
+    size_t free_b = 0, tot_b = 0;
+    if (cudaMemGetInfo(&free_b, &tot_b) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    cudaMemPool_t p = scratch_pool(device);
+    uint64_t reserved = 0, used = 0;
+    if (p && cudaMemPoolGetAttribute(p, cudaMemPoolAttrReservedMemCurrent, &reserved) == cudaSuccess &&
+        cudaMemPoolGetAttribute(p, cudaMemPoolAttrUsedMemCurrent, &used) == cudaSuccess && reserved > used)
+        free_b += (size_t)(reserved - used);
+    return free_b;
 }
 
 static sknn_options merge_options(const sknn_options* o) {
@@ -83,6 +120,14 @@ static sknn_options merge_options(const sknn_options* o) {
     if (d.r_factor <= 0.f) d.r_factor = 0.25f;
     if (d.shard_count <= 1) { d.shard_count = 1; d.shard_rank = 0; }
     return d;
+}
+
+// Is the query array the index's build set (sknn_options.self_query)?
+static bool index_self_query(const sknn_options& o, const void* Q, int64_t nq, const sknn_index* ix) {
+    if (o.self_query < 0) return false;
+    if (nq != ix->t.n) return false;
+    if (o.self_query > 0) return true;
+    return Q == ix->user_ptr;
 }
 
 enum PtrKind { PTR_DEVICE, PTR_HOST, PTR_BAD };
@@ -278,6 +323,11 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
         SKNN_TRY(run_partial(cx, qs, ts, l1, sp, &fell_back));
         full = fell_back;
         if (!fell_back) *path_used = SKNN_PATH_PARTIAL;
+        // the full filter runs instead: its own task list (the partial passes'
+        // 32-query split tasks are only valid for the thread-per-query scan)
+        if (fell_back && scan_tile_size(mapping, ts.dp, k) != tile)
+            SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp, k), k,
+                               scan_resident_warps(cx, mapping, ts.dp, k), lp.shard_rank, lp.shard_count, l1));
     }
     if (full) SKNN_TRY(run_scan(cx, qs, ts, l1, sp));
     mk.scan = tm.mark();
@@ -300,6 +350,7 @@ static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt
     s.dist_recompute = c.dist_recompute;
     s.topk_inserts = c.topk_inserts;
     s.rows_loaded = c.rows_loaded;
+    s.dense_terms = (uint32_t)c.dense_terms;
     s.ms_total = tm.ms(0, mk.end);
     s.ms_build_t = tm.ms(0, mk.bt);
     s.ms_build_q = mk.bq >= 0 ? tm.ms(mk.bt, mk.bq) : 0.f;
@@ -320,7 +371,7 @@ static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt
 // Shared body of sknn_join_ex / sknn_query.
 static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
                             int32_t* out_idx, float* out_dist, const sknn_options* opt_in, sknn_stats* stats,
-                            cudaStream_t stream, const sknn_index* index) {
+                            cudaStream_t stream, const sknn_index* index, bool capturing = false) {
     SKNN_TRY(validate(Q, nq, T ? T : Q, nt, d, k, out_dist));
     if (nq == 0) {
         if (stats) {
@@ -340,11 +391,12 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     cx.stream = stream;
     cx.device = di.device;
     cx.num_sms = di.num_sms;
+    cx.capturing = capturing;
     Timer tm;
     tm.start(stream, stats != nullptr);
     sknn_status st = SKNN_OK;
     const int dp = (d + 3) & ~3;
-    const bool self = index ? (Q == index->user_ptr && nq == index->t.n) : (Q == T && nq == nt);
+    const bool self = index ? index_self_query(o, Q, nq, index) : (Q == T && nq == nt);
     int mapping = choose_mapping(o, di, nq, dp, k);
     int path = o.force_path == SKNN_PATH_BRUTE ? SKNN_PATH_BRUTE : SKNN_PATH_SPARSE;
     Marks mk;
@@ -450,6 +502,114 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     return st;
 }
 
+// ------------------------------------------------------------ CUDA graphs --
+// A whole join is ~25-30 stream-ordered launches with no host round trip, so
+// on small (launch-bound) joins the launch gaps are a visible share of the
+// step. A join whose key (device, pointers, sizes, options) was seen before is
+// recorded ONCE into a CUDA graph (stream capture on a private stream; scratch
+// allocations become graph memory nodes) and replayed with one cudaGraphLaunch
+// afterwards. The graph reads the arrays at the recorded addresses, so a replay
+// on new contents of the same buffers computes the join of the new contents.
+// Only device-pointer calls without stats, outside the partial filter (which
+// sizes its buffer on the host), with a modest scratch footprint.
+struct GraphKey {
+    int device;
+    const void *Q, *T, *oi, *od;
+    int64_t nq, nt;
+    int32_t d, k;
+    sknn_options o;
+    bool operator==(const GraphKey& b) const {
+        return device == b.device && Q == b.Q && T == b.T && oi == b.oi && od == b.od && nq == b.nq && nt == b.nt &&
+               d == b.d && k == b.k && memcmp(&o, &b.o, sizeof(o)) == 0;
+    }
+};
+struct GraphEntry {
+    GraphKey key;
+    cudaGraphExec_t exec = nullptr;  // nullptr: seen once, not yet recorded
+    uint64_t used = 0;
+};
+constexpr int kGraphCache = 8;
+static std::mutex g_graph_mu;
+static GraphEntry g_graphs[kGraphCache];
+static int g_graph_n = 0;
+static uint64_t g_graph_clock = 0;
+
+static cudaStream_t capture_stream(int dev) {
+    static cudaStream_t s[64] = {};
+    if (dev < 0 || dev >= 64) return nullptr;
+    if (!s[dev] && cudaStreamCreateWithFlags(&s[dev], cudaStreamNonBlocking) != cudaSuccess) {
+        cudaGetLastError();
+        s[dev] = nullptr;
+    }
+    return s[dev];
+}
+
+static sknn_status run_join_graphed(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
+                                    int32_t* out_idx, float* out_dist, const sknn_options* opt, sknn_stats* stats,
+                                    cudaStream_t stream) {
+    auto eager = [&]() { return run_join(Q, nq, T, nt, d, k, out_idx, out_dist, opt, stats, stream, nullptr); };
+    if (stats || !Q || !T || !out_dist || nq <= 0 || nt <= 0 || d <= 0 || k <= 0) return eager();
+    const sknn_options o = merge_options(opt);
+    if (o.use_graph < 0 || o.force_path == SKNN_PATH_PARTIAL) return eager();
+    DevInfo di;
+    if (device_info(di) != SKNN_OK) return eager();
+    if (classify(Q, di.device) != PTR_DEVICE || classify(T, di.device) != PTR_DEVICE ||
+        classify(out_dist, di.device) != PTR_DEVICE || (out_idx && classify(out_idx, di.device) != PTR_DEVICE))
+        return eager();
+    const int dp = (d + 3) & ~3;
+    const double footprint = (double)(nq + nt) * (4.0 * dp + 8.0 * k + 64.0);
+    if (footprint > (double)(1u << 30)) return eager();  // large joins are not launch-bound
+    GraphKey key;
+    memset(&key, 0, sizeof(key));
+    key.device = di.device; key.Q = Q; key.T = T; key.oi = out_idx; key.od = out_dist;
+    key.nq = nq; key.nt = nt; key.d = d; key.k = k; key.o = o;
+    std::lock_guard<std::mutex> lk(g_graph_mu);
+    int slot = -1;
+    for (int i = 0; i < g_graph_n; ++i)
+        if (g_graphs[i].key == key) slot = i;
+    if (slot >= 0 && g_graphs[slot].exec) {
+        g_graphs[slot].used = ++g_graph_clock;
+        SKNN_CUDA(cudaGraphLaunch(g_graphs[slot].exec, stream));
+        return SKNN_OK;
+    }
+    if (slot < 0) {  // first sighting: run eagerly, remember the key
+        if (g_graph_n < kGraphCache) {
+            slot = g_graph_n++;
+        } else {
+            slot = 0;
+            for (int i = 1; i < kGraphCache; ++i)
+                if (g_graphs[i].used < g_graphs[slot].used) slot = i;
+            if (g_graphs[slot].exec) cudaGraphExecDestroy(g_graphs[slot].exec);
+        }
+        g_graphs[slot].key = key;
+        g_graphs[slot].exec = nullptr;
+        g_graphs[slot].used = ++g_graph_clock;
+        return eager();
+    }
+    // second sighting: record the join once, then launch the graph
+    cudaStream_t cap = capture_stream(di.device);
+    if (!cap) return eager();
+    if (cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+        cudaGetLastError();
+        return eager();
+    }
+    sknn_status st = run_join(Q, nq, T, nt, d, k, out_idx, out_dist, opt, nullptr, cap, nullptr, true);
+    cudaGraph_t g = nullptr;
+    cudaError_t e = cudaStreamEndCapture(cap, &g);
+    cudaGraphExec_t exec = nullptr;
+    if (st == SKNN_OK && e == cudaSuccess && g) e = cudaGraphInstantiate(&exec, g, 0);
+    if (g) cudaGraphDestroy(g);
+    if (st != SKNN_OK || e != cudaSuccess || !exec) {
+        cudaGetLastError();
+        g_graphs[slot].used = ++g_graph_clock;  // stays "seen": try to record again next time
+        return eager();
+    }
+    g_graphs[slot].exec = exec;
+    g_graphs[slot].used = ++g_graph_clock;
+    SKNN_CUDA(cudaGraphLaunch(exec, stream));
+    return SKNN_OK;
+}
+
 }  // namespace sknn
 
 using namespace sknn;
@@ -470,13 +630,13 @@ void sknn_options_default(sknn_options* o) {
 
 sknn_status sknn_join(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k, int32_t* out_idx,
                       float* out_dist, sknn_stream_t stream) {
-    return run_join(Q, nq, T, nt, d, k, out_idx, out_dist, nullptr, nullptr, (cudaStream_t)stream, nullptr);
+    return run_join_graphed(Q, nq, T, nt, d, k, out_idx, out_dist, nullptr, nullptr, (cudaStream_t)stream);
 }
 
 sknn_status sknn_join_ex(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
                          int32_t* out_idx, float* out_dist, const sknn_options* opt, sknn_stats* stats,
                          sknn_stream_t stream) {
-    return run_join(Q, nq, T, nt, d, k, out_idx, out_dist, opt, stats, (cudaStream_t)stream, nullptr);
+    return run_join_graphed(Q, nq, T, nt, d, k, out_idx, out_dist, opt, stats, (cudaStream_t)stream);
 }
 
 sknn_status sknn_build(const float* T, int64_t nt, int32_t d, const sknn_options* opt, sknn_index** out,
@@ -535,8 +695,8 @@ sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq, int3
         const sknn_options o = merge_options(opt ? opt : &index->opt);
         int64_t B = o.query_batch;
         if (B <= 0) {
-            size_t free_b = 0, tot_b = 0;
-            if (cudaMemGetInfo(&free_b, &tot_b) != cudaSuccess) return fail(SKNN_ERR_CUDA, "cudaMemGetInfo failed");
+            const size_t free_b = usable_free_bytes(index->device);
+            if (free_b == 0) return fail(SKNN_ERR_CUDA, "cudaMemGetInfo failed");
             // per query: input row + output row + clustered copy, center distances and scan state (generous)
             const double per_q = 4.0 * d + 8.0 * k + 2.0 * (4.0 * ((d + 3) & ~3) + 16.0) + 8.0 * k;
             B = (int64_t)(0.4 * (double)free_b / per_q);
@@ -557,6 +717,7 @@ sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq, int3
                     acc.center_evals += sb.center_evals; acc.cand_pairs += sb.cand_pairs;
                     acc.dense_pairs += sb.dense_pairs; acc.dist_recompute += sb.dist_recompute;
                     acc.topk_inserts += sb.topk_inserts; acc.rows_loaded += sb.rows_loaded;
+                    acc.dense_terms = std::max(acc.dense_terms, sb.dense_terms);
                     acc.ms_total += sb.ms_total; acc.ms_build_t += sb.ms_build_t; acc.ms_build_q += sb.ms_build_q;
                     acc.ms_level1 += sb.ms_level1; acc.ms_sparse += sb.ms_sparse; acc.ms_dense += sb.ms_dense;
                     acc.ms_final += sb.ms_final; acc.kernel_launches += sb.kernel_launches;
@@ -628,6 +789,60 @@ sknn_status sknn_index_export(const sknn_index* ix, int32_t* off, int32_t* orig,
     return SKNN_OK;
 }
 
+sknn_status sknn_index_arrays(const sknn_index* ix, void** ptr, size_t* bytes) {
+    if (!ix || !ptr || !bytes) return fail(SKNN_ERR_INVALID_ARG, "NULL pointer");
+    const Side& t = ix->t;
+    void* p[SKNN_INDEX_ARRAYS] = {t.rows, t.dist, t.orig, t.off, t.centers, t.radius, t.tinfo};
+    size_t b[SKNN_INDEX_ARRAYS] = {sizeof(float) * (size_t)t.n * t.dp, sizeof(float) * (size_t)t.n,
+                                   sizeof(int32_t) * (size_t)t.n, sizeof(int32_t) * (size_t)(t.m + 1),
+                                   sizeof(float) * (size_t)t.m * t.dp, sizeof(float) * (size_t)t.m,
+                                   sizeof(int4) * (size_t)t.m};
+    for (int i = 0; i < SKNN_INDEX_ARRAYS; ++i) {
+        ptr[i] = p[i];
+        bytes[i] = b[i];
+    }
+    return SKNN_OK;
+}
+
+sknn_status sknn_index_create(int64_t nt, int32_t d, int32_t mt, const sknn_options* opt, sknn_index** out) {
+    if (!out) return fail(SKNN_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    if (nt <= 0 || nt >= (int64_t(1) << 31) || d <= 0 || mt <= 0 || mt > nt || mt > kMaxClusters)
+        return fail(SKNN_ERR_INVALID_ARG, "bad index geometry");
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    sknn_index* ix = new (std::nothrow) sknn_index();
+    if (!ix) return fail(SKNN_ERR_OOM, "host allocation of the index failed");
+    ix->device = di.device;
+    ix->user_ptr = nullptr;
+    ix->opt = merge_options(opt);
+    Side& t = ix->t;
+    t.n = nt; t.d = d; t.dp = (d + 3) & ~3; t.m = mt; t.owned = true;
+    Ctx cx;
+    cx.stream = nullptr;
+    cx.device = di.device;
+    cx.num_sms = di.num_sms;
+    sknn_status st = SKNN_OK;
+    do {
+        if ((st = cx.alloc_persistent((void**)&t.rows, sizeof(float) * nt * t.dp)) != SKNN_OK) break;
+        if ((st = cx.alloc_persistent((void**)&t.dist, sizeof(float) * nt)) != SKNN_OK) break;
+        if ((st = cx.alloc_persistent((void**)&t.orig, sizeof(int32_t) * nt)) != SKNN_OK) break;
+        if ((st = cx.alloc_persistent((void**)&t.off, sizeof(int32_t) * (mt + 1))) != SKNN_OK) break;
+        if ((st = cx.alloc_persistent((void**)&t.centers, sizeof(float) * mt * t.dp)) != SKNN_OK) break;
+        if ((st = cx.alloc_persistent((void**)&t.radius, sizeof(float) * mt)) != SKNN_OK) break;
+        if ((st = cx.alloc_persistent((void**)&t.tinfo, sizeof(int4) * mt)) != SKNN_OK) break;
+        cudaError_t e = cudaStreamSynchronize(nullptr);
+        if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("index allocation: ") + cudaGetErrorString(e));
+    } while (0);
+    if (st != SKNN_OK) {
+        cx.free_all();
+        delete ix;
+        return st;
+    }
+    *out = ix;
+    return SKNN_OK;
+}
+
 sknn_status sknn_debug_level1(const sknn_index* ix, const float* Q, int64_t nq, int32_t k, const sknn_options* opt,
                               int32_t* mq_out, int32_t* q_cluster, float* ub, int32_t* cand_count, int32_t* cand,
                               int64_t cand_capacity) {
@@ -642,7 +857,7 @@ sknn_status sknn_debug_level1(const sknn_index* ix, const float* Q, int64_t nq, 
     cx.num_sms = di.num_sms;
     sknn_status st = SKNN_OK;
     const Side& ts = ix->t;
-    const bool self = (Q == ix->user_ptr && nq == ts.n);
+    const bool self = index_self_query(o, Q, nq, ix);
     Side qs_local;
     const Side* qs = &ts;
     Level1 l1;

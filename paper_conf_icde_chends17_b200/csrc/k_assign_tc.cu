@@ -22,50 +22,16 @@
 
 #include "sknn_internal.cuh"
 #include "sknn_launch.h"
+#include "tc_ptx.cuh"
 
 namespace sknn {
 
 constexpr int kTcM = 128;   // points per CTA (TMEM lanes)
 constexpr int kTcN = 128;   // centers per chunk (TMEM columns per accumulator)
 
-__device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ uint64_t desc_kmajor(uint32_t saddr, uint32_t sbo) {
-    return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)(128u >> 4) << 16) | ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) |
-           ((uint64_t)1 << 46);
-}
-
-__device__ __forceinline__ void mma_bf16_f32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d),
-        "l"(a), "l"(b), "r"(idesc), "r"(acc));
-}
-
-__device__ __forceinline__ void wait_parity(uint32_t bar, uint32_t ph) {
-    asm volatile(
-        "{\n\t.reg .pred P1;\n\tW_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-        "@!P1 bra W_%=;\n\t}\n" ::"r"(bar),
-        "r"(ph)
-        : "memory");
-}
-
-__device__ __forceinline__ void ld32(uint32_t taddr, uint32_t (&r)[32]) {
-    asm volatile(
-        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
-          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
-          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
-        : "r"(taddr));
-    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-}
-
-__host__ __device__ constexpr uint32_t idesc_bf16_m128(int n) {
-    return (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(n >> 3) << 17) | (uint32_t(kTcM >> 4) << 24);
-}
+using tc::desc_kmajor;
+using tc::smem_u32;
+constexpr uint32_t idesc_bf16_m128(int n) { return tc::idesc_bf16(kTcM, n); }
 
 // o = mean of the m centers: one CTA per column, fixed-order tree (deterministic)
 __global__ void k_center_mean(const float* __restrict__ centers, int m, int dp, float* __restrict__ o) {
@@ -139,16 +105,14 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
     const uint32_t sbo = (uint32_t)kp * 16u;
 
     if (warp == 0) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(&s_tmem)),
-                     "r"(2u * kTcN));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        tc::tmem_alloc(&s_tmem, 2u * kTcN);
     }
     if (tid == 0) {
         for (int i = 0; i < 2; ++i) {
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar_full[i])));
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar_mma[i])));
+            tc::mbar_init(smem_u32(&bar_full[i]), 1);
+            tc::mbar_init(smem_u32(&bar_mma[i]), 1);
         }
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        tc::mbar_fence_init();
     }
     // stage A = x - o (bf16) for the CTA's 128 points
     const int64_t row0 = (int64_t)blockIdx.x * kTcM;
@@ -171,43 +135,35 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
             *reinterpret_cast<uint4*>(sA + off) = make_uint4(h[0], h[1], h[2], h[3]);
         }
     }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    tc::fence_proxy_async();  // generic-proxy smem writes -> visible to the tensor core
+    tc::fence_before();
     __syncthreads();
-    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    tc::fence_after();
     const uint32_t tmem = s_tmem;
     const uint32_t idesc = idesc_bf16_m128(kTcN);
 
     auto issue_copy = [&](int chunk, int buf) {
-        const uint32_t bar = su32(&bar_full[buf]);
+        const uint32_t bar = smem_u32(&bar_full[buf]);
         const uint32_t bytes = b_bytes + kTcN * 4;
-        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+        tc::expect_tx(bar, bytes);
         const unsigned char* src = reinterpret_cast<const unsigned char*>(cbf) + (size_t)chunk * b_bytes;
-        asm volatile(
-            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(su32(sB(buf))),
-            "l"(src), "r"(b_bytes), "r"(bar)
-            : "memory");
-        asm volatile(
-            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(su32(sBn(buf))),
-            "l"(bn + (size_t)chunk * kTcN), "r"((uint32_t)(kTcN * 4)), "r"(bar)
-            : "memory");
+        tc::bulk_g2s(smem_u32(sB(buf)), src, b_bytes, bar);
+        tc::bulk_g2s(smem_u32(sBn(buf)), bn + (size_t)chunk * kTcN, (uint32_t)(kTcN * 4), bar);
     };
     auto issue_mma = [&](int buf) {
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const uint32_t aB = su32(sA), bB = su32(sB(buf));
+        tc::fence_after();
+        const uint32_t aB = smem_u32(sA), bB = smem_u32(sB(buf));
         for (int s = 0; s < kp / 16; ++s)
-            mma_bf16_f32(tmem + (uint32_t)(buf * kTcN), desc_kmajor(aB + s * 256u, sbo), desc_kmajor(bB + s * 256u, sbo),
+            tc::mma_bf16(tmem + (uint32_t)(buf * kTcN), desc_kmajor(aB + s * 256u, sbo), desc_kmajor(bB + s * 256u, sbo),
                          idesc, s > 0);
-        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-                         su32(&bar_mma[buf]))
-                     : "memory");
+        tc::mma_commit(smem_u32(&bar_mma[buf]));
     };
 
     uint32_t ph_full[2] = {0, 0}, ph_mma[2] = {0, 0};
     if (tid == 0) {
         issue_copy(0, 0);
         if (nchunks > 1) issue_copy(1, 1);
-        wait_parity(su32(&bar_full[0]), 0);
+        tc::mbar_wait(smem_u32(&bar_full[0]), 0);
         issue_mma(0);
     }
     ph_full[0] = 1;
@@ -220,13 +176,13 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
         // issue the next chunk's MMA as soon as its copy landed (overlaps this epilogue)
         if (tid == 0 && c + 1 < nchunks) {
             const int nb = (c + 1) & 1;
-            wait_parity(su32(&bar_full[nb]), ph_full[nb]);
+            tc::mbar_wait(smem_u32(&bar_full[nb]), ph_full[nb]);
             issue_mma(nb);
         }
         if (c + 1 < nchunks) ph_full[(c + 1) & 1] ^= 1u;
-        wait_parity(su32(&bar_mma[buf]), ph_mma[buf]);
+        tc::mbar_wait(smem_u32(&bar_mma[buf]), ph_mma[buf]);
         ph_mma[buf] ^= 1u;
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        tc::fence_after();
         const float* bnv = sBn(buf);
         // per 32 columns: the scores, their minimum by a min tree (one FMNMX
         // per score) and, only when it beats the running best, the lowest
@@ -235,7 +191,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
         for (int cb = 0; cb < 2; ++cb) {
             const int col = half * 64 + cb * 32;
             uint32_t v[32];
-            ld32(trow + (uint32_t)(buf * kTcN + col), v);
+            tc::tmem_ld32(trow + (uint32_t)(buf * kTcN + col), v);
             float sc[32];
             const float4* bn4 = reinterpret_cast<const float4*>(bnv + col);
 #pragma unroll
@@ -261,7 +217,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
                 bi = c * kTcN + col + jm;
             }
         }
-        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        tc::fence_before();
         __syncthreads();  // buffer `buf` (smem + TMEM) is free again
         if (tid == 0 && c + 2 < nchunks) issue_copy(c + 2, buf);
     }
@@ -286,9 +242,9 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
         if (counts) atomicAdd(counts + bi, 1);
         if (sums) fx_accumulate(sums + (int64_t)bi * dp, xr, dp, *fx);
     }
-    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    tc::fence_before();
     __syncthreads();
-    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(2u * kTcN));
+    if (warp == 0) tc::tmem_dealloc(tmem, 2u * kTcN);
 }
 
 bool assign_tc_supported(int dp) { return dp >= 8 && ((dp + 15) & ~15) <= 256; }

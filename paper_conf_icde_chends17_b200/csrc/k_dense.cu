@@ -33,70 +33,25 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <math.h>
+#include <stdlib.h>
 #include <stdint.h>
 
 #include "k_scan_common.cuh"
+#include "tc_ptx.cuh"
 
 namespace sknn {
 
 constexpr int kDenseM = 128;
 
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t sbo) {
-    return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)(128u >> 4) << 16) | ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) |
-           ((uint64_t)1 << 46);  // LBO 128 B, descriptor version 1 (sm_100), SWIZZLE_NONE
-}
-
-// kind::f16 instruction descriptor: BF16 x BF16 -> F32, both K-major, M = 128
-__host__ __device__ constexpr uint32_t umma_idesc_bf16(int n) {
-    return (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(n >> 3) << 17) | (uint32_t(kDenseM >> 4) << 24);
-}
-
-__device__ __forceinline__ void umma_bf16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(tmem_d),
-        "l"(a), "l"(b), "r"(idesc), "r"(acc));
-}
-
-__device__ __forceinline__ void umma_commit(uint32_t bar) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t phase) {
-    asm volatile(
-        "{\n\t.reg .pred P1;\n\tWAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-        "@!P1 bra WAIT_%=;\n\t}\n" ::"r"(bar),
-        "r"(phase)
-        : "memory");
-}
-
-__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-                 "l"(src), "r"(bytes), "r"(bar)
-                 : "memory");
-}
-
-__device__ __forceinline__ void expect_tx(uint32_t bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-}
-
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
-    asm volatile(
-        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
-          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
-          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
-        : "r"(taddr));
-    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-}
-
-__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+using tc::smem_u32;
+using tc::mbar_wait;
+using tc::bulk_g2s;
+using tc::expect_tx;
+using tc::tmem_ld32;
+using tc::fence_before;
+using tc::fence_after;
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t sbo) { return tc::desc_kmajor(saddr, sbo); }
+__host__ __device__ constexpr uint32_t umma_idesc_bf16(int n) { return tc::idesc_bf16(kDenseM, n); }
 
 // ------------------------------------------------------ tile conversion --
 // rintf of the mean center: the common origin o of both point sets
@@ -140,12 +95,13 @@ __global__ void __launch_bounds__(256) k_to_tiles(const float* __restrict__ rows
                                                   const float* __restrict__ o, float nscale,
                                                   __nv_bfloat16* __restrict__ hi, __nv_bfloat16* __restrict__ lo,
                                                   float* __restrict__ norm, float* __restrict__ norm_raw,
-                                                  int* __restrict__ lo_flag) {
+                                                  int* __restrict__ lo_flag, int* __restrict__ amax_flag) {
     const int c = blockIdx.x;
     const int lo0 = off[c], size = off[c + 1] - lo0, p0 = offp[c];
     const int c8n = kp / 8;
     const size_t sbo = (size_t)kp * 16;
     bool nz = false;
+    float amax = 0.f;  // max |x - o| over the side (exact-path test)
     for (int w = threadIdx.x; w < size * c8n; w += blockDim.x) {
         const int r = w / c8n, c8 = w % c8n;
         const float* src = rows + (int64_t)(lo0 + r) * dp;
@@ -157,6 +113,7 @@ __global__ void __launch_bounds__(256) k_to_tiles(const float* __restrict__ rows
             for (int e = 0; e < 2; ++e) {
                 const int kk = c8 * 8 + 2 * i + e;
                 v[e] = kk < dp ? src[kk] - o[kk] : 0.f;
+                amax = fmaxf(amax, fabsf(v[e]));
             }
             const __nv_bfloat16 h0 = __float2bfloat16_rn(v[0]), h1 = __float2bfloat16_rn(v[1]);
             const __nv_bfloat16 l0 = __float2bfloat16_rn(v[0] - __bfloat162float(h0));
@@ -181,6 +138,16 @@ __global__ void __launch_bounds__(256) k_to_tiles(const float* __restrict__ rows
         if (norm_raw) norm_raw[p0 + r] = s;
     }
     if (__syncthreads_or(nz) && threadIdx.x == 0) atomicOr(lo_flag, 1);
+    for (int o = 16; o > 0; o >>= 1) amax = fmaxf(amax, __shfl_xor_sync(0xffffffffu, amax, o));
+    if ((threadIdx.x & 31) == 0 && amax > 0.f) atomicMax(amax_flag, __float_as_int(amax));  // >= 0: int order
+}
+
+// self-join: the query side's flags are the target side's
+__global__ void k_copy_flags(int* f) {
+    if (threadIdx.x == 0) {
+        f[0] = f[1];
+        f[2] = f[3];
+    }
 }
 
 __global__ void k_fill_f(float* __restrict__ p, int64_t n, float v) {
@@ -202,7 +169,8 @@ struct DenseArgs {
     const unsigned char* thi;
     const unsigned char* tlo;
     const float* tn;       // ||b||^2 (1 - eps), +inf on padding rows
-    const int* lo_flag;    // [2]: query side, target side has a nonzero lo part
+    const int* lo_flag;    // [4]: query side, target side has a nonzero lo part; max |x - o| bits of each side
+    const float* tn_raw;   // ||b||^2 unscaled, +inf on padding rows (exact variant)
     const float* ub;
     const int32_t* dcand;
     const int32_t* dcount;
@@ -246,6 +214,18 @@ struct ChunkIter {
     __device__ __forceinline__ bool valid() const { return ci < nd; }
 };
 
+// Exact integer tiles: when neither side has a nonzero bf16 lo part (the
+// re-centred coordinates are integers |x - o| <= 256, exact in bf16) and
+// dp (A + B)^2 < 2^24 (A, B = max |x - o| per side), every product and every
+// partial sum of a.b, ||a||^2 and ||b||^2 is an integer below 2^24, so the
+// fp32 MMA result and d2 = ||a||^2 + ||b||^2 - 2 a.b are EXACT and equal the
+// shared SIMT formula's d2 bit for bit: no screen slack, no recompute.
+__device__ __forceinline__ bool dense_exact_ok(const int* flags, int dp) {
+    if (flags[0] | flags[1]) return false;
+    const double s = (double)__int_as_float(flags[2]) + (double)__int_as_float(flags[3]);
+    return (double)dp * s * s < 16777216.0;
+}
+
 template <int KMAX, int NCH>
 __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
     extern __shared__ __align__(128) unsigned char smem[];
@@ -261,27 +241,27 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
     __shared__ uint32_t s_tmem;
     __shared__ int s_tile;
 
+    if (dense_exact_ok(a.lo_flag, a.dp)) return;  // k_dense_exact handles this join
     const int tid = threadIdx.x, warp = tid >> 5;
     if (warp == 0) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&s_tmem)),
-                     "r"((uint32_t)(2 * NCH)));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        tc::tmem_alloc(&s_tmem, (uint32_t)(2 * NCH));
     }
     if (tid == 0) {
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&bar_a)));
+        tc::mbar_init(smem_u32(&bar_a), 1);
         for (int i = 0; i < 2; ++i) {
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&bar_full[i])));
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&bar_mma[i])));
+            tc::mbar_init(smem_u32(&bar_full[i]), 1);
+            tc::mbar_init(smem_u32(&bar_mma[i]), 1);
         }
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        tc::mbar_fence_init();
     }
-    tc_fence_before();
+    fence_before();
     __syncthreads();
-    tc_fence_after();
+    fence_after();
     const uint32_t tmem = s_tmem;
     const uint32_t tmem_row = tmem + ((uint32_t)(warp * 32) << 16);
     const uint32_t idesc = umma_idesc_bf16(NCH);
     const bool loA = a.lo_flag[0] != 0, loB = a.lo_flag[1] != 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) atomicMax(&a.counters->dense_terms, 1ull + loA + loB);
     const uint32_t bstage = loB ? 2 * b_bytes : b_bytes;  // bytes moved per B chunk
     const float INF = __int_as_float(0x7f800000);
     const float rel_k = 1.f + (float)(KP + 2) * 1.1920929e-7f;  // (K+2) 2^-23
@@ -299,17 +279,17 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
         bulk_g2s(smem_u32(s_tn + buf * NCH), a.tn + p, NCH * 4, bar);
     };
     auto issue_mma = [&](int buf) {
-        tc_fence_after();
+        fence_after();
         const uint32_t aH = smem_u32(sA), aL = smem_u32(sA + a_bytes);
         const uint32_t bH = smem_u32(sB + buf * b_bytes), bL = smem_u32(sB + (2 + buf) * b_bytes);
         const uint32_t d = tmem + (uint32_t)(buf * NCH);
         for (int s = 0; s < KP / 16; ++s) {
             const uint32_t ko = (uint32_t)s * 256u;
-            umma_bf16(d, umma_desc(aH + ko, sbo), umma_desc(bH + ko, sbo), idesc, s > 0);
-            if (loB) umma_bf16(d, umma_desc(aH + ko, sbo), umma_desc(bL + ko, sbo), idesc, 1);
-            if (loA) umma_bf16(d, umma_desc(aL + ko, sbo), umma_desc(bH + ko, sbo), idesc, 1);
+            tc::mma_bf16(d, umma_desc(aH + ko, sbo), umma_desc(bH + ko, sbo), idesc, s > 0);
+            if (loB) tc::mma_bf16(d, umma_desc(aH + ko, sbo), umma_desc(bL + ko, sbo), idesc, 1);
+            if (loA) tc::mma_bf16(d, umma_desc(aL + ko, sbo), umma_desc(bH + ko, sbo), idesc, 1);
         }
-        umma_commit(smem_u32(&bar_mma[buf]));
+        tc::mma_commit(smem_u32(&bar_mma[buf]));
     };
 
     for (;;) {
@@ -365,7 +345,7 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
             if (has_next) ph_full[buf ^ 1] ^= 1u;
             mbar_wait(smem_u32(&bar_mma[buf]), ph_mma[buf]);
             ph_mma[buf] ^= 1u;
-            tc_fence_after();
+            fence_after();
             const int nb = min(NCH, cons.size - cons.c * NCH);
             const int j0 = __ldg(a.toff + cons.tc) + cons.c * NCH;  // real (unpadded) first target
             const float* tnv = s_tn + buf * NCH;
@@ -402,7 +382,7 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
                 }
             }
             if (active) covered += (unsigned long long)nb;
-            tc_fence_before();
+            fence_before();
             __syncthreads();  // stage `buf` (smem) and accumulator `buf` (TMEM) are free
             if (tid == 0 && prod.valid()) {
                 issue_b(prod, buf);
@@ -421,10 +401,289 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
     }
     add_counter(&a.counters->evals_dense, covered);
     add_counter(&a.counters->dist_recompute, recomputed);
-    tc_fence_before();
+    fence_before();
     __syncthreads();
     if (warp == 0)
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)(2 * NCH)));
+        tc::tmem_dealloc(tmem, (uint32_t)(2 * NCH));
+}
+
+// ------------------------------------------------------ exact dense tiles --
+// Warp-specialised: warp 8 (one elected thread) is the producer -- tile
+// scheduler, bulk copies of the A tile (128 queries) and of the NCH-target B
+// chunks through a kExStages ring, tcgen05.mma of each chunk into one of
+// kExAcc TMEM accumulators; warps 0-7 are the epilogue -- two threads per query
+// row (TMEM lanes 32 (w % 4) .. + 31), each over one half of the chunk's
+// columns, with its own register top-k; the two halves share their k-th
+// distance through shared memory (the smaller of two subsets' k-th distances
+// is still >= the row's true k-th) and are merged when the tile ends.
+// Barriers: full[s] (chunk landed), sfree[s] (its MMA done: stage reusable),
+// mma[c] (accumulator ready), afree[c] (epilogue done with it: count 8 warps),
+// tfull/tfree[2] (tile id slots). The target norms of a chunk sit in a ring
+// of kExStages + kExAcc slots, so a slot is reloaded only after the epilogue
+// released the chunk that used it (sfree(g + kExAcc) implies afree(g)).
+constexpr int kExNCH = 128;
+constexpr int kExEpiWarps = 8;
+constexpr int kExThreads = (kExEpiWarps + 1) * 32;
+constexpr int kExStages = 3;
+constexpr int kExAcc = 2;
+constexpr int kExTn = kExStages + kExAcc;
+
+__host__ __device__ constexpr int dense_exact_min_blocks(int kmax) { return 1; }
+
+template <int KMAX>
+__global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_dense_exact(DenseArgs a) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    if (!dense_exact_ok(a.lo_flag, a.dp)) return;  // the split-precision k_dense handles this join
+    constexpr int NCH = kExNCH;
+    const int KP = a.kp;
+    const uint32_t sbo = (uint32_t)KP * 16u;
+    const uint32_t a_bytes = (uint32_t)kDenseM * KP * 2, b_bytes = (uint32_t)NCH * KP * 2;
+    unsigned char* sA = smem;
+    unsigned char* sB = smem + a_bytes;                                       // [kExStages][b_bytes]
+    float* s_tn = reinterpret_cast<float*>(sB + kExStages * (size_t)b_bytes);  // [kExTn][NCH]
+    __shared__ __align__(8) uint64_t bar_a, bar_full[kExStages], bar_sfree[kExStages], bar_mma[kExAcc],
+        bar_afree[kExAcc], bar_tfull[2], bar_tfree[2];
+    __shared__ uint32_t s_tmem;
+    __shared__ int s_tile[2];
+    __shared__ unsigned long long s_kth[2][kDenseM];  // {k-th d2 bits, tile seq} per half and row
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    if (blockIdx.x == 0 && tid == 0) atomicMax(&a.counters->dense_terms, 1ull);
+    if (warp == kExEpiWarps) tc::tmem_alloc(&s_tmem, (uint32_t)(kExAcc * NCH));
+    if (tid == 0) {
+        tc::mbar_init(smem_u32(&bar_a), 1);
+        for (int i = 0; i < kExStages; ++i) {
+            tc::mbar_init(smem_u32(&bar_full[i]), 1);
+            tc::mbar_init(smem_u32(&bar_sfree[i]), 1);
+        }
+        for (int i = 0; i < kExAcc; ++i) {
+            tc::mbar_init(smem_u32(&bar_mma[i]), 1);
+            tc::mbar_init(smem_u32(&bar_afree[i]), kExEpiWarps);
+        }
+        for (int i = 0; i < 2; ++i) {
+            tc::mbar_init(smem_u32(&bar_tfull[i]), 1);
+            tc::mbar_init(smem_u32(&bar_tfree[i]), kExEpiWarps);
+        }
+        tc::mbar_fence_init();
+    }
+    for (int i = tid; i < 2 * kDenseM; i += blockDim.x) (&s_kth[0][0])[i] = ~0ull;
+    fence_before();
+    __syncthreads();
+    fence_after();
+    const uint32_t tmem = s_tmem;
+    const int ntiles = *a.ntiles;
+
+    if (warp == kExEpiWarps) {
+        // ------------------------------------------------------- producer --
+        if (lane == 0) {
+            const uint32_t idesc = tc::idesc_bf16(kDenseM, NCH);
+            uint32_t ph_a = 0;
+            uint32_t g = 0;          // global chunk sequence (both roles count it identically)
+            int last_acc = -1;
+            uint32_t last_ph = 0;
+            for (int t = 0;; ++t) {
+                const int slot = t & 1;
+                if (t >= 2) mbar_wait(smem_u32(&bar_tfree[slot]), ((t >> 1) - 1) & 1);
+                const int tile = atomicAdd(a.counter, 1);
+                *(volatile int*)&s_tile[slot] = tile;
+                tc::mbar_arrive(smem_u32(&bar_tfull[slot]));
+                if (tile >= ntiles) break;
+                const int2 tl = a.tiles[tile];
+                const int qc = tl.x;
+                const size_t qp = (size_t)a.qoffp[qc] + tl.y;
+                // the A tile is reloaded once every MMA of the previous tile is done
+                if (last_acc >= 0) mbar_wait(smem_u32(&bar_mma[last_acc]), last_ph);
+                expect_tx(smem_u32(&bar_a), a_bytes);
+                bulk_g2s(smem_u32(sA), a.qhi + (qp >> 3) * sbo, a_bytes, smem_u32(&bar_a));
+                ChunkIter<NCH> ld, mm;
+                ld.start(a, qc);
+                mm.start(a, qc);
+                uint32_t lg = g;  // load cursor, runs up to kExStages chunks ahead of the MMA cursor
+                auto issue_load = [&]() {
+                    const int s = lg % kExStages;
+                    if (lg >= (uint32_t)kExStages) mbar_wait(smem_u32(&bar_sfree[s]), ((lg / kExStages) - 1) & 1);
+                    const uint32_t bar = smem_u32(&bar_full[s]);
+                    expect_tx(bar, b_bytes + NCH * 4);
+                    const size_t p = (size_t)__ldg(a.toffp + ld.tc) + (size_t)ld.c * NCH;
+                    bulk_g2s(smem_u32(sB + (size_t)s * b_bytes), a.thi + (p >> 3) * sbo, b_bytes, bar);
+                    bulk_g2s(smem_u32(s_tn + (lg % kExTn) * NCH), a.tn_raw + p, NCH * 4, bar);
+                    ++lg;
+                    ld.advance(a);
+                };
+                bool a_ready = false;
+                for (; mm.valid(); mm.advance(a), ++g) {
+                    while (ld.valid() && lg < g + kExStages) issue_load();
+                    if (!a_ready) {
+                        mbar_wait(smem_u32(&bar_a), ph_a);
+                        ph_a ^= 1u;
+                        a_ready = true;
+                    }
+                    const int s = g % kExStages, c = g % kExAcc;
+                    mbar_wait(smem_u32(&bar_full[s]), (g / kExStages) & 1);
+                    if (g >= (uint32_t)kExAcc) mbar_wait(smem_u32(&bar_afree[c]), ((g / kExAcc) - 1) & 1);
+                    fence_after();
+                    const uint32_t aB = smem_u32(sA), bB = smem_u32(sB + (size_t)s * b_bytes);
+                    const uint32_t d = tmem + (uint32_t)(c * NCH);
+                    for (int ks = 0; ks < KP / 16; ++ks)
+                        tc::mma_bf16(d, umma_desc(aB + ks * 256u, sbo), umma_desc(bB + ks * 256u, sbo), idesc, ks > 0);
+                    tc::mma_commit(smem_u32(&bar_mma[c]));
+                    tc::mma_commit(smem_u32(&bar_sfree[s]));
+                    last_acc = c;
+                    last_ph = (g / kExAcc) & 1;
+                }
+            }
+        }
+    } else {
+        // ------------------------------------------------------- epilogue --
+        const int quarter = warp & 3, half = warp >> 2;
+        const int row = quarter * 32 + lane;
+        const uint32_t trow = tmem + ((uint32_t)(quarter * 32) << 16);
+        const float INF = __int_as_float(0x7f800000);
+        uint32_t g = 0;
+        unsigned long long covered = 0;
+        for (int t = 0;; ++t) {
+            const int slot = t & 1;
+            mbar_wait(smem_u32(&bar_tfull[slot]), (t >> 1) & 1);
+            const int tile = *(volatile int*)&s_tile[slot];
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(smem_u32(&bar_tfree[slot]));
+            if (tile >= ntiles) break;
+            const int2 tl = a.tiles[tile];
+            const int qc = tl.x;
+            const int qlo = a.qoff[qc], qsz = a.qoff[qc + 1] - qlo;
+            const bool active = tl.y + row < qsz;
+            const int qpos = qlo + tl.y + (active ? row : 0);
+            const size_t qp = (size_t)a.qoffp[qc] + tl.y;
+            const float na = active ? __ldg(a.qn + qp + row) : 0.f;
+            RegTopK<KMAX> top;
+            top.init(a.k);
+            key_t kth = top.kth();
+            const float ub = a.ub[qc];
+            float kth2 = __fmul_ru(ub, ub);
+            const unsigned long long tag = (unsigned long long)(unsigned)t;
+            volatile unsigned long long* mine = &s_kth[half][row];
+            volatile unsigned long long* other = &s_kth[half ^ 1][row];
+            *mine = ((unsigned long long)__float_as_uint(kth2) << 32) | tag;
+            ChunkIter<NCH> it;
+            it.start(a, qc);
+            for (; it.valid(); it.advance(a), ++g) {
+                const int c = g % kExAcc;
+                // the chunk's target norms landed before the producer issued its MMA
+                // (it waited on full[s]); mma[c] completing orders them before us. The
+                // epilogue must NOT wait on full[s] itself: that barrier may already
+                // be one phase further (the stage is refilled once the MMA is done).
+                mbar_wait(smem_u32(&bar_mma[c]), (g / kExAcc) & 1);
+                fence_after();
+                const int nb = min(NCH, it.size - it.c * NCH);
+                const int j0 = __ldg(a.toff + it.tc) + it.c * NCH;  // real (unpadded) first target
+                const float* tn = s_tn + (g % kExTn) * NCH;
+                float lim = kth2;
+                const unsigned long long ot = *other;
+                if ((ot & 0xffffffffull) == tag) lim = fminf(lim, __uint_as_float((uint32_t)(ot >> 32)));
+                float thr = __fsub_ru(lim, na);  // keep t = ||b||^2 - 2 a.b iff t <= lim - ||a||^2
+#pragma unroll 1
+                for (int cb = 0; cb < NCH / 32; ++cb) {  // 16-column blocks of this half
+                    const int col = half * (NCH / 2) + cb * 16;
+                    if (col >= nb) break;  // warp-uniform
+                    uint32_t v[16];
+                    tc::tmem_ld16(trow + (uint32_t)(c * NCH + col), v);
+                    float tt[16];
+                    const float4* tn4 = reinterpret_cast<const float4*>(tn + col);
+#pragma unroll
+                    for (int j4 = 0; j4 < 4; ++j4) {
+                        const float4 b4 = tn4[j4];
+                        tt[4 * j4 + 0] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 0]), b4.x);
+                        tt[4 * j4 + 1] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 1]), b4.y);
+                        tt[4 * j4 + 2] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 2]), b4.z);
+                        tt[4 * j4 + 3] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 3]), b4.w);
+                    }
+                    if (col + 16 > nb) {  // columns past the cluster's last target (next cluster's rows)
+#pragma unroll
+                        for (int j = 0; j < 16; ++j)
+                            if (col + j >= nb) tt[j] = INF;
+                    }
+                    float mn[8];
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) mn[j] = fminf(tt[j], tt[j + 8]);
+#pragma unroll
+                    for (int w2 = 4; w2 > 0; w2 >>= 1)
+#pragma unroll
+                        for (int j = 0; j < w2; ++j) mn[j] = fminf(mn[j], mn[j + w2]);
+                    if (active && mn[0] <= thr) {
+                        unsigned m = 0;
+#pragma unroll
+                        for (int j = 0; j < 16; ++j) m |= (tt[j] <= thr ? 1u : 0u) << j;
+                        while (m) {
+                            const int j = __ffs(m) - 1;
+                            m &= m - 1;
+                            float tj = tt[0];
+#pragma unroll
+                            for (int u = 1; u < 16; ++u)
+                                if (u == j) tj = tt[u];
+                            const float d2 = tj + na;  // exact (integer < 2^24)
+                            if (d2 <= kth2) {
+                                const key_t key = make_key(d2, __ldg(a.torig + j0 + col + j));
+                                if (key < kth) {
+                                    top.insert(key);
+                                    kth = top.kth();
+                                    if (key_d2(kth) < kth2) {
+                                        kth2 = key_d2(kth);
+                                        thr = __fsub_ru(fminf(lim, kth2), na);
+                                    }
+                                }
+                            }
+                        }
+                    }
+                }
+                fence_before();
+                __syncwarp();
+                if (lane == 0) tc::mbar_arrive(smem_u32(&bar_afree[c]));  // accumulator c may be overwritten
+                *mine = ((unsigned long long)__float_as_uint(kth2) << 32) | tag;
+                if (active && half == 0) covered += (unsigned long long)nb;
+            }
+            // merge the two halves' lists of each row (keys are distinct: disjoint columns)
+            key_t* orow = a.topk_out + (int64_t)qpos * a.k;
+            if (active && half == 1) {
+#pragma unroll
+                for (int q = 0; q < KMAX; ++q) {
+                    const int r = q - (KMAX - a.k);
+                    if (r >= 0) orow[r] = top.a[q];
+                }
+            }
+            tc::bar_sync(1, kExEpiWarps * 32);
+            if (active && half == 0) {
+                for (int r = 0; r < a.k; ++r) {
+                    const key_t key = orow[r];
+                    if (key < kth) {
+                        top.insert(key);
+                        kth = top.kth();
+                    }
+                }
+#pragma unroll
+                for (int q = 0; q < KMAX; ++q) {
+                    const int r = q - (KMAX - a.k);
+                    if (r >= 0) orow[r] = top.a[q];
+                }
+            }
+        }
+        // counters: warps of half 0 only (all 32 lanes of a warp call add_counter)
+        if (half == 0) add_counter(&a.counters->evals_dense, covered);
+    }
+    fence_before();
+    __syncthreads();
+    if (warp == kExEpiWarps) tc::tmem_dealloc(tmem, (uint32_t)(kExAcc * kExNCH));
+}
+
+template <int KMAX>
+static sknn_status launch_dense_exact_k(Ctx& cx, const DenseArgs& a) {
+    const size_t smem = (size_t)kDenseM * a.kp * 2 + kExStages * (size_t)kExNCH * a.kp * 2 + kExTn * kExNCH * 4;
+    SKNN_CUDA(cudaFuncSetAttribute(k_dense_exact<KMAX>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_dense_exact<KMAX>, kExThreads, smem);
+    per_sm = std::max(1, std::min(per_sm, 512 / (kExAcc * kExNCH)));  // TMEM columns per SM
+    k_dense_exact<KMAX><<<per_sm * cx.num_sms, kExThreads, smem, cx.stream>>>(a);
+    cx.launched();
+    return cx.check_launch("dense tiles (exact)");
 }
 
 template <int KMAX, int NCH>
@@ -447,6 +706,16 @@ static sknn_status launch_dense_n(Ctx& cx, const DenseArgs& a) {
     return launch_dense_k<32, NCH>(cx, a);
 }
 
+// Both variants are launched; each reads the device-side exactness test
+// (dense_exact_ok) and the one that does not apply exits at once, so the
+// choice needs no host read-back (the join stays stream-ordered).
+static sknn_status launch_dense_exact(Ctx& cx, const DenseArgs& a) {
+    if (a.k <= 8) return launch_dense_exact_k<8>(cx, a);
+    if (a.k <= 16) return launch_dense_exact_k<16>(cx, a);
+    if (a.k <= 24) return launch_dense_exact_k<24>(cx, a);
+    return launch_dense_exact_k<32>(cx, a);
+}
+
 int dense_kp(int dp) { return (dp + 15) & ~15; }
 bool dense_supported(int dp) { return dense_kp(dp) <= 256; }
 
@@ -461,7 +730,7 @@ struct DenseSide {
 };
 
 static sknn_status convert_side(Ctx& cx, const Side& sd, int kp, const float* o, float nscale, bool want_raw,
-                                int* lo_flag, DenseSide& out) {
+                                int* lo_flag, int* amax_flag, DenseSide& out) {
     const int m = sd.m;
     int32_t* cnt8;
     SKNN_TRY(cx.alloc_scratch((void**)&out.offp, sizeof(int32_t) * (m + 1)));
@@ -489,7 +758,8 @@ static sknn_status convert_side(Ctx& cx, const Side& sd, int kp, const float* o,
     }
     k_to_tiles<<<m, 256, 0, cx.stream>>>(sd.rows, sd.off, out.offp, sd.dp, kp, o, nscale,
                                         reinterpret_cast<__nv_bfloat16*>(out.hi),
-                                        reinterpret_cast<__nv_bfloat16*>(out.lo), out.norm, out.norm_raw, lo_flag);
+                                        reinterpret_cast<__nv_bfloat16*>(out.lo), out.norm, out.norm_raw, lo_flag,
+                                        amax_flag);
     cx.launched();
     return cx.check_launch("dense tile conversion");
 }
@@ -521,26 +791,30 @@ sknn_status run_dense(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1,
     const float eps_tc = dense_eps(ts.dp);
     const bool self = &qs == &ts;
     const float* o = p.origin;
+    // flags: [0] query lo part nonzero, [1] target lo part nonzero, [2] / [3]
+    // max |x - o| (float bits) of the query / target side
     int* lo_flag;
-    SKNN_TRY(cx.alloc_scratch((void**)&lo_flag, sizeof(int) * 2));
-    SKNN_CUDA(cudaMemsetAsync(lo_flag, 0, sizeof(int) * 2, cx.stream));
+    SKNN_TRY(cx.alloc_scratch((void**)&lo_flag, sizeof(int) * 4));
+    SKNN_CUDA(cudaMemsetAsync(lo_flag, 0, sizeof(int) * 4, cx.stream));
     DenseSide tq, tt;
-    SKNN_TRY(convert_side(cx, ts, kp, o, 1.f - eps_tc, self, lo_flag + 1, tt));
+    SKNN_TRY(convert_side(cx, ts, kp, o, 1.f - eps_tc, true, lo_flag + 1, lo_flag + 3, tt));
     if (self) {
         tq = tt;
         tq.norm = tt.norm_raw;
-        SKNN_CUDA(cudaMemcpyAsync(lo_flag, lo_flag + 1, sizeof(int), cudaMemcpyDeviceToDevice, cx.stream));
+        k_copy_flags<<<1, 32, 0, cx.stream>>>(lo_flag);
+        cx.launched();
     } else {
-        SKNN_TRY(convert_side(cx, qs, kp, o, 1.f, false, lo_flag, tq));
+        SKNN_TRY(convert_side(cx, qs, kp, o, 1.f, false, lo_flag, lo_flag + 2, tq));
     }
     DenseArgs a{};
     a.qrows = qs.rows; a.qoff = qs.off; a.qoffp = tq.offp; a.qhi = tq.hi; a.qlo = tq.lo; a.qn = tq.norm;
     a.trows = ts.rows; a.torig = ts.orig; a.toff = ts.off; a.toffp = tt.offp; a.thi = tt.hi; a.tlo = tt.lo;
-    a.tn = tt.norm; a.lo_flag = lo_flag;
+    a.tn = tt.norm; a.tn_raw = tt.norm_raw; a.lo_flag = lo_flag;
     a.ub = l1.ub; a.dcand = l1.dcand; a.dcount = l1.dcount;
     a.tiles = l1.dtiles; a.ntiles = l1.dntiles; a.counter = l1.dntiles + 1;
     a.mt = ts.m; a.dp = ts.dp; a.kp = kp; a.k = p.k; a.eps_tc = eps_tc;
     a.topk_out = p.topk_out; a.counters = p.counters;
+    if (!getenv("SKNN_DENSE_SPLIT_ONLY")) SKNN_TRY(launch_dense_exact(cx, a));  // ablation: split path only
     if (kp <= 64) return launch_dense_n<128>(cx, a);
     return launch_dense_n<64>(cx, a);
 }

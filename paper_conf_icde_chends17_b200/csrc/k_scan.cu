@@ -72,16 +72,49 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
             float theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
             const float rown = __ldg(a.qdist + qpos);  // d(q, c_q)
             const float* cD = a.cand_D + (int64_t)qc * a.mt;
-            for (int c = 0; c < ncand; ++c) {
-                const int tc = __ldg(cl + c);
-                // per-query 2-landmark bound (Eq. 3), then the empty-window checks
-                const int4 ti = __ldg(a.tinfo + tc);  // {lo, hi, r_t, smallest member distance}
-                const float D = __ldg(cD + c), rt = __int_as_float(ti.z);
+            // the per-query 2-landmark bound (Eq. 3) of 32 candidates at once, one
+            // per lane (ascending D is kept: survivors are taken lowest lane first);
+            // a survivor is re-tested with the theta reached when its turn comes
+            for (int c0 = 0; c0 < ncand; c0 += 32) {
+                const int cme = c0 + lane;
+                int tcl = 0;
+                int4 til = make_int4(0, 0, 0, 0);
+                float Dl = 0.f;
+                bool okl = false;
+                if (cme < ncand) {
+                    tcl = __ldg(cl + cme);
+                    til = __ldg(a.tinfo + tcl);  // {lo, hi, r_t, smallest member distance}
+                    Dl = __ldg(cD + cme);
+                    const float rtl = __int_as_float(til.z);
+                    okl = ti_keep(Dl - rown - rtl, theta, Dl + rown + rtl, a.eta);
+                }
+                unsigned pend = __ballot_sync(0xffffffffu, okl);
+              while (pend) {
+                const int src = __ffs(pend) - 1;
+                pend &= pend - 1;
+                const int tc = __shfl_sync(0xffffffffu, tcl, src);
+                int4 ti;
+                ti.x = __shfl_sync(0xffffffffu, til.x, src);
+                ti.y = __shfl_sync(0xffffffffu, til.y, src);
+                ti.z = __shfl_sync(0xffffffffu, til.z, src);
+                ti.w = __shfl_sync(0xffffffffu, til.w, src);
+                const float D = __shfl_sync(0xffffffffu, Dl, src), rt = __int_as_float(ti.z);
                 if (!ti_keep(D - rown - rt, theta, D + rown + rt, a.eta)) continue;
                 const int lo = ti.x, hi = ti.y;
                 float dq2;
-                if constexpr (DP > 0) dq2 = d2_reg<DP>(q, a.tcent + (int64_t)tc * DP);
-                else dq2 = d2_rows(sq, a.tcent + (int64_t)tc * dp, dp);
+                if constexpr (DP > 0) {
+                    dq2 = d2_reg<DP>(q, a.tcent + (int64_t)tc * DP);
+                } else {
+                    // runtime dp: lanes split the dimensions (coalesced center row),
+                    // a fixed reduction tree, lane 0's sum broadcast (warp-uniform dq;
+                    // a bound input, so any fp32 order is covered by the R7 slack)
+                    const float4* c4 = reinterpret_cast<const float4*>(a.tcent + (int64_t)tc * dp);
+                    const float4* q4 = reinterpret_cast<const float4*>(sq);
+                    float part = 0.f;
+                    for (int v = lane; v < dp / 4; v += 32) part = d2_acc4(part, q4[v], __ldg(c4 + v));
+                    for (int o = 16; o > 0; o >>= 1) part += __shfl_down_sync(0xffffffffu, part, o);
+                    dq2 = __shfl_sync(0xffffffffu, part, 0);
+                }
                 const float dq = __fsqrt_rn(dq2);
                 if (lane == 0) ++cevals;
                 if (!ti_keep(dq - rt, theta, dq + rt, a.eta)) continue;
@@ -117,6 +150,7 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
                     theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
                     if (bm) break;
                 }
+              }
             }
             if (lane >= 32 - a.k) write_result(a, __ldg(a.qorig + qpos), lane - (32 - a.k), mine);
         }
@@ -606,79 +640,103 @@ __global__ void __launch_bounds__(256) k_merge_split(ScanArgs a, const int4* __r
 }
 
 // --------------------------------------------------------- merge partials --
-// Warp per query: P sorted lists of k (d2, idx) keys -> the k smallest
-// (the paper's final merge of per-thread sorted heaps, across ranks).
+// Warp per query, P sorted lists of k (d2, idx) keys -> the k smallest (the
+// paper's final merge of per-thread sorted heaps, across ranks).
+// A list is K = 32 R keys (+inf past k), key j in register j / 32 of lane
+// j % 32, read coalesced. Merging the running list A with the next list B
+// keeps the K smallest of their union with a bitonic step: C_j = min(A_j,
+// B_{K-1-j}) holds exactly the K smallest keys as a bitonic sequence, which
+// log2 K half-cleaner stages sort (distances >= 32 inside a lane's
+// registers, < 32 by shuffles). (P - 1) (1 + log2 K) compare-exchanges per
+// query instead of one warp insert per key.
+__device__ __forceinline__ key_t shfl_key(key_t v, int src) {
+    return (key_t)__shfl_sync(0xffffffffu, (unsigned long long)v, src);
+}
+__device__ __forceinline__ key_t shfl_xor_key(key_t v, int m) {
+    return (key_t)__shfl_xor_sync(0xffffffffu, (unsigned long long)v, m);
+}
+
+template <int R>
+__device__ __forceinline__ void load_list(key_t (&v)[R], const int32_t* __restrict__ pidx,
+                                          const float* __restrict__ pd2, int64_t row, int k, int lane) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int j = r * 32 + lane;
+        v[r] = j < k ? make_key(__ldg(pd2 + row + j), __ldg(pidx + row + j)) : kInfKey;
+    }
+}
+
+// sort a bitonic sequence of 32 R keys ascending (key j at reg j / 32, lane j % 32)
+template <int R>
+__device__ __forceinline__ void bitonic_clean(key_t (&v)[R], int lane) {
+#pragma unroll
+    for (int h = R / 2; h >= 1; h >>= 1)  // distances 32 h: registers r and r + h of one lane
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+            if ((r & h) == 0) {
+                const key_t x = v[r], y = v[r + h];
+                v[r] = x < y ? x : y;
+                v[r + h] = x < y ? y : x;
+            }
+#pragma unroll
+    for (int m = 16; m >= 1; m >>= 1) {  // distances < 32: lanes l and l ^ m
+        const bool upper = (lane & m) != 0;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const key_t o = shfl_xor_key(v[r], m);
+            v[r] = upper ? (v[r] < o ? o : v[r]) : (v[r] < o ? v[r] : o);
+        }
+    }
+}
+
+template <int R>
 __global__ void __launch_bounds__(256) k_merge(const int32_t* __restrict__ pidx, const float* __restrict__ pd2, int P,
                                                int64_t nq, int k, int32_t* __restrict__ out_idx,
                                                float* __restrict__ out_dist, int out_squared) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     for (int64_t qi = (int64_t)blockIdx.x * 8 + warp; qi < nq; qi += (int64_t)gridDim.x * 8) {
-        key_t mine = (lane < 32 - k) ? kNegKey : kInfKey;
-        key_t kth = kInfKey;
-        for (int p = 0; p < P; ++p) {
-            const int64_t row = ((int64_t)p * nq + qi) * k;
-            key_t key = kInfKey;
-            if (lane < k) key = make_key(pd2[row + lane], pidx[row + lane]);
-            unsigned cm = __ballot_sync(0xffffffffu, key < kth);
-            while (cm) {
-                const int src = __ffs(cm) - 1;
-                const key_t kk = __shfl_sync(0xffffffffu, key, src);
-                mine = warp_insert(mine, kk, lane);
-                kth = __shfl_sync(0xffffffffu, mine, 31);
-                cm &= ~(1u << src);
-                cm &= __ballot_sync(0xffffffffu, key < kth);
+        key_t A[R], B[R];
+        load_list<R>(A, pidx, pd2, qi * k, k, lane);
+        if (P > 1) load_list<R>(B, pidx, pd2, (nq + qi) * k, k, lane);
+        for (int p = 1; p < P; ++p) {
+            key_t Bn[R];
+            if (p + 1 < P) load_list<R>(Bn, pidx, pd2, ((int64_t)(p + 1) * nq + qi) * k, k, lane);  // prefetch
+            // C_j = min(A_j, B_{K-1-j}); j = 32 r + l  <->  K-1-j = 32 (R-1-r) + (31-l)
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+                const key_t b = shfl_key(B[R - 1 - r], 31 - lane);
+                A[r] = b < A[r] ? b : A[r];
+            }
+            bitonic_clean<R>(A, lane);
+            if (p + 1 < P) {
+#pragma unroll
+                for (int r = 0; r < R; ++r) B[r] = Bn[r];
             }
         }
-        if (lane >= 32 - k) {
-            const int r = lane - (32 - k);
-            const int64_t o = qi * k + r;
-            const float d2 = key_d2(mine);
-            out_dist[o] = out_squared ? d2 : __fsqrt_rn(d2);
-            if (out_idx) out_idx[o] = key_idx(mine);
-        }
-    }
-}
-
-// k > 32: one thread per query, P-way merge of the sorted lists by repeated
-// selection of the smallest head (O(k P) per query).
-__global__ void k_merge_big(const int32_t* __restrict__ pidx, const float* __restrict__ pd2, int P, int64_t nq, int k,
-                            int32_t* __restrict__ out_idx, float* __restrict__ out_dist, int out_squared) {
-    int head[16];
-    for (int64_t qi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; qi < nq; qi += (int64_t)gridDim.x * blockDim.x) {
-        for (int p = 0; p < P; ++p) head[p] = 0;
-        for (int r = 0; r < k; ++r) {
-            key_t best = kInfKey;
-            int bp = 0;
-            for (int p = 0; p < P; ++p) {
-                if (head[p] >= k) continue;
-                const int64_t e = ((int64_t)p * nq + qi) * k + head[p];
-                const key_t key = make_key(pd2[e], pidx[e]);
-                if (key < best) { best = key; bp = p; }
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const int j = r * 32 + lane;
+            if (j < k) {
+                const int64_t o = qi * k + j;
+                const float d2 = key_d2(A[r]);
+                out_dist[o] = out_squared ? d2 : __fsqrt_rn(d2);
+                if (out_idx) out_idx[o] = key_idx(A[r]);
             }
-            head[bp] += 1;
-            const int64_t o = qi * k + r;
-            const float d2 = key_d2(best);
-            out_dist[o] = out_squared ? d2 : __fsqrt_rn(d2);
-            if (out_idx) out_idx[o] = key_idx(best);
         }
     }
 }
 
 sknn_status run_merge(Ctx& cx, const int32_t* part_idx, const float* part_d2, int P, int64_t nq, int k,
                       int32_t* out_idx, float* out_dist, int out_squared) {
-    if (k > 32) {
-        if (P > 16) {
-            set_last_error("sknn_merge_partials: k > 32 supports at most 16 partial lists");
-            return SKNN_ERR_UNSUPPORTED;
-        }
-        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((nq + 255) / 256, (int64_t)cx.num_sms * 8));
-        k_merge_big<<<grid, 256, 0, cx.stream>>>(part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared);
-        cx.launched();
-        return cx.check_launch("merge");
-    }
     int64_t blocks = (nq + 7) / 8;
-    int grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)cx.num_sms * 8));
-    k_merge<<<grid, 256, 0, cx.stream>>>(part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared);
+    int grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)cx.num_sms * 16));
+#define SKNN_MERGE(R) k_merge<R><<<grid, 256, 0, cx.stream>>>(part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared)
+    if (k <= 32) SKNN_MERGE(1);
+    else if (k <= 64) SKNN_MERGE(2);
+    else if (k <= 128) SKNN_MERGE(4);
+    else if (k <= 256) SKNN_MERGE(8);
+    else SKNN_MERGE(16);
+#undef SKNN_MERGE
     cx.launched();
     return cx.check_launch("merge");
 }

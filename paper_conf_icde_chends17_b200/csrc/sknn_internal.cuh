@@ -143,7 +143,7 @@ struct Side {
 
 struct Counters {  // device-side counters (sknn_stats)
     unsigned long long evals_sparse, evals_dense, evals_brute, center_evals, cand_pairs, dense_pairs, dist_recompute,
-        topk_inserts, rows_loaded;
+        topk_inserts, rows_loaded, dense_terms;
 };
 
 }  // namespace sknn

@@ -31,6 +31,15 @@ void set_last_error(const std::string& msg);
         }                                                                                  \
     } while (0)
 
+// The library's private stream-ordered memory pool of a device (api.cu):
+// scratch and index arrays come from it, so its retention policy (up to
+// kPoolRetainBytes kept between calls) never touches the device's default
+// pool that other users of the process allocate from.
+cudaMemPool_t scratch_pool(int device);
+// free device memory usable by this library: cudaMemGetInfo's free bytes plus
+// the private pool's reserved-but-unused bytes
+size_t usable_free_bytes(int device);
+
 struct Ctx {
     cudaStream_t stream = nullptr;
     int device = 0;
@@ -41,9 +50,14 @@ struct Ctx {
 
     void launched() { ++launches; }
 
+    bool capturing = false;  // recording a CUDA graph: allocations become graph memory nodes
+    cudaError_t raw_alloc(void** p, size_t bytes) {
+        if (capturing) return cudaMallocAsync(p, bytes, stream);
+        return cudaMallocFromPoolAsync(p, bytes, scratch_pool(device), stream);
+    }
     sknn_status alloc_scratch(void** p, size_t bytes) {
         if (bytes == 0) bytes = 16;
-        cudaError_t e = cudaMallocAsync(p, bytes, stream);
+        cudaError_t e = raw_alloc(p, bytes);
         if (e != cudaSuccess) {
             set_last_error(std::string("cudaMallocAsync(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
             return SKNN_ERR_OOM;
@@ -53,7 +67,7 @@ struct Ctx {
     }
     sknn_status alloc_persistent(void** p, size_t bytes) {
         if (bytes == 0) bytes = 16;
-        cudaError_t e = cudaMallocAsync(p, bytes, stream);
+        cudaError_t e = raw_alloc(p, bytes);
         if (e != cudaSuccess) {
             set_last_error(std::string("cudaMallocAsync(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
             return SKNN_ERR_OOM;

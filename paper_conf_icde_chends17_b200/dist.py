@@ -75,6 +75,42 @@ def join_query_sharded(Q, T, k: int, *, group=None, self_join: bool | None = Non
     return idx, dst
 
 
+def build_index_broadcast(T, *, group=None, src: int = 0, build=None, create=None, **opts):
+    """Query-sharded mode, index built ONCE: rank `src` clusters T (sknn_build)
+    and every other rank receives the index arrays by torch.distributed
+    broadcast (NCCL over NVLink) into an empty index of the same geometry
+    (sknn_index_create) -- instead of every rank rebuilding it (SURVEY §8(e)
+    "Measure both"). Returns the rank's Index; query it with self_query=1
+    for a self-join. `build`/`create` may be injected (tests)."""
+    from . import Index
+    world, rank = _world(group)
+    build = build or (lambda X, **o: Index(X, **o))
+    create = create or (lambda nt, d, mt, **o: Index.create(nt, d, mt, **o))
+    if rank == src:
+        ix = build(T, **opts)
+        inf = ix.info()
+        geom = torch.tensor([inf["nt"], inf["d"], inf["mt"]], dtype=torch.int64, device=T.device)
+    else:
+        geom = torch.zeros(3, dtype=torch.int64, device=T.device)
+    if world > 1:
+        dist.broadcast(geom, src, group=group)
+    if rank != src:
+        ix = create(int(geom[0]), int(geom[1]), int(geom[2]), **opts)
+    if world > 1:
+        for buf in ix.arrays():
+            dist.broadcast(buf, src, group=group)
+    return ix
+
+
+def join_query_sharded_index(index, Q, k: int, *, group=None, out=None, **opts):
+    """Query-sharded self-join against a shared index (build_index_broadcast):
+    each rank runs sknn_query over the query clusters c with c % P == rank;
+    no data-path collective. Returns the full-size buffers (rows of other
+    ranks untouched)."""
+    world, rank = _world(group)
+    return index.query(Q, k, out=out, self_query=1, shard_rank=rank, shard_count=world, **opts)
+
+
 def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, local_join=None, merge=None,
                         out_squared: bool = False, exchange: str = "all_gather", gather: bool = True, **opts):
     """Target-sharded join: local partial lists of every query against this

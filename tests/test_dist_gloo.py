@@ -124,3 +124,62 @@ def test_two_rank_gloo_matches_single_join():
         np.testing.assert_array_equal(qd, rdist)
         np.testing.assert_array_equal(si, sidx)      # self-join, cluster-interleaved shards
         np.testing.assert_array_equal(sd, sdist_)
+
+
+class _FakeIndex:
+    """CPU stand-in for sknn.Index with the same build/create/info/arrays
+    surface (the orchestration of build_index_broadcast is what is tested)."""
+
+    def __init__(self, arrays, nt, d, mt):
+        self._arr, self.nt, self.d, self.mt = arrays, nt, d, mt
+
+    def info(self):
+        return dict(nt=self.nt, d=self.d, mt=self.mt)
+
+    def arrays(self):
+        return self._arr
+
+
+def _fake_build(X, **_):
+    n, d = X.shape
+    mt = 7
+    g = torch.Generator().manual_seed(5)
+    arrs = [torch.randint(0, 255, (nb,), dtype=torch.uint8, generator=g)
+            for nb in (n * d * 4, n * 4, n * 4, (mt + 1) * 4, mt * d * 4, mt * 4, mt * 16)]
+    return _FakeIndex(arrs, n, d, mt)
+
+
+def _fake_create(nt, d, mt, **_):
+    arrs = [torch.zeros(nb, dtype=torch.uint8) for nb in (nt * d * 4, nt * 4, nt * 4, (mt + 1) * 4, mt * d * 4,
+                                                         mt * 4, mt * 16)]
+    return _FakeIndex(arrs, nt, d, mt)
+
+
+def _bcast_worker(rank, world, port, results):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icde_chends17_b200 import dist as sdist
+    try:
+        X = torch.from_numpy(datagen.c1_uniform_int(50))
+        ix = sdist.build_index_broadcast(X, build=_fake_build, create=_fake_create)
+        results[rank] = (ix.info(), [a.numpy().copy() for a in ix.arrays()])
+    finally:
+        dist.destroy_process_group()
+
+
+def test_build_index_broadcast_two_ranks():
+    """Build once on rank 0, broadcast the index geometry and every array:
+    rank 1 ends with an identical index (the query-sharded mode's alternative
+    to replicated builds)."""
+    world = 2
+    port = _free_port()
+    mgr = mp.Manager()
+    results = mgr.dict()
+    mp.spawn(_bcast_worker, args=(world, port, results), nprocs=world, join=True)
+    i0, a0 = results[0]
+    i1, a1 = results[1]
+    assert i0 == i1 == dict(nt=50, d=4, mt=7)
+    assert len(a0) == len(a1) == 7
+    for x, y in zip(a0, a1):
+        np.testing.assert_array_equal(x, y)

@@ -566,3 +566,154 @@ def test_member_sort_bucket_boundaries(sknn, n):
     idx, dist, _ = run(sknn, X, X, k, True, n_clusters_t=1)
     ridx, rdist = oracle.knn_join(X, X, k)
     assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+def _graph_join(sknn, dQ, dT, k, oi, od, **opts):
+    sknn.join(dQ, dT, k, out=(oi, od), **opts)
+    torch.cuda.synchronize()
+    return oi.cpu().numpy().copy(), od.cpu().numpy().copy()
+
+
+def test_graph_replay_matches_eager(sknn):
+    """Repeated stats-free joins on the same buffers run as a recorded CUDA
+    graph (first call eager, second recorded, then replayed): every call equals
+    the eager join bit for bit, and a replay after new contents are written
+    into the same buffers computes the join of the new contents."""
+    Q, T, k, sj = datagen.workload("C2", 0.1)
+    n = Q.shape[0]
+    dQ = dev(Q)
+    oi = torch.empty((n, k), dtype=torch.int32, device="cuda")
+    od = torch.empty((n, k), dtype=torch.float32, device="cuda")
+    ri, rd = sknn.join(dQ, dQ, k, use_graph=-1)
+    ri, rd = ri.cpu().numpy(), rd.cpu().numpy()
+    for _ in range(4):
+        gi, gd = _graph_join(sknn, dQ, dQ, k, oi, od)
+        np.testing.assert_array_equal(gi, ri)
+        np.testing.assert_array_equal(gd.view(np.uint32), rd.view(np.uint32))
+    Q2 = np.ascontiguousarray(Q[::-1] * np.float32(1.5))
+    dQ.copy_(torch.from_numpy(Q2))
+    gi, gd = _graph_join(sknn, dQ, dQ, k, oi, od)
+    ri2, rd2 = sknn.join(dQ, dQ, k, use_graph=-1)
+    np.testing.assert_array_equal(gi, ri2.cpu().numpy())
+    np.testing.assert_array_equal(gd.view(np.uint32), rd2.cpu().numpy().view(np.uint32))
+    _, odist = oracle.knn_join(Q2, Q2, k)
+    assert_knn_tolerant(Q2, Q2, gi, gd, odist)
+
+
+def test_graph_replay_integer_bitexact(sknn):
+    """C1 and a Q != T integer join through graph replays: bit-exact vs the oracle."""
+    for name, scale in (("C1", 1.0), ("C5", 0.002)):
+        Q, T, k, sj = datagen.workload(name, scale)
+        dQ = dev(Q)
+        dT = dQ if sj else dev(T)
+        oi = torch.empty((Q.shape[0], k), dtype=torch.int32, device="cuda")
+        od = torch.empty((Q.shape[0], k), dtype=torch.float32, device="cuda")
+        ridx, rdist = oracle.knn_join(Q, T, k)
+        for _ in range(3):
+            gi, gd = _graph_join(sknn, dQ, dT, k, oi, od)
+            assert_knn_bitexact(gi, gd, ridx, rdist)
+
+
+@pytest.mark.slow
+def test_c2_full_size_graph_path_sampled(sknn):
+    """C2 at full size in exactly bench.py's timed launch configuration (no
+    stats, repeated calls on the same buffers -> CUDA graph replay): a seeded
+    sample of queries checked against the oracle one by one."""
+    Q, T, k, sj = datagen.workload("C2")
+    n = Q.shape[0]
+    dQ = dev(Q)
+    oi = torch.empty((n, k), dtype=torch.int32, device="cuda")
+    od = torch.empty((n, k), dtype=torch.float32, device="cuda")
+    for _ in range(3):
+        gi, gd = _graph_join(sknn, dQ, dQ, k, oi, od)
+    rng = np.random.default_rng(7)
+    s = rng.choice(n, 2000, replace=False)
+    _, rdist = oracle.knn_join(Q[s], T, k)
+    assert_knn_tolerant(Q[s], T, gi[s], gd[s], rdist)
+
+
+def test_dense_exact_integer_path(sknn):
+    """Integer inputs inside the exactness bound (no bf16 lo part, dp (A+B)^2 <
+    2^24): the dense tiles run the exact variant -- the tensor-core d2 IS the
+    key, nothing is recomputed -- and stay bit-identical to the oracle,
+    including ties (equal-norm sphere) and every k bucket."""
+    Q, T, k, sj = datagen.workload("C4", 0.004)
+    idx, dist, st = run(sknn, Q, T, k, sj, force_path="dense")
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    assert st["dist_evals_dense"] > 0 and st["dist_recompute"] == 0
+    X = datagen.sphere_ties()
+    Qs = np.concatenate([np.zeros((5, 4), np.float32), X[::7]], axis=0)
+    for kk in (1, 8, 13, 16, 20, 24, 31, 32):
+        i2, d2_, st2 = run(sknn, Qs, X, kk, False, force_path="dense")
+        r2, rd2 = oracle.knn_join(Qs, X, kk)
+        assert_knn_bitexact(i2, d2_, r2, rd2)
+        assert st2["dist_recompute"] == 0
+
+
+@pytest.mark.parametrize("hi,d", [(4000, 20), (600, 16)])
+def test_dense_split_precision_fallback(sknn, hi, d):
+    """Integer inputs outside the exactness bound (coordinates whose re-centred
+    values need a bf16 lo part, or dp (A+B)^2 >= 2^24) take the split-precision
+    screen + exact recompute variant; still bit-identical to the oracle."""
+    rng = np.random.default_rng(hi + d)
+    centers = rng.integers(0, hi, size=(20, d))
+    T = (centers[rng.integers(0, 20, 3000)] + rng.integers(-hi // 20, hi // 20 + 1, size=(3000, d)))
+    T = np.clip(T, 0, hi).astype(np.float32)
+    Q = np.clip(centers[rng.integers(0, 20, 500)] + rng.integers(-hi // 20, hi // 20 + 1, size=(500, d)), 0,
+                hi).astype(np.float32)
+    k = 16
+    idx, dist, st = run(sknn, Q, T, k, False, force_path="dense")
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    assert st["dist_evals_dense"] > 0 and st["dist_recompute"] > 0
+
+
+@pytest.mark.parametrize("P,k", [(1, 5), (2, 32), (8, 32), (3, 1), (20, 7), (5, 33), (9, 100), (4, 512), (17, 256)])
+def test_merge_partials_bitonic(sknn, P, k):
+    """sknn_merge_partials (bitonic warp merge) on P sorted lists with many
+    equal distances across lists: the k smallest (d2, idx) keys, compared with
+    a lexicographic sort of the concatenated lists (np.lexsort)."""
+    rng = np.random.default_rng(P * 1000 + k)
+    nq = 700
+    d2 = np.sort(rng.integers(0, 50, size=(P, nq, k)).astype(np.float32), axis=2)
+    idx = (np.arange(k, dtype=np.int64)[None, None, :] + np.arange(P)[:, None, None] * 100_000 +
+           rng.integers(0, 1000, size=(1, nq, 1)) * 0).astype(np.int32)
+    oi, od = sknn.merge_partials(torch.from_numpy(idx).cuda(), torch.from_numpy(d2).cuda(), k, out_squared=True)
+    torch.cuda.synchronize()
+    oi, od = oi.cpu().numpy(), od.cpu().numpy()
+    I = idx.transpose(1, 0, 2).reshape(nq, -1)
+    D = d2.transpose(1, 0, 2).reshape(nq, -1)
+    for q in range(nq):
+        order = np.lexsort((I[q], D[q]))[:k]
+        np.testing.assert_array_equal(oi[q], I[q][order])
+        np.testing.assert_array_equal(od[q], D[q][order])
+
+
+def test_index_create_and_share_arrays(sknn):
+    """sknn_index_create + sknn_index_arrays (the build-once-and-broadcast
+    path): an empty index filled with another index's arrays answers queries
+    and self-queries (self_query=1, query sharding included) bit-identically."""
+    Q, T, k, sj = datagen.workload("C3int", 0.05)
+    dT = dev(T)
+    ix = sknn.Index(dT)
+    inf = ix.info()
+    ix2 = sknn.Index.create(inf["nt"], inf["d"], inf["mt"])
+    for src, dst in zip(ix.arrays(), ix2.arrays()):
+        assert src.numel() == dst.numel()
+        dst.copy_(src)
+    torch.cuda.synchronize()
+    dQ = dev(Q[:500] + 1.0)
+    a = ix.query(dQ, k)
+    b = ix2.query(dQ, k)
+    np.testing.assert_array_equal(a[0].cpu().numpy(), b[0].cpu().numpy())
+    np.testing.assert_array_equal(a[1].cpu().numpy(), b[1].cpu().numpy())
+    ridx, rdist = oracle.knn_join(T, T, k)
+    oi = torch.full((T.shape[0], k), -1, dtype=torch.int32, device="cuda")
+    od = torch.zeros((T.shape[0], k), dtype=torch.float32, device="cuda")
+    for r in range(3):
+        ix2.query(dT, k, out=(oi, od), self_query=1, shard_rank=r, shard_count=3)
+    torch.cuda.synchronize()
+    assert_knn_bitexact(oi.cpu().numpy(), od.cpu().numpy(), ridx, rdist)
+    ix.close()
+    ix2.close()
