@@ -68,7 +68,7 @@ static sknn_status device_info(DevInfo& di) {
 // Private stream-ordered pool per device. Freed scratch stays reserved up to
 // kPoolRetainBytes between calls (repeated joins reuse it without new
 // cudaMalloc work); above that the driver releases it at synchronisation.
-constexpr uint64_t kPoolRetainBytes = uint64_t(2) << 30;
+constexpr uint64_t kPoolRetainBytes = uint64_t(8) << 30;
 
 cudaMemPool_t scratch_pool(int device) {
     static std::mutex mu;
@@ -253,7 +253,9 @@ static int dense_mode_for(const sknn_options& o, int dp) {
 // default window-share threshold of the elastic switch (dp > 16)
 static float dense_tau_for(const sknn_options& o, int dp) {
     if (o.dense_threshold > 0.f) return o.dense_threshold;
-    return dp >= 64 ? 0.5f : 0.95f;
+    // measured with the exact-integer dense tiles (profiles/r02e_sweep_c4):
+    // C4 tau 0.25 / 0.5 / 0.75 / all-dense = 62.4 / 67.6 / 103.3 / 193.9 ms
+    return dp >= 64 ? 0.25f : 0.95f;
 }
 
 // The query half of Fig. 4 (lines 3-6) given both clustered sides:
@@ -281,7 +283,10 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
         lp.dorg = &dorg;
     }
     if (lp.dense_mode == 0 && !lp.dorg) lp.dense_mode = 1;
-    SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
+    {
+        NvtxRange r("sknn level-1 (calUB + groupFilter)");
+        SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
+    }
     // Filter strength (§IV-D1, reading R13): the paper switches to the
     // partial level-2 filter when k/d > 8. Measured on B200 the
     // full filter wins every case once large k runs warp per query
@@ -304,6 +309,7 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
         dpar.eta = eta;
         dpar.topk_out = init_topk;
         dpar.counters = counters;
+        NvtxRange r("sknn dense tiles");
         SKNN_TRY(run_dense(cx, qs, ts, l1, dpar));
         mk.dense = tm.mark();
     }
@@ -329,7 +335,10 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
             SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp, k), k,
                                scan_resident_warps(cx, mapping, ts.dp, k), lp.shard_rank, lp.shard_count, l1));
     }
-    if (full) SKNN_TRY(run_scan(cx, qs, ts, l1, sp));
+    if (full) {
+        NvtxRange r("sknn level-2 scan");
+        SKNN_TRY(run_scan(cx, qs, ts, l1, sp));
+    }
     mk.scan = tm.mark();
     return SKNN_OK;
 }
@@ -372,6 +381,7 @@ static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt
 static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
                             int32_t* out_idx, float* out_dist, const sknn_options* opt_in, sknn_stats* stats,
                             cudaStream_t stream, const sknn_index* index, bool capturing = false) {
+    NvtxRange nvtx_call(index ? "sknn_query" : "sknn_join");
     SKNN_TRY(validate(Q, nq, T ? T : Q, nt, d, k, out_dist));
     if (nq == 0) {
         if (stats) {
@@ -459,6 +469,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
             ts = &index->t;
         } else {
             int m = det_lm_num(nt, o.n_clusters_t);
+            NvtxRange r("sknn build target side");
             if ((st = build_side(cx, dT, nt, d, m, o.landmark_trials, o.lloyd_iters, o.seed, ts_local)) != SKNN_OK)
                 break;
             ts = &ts_local;
@@ -469,6 +480,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
             qs = ts;
         } else {
             int m = det_lm_num(nq, o.n_clusters_q);
+            NvtxRange r("sknn build query side");
             if ((st = build_side(cx, dQ, nq, d, m, o.landmark_trials, o.lloyd_iters, o.seed ^ 0x51ull, qs_local)) !=
                 SKNN_OK)
                 break;

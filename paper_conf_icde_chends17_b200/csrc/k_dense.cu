@@ -189,26 +189,32 @@ struct DenseArgs {
 // per-tile chunk sequence: every dense candidate cluster in NCH-target chunks
 template <int NCH>
 struct ChunkIter {
+    // the chunks of each dense candidate cluster are visited LAST first: the
+    // members are stored by distance to their center descending (R11), so
+    // the tail holds the members nearest the center, which for most queries
+    // of a near cluster are the near targets -- the k-th distance tightens
+    // early and far fewer keys enter the top-k (measured: C4 dense stage)
     const int32_t* dl;
-    int nd, ci, c, nch, tc, size;
+    int nd, ci, c, r, nch, tc, size;
     __device__ __forceinline__ void start(const DenseArgs& a, int qc) {
         dl = a.dcand + (int64_t)qc * a.mt;
         nd = a.dcount[qc];
         ci = -1;
-        c = 0;
+        r = 0;
         nch = 0;
         advance(a);
     }
     // moves to the next chunk; false when exhausted
     __device__ __forceinline__ bool advance(const DenseArgs& a) {
-        ++c;
-        while (c >= nch) {
+        ++r;
+        while (r >= nch) {
             if (++ci >= nd) return false;
             tc = __ldg(dl + ci);
             size = __ldg(a.toff + tc + 1) - __ldg(a.toff + tc);
             nch = (size + NCH - 1) / NCH;
-            c = 0;
+            r = 0;
         }
+        c = nch - 1 - r;
         return true;
     }
     __device__ __forceinline__ bool valid() const { return ci < nd; }
@@ -362,8 +368,8 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
                 }
                 if (cb * 32 + 32 > nb) mask &= (1u << (nb - cb * 32)) - 1u;
                 while (mask) {
-                    const int j = __ffs(mask) - 1;
-                    mask &= mask - 1;
+                    const int j = 31 - __clz(mask);  // highest column first (nearer the center)
+                    mask &= ~(1u << j);
                     const int jj = j0 + cb * 32 + j;
                     const float d2 = d2_rows(qrow, a.trows + (int64_t)jj * dp, dp);
                     ++recomputed;
@@ -613,9 +619,9 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
                         unsigned m = 0;
 #pragma unroll
                         for (int j = 0; j < 16; ++j) m |= (tt[j] <= thr ? 1u : 0u) << j;
-                        while (m) {
-                            const int j = __ffs(m) - 1;
-                            m &= m - 1;
+                        while (m) {  // highest column first (members nearer the center)
+                            const int j = 31 - __clz(m);
+                            m &= ~(1u << j);
                             float tj = tt[0];
 #pragma unroll
                             for (int u = 1; u < 16; ++u)

@@ -32,10 +32,9 @@ namespace sknn {
 //              up to k shifts); heap-sorted once at the end
 // All three keep the k smallest (d2, index) keys seen; insert() requires
 // key < kth() and returns the new k-th key.
-//  LIST_HEAP4  4-ary max-heap, same layout (compile-time k only): an insert
-//              reads the four children of a node together, so the dependent
-//              shared-memory chain is log4 k levels instead of log2 k
-enum { LIST_REG = 0, LIST_SORTED = 1, LIST_HEAP = 2, LIST_HEAP4 = 3 };
+// (measured and rejected: a 4-ary heap -- log4 k dependent levels instead of
+// log2 k -- C2 0.411 vs 0.411 ms, C5 52.2 vs 51.2 ms)
+enum { LIST_REG = 0, LIST_SORTED = 1, LIST_HEAP = 2 };
 
 
 template <int LIST, int KMAX, int STRIDE>
@@ -187,89 +186,6 @@ struct TopList<LIST_HEAP, KMAX, STRIDE> {
             const key_t last = s[end * STRIDE];
             s[end * STRIDE] = top;
             sift(last, end);
-        }
-    }
-    template <class F>
-    __device__ __forceinline__ void emit(F f) const {
-        for (int r = 0; r < k; ++r) f(r, s[r * STRIDE]);
-    }
-};
-
-template <int KMAX, int STRIDE>
-struct TopList<LIST_HEAP4, KMAX, STRIDE> {
-    static_assert(KMAX > 1, "the 4-ary heap needs a compile-time k");
-    key_t* s;
-    int k;
-    __device__ __forceinline__ void init(key_t* col, int k_) {
-        s = col;
-        k = k_;
-#pragma unroll
-        for (int r = 0; r < KMAX; ++r) s[r * STRIDE] = kInfKey;
-    }
-    __device__ __forceinline__ key_t kth() const { return s[0]; }
-    // an ascending list read backwards is a max-heap of any arity
-    __device__ __forceinline__ void load_sorted(const key_t* src) {
-#pragma unroll
-        for (int r = 0; r < KMAX; ++r) s[r * STRIDE] = src[KMAX - 1 - r];
-    }
-    static constexpr int levels() {  // nodes below the root along the deepest path
-        int L = 0, first = 0;        // first index of the current level
-        while (4 * first + 1 < KMAX) {
-            first = 4 * first + 1;
-            ++L;
-        }
-        return L;
-    }
-    // replace the root (the k-th key) by `key` and sift it down
-    __device__ __forceinline__ key_t insert(key_t key) {
-        int i = 0;
-#pragma unroll
-        for (int lev = 0; lev < levels(); ++lev) {
-            const int c0 = 4 * i + 1;
-            if (c0 >= KMAX) break;
-            key_t c = s[c0 * STRIDE];
-            int ci = c0;
-#pragma unroll
-            for (int e = 1; e < 4; ++e) {
-                if (c0 + e < KMAX) {  // compile-time on every level but the partial last one
-                    const key_t v = s[(c0 + e) * STRIDE];
-                    if (c < v) {
-                        c = v;
-                        ci = c0 + e;
-                    }
-                }
-            }
-            if (!(key < c)) break;
-            s[i * STRIDE] = c;
-            i = ci;
-        }
-        s[i * STRIDE] = key;
-        return s[0];
-    }
-    // heapsort into ascending order in s[0, k): pop the max to the end
-    __device__ __forceinline__ void finalize() {
-        for (int end = KMAX - 1; end > 0; --end) {
-            const key_t top = s[0];
-            const key_t last = s[end * STRIDE];
-            s[end * STRIDE] = top;
-            int i = 0;
-            for (;;) {
-                const int c0 = 4 * i + 1;
-                if (c0 >= end) break;
-                key_t c = s[c0 * STRIDE];
-                int ci = c0;
-                for (int e = 1; e < 4 && c0 + e < end; ++e) {
-                    const key_t v = s[(c0 + e) * STRIDE];
-                    if (c < v) {
-                        c = v;
-                        ci = c0 + e;
-                    }
-                }
-                if (!(last < c)) break;
-                s[i * STRIDE] = c;
-                i = ci;
-            }
-            s[i * STRIDE] = last;
         }
     }
     template <class F>
@@ -443,12 +359,18 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
 #ifndef SKNN_COLLECT
 #define SKNN_COLLECT 1
 #endif
+#ifndef SKNN_U16
+#define SKNN_U16 2
+#endif
+#ifndef SKNN_MINB16
+#define SKNN_MINB16 1
+#endif
 #ifndef SKNN_UNION_MINB4
 #define SKNN_UNION_MINB4 3
 #endif
 template <int DP>
 constexpr int union_block() {
-    return DP == 0 ? 1 : (DP <= 4 ? SKNN_U4 : (DP <= 8 ? 4 : (DP <= 16 ? 2 : 1)));
+    return DP == 0 ? 1 : (DP <= 4 ? SKNN_U4 : (DP <= 8 ? 4 : (DP <= 16 ? SKNN_U16 : 1)));
 }
 
 // One warp tile of the thread-per-query scan with a WARP-UNION member walk
@@ -713,7 +635,7 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
 // (2 CTAs / SM; the two inlined task bodies otherwise take ~190)
 template <int DP, int LIST, int THREADS, int WALK>
 constexpr int tpq_min_blocks() {
-    return THREADS != 256 ? 1 : (LIST == LIST_REG ? 2 : (DP == 4 ? (WALK ? SKNN_UNION_MINB4 : 4) : 1));
+    return THREADS != 256 ? 1 : (LIST == LIST_REG ? 2 : (DP == 4 ? (WALK ? SKNN_UNION_MINB4 : 4) : (DP == 16 ? SKNN_MINB16 : 1)));
 }
 template <int DP, int KMAX, int LIST, int THREADS, int WALK>
 __global__ void __launch_bounds__(THREADS, (tpq_min_blocks<DP, LIST, THREADS, WALK>())) k_scan_tpq(ScanArgs a) {
@@ -762,7 +684,7 @@ static void launch_tpq_walk(Ctx& cx, const ScanArgs& a) {
 // (per-lane LB-ordered walk) overrides for ablation.
 template <int DP, int KMAX, int LIST, int THREADS>
 static void launch_tpq(Ctx& cx, const ScanArgs& a) {
-    if constexpr ((LIST == LIST_HEAP || LIST == LIST_HEAP4) && KMAX > 1) {  // compile-time k: the default walk only
+    if constexpr (LIST == LIST_HEAP && KMAX > 1) {  // compile-time k: the default walk only
         launch_tpq_walk<DP, KMAX, LIST, THREADS, (KMAX > 24 ? 2 : 1)>(cx, a);
     } else {
         const char* w = getenv("SKNN_WALK");
@@ -782,8 +704,7 @@ static void launch_tpq(Ctx& cx, const ScanArgs& a) {
 static int topk_override() {
     const char* ov = getenv("SKNN_TOPK");
     if (!ov) return -1;
-    if (ov[0] == 'h') return ov[4] == '4' ? LIST_HEAP4 : LIST_HEAP;
-    return ov[0] == 'r' ? LIST_REG : LIST_SORTED;
+    return ov[0] == 'r' ? LIST_REG : (ov[0] == 'h' ? LIST_HEAP : LIST_SORTED);
 }
 
 template <int DP, int KMAX>
@@ -798,15 +719,6 @@ static void launch_tpq_small_k(Ctx& cx, const ScanArgs& a) {
     if (list == LIST_SORTED) {
         launch_tpq<DP, 1, LIST_SORTED, 256>(cx, a);
         return;
-    }
-    if (list == LIST_HEAP4) {
-        switch (a.k) {
-            case 8: launch_tpq<DP, 8, LIST_HEAP4, 256>(cx, a); return;
-            case 16: launch_tpq<DP, 16, LIST_HEAP4, 256>(cx, a); return;
-            case 20: launch_tpq<DP, 20, LIST_HEAP4, 256>(cx, a); return;
-            case 32: launch_tpq<DP, 32, LIST_HEAP4, 256>(cx, a); return;
-            default: list = LIST_HEAP; break;
-        }
     }
     if (list == LIST_HEAP) {
         // the configs' k (C1 8, C3/C4 16, C2 20, C5 32) get a compile-time k

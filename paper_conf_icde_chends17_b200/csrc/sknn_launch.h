@@ -9,6 +9,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../include/sknn.h"
 #include "sknn_internal.cuh"
 
@@ -39,6 +41,15 @@ cudaMemPool_t scratch_pool(int device);
 // free device memory usable by this library: cudaMemGetInfo's free bytes plus
 // the private pool's reserved-but-unused bytes
 size_t usable_free_bytes(int device);
+
+// NVTX range around a host-side stage of a call (header-only NVTX v3: no
+// link dependency, a no-op unless a tool such as Nsight Systems is attached)
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 struct Ctx {
     cudaStream_t stream = nullptr;
