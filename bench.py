@@ -324,6 +324,8 @@ def main():
     ap.add_argument("--config", default="C2")
     ap.add_argument("--mode", default="query", choices=["query", "target"])
     ap.add_argument("--exchange", default="all_to_all", choices=["all_to_all", "all_gather"])
+    ap.add_argument("--global-ub", action="store_true",
+                    help="target mode: prune every shard with the global level-1 bound (all-reduce MIN)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -393,13 +395,13 @@ def main():
                              index_base=int(tlo), **opts)
 
         def step():
-            if ws == 1:
+            if ws == 1 and not args.global_ub:
                 local_join()
             else:
                 sdist.join_target_sharded(Q, Tshard, k, tlo, group=group, exchange=args.exchange, gather=False,
-                                          **opts)
-        parallelism = "target-sharded x%d (%s exchange of partial k-lists + exact merge)" % (
-            ws, args.exchange if ws > 1 else "no")
+                                          global_ub=args.global_ub, **opts)
+        parallelism = "target-sharded x%d (%s exchange of partial k-lists + exact merge%s)" % (
+            ws, args.exchange if ws > 1 else "no", ", global level-1 bound" if args.global_ub else "")
         nq_rank = nq
 
     for _ in range(args.warmup):

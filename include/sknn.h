@@ -117,9 +117,17 @@ typedef struct {
                               /*   0 = auto: yes iff Q is the SAME POINTER and size as the build    */
                               /*   input -- the build buffer must then still be alive and unchanged */
                               /*   (a freed-and-reused address would silently answer for old rows) */
+    int32_t pad1;
+    const float* ub_in;       /* optional DEVICE [mq] upper bounds of the query clusters' k-th    */
+                              /*   distance (e.g. sknn_level1_bounds of every target shard, min  */
+                              /*   over ranks); level-1 takes min(its calUB, ub_in[qc]). Only    */
+                              /*   meaningful with the query side of sknn_join_indexed / the same */
+                              /*   query clustering; rows may then hold fewer than k real entries */
+                              /*   (placeholders: distance +inf, index -1) -- for partial lists  */
     int32_t use_graph;        /* sknn_join_ex on device pointers without stats: 0 = auto (replay a */
                               /*   captured CUDA graph of the whole join when the same shapes,     */
                               /*   pointers and options repeat), -1 = never                         */
+    int32_t pad2;
 } sknn_options;
 
 /* Counters and per-stage times of one call (filled only when a non-NULL
@@ -268,6 +276,24 @@ sknn_status sknn_index_arrays(const sknn_index* index, void** ptr, size_t* bytes
  * sknn_options.self_query = 1. */
 sknn_status sknn_index_create(int64_t nt, int32_t d, int32_t mt, const sknn_options* opt,
                               sknn_index** out);
+
+/* Join of two prebuilt indexes: the query index (sknn_build over Q, whose
+ * clustering is then reused, P:L241 Step 1 for Q) against the target index
+ * (Steps 2-3, Fig. 4 lines 3-6). Output rows in the query index's original row
+ * order. This is the target-sharded mode's building block: every rank clusters
+ * Q identically (seeded), exchanges level-1 bounds (sknn_level1_bounds) and
+ * joins with opt->ub_in = the minimum over ranks. Device outputs. */
+sknn_status sknn_join_indexed(const sknn_index* qindex, const sknn_index* tindex, int32_t k,
+                              int32_t* out_idx, float* out_dist, const sknn_options* opt,
+                              sknn_stats* stats, sknn_stream_t stream);
+
+/* Level-1 upper bounds (calUB) of every query cluster of qindex
+ * against tindex: ub_out DEVICE [mq] (mq = sknn_index_info(qindex).mt),
+ * +inf for an empty query cluster. Each value bounds the k-th nearest
+ * distance of every member of the cluster among tindex's points, hence among
+ * any superset of them (the minimum over target shards is a global bound). */
+sknn_status sknn_level1_bounds(const sknn_index* qindex, const sknn_index* tindex, int32_t k,
+                               const sknn_options* opt, float* ub_out, sknn_stream_t stream);
 
 /* Level-1 products of a query against an index, to HOST buffers (testing):
  * q_cluster [nq] cluster of each query, ub [mq] the inflated upper bound of

@@ -33,7 +33,8 @@ MAX_K = 512
 ABI_SYMBOLS = ["sknn_options_default", "sknn_join", "sknn_join_ex", "sknn_build", "sknn_query",
                "sknn_merge_partials", "sknn_index_free", "sknn_index_info", "sknn_index_export",
                "sknn_debug_level1", "sknn_config_decide", "sknn_error_string", "sknn_last_error",
-               "sknn_version", "sknn_index_arrays", "sknn_index_create"]
+               "sknn_version", "sknn_index_arrays", "sknn_index_create", "sknn_join_indexed",
+               "sknn_level1_bounds"]
 INDEX_ARRAYS = ("rows", "dist", "orig", "off", "centers", "radius", "tinfo")
 
 
@@ -50,7 +51,8 @@ class Options(ctypes.Structure):
                 ("mapping", ctypes.c_int32), ("dense_threshold", ctypes.c_float), ("r_factor", ctypes.c_float),
                 ("out_squared", ctypes.c_int32), ("pad0", ctypes.c_int32), ("index_base", ctypes.c_int64),
                 ("shard_rank", ctypes.c_int32), ("shard_count", ctypes.c_int32), ("query_batch", ctypes.c_int64),
-                ("self_query", ctypes.c_int32), ("use_graph", ctypes.c_int32)]
+                ("self_query", ctypes.c_int32), ("pad1", ctypes.c_int32), ("ub_in", ctypes.c_void_p),
+                ("use_graph", ctypes.c_int32), ("pad2", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -126,10 +128,14 @@ def lib():
             L.sknn_last_error.restype = ctypes.c_char_p
             L.sknn_version.restype = _i32
             L.sknn_index_arrays.argtypes = [_vp, ctypes.POINTER(_vp), ctypes.POINTER(ctypes.c_size_t)]
+            L.sknn_join_indexed.argtypes = [_vp, _vp, _i32, _vp, _vp, ctypes.POINTER(Options),
+                                            ctypes.POINTER(Stats), _vp]
+            L.sknn_level1_bounds.argtypes = [_vp, _vp, _i32, ctypes.POINTER(Options), _vp, _vp]
             L.sknn_index_create.argtypes = [_i64, _i32, _i32, ctypes.POINTER(Options), ctypes.POINTER(_vp)]
             for fn in ("sknn_join", "sknn_join_ex", "sknn_build", "sknn_query", "sknn_merge_partials",
                        "sknn_index_free", "sknn_index_info", "sknn_index_export", "sknn_debug_level1",
-                       "sknn_config_decide", "sknn_index_arrays", "sknn_index_create"):
+                       "sknn_config_decide", "sknn_index_arrays", "sknn_index_create", "sknn_join_indexed",
+                       "sknn_level1_bounds"):
                 getattr(L, fn).restype = _i32
             _lib = L
     return _lib
@@ -150,6 +156,8 @@ def make_options(**kw) -> Options:
             val = PATH[val]
         if key == "mapping" and isinstance(val, str):
             val = MAPPING[val]
+        if key == "ub_in" and hasattr(val, "data_ptr"):  # a CUDA float32 tensor [mq]
+            val = val.data_ptr()
         if not hasattr(o, key):
             raise TypeError("unknown option %r" % key)
         setattr(o, key, val)
@@ -371,6 +379,40 @@ def _device_bytes(ptr, nbytes, device, owner):
 
 def build(T, **opts) -> Index:
     return Index(T, **opts)
+
+
+def join_indexed(qindex: Index, tindex: Index, k: int, *, stream=None, stats: bool = False, out=None, **opts):
+    """The query index's points against the target index (sknn_join_indexed):
+    (idx, dist) [nq, k] on the device, rows in the query set's original order."""
+    import torch
+    nq = qindex.nt
+    dev = torch.device("cuda", torch.cuda.current_device())
+    if out is not None:
+        idx, dist = out
+    else:
+        idx = torch.empty((nq, k), dtype=torch.int32, device=dev)
+        dist = torch.empty((nq, k), dtype=torch.float32, device=dev)
+    o = make_options(**opts)
+    st = Stats()
+    st.struct_size = ctypes.sizeof(Stats)
+    _check(lib().sknn_join_indexed(qindex._handle, tindex._handle, k, idx.data_ptr() if idx is not None else None,
+                                   dist.data_ptr(), ctypes.byref(o), ctypes.byref(st) if stats else None,
+                                   _stream_ptr(stream, dev)))
+    if stats:
+        return idx, dist, st.to_dict()
+    return idx, dist
+
+
+def level1_bounds(qindex: Index, tindex: Index, k: int, *, stream=None, **opts):
+    """Level-1 calUB of every query cluster of qindex against tindex
+    (sknn_level1_bounds): a CUDA float32 tensor [mq]."""
+    import torch
+    dev = torch.device("cuda", torch.cuda.current_device())
+    ub = torch.empty(qindex.info()["mt"], dtype=torch.float32, device=dev)
+    o = make_options(**opts)
+    _check(lib().sknn_level1_bounds(qindex._handle, tindex._handle, k, ctypes.byref(o), ub.data_ptr(),
+                                    _stream_ptr(stream, dev)))
+    return ub
 
 
 def merge_partials(part_idx, part_d2, k: int, *, out_squared: bool = False, stream=None, out=None):

@@ -272,6 +272,7 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     lp.shard_count = o.shard_count > 1 ? o.shard_count : 1;
     lp.dense_mode = dense_mode_for(o, ts.dp);
     lp.dense_tau = dense_tau_for(o, ts.dp);
+    lp.ub_in = o.ub_in;
     if (lp.dense_mode == 2 && (!dense_supported(ts.dp) || k > 32)) {
         set_last_error("force_path = DENSE needs d <= 256 and k <= 32");
         return SKNN_ERR_UNSUPPORTED;
@@ -380,8 +381,12 @@ static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt
 // Shared body of sknn_join_ex / sknn_query.
 static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
                             int32_t* out_idx, float* out_dist, const sknn_options* opt_in, sknn_stats* stats,
-                            cudaStream_t stream, const sknn_index* index, bool capturing = false) {
-    NvtxRange nvtx_call(index ? "sknn_query" : "sknn_join");
+                            cudaStream_t stream, const sknn_index* index, bool capturing = false,
+                            const sknn_index* qindex = nullptr) {
+    NvtxRange nvtx_call(qindex ? "sknn_join_indexed" : (index ? "sknn_query" : "sknn_join"));
+    // a query index supplies the clustered query side (Q is not read)
+    static const float kNoQ = 0.f;
+    if (qindex) Q = &kNoQ;
     SKNN_TRY(validate(Q, nq, T ? T : Q, nt, d, k, out_dist));
     if (nq == 0) {
         if (stats) {
@@ -406,7 +411,7 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     tm.start(stream, stats != nullptr);
     sknn_status st = SKNN_OK;
     const int dp = (d + 3) & ~3;
-    const bool self = index ? index_self_query(o, Q, nq, index) : (Q == T && nq == nt);
+    const bool self = qindex ? qindex == index : (index ? index_self_query(o, Q, nq, index) : (Q == T && nq == nt));
     int mapping = choose_mapping(o, di, nq, dp, k);
     int path = o.force_path == SKNN_PATH_BRUTE ? SKNN_PATH_BRUTE : SKNN_PATH_SPARSE;
     Marks mk;
@@ -421,8 +426,10 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     Counters* counters = nullptr;
     do {
         const void* tmp;
-        if ((st = stage_in(cx, Q, sizeof(float) * nq * d, &tmp, &q_host)) != SKNN_OK) break;
-        dQ = (const float*)tmp;
+        if (!qindex) {
+            if ((st = stage_in(cx, Q, sizeof(float) * nq * d, &tmp, &q_host)) != SKNN_OK) break;
+            dQ = (const float*)tmp;
+        }
         if (!index) {
             if (self) {
                 dT = dQ;
@@ -478,6 +485,8 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
         const Side* qs;
         if (self) {
             qs = ts;
+        } else if (qindex) {
+            qs = &qindex->t;
         } else {
             int m = det_lm_num(nq, o.n_clusters_q);
             NvtxRange r("sknn build query side");
@@ -746,6 +755,45 @@ sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq, int3
         }
     }
     return run_join(Q, nq, nullptr, index->t.n, d, k, out_idx, out_dist, opt, stats, (cudaStream_t)stream, index);
+}
+
+sknn_status sknn_join_indexed(const sknn_index* qindex, const sknn_index* tindex, int32_t k, int32_t* out_idx,
+                              float* out_dist, const sknn_options* opt, sknn_stats* stats, sknn_stream_t stream) {
+    if (!qindex || !tindex) return fail(SKNN_ERR_INVALID_ARG, "index is NULL");
+    if (qindex->t.d != tindex->t.d) return fail(SKNN_ERR_INVALID_ARG, "query and target dimensions differ");
+    if (qindex->device != tindex->device) return fail(SKNN_ERR_WRONG_DEVICE, "indexes on different devices");
+    return run_join(nullptr, qindex->t.n, nullptr, tindex->t.n, tindex->t.d, k, out_idx, out_dist, opt, stats,
+                    (cudaStream_t)stream, tindex, false, qindex);
+}
+
+sknn_status sknn_level1_bounds(const sknn_index* qindex, const sknn_index* tindex, int32_t k, const sknn_options* opt,
+                               float* ub_out, sknn_stream_t stream) {
+    if (!qindex || !tindex || !ub_out) return fail(SKNN_ERR_INVALID_ARG, "NULL pointer");
+    if (qindex->t.d != tindex->t.d) return fail(SKNN_ERR_INVALID_ARG, "query and target dimensions differ");
+    if (k <= 0 || (int64_t)k > tindex->t.n || k > SKNN_MAX_K) return fail(SKNN_ERR_INVALID_ARG, "bad k");
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    if (qindex->device != di.device || tindex->device != di.device)
+        return fail(SKNN_ERR_WRONG_DEVICE, "index built on another device");
+    if (classify(ub_out, di.device) != PTR_DEVICE) return fail(SKNN_ERR_NOT_DEVICE_PTR, "ub_out must be device memory");
+    const sknn_options o = merge_options(opt);
+    Ctx cx;
+    cx.stream = (cudaStream_t)stream;
+    cx.device = di.device;
+    cx.num_sms = di.num_sms;
+    Level1 l1;
+    Level1Params lp;
+    lp.k = k;
+    lp.eta = rounding_eta(tindex->t.d);
+    lp.dense_mode = 1;
+    lp.ub_in = o.ub_in;
+    sknn_status st = run_level1(cx, qindex->t, tindex->t, lp, l1, nullptr);
+    if (st == SKNN_OK) {
+        cudaError_t e = cudaMemcpyAsync(ub_out, l1.ub, sizeof(float) * qindex->t.m, cudaMemcpyDeviceToDevice, cx.stream);
+        if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("level-1 bounds copy: ") + cudaGetErrorString(e));
+    }
+    cx.free_all();
+    return st;
 }
 
 sknn_status sknn_merge_partials(const int32_t* part_idx, const float* part_d2, int32_t P, int64_t nq, int32_t k,

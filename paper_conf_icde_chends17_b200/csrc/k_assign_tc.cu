@@ -6,10 +6,14 @@
 // RECORDED member-center distance to be exact, not the nearest center), so the
 // nearest center is chosen from
 //     score_j = ||b_j||^2 - 2 a.b_j,   a = x - o, b_j = c_j - o   (o = mean center)
-// with a and b rounded to bf16 and a.b_j accumulated in fp32 by tcgen05.mma
-// (kind::f16, M = 128 points x N = 128 centers per MMA, K = d padded to 16);
-// ||a||^2 is the same for every j and drops out of the argmin. The exact fp32
-// distance to the chosen center (the shared d2 formula) is then recomputed.
+// with a and b rounded to bf16 and the whole score produced by tcgen05.mma
+// (kind::f16, M = 128 points x N = 128 centers per MMA, fp32 accumulation):
+// K is augmented by two columns, a' = [a, 1, 1], b'_j = [-2 b_j, hi_j, lo_j]
+// with hi + lo the bf16 split of ||b_j||^2 (of the rounded b_j), so
+// a'.b'_j = ||b_j||^2 - 2 a.b_j and the epilogue is a plain min (one FMNMX per
+// score). ||a||^2 is the same for every j and drops out of the argmin. The
+// exact fp32 distance to the chosen center (the shared d2 formula) is then
+// recomputed.
 //
 // Data movement: the centers are pre-converted once per pass into the UMMA
 // canonical K-major layout (8-row x 16-byte core matrices), chunk by chunk, so a
@@ -48,79 +52,97 @@ __global__ void k_center_mean(const float* __restrict__ centers, int m, int dp, 
     if (threadIdx.x == 0) o[c] = (float)(red[0] / m);
 }
 
-// centers -> bf16 (c - o) in chunked core-matrix layout + ||b||^2 of the rounded values
+// centers -> b' = [-2 (c - o), hi, lo] (bf16) in chunked core-matrix layout,
+// hi + lo = ||bf16(c - o)||^2; padding centers get hi = +inf (score +inf)
 __global__ void k_centers_to_tc(const float* __restrict__ centers, int m, int mpad, int dp, int kp,
-                                const float* __restrict__ o, __nv_bfloat16* __restrict__ out, float* __restrict__ bn) {
+                                const float* __restrict__ o, __nv_bfloat16* __restrict__ out) {
     const int c8n = kp / 8;
-    const int64_t total = (int64_t)mpad * c8n;
-    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < total; w += (int64_t)gridDim.x * blockDim.x) {
-        const int j = (int)(w / c8n), c8 = (int)(w % c8n);
-        uint32_t h[4];
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-            float v0 = 0.f, v1 = 0.f;
-            const int k0 = c8 * 8 + 2 * i;
-            if (j < m && k0 < dp) v0 = centers[(int64_t)j * dp + k0] - o[k0];
-            if (j < m && k0 + 1 < dp) v1 = centers[(int64_t)j * dp + k0 + 1] - o[k0 + 1];
-            h[i] = (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v0)) |
-                   ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v1)) << 16);
-        }
-        const int chunk = j / kTcN, r = j % kTcN;
-        const size_t off = (size_t)chunk * kTcN * kp * 2 + (size_t)(r >> 3) * kp * 16 + (size_t)c8 * 128 + (size_t)(r & 7) * 16;
-        *reinterpret_cast<uint4*>(reinterpret_cast<unsigned char*>(out) + off) = make_uint4(h[0], h[1], h[2], h[3]);
-    }
+    const float INF = __int_as_float(0x7f800000);
     for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < mpad; j += gridDim.x * blockDim.x) {
-        float s = __int_as_float(0x7f800000);
-        if (j < m) {
-            s = 0.f;
+        float nb = 0.f;
+        if (j < m)
             for (int k = 0; k < dp; ++k) {
                 const float v = __bfloat162float(__float2bfloat16_rn(centers[(int64_t)j * dp + k] - o[k]));
-                s = __fmaf_rn(v, v, s);
+                nb = __fmaf_rn(v, v, nb);
             }
+        const __nv_bfloat16 hi = __float2bfloat16_rn(j < m ? nb : INF);
+        const __nv_bfloat16 lo = __float2bfloat16_rn(j < m ? nb - __bfloat162float(hi) : 0.f);
+        const int chunk = j / kTcN, r = j % kTcN;
+        for (int c8 = 0; c8 < c8n; ++c8) {
+            uint32_t h[4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                __nv_bfloat16 e[2];
+#pragma unroll
+                for (int t = 0; t < 2; ++t) {
+                    const int k0 = c8 * 8 + 2 * i + t;
+                    float v = 0.f;
+                    if (j < m && k0 < dp) v = -2.f * __bfloat162float(__float2bfloat16_rn(centers[(int64_t)j * dp + k0] - o[k0]));
+                    e[t] = __float2bfloat16_rn(v);  // exact: -2 times a bf16 value
+                    if (k0 == dp) e[t] = hi;
+                    if (k0 == dp + 1) e[t] = lo;
+                }
+                h[i] = (uint32_t)__bfloat16_as_ushort(e[0]) | ((uint32_t)__bfloat16_as_ushort(e[1]) << 16);
+            }
+            const size_t off = (size_t)chunk * kTcN * kp * 2 + (size_t)(r >> 3) * kp * 16 + (size_t)c8 * 128 + (size_t)(r & 7) * 16;
+            *reinterpret_cast<uint4*>(reinterpret_cast<unsigned char*>(out) + off) = make_uint4(h[0], h[1], h[2], h[3]);
         }
-        bn[j] = s;
     }
 }
 
-// One CTA = 128 points, 8 warps: warps w and w + 4 read the same 32 TMEM lanes
-// (points) and split each chunk's 128 columns in halves. Streams every center
-// chunk through a 2-deep bulk-copy ring.
-constexpr int kTcThreads = 256;
+// One CTA = 256 points (two 128-row A tiles sharing every B chunk, so each
+// center chunk read from L2 feeds two MMAs), 9 warps, warp-specialised:
+//  * warp 8, one elected thread: the producer -- streams the center chunks
+//    through a kStages-deep bulk-copy ring and issues, per chunk, the MMAs of
+//    both A tiles into one of two accumulator pairs (TMEM: 2 x 2 x 128 = 512
+//    columns, one CTA per SM); a stage is refilled as soon as its MMAs are done
+//    (sfree), an accumulator pair as soon as the epilogue released it (afree);
+//  * warps 0-7: the epilogue -- thread (w, lane) owns row 32 (w % 4) + lane of
+//    both A tiles and half w / 4 of the chunk's 128 columns: per 32 columns one
+//    tcgen05.ld and a min tree (one FMNMX per score), the argmin index only on
+//    improvement (lowest column on ties).
+constexpr int kTcEpiWarps = 8;
+constexpr int kTcThreads = (kTcEpiWarps + 1) * 32;
+constexpr int kTcPts = 2 * kTcM;  // points per CTA
+constexpr int kTcMaxStages = 6;
+
 __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __restrict__ Xp, int64_t n, int dp, int kp,
                                                        const float* __restrict__ o,
-                                                       const __nv_bfloat16* __restrict__ cbf,
-                                                       const float* __restrict__ bn, int m, int nchunks,
-                                                       const float* __restrict__ centers,
+                                                       const __nv_bfloat16* __restrict__ cbf, int m, int nchunks,
+                                                       int nstages, const float* __restrict__ centers,
                                                        int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
                                                        long long* __restrict__ sums, const double* __restrict__ fx,
                                                        int32_t* __restrict__ counts, int stride) {
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t a_bytes = (uint32_t)kTcM * kp * 2, b_bytes = (uint32_t)kTcN * kp * 2;
-    unsigned char* sA = smem;
-    auto sB = [&](int b) { return smem + a_bytes + (uint32_t)b * b_bytes; };
-    auto sBn = [&](int b) { return reinterpret_cast<float*>(smem + a_bytes + 2 * b_bytes) + b * kTcN; };
-    __shared__ __align__(8) uint64_t bar_full[2], bar_mma[2];
+    unsigned char* sA = smem;                     // [2][a_bytes]
+    unsigned char* sB0 = smem + 2 * (size_t)a_bytes;  // [nstages][b_bytes]
+    __shared__ __align__(8) uint64_t bar_full[kTcMaxStages], bar_sfree[kTcMaxStages], bar_mma[2], bar_afree[2];
     __shared__ uint32_t s_tmem;
-    const int tid = threadIdx.x, warp = tid >> 5;
+    __shared__ float s_best[2][kTcM];
+    __shared__ int s_bi[2][kTcM];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const uint32_t sbo = (uint32_t)kp * 16u;
 
-    if (warp == 0) {
-        tc::tmem_alloc(&s_tmem, 2u * kTcN);
-    }
+    if (warp == kTcEpiWarps) tc::tmem_alloc(&s_tmem, 4u * kTcN);
     if (tid == 0) {
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < nstages; ++i) {
             tc::mbar_init(smem_u32(&bar_full[i]), 1);
+            tc::mbar_init(smem_u32(&bar_sfree[i]), 1);
+        }
+        for (int i = 0; i < 2; ++i) {
             tc::mbar_init(smem_u32(&bar_mma[i]), 1);
+            tc::mbar_init(smem_u32(&bar_afree[i]), kTcEpiWarps);
         }
         tc::mbar_fence_init();
     }
-    // stage A = x - o (bf16) for the CTA's 128 points
-    const int64_t row0 = (int64_t)blockIdx.x * kTcM;
+    // stage A' = [x - o, 1, 1] (bf16) for the CTA's 256 points (both tiles)
+    const int64_t row0 = (int64_t)blockIdx.x * kTcPts;
     {
         const int c8n = kp / 8;
-        for (int w = tid; w < kTcM * c8n; w += blockDim.x) {
-            const int r = w / c8n, c8 = w % c8n;
-            const int64_t i = (row0 + r) * stride;
+        for (int w = tid; w < kTcPts * c8n; w += blockDim.x) {
+            const int rr = w / c8n, c8 = w % c8n;
+            const int64_t i = (row0 + rr) * stride;
             uint32_t h[4];
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
@@ -128,10 +150,13 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
                 const int k0 = c8 * 8 + 2 * e;
                 if (i < n && k0 < dp) v0 = Xp[i * dp + k0] - o[k0];
                 if (i < n && k0 + 1 < dp) v1 = Xp[i * dp + k0 + 1] - o[k0 + 1];
+                if (k0 == dp || k0 == dp + 1) v0 = 1.f;          // a' = [a, 1, 1]
+                if (k0 + 1 == dp || k0 + 1 == dp + 1) v1 = 1.f;
                 h[e] = (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v0)) |
                        ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v1)) << 16);
             }
-            const uint32_t off = (uint32_t)(r >> 3) * sbo + (uint32_t)c8 * 128u + (uint32_t)(r & 7) * 16u;
+            const int t = rr >> 7, r = rr & 127;
+            const uint32_t off = (uint32_t)t * a_bytes + (uint32_t)(r >> 3) * sbo + (uint32_t)c8 * 128u + (uint32_t)(r & 7) * 16u;
             *reinterpret_cast<uint4*>(sA + off) = make_uint4(h[0], h[1], h[2], h[3]);
         }
     }
@@ -140,139 +165,136 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
     __syncthreads();
     tc::fence_after();
     const uint32_t tmem = s_tmem;
-    const uint32_t idesc = idesc_bf16_m128(kTcN);
 
-    auto issue_copy = [&](int chunk, int buf) {
-        const uint32_t bar = smem_u32(&bar_full[buf]);
-        const uint32_t bytes = b_bytes + kTcN * 4;
-        tc::expect_tx(bar, bytes);
-        const unsigned char* src = reinterpret_cast<const unsigned char*>(cbf) + (size_t)chunk * b_bytes;
-        tc::bulk_g2s(smem_u32(sB(buf)), src, b_bytes, bar);
-        tc::bulk_g2s(smem_u32(sBn(buf)), bn + (size_t)chunk * kTcN, (uint32_t)(kTcN * 4), bar);
-    };
-    auto issue_mma = [&](int buf) {
-        tc::fence_after();
-        const uint32_t aB = smem_u32(sA), bB = smem_u32(sB(buf));
-        for (int s = 0; s < kp / 16; ++s)
-            tc::mma_bf16(tmem + (uint32_t)(buf * kTcN), desc_kmajor(aB + s * 256u, sbo), desc_kmajor(bB + s * 256u, sbo),
-                         idesc, s > 0);
-        tc::mma_commit(smem_u32(&bar_mma[buf]));
-    };
-
-    uint32_t ph_full[2] = {0, 0}, ph_mma[2] = {0, 0};
-    if (tid == 0) {
-        issue_copy(0, 0);
-        if (nchunks > 1) issue_copy(1, 1);
-        tc::mbar_wait(smem_u32(&bar_full[0]), 0);
-        issue_mma(0);
-    }
-    ph_full[0] = 1;
-    float best = __int_as_float(0x7f800000);
-    int bi = 0;
-    const int half = warp >> 2;  // columns [64 * half, 64 * half + 64) of every chunk
-    const uint32_t trow = tmem + ((uint32_t)((warp & 3) * 32) << 16);
-    for (int c = 0; c < nchunks; ++c) {
-        const int buf = c & 1;
-        // issue the next chunk's MMA as soon as its copy landed (overlaps this epilogue)
-        if (tid == 0 && c + 1 < nchunks) {
-            const int nb = (c + 1) & 1;
-            tc::mbar_wait(smem_u32(&bar_full[nb]), ph_full[nb]);
-            issue_mma(nb);
+    float best[2] = {__int_as_float(0x7f800000), __int_as_float(0x7f800000)};
+    int bi[2] = {0, 0};
+    const int half = (warp >> 2) & 1;  // columns [64 half, 64 half + 64) of every chunk
+    if (warp == kTcEpiWarps) {
+        // ------------------------------------------------------- producer --
+        if (lane == 0) {
+            const uint32_t idesc = idesc_bf16_m128(kTcN);
+            const uint32_t aB[2] = {smem_u32(sA), smem_u32(sA + a_bytes)};
+            int lc = 0;  // load cursor
+            for (int c = 0; c < nchunks; ++c) {
+                for (; lc < nchunks && lc < c + nstages; ++lc) {
+                    const int s = lc % nstages;
+                    if (lc >= nstages) tc::mbar_wait(smem_u32(&bar_sfree[s]), ((lc / nstages) - 1) & 1);
+                    tc::expect_tx(smem_u32(&bar_full[s]), b_bytes);
+                    tc::bulk_g2s(smem_u32(sB0 + (size_t)s * b_bytes),
+                                 reinterpret_cast<const unsigned char*>(cbf) + (size_t)lc * b_bytes, b_bytes,
+                                 smem_u32(&bar_full[s]));
+                }
+                const int s = c % nstages, buf = c & 1;
+                tc::mbar_wait(smem_u32(&bar_full[s]), (c / nstages) & 1);
+                if (c >= 2) tc::mbar_wait(smem_u32(&bar_afree[buf]), ((c >> 1) - 1) & 1);
+                tc::fence_after();
+                const uint32_t bB = smem_u32(sB0 + (size_t)s * b_bytes);
+#pragma unroll
+                for (int t = 0; t < 2; ++t) {
+                    const uint32_t d = tmem + (uint32_t)((buf * 2 + t) * kTcN);
+                    for (int ks = 0; ks < kp / 16; ++ks)
+                        tc::mma_bf16(d, desc_kmajor(aB[t] + ks * 256u, sbo), desc_kmajor(bB + ks * 256u, sbo), idesc,
+                                     ks > 0);
+                }
+                tc::mma_commit(smem_u32(&bar_mma[buf]));
+                tc::mma_commit(smem_u32(&bar_sfree[s]));
+            }
         }
-        if (c + 1 < nchunks) ph_full[(c + 1) & 1] ^= 1u;
-        tc::mbar_wait(smem_u32(&bar_mma[buf]), ph_mma[buf]);
-        ph_mma[buf] ^= 1u;
-        tc::fence_after();
-        const float* bnv = sBn(buf);
-        // per 32 columns: the scores, their minimum by a min tree (one FMNMX
-        // per score) and, only when it beats the running best, the lowest
-        // column holding it (a strict running argmin over increasing columns)
+    } else {
+        // ------------------------------------------------------- epilogue --
+        const uint32_t trow = tmem + ((uint32_t)((warp & 3) * 32) << 16);
+        for (int c = 0; c < nchunks; ++c) {
+            const int buf = c & 1;
+            tc::mbar_wait(smem_u32(&bar_mma[buf]), (c >> 1) & 1);
+            tc::fence_after();
+#pragma unroll
+            for (int t = 0; t < 2; ++t) {
 #pragma unroll 1
-        for (int cb = 0; cb < 2; ++cb) {
-            const int col = half * 64 + cb * 32;
-            uint32_t v[32];
-            tc::tmem_ld32(trow + (uint32_t)(buf * kTcN + col), v);
-            float sc[32];
-            const float4* bn4 = reinterpret_cast<const float4*>(bnv + col);
+                for (int cb = 0; cb < 2; ++cb) {
+                    const int col = half * 64 + cb * 32;
+                    uint32_t v[32];
+                    tc::tmem_ld32(trow + (uint32_t)((buf * 2 + t) * kTcN + col), v);
+                    float mn[16];
 #pragma unroll
-            for (int j4 = 0; j4 < 8; ++j4) {
-                const float4 b4 = bn4[j4];
-                sc[4 * j4 + 0] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 0]), b4.x);
-                sc[4 * j4 + 1] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 1]), b4.y);
-                sc[4 * j4 + 2] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 2]), b4.z);
-                sc[4 * j4 + 3] = __fmaf_rn(-2.f, __uint_as_float(v[4 * j4 + 3]), b4.w);
+                    for (int j = 0; j < 16; ++j) mn[j] = fminf(__uint_as_float(v[j]), __uint_as_float(v[j + 16]));
+#pragma unroll
+                    for (int w2 = 8; w2 > 0; w2 >>= 1)
+#pragma unroll
+                        for (int j = 0; j < w2; ++j) mn[j] = fminf(mn[j], mn[j + w2]);
+                    if (mn[0] < best[t]) {  // the lowest column holding the new best
+                        int jm = 31;
+#pragma unroll
+                        for (int j = 31; j >= 0; --j) jm = (__uint_as_float(v[j]) == mn[0]) ? j : jm;
+                        best[t] = mn[0];
+                        bi[t] = c * kTcN + col + jm;
+                    }
+                }
             }
-            float t[16];
+            tc::fence_before();
+            __syncwarp();
+            if (lane == 0) tc::mbar_arrive(smem_u32(&bar_afree[buf]));  // accumulator pair may be overwritten
+        }
+        if (half == 1) {
 #pragma unroll
-            for (int j = 0; j < 16; ++j) t[j] = fminf(sc[j], sc[j + 16]);
-#pragma unroll
-            for (int w = 8; w > 0; w >>= 1)
-#pragma unroll
-                for (int j = 0; j < w; ++j) t[j] = fminf(t[j], t[j + w]);
-            if (t[0] < best) {  // the lowest column holding the new best
-                int jm = 31;
-#pragma unroll
-                for (int j = 31; j >= 0; --j) jm = (sc[j] == t[0]) ? j : jm;
-                best = t[0];
-                bi = c * kTcN + col + jm;
+            for (int t = 0; t < 2; ++t) {
+                s_best[t][(warp & 3) * 32 + lane] = best[t];
+                s_bi[t][(warp & 3) * 32 + lane] = bi[t];
             }
         }
-        tc::fence_before();
-        __syncthreads();  // buffer `buf` (smem + TMEM) is free again
-        if (tid == 0 && c + 2 < nchunks) issue_copy(c + 2, buf);
-    }
-    // merge the two column halves (the lower column wins ties)
-    __shared__ float s_best[kTcM];
-    __shared__ int s_bi[kTcM];
-    if (half == 1) {
-        s_best[tid - kTcM] = best;
-        s_bi[tid - kTcM] = bi;
     }
     __syncthreads();
-    const int64_t i = (row0 + tid) * stride;
-    if (half == 0 && i < n) {
-        const float ob = s_best[tid];
-        const int obi = s_bi[tid];
-        if (ob < best || (ob == best && obi < bi)) bi = obi;
-        const float* xr = Xp + i * dp;
-        bi = min(bi, m - 1);
-        const float d2 = d2_rows(xr, centers + (int64_t)bi * dp, dp);  // exact fp32, shared formula
-        if (cid_out) cid_out[i] = bi;
-        if (dist_out) dist_out[i] = __fsqrt_rn(d2);
-        if (counts) atomicAdd(counts + bi, 1);
-        if (sums) fx_accumulate(sums + (int64_t)bi * dp, xr, dp, *fx);
+    if (warp < kTcEpiWarps && half == 0) {
+        const int r = (warp & 3) * 32 + lane;
+#pragma unroll
+        for (int t = 0; t < 2; ++t) {
+            const int64_t i = (row0 + t * kTcM + r) * stride;
+            if (i >= n) continue;
+            int b = bi[t];
+            const float ob = s_best[t][r];
+            const int obi = s_bi[t][r];
+            if (ob < best[t] || (ob == best[t] && obi < b)) b = obi;  // the lower column wins ties
+            const float* xr = Xp + i * dp;
+            b = min(b, m - 1);
+            const float d2 = d2_rows(xr, centers + (int64_t)b * dp, dp);  // exact fp32, shared formula
+            if (cid_out) cid_out[i] = b;
+            if (dist_out) dist_out[i] = __fsqrt_rn(d2);
+            if (counts) atomicAdd(counts + b, 1);
+            if (sums) fx_accumulate(sums + (int64_t)b * dp, xr, dp, *fx);
+        }
     }
     tc::fence_before();
     __syncthreads();
-    if (warp == 0) tc::tmem_dealloc(tmem, 2u * kTcN);
+    if (warp == kTcEpiWarps) tc::tmem_dealloc(tmem, 4u * kTcN);
 }
 
-bool assign_tc_supported(int dp) { return dp >= 8 && ((dp + 15) & ~15) <= 256; }
+// K = dp + 2 augmented columns, padded to the MMA's K step of 16
+static int assign_tc_kp(int dp) { return (dp + 2 + 15) & ~15; }
+bool assign_tc_supported(int dp) { return dp >= 8 && assign_tc_kp(dp) <= 208; }  // 2 A tiles + 2 B stages <= 227 KB
 
 sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m, int32_t* cid,
                           float* dist, long long* sums, const double* fx, int32_t* counts, int stride) {
-    const int kp = (dp + 15) & ~15;
+    const int kp = assign_tc_kp(dp);
     const int nchunks = (m + kTcN - 1) / kTcN;
     const int mpad = nchunks * kTcN;
     float* o;
     __nv_bfloat16* cbf;
-    float* bn;
     SKNN_TRY(cx.alloc_scratch((void**)&o, sizeof(float) * dp));
     SKNN_TRY(cx.alloc_scratch((void**)&cbf, (size_t)mpad * kp * 2));
-    SKNN_TRY(cx.alloc_scratch((void**)&bn, sizeof(float) * mpad));
     k_center_mean<<<dp, 256, 0, cx.stream>>>(centers, m, dp, o);
     cx.launched();
-    const int64_t work = (int64_t)mpad * (kp / 8);
-    k_centers_to_tc<<<(int)std::min<int64_t>((work + 255) / 256, 148 * 8), 256, 0, cx.stream>>>(centers, m, mpad, dp, kp,
-                                                                                                o, cbf, bn);
+    k_centers_to_tc<<<(int)std::min<int64_t>((mpad + 255) / 256, 148 * 8), 256, 0, cx.stream>>>(centers, m, mpad, dp, kp,
+                                                                                                o, cbf);
     cx.launched();
-    // >= 90 KB keeps at most two CTAs per SM: each holds 256 of the 512 TMEM columns
-    const size_t smem = std::max<size_t>((size_t)kTcM * kp * 2 + 2 * (size_t)kTcN * kp * 2 + 2 * kTcN * 4, 90 * 1024);
+    // two A tiles + as many B stages as fit (<= 6) in ~200 KB; the 512 TMEM
+    // columns keep one CTA per SM (>= 116 KB of shared memory enforces it)
+    const size_t a_bytes = (size_t)kTcM * kp * 2, b_bytes = (size_t)kTcN * kp * 2;
+    const int nstages = (int)std::max<size_t>(2, std::min<size_t>(kTcMaxStages, (200 * 1024 - 2 * a_bytes) / b_bytes));
+    const size_t smem = std::max<size_t>(2 * a_bytes + nstages * b_bytes, 116 * 1024);
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-    const int64_t grid = ((n + stride - 1) / stride + kTcM - 1) / kTcM;
-    k_assign_tc<<<(unsigned)grid, kTcThreads, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, bn, m, nchunks, centers, cid, dist,
-                                                          sums, fx, counts, stride);
+    const int64_t grid = ((n + stride - 1) / stride + kTcPts - 1) / kTcPts;
+    k_assign_tc<<<(unsigned)grid, kTcThreads, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, m, nchunks, nstages, centers,
+                                                                cid, dist, sums, fx, counts, stride);
     cx.launched();
     return cx.check_launch("assign (tensor cores)");
 }

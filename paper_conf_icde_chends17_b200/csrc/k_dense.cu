@@ -424,9 +424,9 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
 // is still >= the row's true k-th) and are merged when the tile ends.
 // Barriers: full[s] (chunk landed), sfree[s] (its MMA done: stage reusable),
 // mma[c] (accumulator ready), afree[c] (epilogue done with it: count 8 warps),
-// tfull/tfree[2] (tile id slots). The target norms of a chunk sit in a ring
-// of kExStages + kExAcc slots, so a slot is reloaded only after the epilogue
-// released the chunk that used it (sfree(g + kExAcc) implies afree(g)).
+// tfull/tfree[2] (tile id slots). The target norms of a chunk land with it in
+// a ring of kExTn slots (not in the B stage: a stage is reusable as soon as
+// its MMA completed), each released by the epilogue through tnfree[slot].
 constexpr int kExNCH = 128;
 constexpr int kExEpiWarps = 8;
 constexpr int kExThreads = (kExEpiWarps + 1) * 32;
@@ -448,7 +448,7 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
     unsigned char* sB = smem + a_bytes;                                       // [kExStages][b_bytes]
     float* s_tn = reinterpret_cast<float*>(sB + kExStages * (size_t)b_bytes);  // [kExTn][NCH]
     __shared__ __align__(8) uint64_t bar_a, bar_full[kExStages], bar_sfree[kExStages], bar_mma[kExAcc],
-        bar_afree[kExAcc], bar_tfull[2], bar_tfree[2];
+        bar_afree[kExAcc], bar_tfull[2], bar_tfree[2], bar_tnfree[kExTn];
     __shared__ uint32_t s_tmem;
     __shared__ int s_tile[2];
     __shared__ unsigned long long s_kth[2][kDenseM];  // {k-th d2 bits, tile seq} per half and row
@@ -470,6 +470,7 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
             tc::mbar_init(smem_u32(&bar_tfull[i]), 1);
             tc::mbar_init(smem_u32(&bar_tfree[i]), kExEpiWarps);
         }
+        for (int i = 0; i < kExTn; ++i) tc::mbar_init(smem_u32(&bar_tnfree[i]), kExEpiWarps);
         tc::mbar_fence_init();
     }
     for (int i = tid; i < 2 * kDenseM; i += blockDim.x) (&s_kth[0][0])[i] = ~0ull;
@@ -509,10 +510,12 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
                     const int s = lg % kExStages;
                     if (lg >= (uint32_t)kExStages) mbar_wait(smem_u32(&bar_sfree[s]), ((lg / kExStages) - 1) & 1);
                     const uint32_t bar = smem_u32(&bar_full[s]);
+                    const int ts_ = lg % kExTn;  // target-norm slot: free once the epilogue read it
+                    if (lg >= (uint32_t)kExTn) mbar_wait(smem_u32(&bar_tnfree[ts_]), ((lg / kExTn) - 1) & 1);
                     expect_tx(bar, b_bytes + NCH * 4);
                     const size_t p = (size_t)__ldg(a.toffp + ld.tc) + (size_t)ld.c * NCH;
                     bulk_g2s(smem_u32(sB + (size_t)s * b_bytes), a.thi + (p >> 3) * sbo, b_bytes, bar);
-                    bulk_g2s(smem_u32(s_tn + (lg % kExTn) * NCH), a.tn_raw + p, NCH * 4, bar);
+                    bulk_g2s(smem_u32(s_tn + ts_ * NCH), a.tn_raw + p, NCH * 4, bar);
                     ++lg;
                     ld.advance(a);
                 };
@@ -567,24 +570,26 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
             const float ub = a.ub[qc];
             float kth2 = __fmul_ru(ub, ub);
             const unsigned long long tag = (unsigned long long)(unsigned)t;
-            volatile unsigned long long* mine = &s_kth[half][row];
-            volatile unsigned long long* other = &s_kth[half ^ 1][row];
-            *mine = ((unsigned long long)__float_as_uint(kth2) << 32) | tag;
+            // the halves' k-th distances, exchanged with shared-memory atomics (a
+            // reader may see the other's older value: any of them is a valid bound)
+            unsigned long long* mine = &s_kth[half][row];
+            unsigned long long* other = &s_kth[half ^ 1][row];
+            atomicExch(mine, ((unsigned long long)__float_as_uint(kth2) << 32) | tag);
             ChunkIter<NCH> it;
             it.start(a, qc);
             for (; it.valid(); it.advance(a), ++g) {
                 const int c = g % kExAcc;
-                // the chunk's target norms landed before the producer issued its MMA
-                // (it waited on full[s]); mma[c] completing orders them before us. The
-                // epilogue must NOT wait on full[s] itself: that barrier may already
-                // be one phase further (the stage is refilled once the MMA is done).
+                // (the epilogue must NOT wait on full[s]: that barrier may already be
+                // one phase further -- the stage is refilled once the MMA is done)
                 mbar_wait(smem_u32(&bar_mma[c]), (g / kExAcc) & 1);
                 fence_after();
                 const int nb = min(NCH, it.size - it.c * NCH);
                 const int j0 = __ldg(a.toff + it.tc) + it.c * NCH;  // real (unpadded) first target
+                // target norms ||b||^2 of the chunk (landed with the chunk: the producer
+                // waited on full[s] before the MMA we waited on); +inf on padding rows
                 const float* tn = s_tn + (g % kExTn) * NCH;
                 float lim = kth2;
-                const unsigned long long ot = *other;
+                const unsigned long long ot = atomicOr(other, 0ull);
                 if ((ot & 0xffffffffull) == tag) lim = fminf(lim, __uint_as_float((uint32_t)(ot >> 32)));
                 float thr = __fsub_ru(lim, na);  // keep t = ||b||^2 - 2 a.b iff t <= lim - ||a||^2
 #pragma unroll 1
@@ -643,8 +648,11 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
                 }
                 fence_before();
                 __syncwarp();
-                if (lane == 0) tc::mbar_arrive(smem_u32(&bar_afree[c]));  // accumulator c may be overwritten
-                *mine = ((unsigned long long)__float_as_uint(kth2) << 32) | tag;
+                if (lane == 0) {
+                    tc::mbar_arrive(smem_u32(&bar_afree[c]));             // accumulator c may be overwritten
+                    tc::mbar_arrive(smem_u32(&bar_tnfree[g % kExTn]));    // and the chunk's norm slot
+                }
+                atomicExch(mine, ((unsigned long long)__float_as_uint(kth2) << 32) | tag);
                 if (active && half == 0) covered += (unsigned long long)nb;
             }
             // merge the two halves' lists of each row (keys are distinct: disjoint columns)

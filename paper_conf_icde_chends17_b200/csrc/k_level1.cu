@@ -190,7 +190,8 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     const float* __restrict__ tcent, const int4* __restrict__ tinfo, const float* __restrict__ tdk,
     const float* __restrict__ tdist, int mt, int dp, int k, float eta, int keys_cap, int shard_rank,
     int shard_count, int dense_mode, float dense_tau, const float* __restrict__ cq_o,
-    const float* __restrict__ ct_o, float dense_eps, float* __restrict__ ub_out, int32_t* __restrict__ cand,
+    const float* __restrict__ ct_o, float dense_eps, const float* __restrict__ ub_in, float* __restrict__ ub_out,
+    int32_t* __restrict__ cand,
     int32_t* __restrict__ cand_count, float* __restrict__ cand_D, int32_t* __restrict__ dcand,
     int32_t* __restrict__ dcount, unsigned long long* __restrict__ work,
     Counters* __restrict__ counters) {
@@ -208,7 +209,9 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     const int qc = blockIdx.x;
     const int qsize = qoff[qc + 1] - qoff[qc];
     if (qsize == 0 || (shard_count > 1 && qc % shard_count != shard_rank)) {
-        if (threadIdx.x == 0) { ub_out[qc] = 0.f; cand_count[qc] = 0; dcount[qc] = 0; work[qc] = 0; }
+        if (threadIdx.x == 0) {  // +inf: neutral for a minimum over ranks (target sharding)
+            ub_out[qc] = __int_as_float(0x7f800000); cand_count[qc] = 0; dcount[qc] = 0; work[qc] = 0;
+        }
         return;
     }
     for (int i = threadIdx.x; i < dp; i += blockDim.x) s_qc[i] = qcent[(int64_t)qc * dp + i];
@@ -273,8 +276,12 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     __syncthreads();
     float Vk = (nv <= kL1Vals) ? block_kth_smallest(s_v, nv, k, s_hist, s_sel, s_small) : Mk;  // overflow: M_k is a valid bound
     if (!(Vk <= Mk)) Vk = Mk;
-    // UB = r_q + V_k, inflated to cover the rounding of the three summed distances (R7)
-    const float UB = __fmul_ru(rq + Vk, 1.f + 2.f * eta);
+    // UB = r_q + V_k, inflated to cover the rounding of the three summed distances (R7).
+    // ub_in: an external bound of the same query cluster (target-sharded mode:
+    // the minimum over ranks of their local UBs -- each bounds the k-th distance
+    // over ALL targets, since a shard's k-th is >= the global k-th)
+    float UB = __fmul_ru(rq + Vk, 1.f + 2.f * eta);
+    if (ub_in) UB = fminf(UB, __ldg(ub_in + qc));
     if (threadIdx.x == 0) {
         ub_out[qc] = UB;
         s_cnt = 0;
@@ -426,7 +433,7 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
                                                   ts.dist, mt, dp, p.k, p.eta, cap, p.shard_rank, p.shard_count,
                                                   p.dense_mode, p.dense_tau, p.dorg ? p.dorg->cq_o : nullptr,
                                                   p.dorg ? p.dorg->ct_o : nullptr, p.dorg ? p.dorg->eps : 0.f,
-                                                  out.ub, out.cand, out.cand_count, out.cand_D,
+                                                  p.ub_in, out.ub, out.cand, out.cand_count, out.cand_D,
                                                   out.dcand, out.dcount, out.work, counters);
     cx.launched();
     return cx.check_launch("level1");

@@ -88,7 +88,9 @@ __device__ __forceinline__ void write_result(const ScanArgs& a, int qorig, int r
     int64_t o = (int64_t)qorig * a.k + r;
     float d2 = key_d2(key);
     a.out_dist[o] = a.out_squared ? d2 : __fsqrt_rn(d2);
-    if (a.out_idx) a.out_idx[o] = (int32_t)(key_idx(key) + a.index_base);
+    // a placeholder (fewer than k targets under an external bound, target-sharded
+    // mode) gets index -1; the merge never selects it over a real key
+    if (a.out_idx) a.out_idx[o] = key == kInfKey ? -1 : (int32_t)(key_idx(key) + a.index_base);
 }
 
 // warp-aggregated counter: one atomic per warp (all 32 lanes must call)

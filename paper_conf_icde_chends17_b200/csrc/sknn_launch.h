@@ -148,6 +148,7 @@ struct Level1Params {
     int shard_rank = 0, shard_count = 1;
     int dense_mode = 0;           // 0 auto (cost model), 1 never, 2 every candidate pair
     float dense_tau = 0.5f;       // auto: dense iff |tc| >= 32 and the expected window share >= tau
+    const float* ub_in = nullptr; // optional [mq] external upper bounds (min'd with the local calUB)
 };
 sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Params& p, Level1& out,
                        Counters* counters);

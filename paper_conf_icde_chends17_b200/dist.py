@@ -8,7 +8,8 @@ SURVEY.md §8(e). Two modes:
   and processes the query clusters c with c % P == rank
   (``sknn_options.shard_rank/shard_count``); otherwise rank r takes the
   contiguous query rows [r*nq/P, (r+1)*nq/P). No data-path collective; the
-  optional result assembly is one all-reduce outside the join.
+  optional result assembly is one collective outside the join (an all-gather of
+  the row slices, or for a self-join one all-reduce of packed (dist, idx) keys).
 * Target sharding: rank r owns T[r*nt/P, (r+1)*nt/P), computes partial k-lists
   of ALL queries with squared distances and global indices (``out_squared``,
   ``index_base``), the partial lists are exchanged with one all-gather over
@@ -49,7 +50,7 @@ def join_query_sharded(Q, T, k: int, *, group=None, self_join: bool | None = Non
                        local_join=None, **opts):
     """Query-sharded join. Returns (idx, dist) for the rank's rows (gather=False:
     full-size buffers with -1 / 0 in rows of other ranks) or the assembled
-    full result on every rank (gather=True, one all-reduce)."""
+    full result on every rank (gather=True, one collective)."""
     world, rank = _world(group)
     local_join = local_join or _cuda_join
     if self_join is None:
@@ -69,9 +70,26 @@ def join_query_sharded(Q, T, k: int, *, group=None, self_join: bool | None = Non
             dst[lo:hi] = d
     if not gather or world == 1:
         return idx, dst
-    # rows are disjoint across ranks: -1 / 0 elsewhere, so MAX / SUM assemble them
-    dist.all_reduce(idx, op=dist.ReduceOp.MAX, group=group)
-    dist.all_reduce(dst, op=dist.ReduceOp.SUM, group=group)
+    if not self_join:
+        # contiguous row slices: one all-gather of the (padded) slices
+        splits = [shard_bounds(nq, world, r) for r in range(world)]
+        cap = max(h - l for l, h in splits)
+        lo, hi = splits[rank]
+        mine = torch.zeros((cap, k, 2), dtype=torch.int32, device=Q.device)
+        mine[:hi - lo, :, 0] = idx[lo:hi]
+        mine[:hi - lo, :, 1] = dst[lo:hi].view(torch.int32)
+        allp = torch.empty((world * cap, k, 2), dtype=torch.int32, device=Q.device)
+        dist.all_gather_into_tensor(allp, mine, group=group)
+        out = torch.cat([allp[r * cap:r * cap + (h - l)] for r, (l, h) in enumerate(splits)])
+        return out[:, :, 0].contiguous(), out[:, :, 1].contiguous().view(torch.float32)
+    # self-join, cluster-interleaved rows: each rank's rows hold (dist bits << 32 |
+    # idx + 1), every other row 0, so ONE all-reduce SUM assembles both arrays
+    own = idx >= 0
+    packed = torch.where(own, (dst.view(torch.int32).to(torch.int64) << 32) | (idx.to(torch.int64) + 1),
+                         torch.zeros((), dtype=torch.int64, device=Q.device))
+    dist.all_reduce(packed, op=dist.ReduceOp.SUM, group=group)
+    idx = ((packed & 0xFFFFFFFF) - 1).to(torch.int32)
+    dst = (packed >> 32).to(torch.int32).view(torch.float32)
     return idx, dst
 
 
@@ -111,8 +129,29 @@ def join_query_sharded_index(index, Q, k: int, *, group=None, out=None, **opts):
     return index.query(Q, k, out=out, self_query=1, shard_rank=rank, shard_count=world, **opts)
 
 
+def target_shard_partials_global_ub(Q, T_shard, k: int, shard_offset: int, *, group=None, qindex=None, **opts):
+    """Partial k-lists of ALL queries against this rank's target shard, pruned
+    with the GLOBAL level-1 bound: every rank clusters Q
+    identically (seeded; or pass a prebuilt `qindex`), computes the calUB of
+    each query cluster against its shard (sknn_level1_bounds), the bounds are
+    combined by one all-reduce MIN (mq floats: a shard's k-th distance is >=
+    the global one, so every rank's bound is a global bound), and the join runs
+    with the tightest one (sknn_join_indexed with ub_in). Rows may hold fewer
+    than k real entries (+inf / -1 placeholders); the merged result is exact.
+    Returns (idx, d2) with global indices."""
+    from . import Index, join_indexed, level1_bounds
+    qix = qindex or Index(Q, **{kk: v for kk, v in opts.items() if kk in ("lloyd_iters", "landmark_trials", "seed",
+                                                                              "n_clusters_t")})
+    tix = Index(T_shard)
+    ub = level1_bounds(qix, tix, k)
+    if dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(ub, op=dist.ReduceOp.MIN, group=group)
+    return join_indexed(qix, tix, k, out_squared=1, index_base=int(shard_offset), ub_in=ub, **opts)[:2]
+
+
 def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, local_join=None, merge=None,
-                        out_squared: bool = False, exchange: str = "all_gather", gather: bool = True, **opts):
+                        out_squared: bool = False, exchange: str = "all_gather", gather: bool = True,
+                        global_ub: bool = False, **opts):
     """Target-sharded join: local partial lists of every query against this
     rank's T_shard (global indices), exchanged and merged exactly.
     exchange="all_gather": every rank merges all nq rows (returns the full
@@ -124,7 +163,10 @@ def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, lo
     merge = merge or _cuda_merge
     nq = Q.shape[0]
     kk = min(k, T_shard.shape[0])
-    pidx, pd2 = local_join(Q, T_shard, kk, out_squared=1, index_base=int(shard_offset), **opts)[:2]
+    if global_ub:  # NEXT-1: prune every shard with the global level-1 bound
+        pidx, pd2 = target_shard_partials_global_ub(Q, T_shard, kk, shard_offset, group=group, **opts)
+    else:
+        pidx, pd2 = local_join(Q, T_shard, kk, out_squared=1, index_base=int(shard_offset), **opts)[:2]
     if kk < k:  # a shard smaller than k: pad with +inf keys (never selected over real ones)
         pad_i = torch.full((nq, k - kk), -1, dtype=torch.int32, device=Q.device)
         pad_d = torch.full((nq, k - kk), float("inf"), dtype=torch.float32, device=Q.device)
