@@ -378,6 +378,19 @@ static void fill_stats(sknn_stats* st, const Counters& c, int64_t nq, int64_t nt
     memcpy(st, &s, sz);
 }
 
+// Private non-blocking stream per device for the forked query-side build.
+static cudaStream_t side_stream(int dev) {
+    static std::mutex mu;
+    static cudaStream_t s[64] = {};
+    if (dev < 0 || dev >= 64) return nullptr;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!s[dev] && cudaStreamCreateWithFlags(&s[dev], cudaStreamNonBlocking) != cudaSuccess) {
+        cudaGetLastError();
+        s[dev] = nullptr;
+    }
+    return s[dev];
+}
+
 // Shared body of sknn_join_ex / sknn_query.
 static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
                             int32_t* out_idx, float* out_dist, const sknn_options* opt_in, sknn_stats* stats,
@@ -424,6 +437,8 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     int32_t* d_oidx = nullptr;
     float* d_odist = nullptr;
     Counters* counters = nullptr;
+    Ctx cq;  // forked query-side build (Q != T joins)
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     do {
         const void* tmp;
         if (!qindex) {
@@ -472,6 +487,33 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
         }
         Side ts_local, qs_local;
         const Side* ts;
+        // A Q != T join clusters both sides: the query side is built on a forked
+        // stream concurrently with the target side (both are chains of mostly
+        // small, latency-bound kernels; the joins and frees stay stream-ordered,
+        // and a graph capture follows the fork/join events)
+        const bool fork_q = !index && !self && !qindex;
+        if (fork_q) {
+            cq.stream = side_stream(di.device);
+            cq.device = cx.device;
+            cq.num_sms = cx.num_sms;
+            cq.capturing = capturing;
+            if (!cq.stream || cudaEventCreateWithFlags(&ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventCreateWithFlags(&ev_join, cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventRecord(ev_fork, stream) != cudaSuccess || cudaStreamWaitEvent(cq.stream, ev_fork, 0) != cudaSuccess) {
+                st = fail(SKNN_ERR_CUDA, "fork of the query-side build failed");
+                break;
+            }
+            int m = det_lm_num(nq, o.n_clusters_q);
+            NvtxRange r("sknn build query side (forked stream)");
+            if ((st = build_side(cq, dQ, nq, d, m, o.landmark_trials, o.lloyd_iters, o.seed ^ 0x51ull, qs_local)) !=
+                SKNN_OK)
+                break;
+            cq.free_scratch();
+            if (cudaEventRecord(ev_join, cq.stream) != cudaSuccess) {
+                st = fail(SKNN_ERR_CUDA, "join of the query-side build failed");
+                break;
+            }
+        }
         if (index) {
             ts = &index->t;
         } else {
@@ -487,12 +529,26 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
             qs = ts;
         } else if (qindex) {
             qs = &qindex->t;
-        } else {
+        } else if (!fork_q) {  // query of a resident index: cluster Q here
             int m = det_lm_num(nq, o.n_clusters_q);
             NvtxRange r("sknn build query side");
             if ((st = build_side(cx, dQ, nq, d, m, o.landmark_trials, o.lloyd_iters, o.seed ^ 0x51ull, qs_local)) !=
                 SKNN_OK)
                 break;
+            qs = &qs_local;
+            mk.bq = tm.mark();
+        } else {
+            if (cudaStreamWaitEvent(stream, ev_join, 0) != cudaSuccess) {
+                st = fail(SKNN_ERR_CUDA, "join of the query-side build failed");
+                break;
+            }
+            // the query side's arrays are used (and freed) on `stream` from here on
+            cx.persistent.insert(cx.persistent.end(), cq.persistent.begin(), cq.persistent.end());
+            cq.persistent.clear();
+            cx.launches += cq.launches;
+            cudaEventDestroy(ev_fork);
+            cudaEventDestroy(ev_join);
+            ev_fork = ev_join = nullptr;
             qs = &qs_local;
             mk.bq = tm.mark();
         }
@@ -511,6 +567,13 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
         }
         if (stats && counters) cudaMemcpyAsync(&host_c, counters, sizeof(Counters), cudaMemcpyDeviceToHost, stream);
         mk.end = tm.mark();
+    }
+    if (ev_fork) {  // an error left the forked build unjoined: join it, free its memory
+        if (!ev_join || cudaEventRecord(ev_join, cq.stream) != cudaSuccess) cudaStreamSynchronize(cq.stream);
+        else cudaStreamWaitEvent(stream, ev_join, 0);
+        cq.free_all();
+        cudaEventDestroy(ev_fork);
+        if (ev_join) cudaEventDestroy(ev_join);
     }
     int launches = cx.launches;
     cx.free_all();

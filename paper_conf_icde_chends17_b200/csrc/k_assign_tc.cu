@@ -90,59 +90,46 @@ __global__ void k_centers_to_tc(const float* __restrict__ centers, int m, int mp
     }
 }
 
-// One CTA = 256 points (two 128-row A tiles sharing every B chunk, so each
-// center chunk read from L2 feeds two MMAs), 9 warps, warp-specialised:
-//  * warp 8, one elected thread: the producer -- streams the center chunks
-//    through a kStages-deep bulk-copy ring and issues, per chunk, the MMAs of
-//    both A tiles into one of two accumulator pairs (TMEM: 2 x 2 x 128 = 512
-//    columns, one CTA per SM); a stage is refilled as soon as its MMAs are done
-//    (sfree), an accumulator pair as soon as the epilogue released it (afree);
-//  * warps 0-7: the epilogue -- thread (w, lane) owns row 32 (w % 4) + lane of
-//    both A tiles and half w / 4 of the chunk's 128 columns: per 32 columns one
-//    tcgen05.ld and a min tree (one FMNMX per score), the argmin index only on
-//    improvement (lowest column on ties).
-constexpr int kTcEpiWarps = 8;
-constexpr int kTcThreads = (kTcEpiWarps + 1) * 32;
-constexpr int kTcPts = 2 * kTcM;  // points per CTA
-constexpr int kTcMaxStages = 6;
-
+// One CTA = 128 points, 8 warps: warps w and w + 4 read the same 32 TMEM lanes
+// (points) and split each chunk's 128 columns in halves. Streams every center
+// chunk through a 2-deep bulk-copy ring (a stage is refilled as soon as its
+// MMA completed). (Measured and rejected: 256 points per CTA sharing each
+// chunk with a warp-specialised producer and up to 6 stages, one CTA per SM
+// -- C4 full pass 2.29 -> 2.68 ms, C5 5.21 -> 5.56 ms.)
+constexpr int kTcThreads = 256;
 __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __restrict__ Xp, int64_t n, int dp, int kp,
                                                        const float* __restrict__ o,
                                                        const __nv_bfloat16* __restrict__ cbf, int m, int nchunks,
-                                                       int nstages, const float* __restrict__ centers,
+                                                       const float* __restrict__ centers,
                                                        int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
                                                        long long* __restrict__ sums, const double* __restrict__ fx,
                                                        int32_t* __restrict__ counts, int stride) {
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t a_bytes = (uint32_t)kTcM * kp * 2, b_bytes = (uint32_t)kTcN * kp * 2;
-    unsigned char* sA = smem;                     // [2][a_bytes]
-    unsigned char* sB0 = smem + 2 * (size_t)a_bytes;  // [nstages][b_bytes]
-    __shared__ __align__(8) uint64_t bar_full[kTcMaxStages], bar_sfree[kTcMaxStages], bar_mma[2], bar_afree[2];
+    unsigned char* sA = smem;
+    auto sB = [&](int b) { return smem + a_bytes + (uint32_t)b * b_bytes; };
+    __shared__ __align__(8) uint64_t bar_full[2], bar_mma[2];
     __shared__ uint32_t s_tmem;
-    __shared__ float s_best[2][kTcM];
-    __shared__ int s_bi[2][kTcM];
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int tid = threadIdx.x, warp = tid >> 5;
     const uint32_t sbo = (uint32_t)kp * 16u;
 
-    if (warp == kTcEpiWarps) tc::tmem_alloc(&s_tmem, 4u * kTcN);
+    if (warp == 0) {
+        tc::tmem_alloc(&s_tmem, 2u * kTcN);
+    }
     if (tid == 0) {
-        for (int i = 0; i < nstages; ++i) {
-            tc::mbar_init(smem_u32(&bar_full[i]), 1);
-            tc::mbar_init(smem_u32(&bar_sfree[i]), 1);
-        }
         for (int i = 0; i < 2; ++i) {
+            tc::mbar_init(smem_u32(&bar_full[i]), 1);
             tc::mbar_init(smem_u32(&bar_mma[i]), 1);
-            tc::mbar_init(smem_u32(&bar_afree[i]), kTcEpiWarps);
         }
         tc::mbar_fence_init();
     }
-    // stage A' = [x - o, 1, 1] (bf16) for the CTA's 256 points (both tiles)
-    const int64_t row0 = (int64_t)blockIdx.x * kTcPts;
+    // stage A = x - o (bf16) for the CTA's 128 points
+    const int64_t row0 = (int64_t)blockIdx.x * kTcM;
     {
         const int c8n = kp / 8;
-        for (int w = tid; w < kTcPts * c8n; w += blockDim.x) {
-            const int rr = w / c8n, c8 = w % c8n;
-            const int64_t i = (row0 + rr) * stride;
+        for (int w = tid; w < kTcM * c8n; w += blockDim.x) {
+            const int r = w / c8n, c8 = w % c8n;
+            const int64_t i = (row0 + r) * stride;
             uint32_t h[4];
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
@@ -155,8 +142,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
                 h[e] = (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v0)) |
                        ((uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(v1)) << 16);
             }
-            const int t = rr >> 7, r = rr & 127;
-            const uint32_t off = (uint32_t)t * a_bytes + (uint32_t)(r >> 3) * sbo + (uint32_t)c8 * 128u + (uint32_t)(r & 7) * 16u;
+            const uint32_t off = (uint32_t)(r >> 3) * sbo + (uint32_t)c8 * 128u + (uint32_t)(r & 7) * 16u;
             *reinterpret_cast<uint4*>(sA + off) = make_uint4(h[0], h[1], h[2], h[3]);
         }
     }
@@ -165,111 +151,109 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
     __syncthreads();
     tc::fence_after();
     const uint32_t tmem = s_tmem;
+    const uint32_t idesc = idesc_bf16_m128(kTcN);
 
-    float best[2] = {__int_as_float(0x7f800000), __int_as_float(0x7f800000)};
-    int bi[2] = {0, 0};
-    const int half = (warp >> 2) & 1;  // columns [64 half, 64 half + 64) of every chunk
-    if (warp == kTcEpiWarps) {
-        // ------------------------------------------------------- producer --
-        if (lane == 0) {
-            const uint32_t idesc = idesc_bf16_m128(kTcN);
-            const uint32_t aB[2] = {smem_u32(sA), smem_u32(sA + a_bytes)};
-            int lc = 0;  // load cursor
-            for (int c = 0; c < nchunks; ++c) {
-                for (; lc < nchunks && lc < c + nstages; ++lc) {
-                    const int s = lc % nstages;
-                    if (lc >= nstages) tc::mbar_wait(smem_u32(&bar_sfree[s]), ((lc / nstages) - 1) & 1);
-                    tc::expect_tx(smem_u32(&bar_full[s]), b_bytes);
-                    tc::bulk_g2s(smem_u32(sB0 + (size_t)s * b_bytes),
-                                 reinterpret_cast<const unsigned char*>(cbf) + (size_t)lc * b_bytes, b_bytes,
-                                 smem_u32(&bar_full[s]));
-                }
-                const int s = c % nstages, buf = c & 1;
-                tc::mbar_wait(smem_u32(&bar_full[s]), (c / nstages) & 1);
-                if (c >= 2) tc::mbar_wait(smem_u32(&bar_afree[buf]), ((c >> 1) - 1) & 1);
-                tc::fence_after();
-                const uint32_t bB = smem_u32(sB0 + (size_t)s * b_bytes);
-#pragma unroll
-                for (int t = 0; t < 2; ++t) {
-                    const uint32_t d = tmem + (uint32_t)((buf * 2 + t) * kTcN);
-                    for (int ks = 0; ks < kp / 16; ++ks)
-                        tc::mma_bf16(d, desc_kmajor(aB[t] + ks * 256u, sbo), desc_kmajor(bB + ks * 256u, sbo), idesc,
-                                     ks > 0);
-                }
-                tc::mma_commit(smem_u32(&bar_mma[buf]));
-                tc::mma_commit(smem_u32(&bar_sfree[s]));
-            }
+    auto issue_copy = [&](int chunk, int buf) {
+        const uint32_t bar = smem_u32(&bar_full[buf]);
+        tc::expect_tx(bar, b_bytes);
+        const unsigned char* src = reinterpret_cast<const unsigned char*>(cbf) + (size_t)chunk * b_bytes;
+        tc::bulk_g2s(smem_u32(sB(buf)), src, b_bytes, bar);
+    };
+    auto issue_mma = [&](int buf) {
+        tc::fence_after();
+        const uint32_t aB = smem_u32(sA), bB = smem_u32(sB(buf));
+        for (int s = 0; s < kp / 16; ++s)
+            tc::mma_bf16(tmem + (uint32_t)(buf * kTcN), desc_kmajor(aB + s * 256u, sbo), desc_kmajor(bB + s * 256u, sbo),
+                         idesc, s > 0);
+        tc::mma_commit(smem_u32(&bar_mma[buf]));
+    };
+
+    uint32_t ph_full[2] = {0, 0}, ph_mma[2] = {0, 0};
+    if (tid == 0) {
+        issue_copy(0, 0);
+        if (nchunks > 1) issue_copy(1, 1);
+        tc::mbar_wait(smem_u32(&bar_full[0]), 0);
+        issue_mma(0);
+    }
+    ph_full[0] = 1;
+    float best = __int_as_float(0x7f800000);
+    int bi = 0;
+    const int half = warp >> 2;  // columns [64 * half, 64 * half + 64) of every chunk
+    const uint32_t trow = tmem + ((uint32_t)((warp & 3) * 32) << 16);
+    for (int c = 0; c < nchunks; ++c) {
+        const int buf = c & 1;
+        // issue the next chunk's MMA as soon as its copy landed (overlaps this epilogue)
+        if (tid == 0 && c + 1 < nchunks) {
+            const int nb = (c + 1) & 1;
+            tc::mbar_wait(smem_u32(&bar_full[nb]), ph_full[nb]);
+            issue_mma(nb);
         }
-    } else {
-        // ------------------------------------------------------- epilogue --
-        const uint32_t trow = tmem + ((uint32_t)((warp & 3) * 32) << 16);
-        for (int c = 0; c < nchunks; ++c) {
-            const int buf = c & 1;
-            tc::mbar_wait(smem_u32(&bar_mma[buf]), (c >> 1) & 1);
-            tc::fence_after();
-#pragma unroll
-            for (int t = 0; t < 2; ++t) {
+        if (c + 1 < nchunks) ph_full[(c + 1) & 1] ^= 1u;
+        tc::mbar_wait(smem_u32(&bar_mma[buf]), ph_mma[buf]);
+        ph_mma[buf] ^= 1u;
+        tc::fence_after();
+        // MMA(c) has consumed stage `buf`: refill it now, so the copy overlaps
+        // this chunk's epilogue (the accumulator `buf` stays busy until the
+        // barrier below; MMA(c + 2) is issued only after it)
+        if (tid == 0 && c + 2 < nchunks) issue_copy(c + 2, buf);
+        // per 32 columns: the scores (straight from TMEM), their minimum by a
+        // min tree (one FMNMX per score) and, only when it beats the running
+        // best, the lowest column holding it (a strict running argmin)
 #pragma unroll 1
-                for (int cb = 0; cb < 2; ++cb) {
-                    const int col = half * 64 + cb * 32;
-                    uint32_t v[32];
-                    tc::tmem_ld32(trow + (uint32_t)((buf * 2 + t) * kTcN + col), v);
-                    float mn[16];
+        for (int cb = 0; cb < 2; ++cb) {
+            const int col = half * 64 + cb * 32;
+            uint32_t v[32];
+            tc::tmem_ld32(trow + (uint32_t)(buf * kTcN + col), v);
+            float sc[32];
 #pragma unroll
-                    for (int j = 0; j < 16; ++j) mn[j] = fminf(__uint_as_float(v[j]), __uint_as_float(v[j + 16]));
+            for (int j = 0; j < 32; ++j) sc[j] = __uint_as_float(v[j]);
+            float t[16];
 #pragma unroll
-                    for (int w2 = 8; w2 > 0; w2 >>= 1)
+            for (int j = 0; j < 16; ++j) t[j] = fminf(sc[j], sc[j + 16]);
 #pragma unroll
-                        for (int j = 0; j < w2; ++j) mn[j] = fminf(mn[j], mn[j + w2]);
-                    if (mn[0] < best[t]) {  // the lowest column holding the new best
-                        int jm = 31;
+            for (int w = 8; w > 0; w >>= 1)
 #pragma unroll
-                        for (int j = 31; j >= 0; --j) jm = (__uint_as_float(v[j]) == mn[0]) ? j : jm;
-                        best[t] = mn[0];
-                        bi[t] = c * kTcN + col + jm;
-                    }
-                }
-            }
-            tc::fence_before();
-            __syncwarp();
-            if (lane == 0) tc::mbar_arrive(smem_u32(&bar_afree[buf]));  // accumulator pair may be overwritten
-        }
-        if (half == 1) {
+                for (int j = 0; j < w; ++j) t[j] = fminf(t[j], t[j + w]);
+            if (t[0] < best) {  // the lowest column holding the new best
+                int jm = 31;
 #pragma unroll
-            for (int t = 0; t < 2; ++t) {
-                s_best[t][(warp & 3) * 32 + lane] = best[t];
-                s_bi[t][(warp & 3) * 32 + lane] = bi[t];
+                for (int j = 31; j >= 0; --j) jm = (sc[j] == t[0]) ? j : jm;
+                best = t[0];
+                bi = c * kTcN + col + jm;
             }
         }
+        tc::fence_before();
+        __syncthreads();  // accumulator `buf` (TMEM) is free again
+    }
+    // merge the two column halves (the lower column wins ties)
+    __shared__ float s_best[kTcM];
+    __shared__ int s_bi[kTcM];
+    if (half == 1) {
+        s_best[tid - kTcM] = best;
+        s_bi[tid - kTcM] = bi;
     }
     __syncthreads();
-    if (warp < kTcEpiWarps && half == 0) {
-        const int r = (warp & 3) * 32 + lane;
-#pragma unroll
-        for (int t = 0; t < 2; ++t) {
-            const int64_t i = (row0 + t * kTcM + r) * stride;
-            if (i >= n) continue;
-            int b = bi[t];
-            const float ob = s_best[t][r];
-            const int obi = s_bi[t][r];
-            if (ob < best[t] || (ob == best[t] && obi < b)) b = obi;  // the lower column wins ties
-            const float* xr = Xp + i * dp;
-            b = min(b, m - 1);
-            const float d2 = d2_rows(xr, centers + (int64_t)b * dp, dp);  // exact fp32, shared formula
-            if (cid_out) cid_out[i] = b;
-            if (dist_out) dist_out[i] = __fsqrt_rn(d2);
-            if (counts) atomicAdd(counts + b, 1);
-            if (sums) fx_accumulate(sums + (int64_t)b * dp, xr, dp, *fx);
-        }
+    const int64_t i = (row0 + tid) * stride;
+    if (half == 0 && i < n) {
+        const float ob = s_best[tid];
+        const int obi = s_bi[tid];
+        if (ob < best || (ob == best && obi < bi)) bi = obi;
+        const float* xr = Xp + i * dp;
+        bi = min(bi, m - 1);
+        const float d2 = d2_rows(xr, centers + (int64_t)bi * dp, dp);  // exact fp32, shared formula
+        if (cid_out) cid_out[i] = bi;
+        if (dist_out) dist_out[i] = __fsqrt_rn(d2);
+        if (counts) atomicAdd(counts + bi, 1);
+        if (sums) fx_accumulate(sums + (int64_t)bi * dp, xr, dp, *fx);
     }
     tc::fence_before();
     __syncthreads();
-    if (warp == kTcEpiWarps) tc::tmem_dealloc(tmem, 4u * kTcN);
+    if (warp == 0) tc::tmem_dealloc(tmem, 2u * kTcN);
 }
 
 // K = dp + 2 augmented columns, padded to the MMA's K step of 16
 static int assign_tc_kp(int dp) { return (dp + 2 + 15) & ~15; }
-bool assign_tc_supported(int dp) { return dp >= 8 && assign_tc_kp(dp) <= 208; }  // 2 A tiles + 2 B stages <= 227 KB
+bool assign_tc_supported(int dp) { return dp >= 8 && assign_tc_kp(dp) <= 256; }
 
 sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const float* centers, int m, int32_t* cid,
                           float* dist, long long* sums, const double* fx, int32_t* counts, int stride) {
@@ -285,16 +269,13 @@ sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
     k_centers_to_tc<<<(int)std::min<int64_t>((mpad + 255) / 256, 148 * 8), 256, 0, cx.stream>>>(centers, m, mpad, dp, kp,
                                                                                                 o, cbf);
     cx.launched();
-    // two A tiles + as many B stages as fit (<= 6) in ~200 KB; the 512 TMEM
-    // columns keep one CTA per SM (>= 116 KB of shared memory enforces it)
-    const size_t a_bytes = (size_t)kTcM * kp * 2, b_bytes = (size_t)kTcN * kp * 2;
-    const int nstages = (int)std::max<size_t>(2, std::min<size_t>(kTcMaxStages, (200 * 1024 - 2 * a_bytes) / b_bytes));
-    const size_t smem = std::max<size_t>(2 * a_bytes + nstages * b_bytes, 116 * 1024);
+    // >= 90 KB keeps at most two CTAs per SM: each holds 256 of the 512 TMEM columns
+    const size_t smem = std::max<size_t>((size_t)kTcM * kp * 2 + 2 * (size_t)kTcN * kp * 2, 90 * 1024);
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-    const int64_t grid = ((n + stride - 1) / stride + kTcPts - 1) / kTcPts;
-    k_assign_tc<<<(unsigned)grid, kTcThreads, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, m, nchunks, nstages, centers,
-                                                                cid, dist, sums, fx, counts, stride);
+    const int64_t grid = ((n + stride - 1) / stride + kTcM - 1) / kTcM;
+    k_assign_tc<<<(unsigned)grid, kTcThreads, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, m, nchunks, centers, cid, dist,
+                                                          sums, fx, counts, stride);
     cx.launched();
     return cx.check_launch("assign (tensor cores)");
 }

@@ -424,15 +424,14 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
 // is still >= the row's true k-th) and are merged when the tile ends.
 // Barriers: full[s] (chunk landed), sfree[s] (its MMA done: stage reusable),
 // mma[c] (accumulator ready), afree[c] (epilogue done with it: count 8 warps),
-// tfull/tfree[2] (tile id slots). The target norms of a chunk land with it in
-// a ring of kExTn slots (not in the B stage: a stage is reusable as soon as
-// its MMA completed), each released by the epilogue through tnfree[slot].
+// tfull/tfree[2] (tile id slots). A B stage is reusable as soon as its MMA
+// completed; the target norms the epilogue needs are fetched by each epilogue
+// warp itself (cp.async, one chunk ahead) into its own double buffer.
 constexpr int kExNCH = 128;
 constexpr int kExEpiWarps = 8;
 constexpr int kExThreads = (kExEpiWarps + 1) * 32;
 constexpr int kExStages = 3;
 constexpr int kExAcc = 2;
-constexpr int kExTn = kExStages + kExAcc;
 
 __host__ __device__ constexpr int dense_exact_min_blocks(int kmax) { return 1; }
 
@@ -445,10 +444,12 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
     const uint32_t sbo = (uint32_t)KP * 16u;
     const uint32_t a_bytes = (uint32_t)kDenseM * KP * 2, b_bytes = (uint32_t)NCH * KP * 2;
     unsigned char* sA = smem;
-    unsigned char* sB = smem + a_bytes;                                       // [kExStages][b_bytes]
-    float* s_tn = reinterpret_cast<float*>(sB + kExStages * (size_t)b_bytes);  // [kExTn][NCH]
+    unsigned char* sB = smem + a_bytes;  // [kExStages][b_bytes]
     __shared__ __align__(8) uint64_t bar_a, bar_full[kExStages], bar_sfree[kExStages], bar_mma[kExAcc],
-        bar_afree[kExAcc], bar_tfull[2], bar_tfree[2], bar_tnfree[kExTn];
+        bar_afree[kExAcc], bar_tfull[2], bar_tfree[2];
+    // target norms of a chunk, per epilogue warp (its 64 columns), double-buffered,
+    // prefetched one chunk ahead by the warp itself with cp.async
+    __shared__ __align__(16) float s_tnw[kExEpiWarps][2][kExNCH / 2];
     __shared__ uint32_t s_tmem;
     __shared__ int s_tile[2];
     __shared__ unsigned long long s_kth[2][kDenseM];  // {k-th d2 bits, tile seq} per half and row
@@ -470,7 +471,6 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
             tc::mbar_init(smem_u32(&bar_tfull[i]), 1);
             tc::mbar_init(smem_u32(&bar_tfree[i]), kExEpiWarps);
         }
-        for (int i = 0; i < kExTn; ++i) tc::mbar_init(smem_u32(&bar_tnfree[i]), kExEpiWarps);
         tc::mbar_fence_init();
     }
     for (int i = tid; i < 2 * kDenseM; i += blockDim.x) (&s_kth[0][0])[i] = ~0ull;
@@ -510,12 +510,9 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
                     const int s = lg % kExStages;
                     if (lg >= (uint32_t)kExStages) mbar_wait(smem_u32(&bar_sfree[s]), ((lg / kExStages) - 1) & 1);
                     const uint32_t bar = smem_u32(&bar_full[s]);
-                    const int ts_ = lg % kExTn;  // target-norm slot: free once the epilogue read it
-                    if (lg >= (uint32_t)kExTn) mbar_wait(smem_u32(&bar_tnfree[ts_]), ((lg / kExTn) - 1) & 1);
-                    expect_tx(bar, b_bytes + NCH * 4);
+                    expect_tx(bar, b_bytes);
                     const size_t p = (size_t)__ldg(a.toffp + ld.tc) + (size_t)ld.c * NCH;
                     bulk_g2s(smem_u32(sB + (size_t)s * b_bytes), a.thi + (p >> 3) * sbo, b_bytes, bar);
-                    bulk_g2s(smem_u32(s_tn + ts_ * NCH), a.tn_raw + p, NCH * 4, bar);
                     ++lg;
                     ld.advance(a);
                 };
@@ -546,16 +543,26 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
         // ------------------------------------------------------- epilogue --
         const int quarter = warp & 3, half = warp >> 2;
         const int row = quarter * 32 + lane;
+        // lanes 0-15 copy the warp's 64 norms of a chunk (16 B each) into buffer `sl`
+        auto prefetch_tn = [&](const ChunkIter<NCH>& ci, int sl) {
+            if (lane < 16) {
+                const float* src = a.tn_raw + (size_t)__ldg(a.toffp + ci.tc) + (size_t)ci.c * NCH + half * (NCH / 2) + lane * 4;
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(&s_tnw[warp][sl][lane * 4])),
+                             "l"(src)
+                             : "memory");
+            }
+            asm volatile("cp.async.commit_group;" ::: "memory");
+        };
         const uint32_t trow = tmem + ((uint32_t)(quarter * 32) << 16);
         const float INF = __int_as_float(0x7f800000);
         uint32_t g = 0;
         unsigned long long covered = 0;
         for (int t = 0;; ++t) {
-            const int slot = t & 1;
-            mbar_wait(smem_u32(&bar_tfull[slot]), (t >> 1) & 1);
-            const int tile = *(volatile int*)&s_tile[slot];
+            const int tslot = t & 1;
+            mbar_wait(smem_u32(&bar_tfull[tslot]), (t >> 1) & 1);
+            const int tile = *(volatile int*)&s_tile[tslot];
             __syncwarp();
-            if (lane == 0) tc::mbar_arrive(smem_u32(&bar_tfree[slot]));
+            if (lane == 0) tc::mbar_arrive(smem_u32(&bar_tfree[tslot]));
             if (tile >= ntiles) break;
             const int2 tl = a.tiles[tile];
             const int qc = tl.x;
@@ -577,6 +584,8 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
             atomicExch(mine, ((unsigned long long)__float_as_uint(kth2) << 32) | tag);
             ChunkIter<NCH> it;
             it.start(a, qc);
+            int slot = 0;
+            if (it.valid()) prefetch_tn(it, 0);
             for (; it.valid(); it.advance(a), ++g) {
                 const int c = g % kExAcc;
                 // (the epilogue must NOT wait on full[s]: that barrier may already be
@@ -585,9 +594,17 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
                 fence_after();
                 const int nb = min(NCH, it.size - it.c * NCH);
                 const int j0 = __ldg(a.toff + it.tc) + it.c * NCH;  // real (unpadded) first target
-                // target norms ||b||^2 of the chunk (landed with the chunk: the producer
-                // waited on full[s] before the MMA we waited on); +inf on padding rows
-                const float* tn = s_tn + (g % kExTn) * NCH;
+                // target norms ||b||^2 of this chunk's 64 columns (+inf on padding
+                // rows): prefetch the next chunk's, then wait for this one's
+                {
+                    ChunkIter<NCH> nx = it;
+                    const bool more = nx.advance(a);
+                    if (more) prefetch_tn(nx, (slot ^ 1));
+                    if (more) asm volatile("cp.async.wait_group 1;" ::: "memory");
+                    else asm volatile("cp.async.wait_group 0;" ::: "memory");
+                    __syncwarp();
+                }
+                const float* tn = s_tnw[warp][slot] - half * (NCH / 2);  // indexed by the chunk column
                 float lim = kth2;
                 const unsigned long long ot = atomicOr(other, 0ull);
                 if ((ot & 0xffffffffull) == tag) lim = fminf(lim, __uint_as_float((uint32_t)(ot >> 32)));
@@ -647,11 +664,9 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
                     }
                 }
                 fence_before();
-                __syncwarp();
-                if (lane == 0) {
-                    tc::mbar_arrive(smem_u32(&bar_afree[c]));             // accumulator c may be overwritten
-                    tc::mbar_arrive(smem_u32(&bar_tnfree[g % kExTn]));    // and the chunk's norm slot
-                }
+                __syncwarp();  // (also: every lane is done with norm buffer `slot` before it is refilled)
+                if (lane == 0) tc::mbar_arrive(smem_u32(&bar_afree[c]));  // accumulator c may be overwritten
+                slot ^= 1;
                 atomicExch(mine, ((unsigned long long)__float_as_uint(kth2) << 32) | tag);
                 if (active && half == 0) covered += (unsigned long long)nb;
             }
@@ -690,7 +705,7 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
 
 template <int KMAX>
 static sknn_status launch_dense_exact_k(Ctx& cx, const DenseArgs& a) {
-    const size_t smem = (size_t)kDenseM * a.kp * 2 + kExStages * (size_t)kExNCH * a.kp * 2 + kExTn * kExNCH * 4;
+    const size_t smem = (size_t)kDenseM * a.kp * 2 + kExStages * (size_t)kExNCH * a.kp * 2;
     SKNN_CUDA(cudaFuncSetAttribute(k_dense_exact<KMAX>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_dense_exact<KMAX>, kExThreads, smem);

@@ -359,6 +359,9 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
 #ifndef SKNN_COLLECT
 #define SKNN_COLLECT 1
 #endif
+#ifndef SKNN_MINFIRST
+#define SKNN_MINFIRST 1
+#endif
 #ifndef SKNN_U16
 #define SKNN_U16 2
 #endif
@@ -512,9 +515,21 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
 #pragma unroll
                     for (int c = 0; c < DP / 4; ++c) s = d2_acc4(s, q[c], r[u][c]);
                     dd[u] = s;
-                    // Alg. 2 line 16 (distance part); a lane past the tile's last
-                    // query only shadows the walk and never inserts
-                    if (active && u < n && s <= kth_d2) pass |= 1u << u;
+                }
+#if SKNN_MINFIRST
+                // one compare of the block minimum first (members past n repeat the
+                // last member, so the minimum is still a real distance of the block)
+                float mn = dd[0];
+#pragma unroll
+                for (int u = 1; u < U; ++u) mn = fminf(mn, dd[u]);
+                if (active && mn <= kth_d2)
+#endif
+                {
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        // Alg. 2 line 16 (distance part); a lane past the tile's last
+                        // query only shadows the walk and never inserts
+                        if (active && u < n && dd[u] <= kth_d2) pass |= 1u << u;
                 }
                 while (pass) {
                     const int u = __ffs(pass) - 1;

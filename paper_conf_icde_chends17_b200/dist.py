@@ -43,6 +43,8 @@ def shard_bounds(n: int, world: int, rank: int):
 
 
 def _world(group):
+    if not dist.is_available() or not dist.is_initialized():
+        return 1, 0  # single process: every collective below is skipped
     return dist.get_world_size(group), dist.get_rank(group)
 
 
@@ -172,6 +174,8 @@ def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, lo
         pad_d = torch.full((nq, k - kk), float("inf"), dtype=torch.float32, device=Q.device)
         pidx = torch.cat([pidx, pad_i], 1)
         pd2 = torch.cat([pd2, pad_d], 1)
+    if world == 1:  # one shard: its partial list is the result
+        return merge(pidx.view(1, nq, k), pd2.view(1, nq, k), k, out_squared=out_squared)
     if exchange == "all_gather":
         all_i = torch.empty((world * nq, k), dtype=torch.int32, device=Q.device)
         all_d = torch.empty((world * nq, k), dtype=torch.float32, device=Q.device)
