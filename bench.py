@@ -260,6 +260,14 @@ def roofline_of(st, stage, peaks, nq_r, nt, d, k, ws):
         Rl = float(st.get("rows_loaded", E))
         P = float(st["cand_pairs"]) * (nq_r / max(1.0, st["mq"] / max(1, ws)))
         tile = 32.0 if st["mapping_used"] == 1 else 8.0
+        note = None
+        if st["mapping_used"] != 1:
+            # warp per query: rows_loaded counts every evaluation; the reuse unit of
+            # §8(d) is the 8-query tile (its windows share rows through L1), so the
+            # algorithmic rows are taken as rows_loaded / 8 (the tile's windows
+            # coinciding: a lower bound of their union)
+            Rl /= tile
+            note = "warp-per-query scan: target rows counted once per 8-query tile (rows_loaded / 8)"
         bytes_alg = 4.0 * dpad * nq_r + (4.0 * dpad + 4.0) * Rl + 8.0 * k * nq_r + (4.0 * dpad + 16.0) * P / tile
         flops = 3.0 * d * (E + C) + P * float(np.log2(max(2.0, nt / max(1, st["mt"]))))
         gbs = bytes_alg / (scan_ms / 1e3) / 1e9
@@ -269,6 +277,8 @@ def roofline_of(st, stage, peaks, nq_r, nt, d, k, ws):
             b = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": f_hbm}
         else:
             b = {"bound": "alu", "achieved": tfs, "peak": peaks["fp32_tflops"], "unit": "TFLOP/s", "frac": f_alu}
+        if note:
+            b["note"] = note
         b.update({"kernel": "k_scan_%s (level-2 scan fused with top-k)" % ("tpq" if st["mapping_used"] == 1 else "wpq"),
                   "launch_ms": scan_ms, "algorithmic_bytes": bytes_alg, "algorithmic_flops": flops,
                   "intensity_flop_per_byte": flops / bytes_alg if bytes_alg else None,
@@ -283,8 +293,9 @@ def roofline_of(st, stage, peaks, nq_r, nt, d, k, ws):
         tfs = flops / (dense_ms / 1e3) / 1e12
         pk = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
         out["dense"] = {"bound": "tensor", "achieved": tfs, "peak": pk, "unit": "TFLOP/s", "frac": tfs / pk,
-                        "kernel": "k_dense (tcgen05 bf16 screen + exact fp32 recompute)", "launch_ms": dense_ms,
-                        "algorithmic_flops": flops, "mma_terms": terms}
+                        "kernel": "k_dense (tcgen05 bf16 dense tiles: %s)" % (
+                            "exact integer, no recompute" if terms == 1 else "split-precision screen + exact recompute"),
+                        "launch_ms": dense_ms, "algorithmic_flops": flops, "mma_terms": terms}
     if not out:
         return None
     dom = max(out, key=lambda s: out[s]["launch_ms"])

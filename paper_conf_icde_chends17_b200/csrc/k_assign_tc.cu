@@ -97,10 +97,11 @@ __global__ void k_centers_to_tc(const float* __restrict__ centers, int m, int mp
 // chunk with a warp-specialised producer and up to 6 stages, one CTA per SM
 // -- C4 full pass 2.29 -> 2.68 ms, C5 5.21 -> 5.56 ms.)
 constexpr int kTcThreads = 256;
+constexpr int kTcMaxStages = 6;
 __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __restrict__ Xp, int64_t n, int dp, int kp,
                                                        const float* __restrict__ o,
                                                        const __nv_bfloat16* __restrict__ cbf, int m, int nchunks,
-                                                       const float* __restrict__ centers,
+                                                       int nstages, const float* __restrict__ centers,
                                                        int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
                                                        long long* __restrict__ sums, const double* __restrict__ fx,
                                                        int32_t* __restrict__ counts, int stride) {
@@ -108,7 +109,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
     const uint32_t a_bytes = (uint32_t)kTcM * kp * 2, b_bytes = (uint32_t)kTcN * kp * 2;
     unsigned char* sA = smem;
     auto sB = [&](int b) { return smem + a_bytes + (uint32_t)b * b_bytes; };
-    __shared__ __align__(8) uint64_t bar_full[2], bar_mma[2];
+    __shared__ __align__(8) uint64_t bar_full[kTcMaxStages], bar_mma[2];
     __shared__ uint32_t s_tmem;
     const int tid = threadIdx.x, warp = tid >> 5;
     const uint32_t sbo = (uint32_t)kp * 16u;
@@ -117,10 +118,8 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
         tc::tmem_alloc(&s_tmem, 2u * kTcN);
     }
     if (tid == 0) {
-        for (int i = 0; i < 2; ++i) {
-            tc::mbar_init(smem_u32(&bar_full[i]), 1);
-            tc::mbar_init(smem_u32(&bar_mma[i]), 1);
-        }
+        for (int i = 0; i < nstages; ++i) tc::mbar_init(smem_u32(&bar_full[i]), 1);
+        for (int i = 0; i < 2; ++i) tc::mbar_init(smem_u32(&bar_mma[i]), 1);
         tc::mbar_fence_init();
     }
     // stage A = x - o (bf16) for the CTA's 128 points
@@ -153,29 +152,29 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
     const uint32_t tmem = s_tmem;
     const uint32_t idesc = idesc_bf16_m128(kTcN);
 
-    auto issue_copy = [&](int chunk, int buf) {
+    auto issue_copy = [&](int chunk, int buf) {  // chunk -> B stage buf
         const uint32_t bar = smem_u32(&bar_full[buf]);
         tc::expect_tx(bar, b_bytes);
         const unsigned char* src = reinterpret_cast<const unsigned char*>(cbf) + (size_t)chunk * b_bytes;
         tc::bulk_g2s(smem_u32(sB(buf)), src, b_bytes, bar);
     };
-    auto issue_mma = [&](int buf) {
+    auto issue_mma = [&](int stage, int acc) {  // B stage -> accumulator acc
         tc::fence_after();
-        const uint32_t aB = smem_u32(sA), bB = smem_u32(sB(buf));
+        const uint32_t aB = smem_u32(sA), bB = smem_u32(sB(stage));
         for (int s = 0; s < kp / 16; ++s)
-            tc::mma_bf16(tmem + (uint32_t)(buf * kTcN), desc_kmajor(aB + s * 256u, sbo), desc_kmajor(bB + s * 256u, sbo),
+            tc::mma_bf16(tmem + (uint32_t)(acc * kTcN), desc_kmajor(aB + s * 256u, sbo), desc_kmajor(bB + s * 256u, sbo),
                          idesc, s > 0);
-        tc::mma_commit(smem_u32(&bar_mma[buf]));
+        tc::mma_commit(smem_u32(&bar_mma[acc]));
     };
 
-    uint32_t ph_full[2] = {0, 0}, ph_mma[2] = {0, 0};
+    // chunk c lives in B stage c % nstages (phase (c / nstages) & 1 of its
+    // full barrier) and accumulates into accumulator c & 1
+    uint32_t ph_mma[2] = {0, 0};
     if (tid == 0) {
-        issue_copy(0, 0);
-        if (nchunks > 1) issue_copy(1, 1);
+        for (int c = 0; c < nstages && c < nchunks; ++c) issue_copy(c, c);
         tc::mbar_wait(smem_u32(&bar_full[0]), 0);
-        issue_mma(0);
+        issue_mma(0, 0);
     }
-    ph_full[0] = 1;
     float best = __int_as_float(0x7f800000);
     int bi = 0;
     const int half = warp >> 2;  // columns [64 * half, 64 * half + 64) of every chunk
@@ -184,18 +183,17 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
         const int buf = c & 1;
         // issue the next chunk's MMA as soon as its copy landed (overlaps this epilogue)
         if (tid == 0 && c + 1 < nchunks) {
-            const int nb = (c + 1) & 1;
-            tc::mbar_wait(smem_u32(&bar_full[nb]), ph_full[nb]);
-            issue_mma(nb);
+            const int ns = (c + 1) % nstages;
+            tc::mbar_wait(smem_u32(&bar_full[ns]), ((c + 1) / nstages) & 1);
+            issue_mma(ns, (c + 1) & 1);
         }
-        if (c + 1 < nchunks) ph_full[(c + 1) & 1] ^= 1u;
         tc::mbar_wait(smem_u32(&bar_mma[buf]), ph_mma[buf]);
         ph_mma[buf] ^= 1u;
         tc::fence_after();
-        // MMA(c) has consumed stage `buf`: refill it now, so the copy overlaps
-        // this chunk's epilogue (the accumulator `buf` stays busy until the
-        // barrier below; MMA(c + 2) is issued only after it)
-        if (tid == 0 && c + 2 < nchunks) issue_copy(c + 2, buf);
+        // MMA(c) has consumed B stage c % nstages: refill it now with chunk
+        // c + nstages (the accumulator `buf` stays busy until the barrier below;
+        // MMA(c + 2) is issued only after it)
+        if (tid == 0 && c + nstages < nchunks) issue_copy(c + nstages, c % nstages);
         // per 32 columns: the scores (straight from TMEM), their minimum by a
         // min tree (one FMNMX per score) and, only when it beats the running
         // best, the lowest column holding it (a strict running argmin)
@@ -214,12 +212,18 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
             for (int w = 8; w > 0; w >>= 1)
 #pragma unroll
                 for (int j = 0; j < w; ++j) t[j] = fminf(t[j], t[j + w]);
-            if (t[0] < best) {  // the lowest column holding the new best
-                int jm = 31;
+            // the lowest column holding a new best; a warp-uniform branch (the
+            // compiler otherwise if-converts the 32-step search and runs it for
+            // every block: ncu, 35% of the C5 pass's instructions)
+            const bool better = t[0] < best;
+            if (__any_sync(0xffffffffu, better)) {
+                if (better) {
+                    int jm = 31;
 #pragma unroll
-                for (int j = 31; j >= 0; --j) jm = (sc[j] == t[0]) ? j : jm;
-                best = t[0];
-                bi = c * kTcN + col + jm;
+                    for (int j = 31; j >= 0; --j) jm = (sc[j] == t[0]) ? j : jm;
+                    best = t[0];
+                    bi = c * kTcN + col + jm;
+                }
             }
         }
         tc::fence_before();
@@ -269,12 +273,18 @@ sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
     k_centers_to_tc<<<(int)std::min<int64_t>((mpad + 255) / 256, 148 * 8), 256, 0, cx.stream>>>(centers, m, mpad, dp, kp,
                                                                                                 o, cbf);
     cx.launched();
-    // >= 90 KB keeps at most two CTAs per SM: each holds 256 of the 512 TMEM columns
-    const size_t smem = std::max<size_t>((size_t)kTcM * kp * 2 + 2 * (size_t)kTcN * kp * 2, 90 * 1024);
+    // B ring depth: as many stages (<= 6) as keep two CTAs per SM (each holds 256
+    // of the 512 TMEM columns) within ~110 KB of shared memory, at least 2; a
+    // stage is refilled as soon as its MMA completed, so deeper rings hide the
+    // L2 latency of the chunk loads (measured: C4 / C5 passes)
+    const size_t a_bytes = (size_t)kTcM * kp * 2, b_bytes = (size_t)kTcN * kp * 2;
+    const int nstages =
+        (int)std::max<size_t>(2, std::min<size_t>(kTcMaxStages, (110 * 1024 - a_bytes) / b_bytes));
+    const size_t smem = std::max<size_t>(a_bytes + nstages * b_bytes, 90 * 1024);
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     const int64_t grid = ((n + stride - 1) / stride + kTcM - 1) / kTcM;
-    k_assign_tc<<<(unsigned)grid, kTcThreads, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, m, nchunks, centers, cid, dist,
+    k_assign_tc<<<(unsigned)grid, kTcThreads, smem, cx.stream>>>(Xp, n, dp, kp, o, cbf, m, nchunks, nstages, centers, cid, dist,
                                                           sums, fx, counts, stride);
     cx.launched();
     return cx.check_launch("assign (tensor cores)");

@@ -371,6 +371,18 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
 #ifndef SKNN_UNION_MINB4
 #define SKNN_UNION_MINB4 3
 #endif
+#ifndef SKNN_AB4
+#define SKNN_AB4 2
+#endif
+#ifndef SKNN_AB16
+#define SKNN_AB16 1
+#endif
+// blocks of union_block<DP>() members per alive test of the walk (overshoot
+// past a side's last needed member: at most U * AB - 1 extra evaluations)
+template <int DP>
+constexpr int union_alive_blocks() {
+    return DP == 0 ? 1 : (DP <= 4 ? SKNN_AB4 : (DP <= 16 && DP > 8 ? SKNN_AB16 : 1));
+}
 template <int DP>
 constexpr int union_block() {
     return DP == 0 ? 1 : (DP <= 4 ? SKNN_U4 : (DP <= 8 ? 4 : (DP <= 16 ? SKNN_U16 : 1)));
@@ -605,10 +617,15 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
         bool aliveL = L >= lo && __any_sync(FULL, ok && ti_keep(__ldg(a.tdist + L) - dq, theta,
                                                                  dq + __ldg(a.tdist + L), a.eta));
         unsigned walked = 0;
+        // the alive test (a load of the next member distance + a vote) runs once
+        // per UA = U * AB members; the block is evaluated U members at a time
+        constexpr int AB = union_alive_blocks<DP>();
         while (aliveR || aliveL) {
             if (aliveR) {
-                const int n = min(U, hi - R);
-                eval_block(R, 1, n);
+                const int n = min(U * AB, hi - R);
+#pragma unroll
+                for (int sb = 0; sb < AB; ++sb)
+                    if (sb * U < n) eval_block(R + sb * U, 1, min(U, n - sb * U));
                 refresh();
                 R += n;
                 walked += n;
@@ -617,8 +634,10 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
                 aliveR = R < hi && __any_sync(FULL, ok && ti_keep(dq - dtn, theta, dq + dtn, a.eta));
             }
             if (aliveL) {
-                const int n = min(U, L - lo + 1);
-                eval_block(L, -1, n);
+                const int n = min(U * AB, L - lo + 1);
+#pragma unroll
+                for (int sb = 0; sb < AB; ++sb)
+                    if (sb * U < n) eval_block(L - sb * U, -1, min(U, n - sb * U));
                 refresh();
                 L -= n;
                 walked += n;
