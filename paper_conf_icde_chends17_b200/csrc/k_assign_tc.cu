@@ -23,6 +23,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "sknn_internal.cuh"
 #include "sknn_launch.h"
@@ -273,13 +274,14 @@ sknn_status run_assign_tc(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
     k_centers_to_tc<<<(int)std::min<int64_t>((mpad + 255) / 256, 148 * 8), 256, 0, cx.stream>>>(centers, m, mpad, dp, kp,
                                                                                                 o, cbf);
     cx.launched();
-    // B ring depth: as many stages (<= 6) as keep two CTAs per SM (each holds 256
-    // of the 512 TMEM columns) within ~110 KB of shared memory, at least 2; a
-    // stage is refilled as soon as its MMA completed, so deeper rings hide the
-    // L2 latency of the chunk loads (measured: C4 / C5 passes)
+    // B ring depth: 2 (SKNN_ASSIGN_STAGES = 3..6 for study). Measured: a
+    // 6-deep ring (two CTAs per SM still) is SLOWER on C5 (5.3 -> 5.7 ms per
+    // full pass): the pass is bound by the epilogue's ALU pipe (ncu: ALU 60%,
+    // one FMNMX per score), not by the chunk loads
     const size_t a_bytes = (size_t)kTcM * kp * 2, b_bytes = (size_t)kTcN * kp * 2;
-    const int nstages =
-        (int)std::max<size_t>(2, std::min<size_t>(kTcMaxStages, (110 * 1024 - a_bytes) / b_bytes));
+    const char* es = getenv("SKNN_ASSIGN_STAGES");
+    const int want = es ? std::max(2, std::min(kTcMaxStages, atoi(es))) : 2;
+    const int nstages = (int)std::max<size_t>(2, std::min<size_t>(want, (110 * 1024 - a_bytes) / b_bytes));
     const size_t smem = std::max<size_t>(a_bytes + nstages * b_bytes, 90 * 1024);
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     SKNN_CUDA(cudaFuncSetAttribute(k_assign_tc, cudaFuncAttributePreferredSharedMemoryCarveout, 100));

@@ -258,15 +258,18 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
             float dv[8];
 #pragma unroll
             for (int u = 0; u < 8; ++u) dv[u] = (i0 + u < cnt) ? __ldg(tdist + hi - 1 - i0 - u) : __int_as_float(0x7f800000);
-            bool stop = false;
+            // the bounds grow along the batch: keep its prefix <= M_k with ONE
+            // shared-memory atomic per batch (not one per bound: ncu showed the
+            // CTAs serialised on that counter)
+            int nkeep = 0;
 #pragma unroll
-            for (int u = 0; u < 8; ++u) {
-                const float v = D + dv[u];
-                if (v > Mk) { stop = true; break; }  // later bounds only grow
-                const int pos = atomicAdd(&s_cnt, 1);
-                if (pos < kL1Vals) s_keys[pos] = u64(__float_as_uint(v));
-            }
-            if (stop) break;
+            for (int u = 0; u < 8; ++u) nkeep += (D + dv[u] <= Mk) ? 1 : 0;
+            if (nkeep == 0) break;
+            const int pos = atomicAdd(&s_cnt, nkeep);
+#pragma unroll
+            for (int u = 0; u < 8; ++u)
+                if (u < nkeep && pos + u < kL1Vals) s_keys[pos + u] = u64(__float_as_uint(D + dv[u]));
+            if (nkeep < 8) break;  // later bounds only grow
         }
     }
     __syncthreads();

@@ -401,7 +401,10 @@ static void launch_wpq(Ctx& cx, const ScanArgs& a) {
 // it. SKNN_BIGK_HEAP=1 keeps the heap for every k (ablation).
 bool scan_uses_bigk(int k) { return k > 96 && !getenv("SKNN_BIGK_HEAP"); }
 bool scan_uses_tpq(int mapping, int dp, int k) {
-    return !scan_uses_bigk(k) && ((mapping == SKNN_MAP_THREAD && dp <= 32) || k > 32);
+    // SKNN_TPQ_HIGHD=1 (study): a forced thread mapping also for dp > 32 (the
+    // runtime-dp union walk, query rows re-read from L1, member rows broadcast)
+    static const bool highd = getenv("SKNN_TPQ_HIGHD") != nullptr;
+    return !scan_uses_bigk(k) && ((mapping == SKNN_MAP_THREAD && (dp <= 32 || highd)) || k > 32);
 }
 int scan_tile_size(int mapping, int dp, int k) { return scan_uses_tpq(mapping, dp, k) ? 32 : 8; }
 
