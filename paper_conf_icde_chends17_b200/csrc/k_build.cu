@@ -359,6 +359,7 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
                                                      int nwalk, int32_t* __restrict__ rank_out) {
     const int dp = DP > 0 ? DP : dp_rt;
     const int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * stride;  // Lloyd passes subsample
+    const unsigned live = __ballot_sync(0xffffffffu, i < n);  // lanes that reach the aggregated atomic
     if (i >= n) return;
     const float* xr = Xp + i * dp;
     float4 q[DP > 0 ? DP / 4 : 1];
@@ -411,8 +412,16 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
     if (cid_out) cid_out[i] = best;
     if (dist_out) dist_out[i] = __fsqrt_rn(bd);
     if (counts) {  // rank_out: the member's slot in its cluster (k_scatter_keys needs no atomics)
-        const int r = atomicAdd(counts + best, 1);
-        if (rank_out) rank_out[i] = r;
+        // warp-aggregated: lanes with the same cluster (neighbouring input rows
+        // often share one) take one atomic; slots are sorted away later, so the
+        // order within a group does not matter
+        const int lane = threadIdx.x & 31;
+        const unsigned grp = __match_any_sync(live, best);
+        const int leader = __ffs(grp) - 1;
+        int base = 0;
+        if (lane == leader) base = atomicAdd(counts + best, __popc(grp));
+        base = __shfl_sync(grp, base, leader);
+        if (rank_out) rank_out[i] = base + __popc(grp & ((1u << lane) - 1u));
     }
     if (sums) {
         fx_accumulate(sums + (int64_t)best * dp, xr, dp, *fx);
@@ -668,7 +677,9 @@ __device__ __forceinline__ void warp_segsort(u64* __restrict__ g, int size, floa
 
 // one 256-thread CTA per cluster of at most kMidSeg members: up to kTinySeg
 // members warp 0 sorts in registers (the other warps leave), larger clusters
-// run the bitonic network in 8 KB of shared memory
+// run the bitonic network in 8 KB of shared memory. (Measured and rejected:
+// 8 clusters per CTA, one warp each, with the 257-1024-member ones in a second
+// launch -- C2 25.5 -> 38 us; register sorts up to 512 members -- 62 us.)
 constexpr int kMidSeg = 1024;
 __global__ void __launch_bounds__(256) k_segsort_small(u64* __restrict__ keys, const int32_t* __restrict__ off,
                                                        float* __restrict__ radius) {
@@ -942,6 +953,8 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         if (graph_m != mc) {
             // (measured and rejected: centers staged in shared memory, two-pass
             // bound + compaction, 16 warps per CTA -- C2 29.5 vs 30.5 us)
+            // (measured and rejected: each center's candidates split over 4 warps
+            // merged bitonically -- C2 30 -> 41 us)
             k_center_knn<<<(mc + 7) / 8, 256, 0, s>>>(out.centers, mc, dp, nbr);
             cx.launched();
             graph_m = mc;
@@ -971,8 +984,10 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     const int32_t* prev = nullptr;
     // the D^2 draw only needs the squared distances of a sample: the seeding
     // pass assigns every sstride-th point (others keep distance 0 = never drawn;
-    // C5 seeding pass 3.2 -> ~0.4 ms per side)
-    const int sstride = (int)std::max<int64_t>(1, std::min<int64_t>(8, n / (64LL * std::max(1, m0))));
+    // C5 build 21.2 -> 17.1 ms for both sides, C3 join 3.94 -> 3.65 ms)
+    // (dp <= 32 only: at d = 128 (C4) the sampled seeding let a few clusters grow
+    // large and the warp-per-query scan's tail explode -- measured 25 -> 824 ms)
+    const int sstride = dp <= 32 ? (int)std::max<int64_t>(1, std::min<int64_t>(8, n / (64LL * std::max(1, m0)))) : 1;
     int seed_stride = 1;
     if (m0 < m) {
         SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
