@@ -28,8 +28,16 @@
  *     call is stream-ordered: it enqueues all work on `stream` and returns
  *     without waiting (unless stats are requested); results are valid once
  *     `stream` completes.
- *   - The library never frees caller memory. Scratch is allocated with
- *     cudaMallocAsync on `stream` and released (stream-ordered) before return.
+ *   - The library never frees caller memory. Scratch is allocated from a
+ *     private stream-ordered memory pool of the device (cudaMallocFromPoolAsync
+ *     on `stream`; up to 8 GB of freed scratch stays reserved in that pool
+ *     between calls, the device's default pool is not touched) and released
+ *     (stream-ordered) before return.
+ *   - sknn_join / sknn_join_ex with device pointers and no stats: when the
+ *     same (device, pointers, sizes, options) repeat, the second call records
+ *     the join into a CUDA graph and later calls replay it (one launch); the
+ *     replay reads the CURRENT contents of the recorded buffers, so results
+ *     are always those of the data at call time (opt->use_graph = -1 opts out).
  *   - `stream` is a cudaStream_t (NULL = the legacy default stream).
  *
  * Errors: every function returns an sknn_status; no C++ exception crosses the
@@ -80,7 +88,9 @@ enum {
                           /* fixed at the level-1 UB, every window member's distance stored  */
                           /* in a global survivor buffer, then a k-selection kernel; k <= 512 */
                           /* (falls back to the full filter when the buffer would not fit in */
-                          /* half of the free device memory)                                 */
+                          /* half of the free device memory). It reads the survivor count    */
+                          /* back to size that buffer: the call synchronises `stream` (the   */
+                          /* one host round trip of the library; never taken by auto)         */
 };
 
 /* Level-2 thread mapping override (sknn_options.mapping), §IV-B2 / §IV-D3. */

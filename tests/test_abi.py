@@ -113,3 +113,13 @@ def test_config_decide_matches_oracle_b200(L):
     assert sknn.config_decide(4_000_000, 4_000_000, 16, 32, props=props)["mapping"] == 1
     assert sknn.config_decide(65_554, 65_554, 28, 16, props=props)["mapping"] == 1  # B200 rule: dp <= 32
     assert sknn.config_decide(1_000_000, 1_000_000, 128, 16, props=props)["mapping"] == 2
+
+
+def test_struct_layouts_match_the_header(L):
+    """The ctypes mirrors of sknn_options / sknn_stats have the C sizes
+    (sknn_options_default writes sizeof(sknn_options) into struct_size)."""
+    o = sknn.make_options()
+    assert o.struct_size == ctypes.sizeof(sknn.Options)
+    # sknn_stats: the last field (dense_terms + pad) closes an 8-byte-aligned struct
+    assert ctypes.sizeof(sknn.Stats) % 8 == 0
+    assert sknn.Stats.dense_terms.offset == sknn.Stats.rows_loaded.offset + 8
