@@ -97,7 +97,14 @@ enum {
 enum {
     SKNN_MAP_AUTO = 0,
     SKNN_MAP_THREAD = 1,  /* one thread per query ("query level parallelism")       */
-    SKNN_MAP_WARP = 2     /* one warp per query ("multi-level parallelism")         */
+    SKNN_MAP_WARP = 2,    /* one warp per query ("multi-level parallelism")         */
+    SKNN_MAP_BASIC = 3    /* ablation arm: the basic KNN-TI Sweet KNN starts from     */
+                          /* (Fig. 4 / Alg. 2): one thread per */
+                          /* query in INPUT order (no thread-data remapping, §IV-C1), */
+                          /* every member of a candidate cluster visited from the top */
+                          /* (Alg. 2's continue / break), kNearests a sorted array in */
+                          /* thread-local memory; sparse only, k <= 32, no sharding.  */
+                          /* Same exact result as every other mapping    */
 };
 
 /* Tunables. Zero-initialise and set struct_size = sizeof(sknn_options), or
@@ -137,7 +144,12 @@ typedef struct {
     int32_t use_graph;        /* sknn_join_ex on device pointers without stats: 0 = auto (replay a */
                               /*   captured CUDA graph of the whole join when the same shapes,     */
                               /*   pointers and options repeat), -1 = never                         */
-    int32_t pad2;
+    int32_t shard_policy;     /* query sharding (shard_count > 1): which query clusters a rank owns. */
+                              /*   0 = interleave (c % shard_count == shard_rank);                   */
+                              /*   1 = balanced: every rank runs level-1 over ALL query clusters      */
+                              /*   (replicated) and deals the clusters, heaviest first by |qc| x the */
+                              /*   level-1 scan-work estimate, to ranks in snake order -- identical  */
+                              /*   on every rank (deterministic clustering and integer work sums)     */
 } sknn_options;
 
 /* Counters and per-stage times of one call (filled only when a non-NULL

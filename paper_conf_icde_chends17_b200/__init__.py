@@ -26,7 +26,7 @@ SKNN_OK = 0
 STATUS = {0: "SKNN_OK", -1: "SKNN_ERR_INVALID_ARG", -2: "SKNN_ERR_NOT_DEVICE_PTR", -3: "SKNN_ERR_OOM",
           -4: "SKNN_ERR_CUDA", -5: "SKNN_ERR_UNSUPPORTED", -6: "SKNN_ERR_WRONG_DEVICE"}
 PATH = {"auto": 0, "sparse": 1, "dense": 2, "brute": 3, "partial": 4}
-MAPPING = {"auto": 0, "thread": 1, "warp": 2}
+MAPPING = {"auto": 0, "thread": 1, "warp": 2, "basic": 3}
 MAX_K = 512
 
 # every symbol include/sknn.h declares (tests check the library exports them)
@@ -52,7 +52,7 @@ class Options(ctypes.Structure):
                 ("out_squared", ctypes.c_int32), ("pad0", ctypes.c_int32), ("index_base", ctypes.c_int64),
                 ("shard_rank", ctypes.c_int32), ("shard_count", ctypes.c_int32), ("query_batch", ctypes.c_int64),
                 ("self_query", ctypes.c_int32), ("pad1", ctypes.c_int32), ("ub_in", ctypes.c_void_p),
-                ("use_graph", ctypes.c_int32), ("pad2", ctypes.c_int32)]
+                ("use_graph", ctypes.c_int32), ("shard_policy", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):

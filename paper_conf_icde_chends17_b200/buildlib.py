@@ -49,9 +49,16 @@ def build(force: bool = False, verbose: bool = False, out: str = None) -> str:
         common += ["-Xptxas", "-v"]
     objs = []
     procs = []
+    hdr = glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh")) + \
+        glob.glob(os.path.join(INCLUDE, "*.h")) + [os.path.abspath(__file__)]
+    hdr_t = max(os.path.getmtime(h) for h in hdr)
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src)[:-3] + ".o")
         objs.append(obj)
+        # incremental: an object newer than its source and every header is kept
+        # (flags are part of objdir's name, so a flag change never reuses one)
+        if not force and os.path.exists(obj) and os.path.getmtime(obj) > max(os.path.getmtime(src), hdr_t):
+            continue
         cmd = [NVCC, "-c", src, "-o", obj] + common
         procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
     failed = False

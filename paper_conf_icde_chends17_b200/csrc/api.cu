@@ -207,7 +207,7 @@ struct Timer {
 };
 
 static int choose_mapping(const sknn_options& o, const DevInfo& di, int64_t nq, int dp, int k) {
-    if (o.mapping == SKNN_MAP_THREAD || o.mapping == SKNN_MAP_WARP) return o.mapping;
+    if (o.mapping == SKNN_MAP_THREAD || o.mapping == SKNN_MAP_WARP || o.mapping == SKNN_MAP_BASIC) return o.mapping;
     if (k > 32) return scan_uses_bigk(k) ? SKNN_MAP_WARP : SKNN_MAP_THREAD;  // k_scan_bigk: warp per query
     // Fig. 8 bottom chooses query-level parallelism when
     // |Q| >= r*max_cur and several threads per query otherwise. Measured on
@@ -270,6 +270,14 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     lp.eta = eta;
     lp.shard_rank = o.shard_count > 1 ? o.shard_rank : 0;
     lp.shard_count = o.shard_count > 1 ? o.shard_count : 1;
+    // balanced query sharding: level-1 over every query cluster (replicated),
+    // then the owner deal (run_shard_owner); the partial filter keeps interleave
+    const bool balanced = lp.shard_count > 1 && o.shard_policy == 1 && o.force_path != SKNN_PATH_PARTIAL;
+    const int shard_rank = lp.shard_rank, shard_count = lp.shard_count;
+    if (balanced) {
+        lp.shard_rank = 0;
+        lp.shard_count = 1;
+    }
     lp.dense_mode = dense_mode_for(o, ts.dp);
     lp.dense_tau = dense_tau_for(o, ts.dp);
     lp.ub_in = o.ub_in;
@@ -278,6 +286,14 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
         return SKNN_ERR_UNSUPPORTED;
     }
     if (k > 32) lp.dense_mode = 1;  // the dense tiles keep a register top-k (k <= 32)
+    const bool basic = mapping == SKNN_MAP_BASIC;
+    if (basic) {
+        if (k > 32 || o.force_path == SKNN_PATH_DENSE || o.force_path == SKNN_PATH_PARTIAL || shard_count > 1) {
+            set_last_error("mapping = BASIC (ablation arm) runs the sparse full filter only, k <= 32, unsharded");
+            return SKNN_ERR_UNSUPPORTED;
+        }
+        lp.dense_mode = 1;
+    }
     DenseOrigin dorg;
     if (lp.dense_mode != 1) {
         SKNN_TRY(dense_prepare(cx, qs, ts, dorg));
@@ -288,6 +304,7 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
         NvtxRange r("sknn level-1 (calUB + groupFilter)");
         SKNN_TRY(run_level1(cx, qs, ts, lp, l1, counters));
     }
+    if (balanced) SKNN_TRY(run_shard_owner(cx, qs, l1, shard_rank, shard_count));
     // Filter strength (§IV-D1, reading R13): the paper switches to the
     // partial level-2 filter when k/d > 8. Measured on B200 the
     // full filter wins every case once large k runs warp per query
@@ -297,8 +314,8 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     const bool partial = o.force_path == SKNN_PATH_PARTIAL;
     // the partial filter's passes take 32 queries per warp task (thread per query)
     const int tile = partial ? 32 : scan_tile_size(mapping, ts.dp, k);
-    SKNN_TRY(run_tiles(cx, qs, tile, k, scan_resident_warps(cx, mapping, ts.dp, k),
-                       lp.shard_rank, lp.shard_count, l1));
+    if (!basic)
+        SKNN_TRY(run_tiles(cx, qs, tile, k, scan_resident_warps(cx, mapping, ts.dp, k), shard_rank, shard_count, l1));
     mk.l1 = tm.mark();
     key_t* init_topk = nullptr;
     if (lp.dense_mode != 1) {
@@ -334,9 +351,12 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
         // 32-query split tasks are only valid for the thread-per-query scan)
         if (fell_back && scan_tile_size(mapping, ts.dp, k) != tile)
             SKNN_TRY(run_tiles(cx, qs, scan_tile_size(mapping, ts.dp, k), k,
-                               scan_resident_warps(cx, mapping, ts.dp, k), lp.shard_rank, lp.shard_count, l1));
+                               scan_resident_warps(cx, mapping, ts.dp, k), shard_rank, shard_count, l1));
     }
-    if (full) {
+    if (basic) {
+        NvtxRange r("sknn level-2 scan (basic KNN-TI)");
+        SKNN_TRY(run_scan_basic(cx, qs, ts, l1, sp));
+    } else if (full) {
         NvtxRange r("sknn level-2 scan");
         SKNN_TRY(run_scan(cx, qs, ts, l1, sp));
     }
@@ -395,7 +415,7 @@ static cudaStream_t side_stream(int dev) {
 static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t nt, int32_t d, int32_t k,
                             int32_t* out_idx, float* out_dist, const sknn_options* opt_in, sknn_stats* stats,
                             cudaStream_t stream, const sknn_index* index, bool capturing = false,
-                            const sknn_index* qindex = nullptr) {
+                            const sknn_index* qindex = nullptr, bool defer_sync = false) {
     NvtxRange nvtx_call(qindex ? "sknn_join_indexed" : (index ? "sknn_query" : "sknn_join"));
     // a query index supplies the clustered query side (Q is not read)
     static const float kNoQ = 0.f;
@@ -577,7 +597,9 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     }
     int launches = cx.launches;
     cx.free_all();
-    if (st == SKNN_OK && (stats || oi_host || od_host || q_host || t_host)) {
+    // host buffers are synchronised before returning, unless the caller (the
+    // overlapped out-of-core batches) passed pinned buffers and syncs itself
+    if (st == SKNN_OK && (stats || ((oi_host || od_host || q_host || t_host) && !defer_sync))) {
         cudaError_t e = cudaStreamSynchronize(stream);
         if (e != cudaSuccess) st = fail(SKNN_ERR_CUDA, std::string("kernel execution failed: ") + cudaGetErrorString(e));
     }
@@ -765,6 +787,110 @@ sknn_status sknn_build(const float* T, int64_t nt, int32_t d, const sknn_options
     return SKNN_OK;
 }
 
+// Out-of-core batches, overlapped (NEXT-4): batch b runs on stream s[b % 2]
+// (the caller's stream and one private stream), so batch b's host->device
+// copy and kernels overlap batch b-1's device->host copy. Host buffers the
+// caller did not page-lock go through page-locked staging buffers (a
+// cudaMemcpyAsync into pageable memory blocks the host thread until it
+// completes, which would serialise the batches): rows are staged on the host
+// while the device runs the previous batch, and a batch's results are copied
+// out of staging once its completion event fires. Every batch is the same
+// exact query, so the rows equal one unbatched call.
+static bool pinned_host(const void* p) {
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeHost;
+}
+
+static sknn_status query_batches_overlapped(const sknn_index* index, const float* Q, int64_t nq, int32_t k,
+                                            int32_t* out_idx, float* out_dist, const sknn_options* opt, int64_t B,
+                                            cudaStream_t user) {
+    const int d = index->t.d;
+    const bool q_pin = pinned_host(Q), oi_pin = !out_idx || pinned_host(out_idx), od_pin = pinned_host(out_dist);
+    if (!(q_pin && oi_pin && od_pin)) {  // staging: at most 256 MB of rows per slot (SKNN_OOC_STAGE=1 only)
+        const int64_t row = 4ll * d + 8ll * k;
+        B = std::max<int64_t>(k, std::min<int64_t>(B, (256ll << 20) / row));
+    }
+    cudaStream_t s[2] = {user, nullptr};
+    cudaEvent_t done[2] = {nullptr, nullptr}, start = nullptr;
+    float* sq[2] = {nullptr, nullptr};
+    int32_t* si[2] = {nullptr, nullptr};
+    float* sd[2] = {nullptr, nullptr};
+    int64_t pend_b0[2] = {-1, -1}, pend_nb[2] = {0, 0};
+    sknn_status st = SKNN_OK;
+    auto cuda_ok = [&](cudaError_t e, const char* what) {
+        if (e == cudaSuccess) return true;
+        st = fail(SKNN_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+        return false;
+    };
+    // results of the batch in `slot` (already complete) into the caller's buffers
+    auto finish = [&](int slot) {
+        if (pend_b0[slot] < 0) return;
+        if (!cuda_ok(cudaEventSynchronize(done[slot]), "batch")) return;
+        const int64_t b0 = pend_b0[slot], nb = pend_nb[slot];
+        if (!od_pin) memcpy(out_dist + b0 * k, sd[slot], sizeof(float) * nb * k);
+        if (!oi_pin) memcpy(out_idx + b0 * k, si[slot], sizeof(int32_t) * nb * k);
+        pend_b0[slot] = -1;
+    };
+    do {
+        if (!cuda_ok(cudaStreamCreateWithFlags(&s[1], cudaStreamNonBlocking), "stream")) break;
+        if (!cuda_ok(cudaEventCreateWithFlags(&start, cudaEventDisableTiming), "event")) break;
+        if (!cuda_ok(cudaEventCreateWithFlags(&done[0], cudaEventDisableTiming), "event")) break;
+        if (!cuda_ok(cudaEventCreateWithFlags(&done[1], cudaEventDisableTiming), "event")) break;
+        // the private stream starts after the work the caller queued before the call
+        if (!cuda_ok(cudaEventRecord(start, user), "event")) break;
+        if (!cuda_ok(cudaStreamWaitEvent(s[1], start, 0), "event")) break;
+        for (int i = 0; i < 2 && st == SKNN_OK; ++i) {
+            if (!q_pin) cuda_ok(cudaHostAlloc((void**)&sq[i], sizeof(float) * B * d, cudaHostAllocDefault), "staging");
+            if (!oi_pin && st == SKNN_OK)
+                cuda_ok(cudaHostAlloc((void**)&si[i], sizeof(int32_t) * B * k, cudaHostAllocDefault), "staging");
+            if (!od_pin && st == SKNN_OK)
+                cuda_ok(cudaHostAlloc((void**)&sd[i], sizeof(float) * B * k, cudaHostAllocDefault), "staging");
+        }
+        if (st != SKNN_OK) break;
+        int b = 0;
+        for (int64_t b0 = 0; b0 < nq && st == SKNN_OK; b0 += B, ++b) {
+            const int slot = b & 1;
+            const int64_t nb = std::min(B, nq - b0);
+            finish(slot);  // batch b-2: its staging buffers are free again
+            if (st != SKNN_OK) break;
+            const float* qb = Q + b0 * d;
+            if (!q_pin) {
+                memcpy(sq[slot], qb, sizeof(float) * nb * d);
+                qb = sq[slot];
+            }
+            int32_t* ob = out_idx ? (oi_pin ? out_idx + b0 * k : si[slot]) : nullptr;
+            float* db = od_pin ? out_dist + b0 * k : sd[slot];
+            st = run_join(qb, nb, nullptr, index->t.n, d, k, ob, db, opt, nullptr, s[slot], index, false, nullptr,
+                          /*defer_sync=*/true);
+            if (st != SKNN_OK) break;
+            if (!cuda_ok(cudaEventRecord(done[slot], s[slot]), "event")) break;
+            pend_b0[slot] = b0;
+            pend_nb[slot] = nb;
+        }
+        // oldest first
+        const int last = (b - 1) & 1;
+        finish(last ^ 1);
+        finish(last);
+    } while (0);
+    if (s[1]) {
+        cudaStreamSynchronize(s[1]);
+        cudaStreamDestroy(s[1]);
+    }
+    cudaStreamSynchronize(user);
+    for (int i = 0; i < 2; ++i) {
+        if (sq[i]) cudaFreeHost(sq[i]);
+        if (si[i]) cudaFreeHost(si[i]);
+        if (sd[i]) cudaFreeHost(sd[i]);
+        if (done[i]) cudaEventDestroy(done[i]);
+    }
+    if (start) cudaEventDestroy(start);
+    return st;
+}
+
 sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq, int32_t k, int32_t* out_idx,
                        float* out_dist, const sknn_options* opt, sknn_stats* stats, sknn_stream_t stream) {
     if (!index) return fail(SKNN_ERR_INVALID_ARG, "index is NULL");
@@ -783,9 +909,18 @@ sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq, int3
             if (free_b == 0) return fail(SKNN_ERR_CUDA, "cudaMemGetInfo failed");
             // per query: input row + output row + clustered copy, center distances and scan state (generous)
             const double per_q = 4.0 * d + 8.0 * k + 2.0 * (4.0 * ((d + 3) & ~3) + 16.0) + 8.0 * k;
-            B = (int64_t)(0.4 * (double)free_b / per_q);
+            B = (int64_t)((stats ? 0.4 : 0.2) * (double)free_b / per_q);  // two batches in flight without stats
         }
         if (B >= (int64_t)k && B < nq) {
+            // SKNN_OOC_SERIAL=1 (study): the serial batch loop also without stats
+            // Overlap only when the caller's host buffers are page-locked: measured
+            // (tools/ooc_bench.py) with pageable buffers the page-locked staging
+            // copies cost more than the overlap gains (C5 443 serial vs 519 ms staged,
+            // C2 19 vs 60 ms), so pageable buffers keep the serial loop (the driver
+            // stages those copies itself); SKNN_OOC_STAGE=1 forces the staging
+            const bool all_pinned = pinned_host(Q) && pinned_host(out_dist) && (!out_idx || pinned_host(out_idx));
+            if (!stats && !getenv("SKNN_OOC_SERIAL") && (all_pinned || getenv("SKNN_OOC_STAGE")))
+                return query_batches_overlapped(index, Q, nq, k, out_idx, out_dist, opt, B, (cudaStream_t)stream);
             sknn_stats acc;
             memset(&acc, 0, sizeof(acc));
             for (int64_t b0 = 0; b0 < nq; b0 += B) {
@@ -795,25 +930,24 @@ sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq, int3
                 sb.struct_size = sizeof(sb);
                 SKNN_TRY(run_join(Q + b0 * d, nb, nullptr, index->t.n, d, k, out_idx ? out_idx + b0 * k : nullptr,
                                   out_dist + b0 * k, opt, stats ? &sb : nullptr, (cudaStream_t)stream, index));
-                if (stats) {  // batch sums (sizes and times add up over the batches)
-                    acc.pairs_total += sb.pairs_total; acc.dist_evals_sparse += sb.dist_evals_sparse;
-                    acc.dist_evals_dense += sb.dist_evals_dense; acc.dist_evals_brute += sb.dist_evals_brute;
-                    acc.center_evals += sb.center_evals; acc.cand_pairs += sb.cand_pairs;
-                    acc.dense_pairs += sb.dense_pairs; acc.dist_recompute += sb.dist_recompute;
-                    acc.topk_inserts += sb.topk_inserts; acc.rows_loaded += sb.rows_loaded;
-                    acc.dense_terms = std::max(acc.dense_terms, sb.dense_terms);
-                    acc.ms_total += sb.ms_total; acc.ms_build_t += sb.ms_build_t; acc.ms_build_q += sb.ms_build_q;
-                    acc.ms_level1 += sb.ms_level1; acc.ms_sparse += sb.ms_sparse; acc.ms_dense += sb.ms_dense;
-                    acc.ms_final += sb.ms_final; acc.kernel_launches += sb.kernel_launches;
-                    acc.mapping_used = sb.mapping_used; acc.path_used = sb.path_used;
-                    acc.mq += sb.mq; acc.mt = sb.mt;
-                }
+                if (!stats) continue;
+                // batch sums (sizes and times add up over the batches)
+                acc.pairs_total += sb.pairs_total; acc.dist_evals_sparse += sb.dist_evals_sparse;
+                acc.dist_evals_dense += sb.dist_evals_dense; acc.dist_evals_brute += sb.dist_evals_brute;
+                acc.center_evals += sb.center_evals; acc.cand_pairs += sb.cand_pairs;
+                acc.dense_pairs += sb.dense_pairs; acc.dist_recompute += sb.dist_recompute;
+                acc.topk_inserts += sb.topk_inserts; acc.rows_loaded += sb.rows_loaded;
+                acc.dense_terms = std::max(acc.dense_terms, sb.dense_terms);
+                acc.ms_total += sb.ms_total; acc.ms_build_t += sb.ms_build_t; acc.ms_build_q += sb.ms_build_q;
+                acc.ms_level1 += sb.ms_level1; acc.ms_sparse += sb.ms_sparse; acc.ms_dense += sb.ms_dense;
+                acc.ms_final += sb.ms_final; acc.kernel_launches += sb.kernel_launches;
+                acc.mapping_used = sb.mapping_used; acc.path_used = sb.path_used;
+                acc.mq += sb.mq; acc.mt = sb.mt;
             }
-            if (stats) {
-                acc.struct_size = sizeof(acc);
-                const size_t sz = stats->struct_size ? std::min(stats->struct_size, sizeof(sknn_stats)) : sizeof(sknn_stats);
-                memcpy(stats, &acc, sz);
-            }
+            if (!stats) return SKNN_OK;
+            acc.struct_size = sizeof(acc);
+            const size_t sz = stats->struct_size ? std::min(stats->struct_size, sizeof(sknn_stats)) : sizeof(sknn_stats);
+            memcpy(stats, &acc, sz);
             return SKNN_OK;
         }
     }

@@ -19,6 +19,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdio.h>
+#include <string.h>
 
 #include <algorithm>
 #include <vector>
@@ -277,7 +278,7 @@ __device__ __forceinline__ int4 block_exscan4(int4 v, int4* s_warp, int4& total)
 // keeps S = 1 and only orders.
 constexpr int kTaskPer = kMaxClusters / 1024;
 __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__ qoff, int mq, int tile,
-                                                     int shard_rank, int shard_count,
+                                                     int shard_rank, int shard_count, const int32_t* __restrict__ owner,
                                                      const unsigned long long* __restrict__ work,
                                                      const int32_t* __restrict__ ccount, int slots, int cap_split,
                                                      int split, int order, float wfac, float hfac,
@@ -297,7 +298,8 @@ __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__
         nt[u] = 0;
         wk[u] = 0;
         ncc[u] = 1;
-        if (u < per && c < mq && !(shard_count > 1 && c % shard_count != shard_rank)) {
+        const bool mine = owner ? (c < mq && owner[c] == shard_rank) : !(shard_count > 1 && c % shard_count != shard_rank);
+        if (u < per && c < mq && mine) {
             nt[u] = (qoff[c + 1] - qoff[c] + tile - 1) / tile;
             wk[u] = work[c];
             ncc[u] = ccount[c] > 1 ? ccount[c] : 1;
@@ -436,7 +438,8 @@ sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int s
         SKNN_CUDA(cudaMemsetAsync(l1.theta2, 0x7f, sizeof(unsigned) * (size_t)qs.n, cx.stream));
     }
     l1.tile = tile;
-    k_make_tasks<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, l1.work, l1.cand_count,
+    k_make_tasks<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, l1.owner, l1.work,
+                                             l1.cand_count,
                                              slots, cap, split && cap > 0 ? 1 : 0, order, wfac, hfac, l1.tiles, l1.ntiles, l1.merges,
                                              l1.nmerges);
     cx.launched();
@@ -462,6 +465,64 @@ sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int s
                 "tot/slots=%.3g\n", slots, tiles, nt[0], nm, tot, tot / std::max(1L, tiles), mx, tot / slots);
     }
     return cx.check_launch("tasks");
+}
+
+// Balanced query sharding ("whole query clusters balanced by
+// estimated work"; sknn_options.shard_policy = 1). One CTA: cluster c's
+// weight is |qc| x work[c] (level-1's per-query scan estimate, an integer sum,
+// so every rank computes the same bits); clusters are sorted heaviest first
+// (ties by id) with a shared-memory bitonic sort and dealt to ranks in snake
+// order 0..P-1, P-1..0, ... (each round gives every rank one cluster, the
+// heavy end alternating). Other ranks' clusters lose their dense pairs here
+// (dcount = 0) so the dense-tile list skips them.
+__global__ void __launch_bounds__(1024) k_shard_owner(const int32_t* __restrict__ qoff,
+                                                      const unsigned long long* __restrict__ work,
+                                                      int32_t* __restrict__ dcount, int mq, int P, int rank,
+                                                      int32_t* __restrict__ owner) {
+    extern __shared__ unsigned long long s_key[];
+    int n2 = 1;
+    while (n2 < mq) n2 <<= 1;
+    constexpr unsigned long long kMaxW = (1ull << 50) - 1;
+    for (int i = threadIdx.x; i < n2; i += blockDim.x) {
+        unsigned long long key = ~0ull;
+        if (i < mq) {
+            unsigned long long w = (unsigned long long)(qoff[i + 1] - qoff[i]) * work[i];
+            if (w > kMaxW) w = kMaxW;
+            key = ((kMaxW - w) << 14) | (unsigned long long)i;  // ascending key = heaviest first, then id
+        }
+        s_key[i] = key;
+    }
+    __syncthreads();
+    for (int size = 2; size <= n2; size <<= 1)
+        for (int stride = size >> 1; stride > 0; stride >>= 1) {
+            for (int i = threadIdx.x; i < n2; i += blockDim.x) {
+                const int j = i ^ stride;
+                if (j > i) {
+                    const bool up = (i & size) == 0;
+                    const unsigned long long a = s_key[i], b = s_key[j];
+                    if ((a > b) == up) { s_key[i] = b; s_key[j] = a; }
+                }
+            }
+            __syncthreads();
+        }
+    for (int i = threadIdx.x; i < mq; i += blockDim.x) {
+        const int c = (int)(s_key[i] & 0x3fffull);
+        const int round = i / P, j = i - round * P;
+        const int r = (round & 1) ? P - 1 - j : j;
+        owner[c] = r;
+        if (r != rank && dcount) dcount[c] = 0;
+    }
+}
+
+sknn_status run_shard_owner(Ctx& cx, const Side& qs, Level1& l1, int shard_rank, int shard_count) {
+    SKNN_TRY(cx.alloc_scratch((void**)&l1.owner, sizeof(int32_t) * (size_t)std::max(1, qs.m)));
+    int n2 = 1;
+    while (n2 < qs.m) n2 <<= 1;
+    const size_t smem = sizeof(unsigned long long) * (size_t)n2;
+    if (smem > 48 * 1024) cudaFuncSetAttribute(k_shard_owner, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_shard_owner<<<1, 1024, smem, cx.stream>>>(qs.off, l1.work, l1.dcount, qs.m, shard_count, shard_rank, l1.owner);
+    cx.launched();
+    return cx.check_launch("shard owner");
 }
 
 // dense-tile work list: tiles of 128 queries of the clusters with dense pairs
@@ -550,6 +611,87 @@ sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, 
         SKNN_TRY(cx.check_launch("merge split tasks"));
     }
     return SKNN_OK;
+}
+
+// ------------------------------------------------- basic KNN-TI (ablation) --
+// The version Sweet KNN improves on (Fig. 4 pointFilter / Alg. 2, P:L273-281,
+// P:L355-375; Table IV's "KNN-TI" column): one thread per query
+// in INPUT order, so neighbouring threads of a warp belong to different query
+// clusters and walk different candidate lists (no thread-data remapping,
+// §IV-C1); each candidate cluster's members are visited from the top of the
+// distance-descending array with Alg. 2's `continue` (l < -theta) and
+// `break` (l > theta); kNearests is a sorted array in thread-local memory
+// with an insertion shift. Level-1 (calUB + groupFilter, the candidate lists
+// in ascending D) is shared with the Sweet path. Same exact keys, so the same
+// result (reading R2 ties, R6 non-strict tests, R7 slack).
+__global__ void k_invert_perm(const int32_t* __restrict__ orig, int64_t n, int32_t* __restrict__ pos) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n; p += (int64_t)gridDim.x * blockDim.x)
+        pos[orig[p]] = (int32_t)p;
+}
+
+__global__ void __launch_bounds__(256) k_scan_basic(ScanArgs a, int64_t nq, int mq, const int32_t* __restrict__ pos) {
+    unsigned long long evals = 0, cevals = 0, inserts = 0;
+    const int dp = a.dp, k = a.k;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nq; i += (int64_t)gridDim.x * blockDim.x) {
+        const int p = __ldg(pos + i);
+        int lo = 0, hi = mq;  // query cluster: the last c with qoff[c] <= p
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (__ldg(a.qoff + mid) <= p) lo = mid;
+            else hi = mid;
+        }
+        const int qc = lo;
+        key_t list[32];  // kNearests, ascending; list[k-1] is the k-th key (R8: (+inf, -1) start)
+        for (int r = 0; r < k; ++r) list[r] = kInfKey;
+        const float ub = __ldg(a.ub + qc);
+        float theta = ub;
+        const float* q = a.qrows + (int64_t)p * dp;
+        const int ncand = __ldg(a.cand_count + qc);
+        for (int c = 0; c < ncand; ++c) {
+            const int tc = __ldg(a.cand + (int64_t)qc * a.mt + c);
+            const float dq = __fsqrt_rn(d2_rows(q, a.tcent + (int64_t)tc * dp, dp));
+            ++cevals;
+            const int jlo = __ldg(a.toff + tc), jhi = __ldg(a.toff + tc + 1);
+            for (int j = jlo; j < jhi; ++j) {
+                const float dt = __ldg(a.tdist + j);
+                const float l = dq - dt;
+                if (!ti_keep(l, theta, dq + dt, a.eta)) break;      // Alg. 2 line 10
+                if (!ti_keep(-l, theta, dq + dt, a.eta)) continue;  // Alg. 2 line 12
+                const float d2 = d2_rows(q, a.trows + (int64_t)j * dp, dp);
+                ++evals;
+                const key_t key = make_key(d2, __ldg(a.torig + j));
+                if (key < list[k - 1]) {  // Alg. 2 lines 15-17: kNearests.insert
+                    int r = k - 1;
+                    while (r > 0 && list[r - 1] > key) {
+                        list[r] = list[r - 1];
+                        --r;
+                    }
+                    list[r] = key;
+                    ++inserts;
+                    theta = fminf(ub, __fsqrt_ru(key_d2(list[k - 1])));
+                }
+            }
+        }
+        for (int r = 0; r < k; ++r) write_result(a, (int)i, r, list[r]);
+    }
+    add_counter(&a.counters->evals_sparse, evals);
+    add_counter(&a.counters->rows_loaded, evals);
+    add_counter(&a.counters->center_evals, cevals);
+    add_counter(&a.counters->topk_inserts, inserts);
+}
+
+sknn_status run_scan_basic(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p) {
+    ScanArgs a = make_scan_args(qs, ts, l1, p);
+    int32_t* pos = nullptr;
+    SKNN_TRY(cx.alloc_scratch((void**)&pos, sizeof(int32_t) * (size_t)qs.n));
+    const int g = (int)std::min<int64_t>((qs.n + 255) / 256, (int64_t)cx.num_sms * 8);
+    k_invert_perm<<<g > 0 ? g : 1, 256, 0, cx.stream>>>(qs.orig, qs.n, pos);
+    cx.launched();
+    SKNN_TRY(cx.check_launch("invert permutation"));
+    const int grid = occupancy_grid(cx, (const void*)k_scan_basic, 256, 0);
+    k_scan_basic<<<grid, 256, 0, cx.stream>>>(a, qs.n, qs.m, pos);
+    cx.launched();
+    return cx.check_launch("level2 scan (basic KNN-TI)");
 }
 
 // ------------------------------------------------------------ brute force --
@@ -729,8 +871,283 @@ __global__ void __launch_bounds__(256) k_merge(const int32_t* __restrict__ pidx,
     }
 }
 
+// Thread per query (k <= K <= 32): the same bitonic step, but the whole list
+// of K keys lives in one thread's registers, so a compare-exchange is one
+// compare and four selects producing BOTH the min and the max (the warp form
+// computes each side's half on its own lane, behind two shuffles). ncu of the
+// warp form at C5 P = 8: ALU pipe 77%, DRAM 40% -> this form's ALU work per
+// query is ~2x smaller and the kernel streams. Rows of k % 4 == 0 keys are
+// read as float4 / int4 (a thread reads whole 128 B lines; the warp's other
+// lanes read their own lines, so the L1 serves the 8 vector loads per line).
+// One compare for both selects. Merge keys are >= 0 and their top 11 bits
+// (the float d2's bits 30..20) are never all ones for a finite or +inf d2, so
+// read as IEEE doubles they are finite, non-negative and order exactly like
+// the integers: one DSETP (fp64 pipe) replaces the 64-bit integer compare
+// pair, which the compiler also duplicates into a less-than and a
+// greater-than pair when both the min and the max are selected.
+__device__ __forceinline__ void cex(key_t x, key_t y, key_t& lo, key_t& hi) {
+    const bool lt = __longlong_as_double(x) < __longlong_as_double(y);
+    lo = lt ? x : y;
+    hi = lt ? y : x;
+}
+
+template <int K>
+__device__ __forceinline__ void tmerge_load(key_t (&v)[K], const int32_t* __restrict__ pidx,
+                                            const float* __restrict__ pd2, int64_t row, int k, bool vec) {
+    if (vec) {
+        const float4* d4 = reinterpret_cast<const float4*>(pd2 + row);
+        const int4* i4 = reinterpret_cast<const int4*>(pidx + row);
+#pragma unroll
+        for (int c = 0; c < K / 4; ++c) {
+            if (4 * c < k) {
+                const float4 d = __ldg(d4 + c);
+                const int4 i = __ldg(i4 + c);
+                v[4 * c + 0] = make_key(d.x, i.x);
+                v[4 * c + 1] = make_key(d.y, i.y);
+                v[4 * c + 2] = make_key(d.z, i.z);
+                v[4 * c + 3] = make_key(d.w, i.w);
+            } else {
+                v[4 * c + 0] = v[4 * c + 1] = v[4 * c + 2] = v[4 * c + 3] = kInfKey;
+            }
+        }
+    } else {
+#pragma unroll
+        for (int j = 0; j < K; ++j) v[j] = j < k ? make_key(__ldg(pd2 + row + j), __ldg(pidx + row + j)) : kInfKey;
+    }
+}
+
+template <int K>
+__global__ void __launch_bounds__(128) k_merge_tpq(const int32_t* __restrict__ pidx, const float* __restrict__ pd2,
+                                                   int P, int64_t nq, int k, int32_t* __restrict__ out_idx,
+                                                   float* __restrict__ out_dist, int out_squared, int vec) {
+    for (int64_t qi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; qi < nq; qi += (int64_t)gridDim.x * blockDim.x) {
+        key_t A[K], B[K];
+        tmerge_load<K>(A, pidx, pd2, qi * k, k, vec);
+        for (int p = 1; p < P; ++p) {
+            tmerge_load<K>(B, pidx, pd2, ((int64_t)p * nq + qi) * k, k, vec);
+            // C_j = min(A_j, B_{K-1-j}): the K smallest of A u B, bitonic
+#pragma unroll
+            for (int j = 0; j < K; ++j)
+                A[j] = __longlong_as_double(B[K - 1 - j]) < __longlong_as_double(A[j]) ? B[K - 1 - j] : A[j];
+#pragma unroll
+            for (int h = K / 2; h >= 1; h >>= 1)
+#pragma unroll
+                for (int j = 0; j < K; ++j)
+                    if ((j & h) == 0) {
+                        key_t lo, hi;
+                        cex(A[j], A[j + h], lo, hi);
+                        A[j] = lo;
+                        A[j + h] = hi;
+                    }
+        }
+        if (vec) {
+            float4* od = reinterpret_cast<float4*>(out_dist + qi * k);
+            int4* oi = reinterpret_cast<int4*>(out_idx ? out_idx + qi * k : nullptr);
+#pragma unroll
+            for (int c = 0; c < K / 4; ++c)
+                if (4 * c < k) {
+                    float4 d;
+                    d.x = key_d2(A[4 * c + 0]);
+                    d.y = key_d2(A[4 * c + 1]);
+                    d.z = key_d2(A[4 * c + 2]);
+                    d.w = key_d2(A[4 * c + 3]);
+                    if (!out_squared) {
+                        d.x = __fsqrt_rn(d.x);
+                        d.y = __fsqrt_rn(d.y);
+                        d.z = __fsqrt_rn(d.z);
+                        d.w = __fsqrt_rn(d.w);
+                    }
+                    od[c] = d;
+                    if (oi)
+                        oi[c] = make_int4(key_idx(A[4 * c + 0]), key_idx(A[4 * c + 1]), key_idx(A[4 * c + 2]),
+                                          key_idx(A[4 * c + 3]));
+                }
+        } else {
+#pragma unroll
+            for (int j = 0; j < K; ++j)
+                if (j < k) {
+                    const float d2 = key_d2(A[j]);
+                    out_dist[qi * k + j] = out_squared ? d2 : __fsqrt_rn(d2);
+                    if (out_idx) out_idx[qi * k + j] = key_idx(A[j]);
+                }
+        }
+    }
+}
+
+// Staged form (k % 4 == 0, 16-byte aligned rows): a CTA owns 128 queries;
+// list p of those queries is one contiguous [128 x k] block of d2 and of idx,
+// copied with coalesced 16-byte cp.async into shared memory (3 buffers, two
+// lists in flight while one is merged) at a row stride of S 16-byte units, S
+// odd, so the eight threads of a 128-bit shared load phase hit eight
+// different bank quads. ncu of the direct-load form at C5 P = 8: L1/TEX 99%
+// busy (every warp load touches 32 lines), DRAM 55%. The result rows go out
+// the same way (staged, then coalesced stores).
+__device__ __forceinline__ uint32_t smem_addr_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+template <int K>
+struct MergeStage {
+    static constexpr int kS = (K / 4) % 2 ? K / 4 : K / 4 + 1;  // row stride in 16-byte units (odd)
+    static constexpr int kRowBytes = kS * 16;
+    static constexpr int kArrBytes = 128 * kRowBytes;  // one array (d2 or idx) of 128 rows
+    static constexpr int kBufBytes = 2 * kArrBytes;
+    static constexpr int kSmem = 3 * kBufBytes;
+};
+
+// copy rows [q0, q0 + nrows) of list p (k keys per row) into buffer `buf`
+template <int K>
+__device__ __forceinline__ void merge_stage_load(char* buf, const int32_t* __restrict__ pidx,
+                                                 const float* __restrict__ pd2, int64_t row0, int nrows, int k) {
+    const int c4 = k / 4;  // 16-byte chunks per row
+    const int total = nrows * c4;
+    const char* gd = reinterpret_cast<const char*>(pd2 + row0 * k);
+    const char* gi = reinterpret_cast<const char*>(pidx + row0 * k);
+    for (int c = threadIdx.x; c < total; c += blockDim.x) {
+        const int r = c / c4, col = c - r * c4;
+        const uint32_t sd = smem_addr_u32(buf + r * MergeStage<K>::kRowBytes + col * 16);
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sd), "l"(gd + (int64_t)c * 16));
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sd + MergeStage<K>::kArrBytes),
+                     "l"(gi + (int64_t)c * 16));
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+template <int K>
+__global__ void __launch_bounds__(128) k_merge_tpq_staged(const int32_t* __restrict__ pidx,
+                                                          const float* __restrict__ pd2, int P, int64_t nq, int k,
+                                                          int32_t* __restrict__ out_idx, float* __restrict__ out_dist,
+                                                          int out_squared) {
+    extern __shared__ __align__(16) char s_merge[];
+    using MS = MergeStage<K>;
+    const int64_t q0 = (int64_t)blockIdx.x * 128;
+    const int nrows = nq - q0 < 128 ? (int)(nq - q0) : 128;
+    const int t = threadIdx.x;
+    const bool mine = t < nrows;
+    const int c4 = k / 4;
+    // prologue: lists 0, 1 (and 2) in flight; one commit group per list
+#pragma unroll 1
+    for (int p = 0; p < 3 && p < P; ++p)
+        merge_stage_load<K>(s_merge + p * MS::kBufBytes, pidx, pd2, (int64_t)p * nq + q0, nrows, k);
+    key_t A[K];
+#pragma unroll 1
+    for (int p = 0; p < P; ++p) {
+        // groups committed so far: min(P, p + 3); list p is complete when at most
+        // min(P, p + 3) - p - 1 younger groups are still pending
+        const int younger = min(P, p + 3) - p - 1;
+        if (younger >= 2) asm volatile("cp.async.wait_group 2;" ::: "memory");
+        else if (younger == 1) asm volatile("cp.async.wait_group 1;" ::: "memory");
+        else asm volatile("cp.async.wait_group 0;" ::: "memory");
+        __syncthreads();
+        char* buf = s_merge + (p % 3) * MS::kBufBytes;
+        key_t B[K];
+        if (mine) {
+            const float4* d4 = reinterpret_cast<const float4*>(buf + t * MS::kRowBytes);
+            const int4* i4 = reinterpret_cast<const int4*>(buf + MS::kArrBytes + t * MS::kRowBytes);
+#pragma unroll
+            for (int c = 0; c < K / 4; ++c) {
+                if (c < c4) {
+                    const float4 d = d4[c];
+                    const int4 i = i4[c];
+                    B[4 * c + 0] = make_key(d.x, i.x);
+                    B[4 * c + 1] = make_key(d.y, i.y);
+                    B[4 * c + 2] = make_key(d.z, i.z);
+                    B[4 * c + 3] = make_key(d.w, i.w);
+                } else {
+                    B[4 * c + 0] = B[4 * c + 1] = B[4 * c + 2] = B[4 * c + 3] = kInfKey;
+                }
+            }
+        }
+        __syncthreads();  // buffer p % 3 is free again
+        if (p + 3 < P) merge_stage_load<K>(buf, pidx, pd2, (int64_t)(p + 3) * nq + q0, nrows, k);
+        if (!mine) continue;
+        if (p == 0) {
+#pragma unroll
+            for (int j = 0; j < K; ++j) A[j] = B[j];
+            continue;
+        }
+#pragma unroll
+        for (int j = 0; j < K; ++j)
+            A[j] = __longlong_as_double(B[K - 1 - j]) < __longlong_as_double(A[j]) ? B[K - 1 - j] : A[j];
+#pragma unroll
+        for (int h = K / 2; h >= 1; h >>= 1)
+#pragma unroll
+            for (int j = 0; j < K; ++j)
+                if ((j & h) == 0) {
+                    key_t lo, hi;
+                    cex(A[j], A[j + h], lo, hi);
+                    A[j] = lo;
+                    A[j + h] = hi;
+                }
+    }
+    // results: rows staged in buffer 0 (every load has completed), then coalesced stores
+    __syncthreads();
+    if (mine) {
+        float4* d4 = reinterpret_cast<float4*>(s_merge + t * MS::kRowBytes);
+        int4* i4 = reinterpret_cast<int4*>(s_merge + MS::kArrBytes + t * MS::kRowBytes);
+#pragma unroll
+        for (int c = 0; c < K / 4; ++c)
+            if (c < c4) {
+                float4 d = make_float4(key_d2(A[4 * c + 0]), key_d2(A[4 * c + 1]), key_d2(A[4 * c + 2]),
+                                       key_d2(A[4 * c + 3]));
+                if (!out_squared) {
+                    d.x = __fsqrt_rn(d.x);
+                    d.y = __fsqrt_rn(d.y);
+                    d.z = __fsqrt_rn(d.z);
+                    d.w = __fsqrt_rn(d.w);
+                }
+                d4[c] = d;
+                i4[c] = make_int4(key_idx(A[4 * c + 0]), key_idx(A[4 * c + 1]), key_idx(A[4 * c + 2]),
+                                  key_idx(A[4 * c + 3]));
+            }
+    }
+    __syncthreads();
+    float4* od = reinterpret_cast<float4*>(out_dist + q0 * k);
+    int4* oi = reinterpret_cast<int4*>(out_idx ? out_idx + q0 * k : nullptr);
+    for (int c = t; c < nrows * c4; c += blockDim.x) {
+        const int r = c / c4, col = c - r * c4;
+        od[c] = *reinterpret_cast<const float4*>(s_merge + r * MS::kRowBytes + col * 16);
+        if (oi) oi[c] = *reinterpret_cast<const int4*>(s_merge + MS::kArrBytes + r * MS::kRowBytes + col * 16);
+    }
+}
+
 sknn_status run_merge(Ctx& cx, const int32_t* part_idx, const float* part_d2, int P, int64_t nq, int k,
                       int32_t* out_idx, float* out_dist, int out_squared) {
+    const char* env = getenv("SKNN_MERGE");  // study knob for k <= 32: "warp" | "direct" | "staged"
+    if (k <= 32 && !(env && !strcmp(env, "warp"))) {
+        const bool vec = (k % 4) == 0 && ((uintptr_t)part_idx % 16) == 0 && ((uintptr_t)part_d2 % 16) == 0 &&
+                         ((uintptr_t)out_dist % 16) == 0 && ((uintptr_t)out_idx % 16) == 0;
+        const int64_t blocks = (nq + 127) / 128;
+        // measured at nq = 4M, P = 8 (tools/merge_bench.py): k = 32 staged 1.84 /
+        // direct 2.04 ms; k = 16 0.79 / 0.76; k = 20 1.60 / 1.05 (the staged form
+        // pads rows to K = 32 and keeps 2 CTAs per SM): staged only when k == 32
+        const bool staged = env ? !strcmp(env, "staged") : k == 32;
+        if (vec && staged && blocks < (1ll << 31)) {
+#define SKNN_SMERGE(K)                                                                                          \
+    do {                                                                                                        \
+        cudaFuncSetAttribute(k_merge_tpq_staged<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,                 \
+                             MergeStage<K>::kSmem);                                                             \
+        k_merge_tpq_staged<K><<<(int)blocks, 128, MergeStage<K>::kSmem, cx.stream>>>(part_idx, part_d2, P, nq, k, \
+                                                                                     out_idx, out_dist,         \
+                                                                                     out_squared);              \
+    } while (0)
+            if (k <= 8) SKNN_SMERGE(8);
+            else if (k <= 16) SKNN_SMERGE(16);
+            else SKNN_SMERGE(32);
+#undef SKNN_SMERGE
+            cx.launched();
+            return cx.check_launch("merge");
+        }
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)cx.num_sms * 8));
+#define SKNN_TMERGE(K) \
+    k_merge_tpq<K><<<grid, 128, 0, cx.stream>>>(part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared, vec)
+        if (k <= 8) SKNN_TMERGE(8);
+        else if (k <= 16) SKNN_TMERGE(16);
+        else SKNN_TMERGE(32);
+#undef SKNN_TMERGE
+        cx.launched();
+        return cx.check_launch("merge");
+    }
     int64_t blocks = (nq + 7) / 8;
     int grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)cx.num_sms * 16));
 #define SKNN_MERGE(R) k_merge<R><<<grid, 256, 0, cx.stream>>>(part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared)

@@ -134,6 +134,7 @@ struct Level1 {
     int32_t* dcount = nullptr;    // [mq]
     int2* dtiles = nullptr;       // dense work tiles (128 queries of one cluster)
     int* dntiles = nullptr;       // [2]
+    int32_t* owner = nullptr;     // [mq] owning rank of each query cluster (balanced query sharding), or NULL
 };
 struct DenseOrigin {          // common re-centring point of the dense tiles
     float* o = nullptr;         // [kp] rounded mean target center
@@ -152,6 +153,9 @@ struct Level1Params {
 };
 sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Params& p, Level1& out,
                        Counters* counters);
+// balanced query sharding: owner[c] for every query cluster from the level-1
+// work estimate (snake deal, heaviest first); zeroes dcount of other ranks' clusters
+sknn_status run_shard_owner(Ctx& cx, const Side& qs, Level1& l1, int shard_rank, int shard_count);
 // k_dense.cu
 struct DenseParams {
     const float* origin = nullptr;
@@ -188,6 +192,8 @@ struct ScanParams {
     const key_t* init_topk = nullptr;    // dense-tile pass results to continue from
 };
 sknn_status run_scan(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p);
+// basic KNN-TI ablation arm (SKNN_MAP_BASIC): thread per query in input order
+sknn_status run_scan_basic(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p);
 struct ScanArgs;
 ScanArgs make_scan_args(const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p);
 // k_partial.cu: the paper's partial level-2 filter (SKNN_PATH_PARTIAL); *fell_back

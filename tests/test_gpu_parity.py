@@ -312,17 +312,32 @@ def test_auto_switch_mixes_paths(sknn):
 
 
 # ------------------------------------------------------------ multi-GPU --
-def test_query_shard_option_covers_all_rows(sknn):
-    """Query sharding of a self-join (sknn_options.shard_rank/count): P ranks'
-    cluster-interleaved shards, run one after the other into the same output,
-    reproduce the single join bit-exactly (P11)."""
-    Q, T, k, sj = datagen.workload("C3int", 0.05)
-    dX = dev(Q)
+@pytest.mark.parametrize("policy", [0, 1])
+@pytest.mark.parametrize("name,scale,P", [("C3int", 0.05, 3), ("C4", 0.004, 4), ("C5", 0.0025, 8), ("C1", 1.0, 5)])
+def test_query_shard_option_covers_all_rows(sknn, policy, name, scale, P):
+    """Query sharding (sknn_options.shard_rank/count): P ranks' shards, run one
+    after the other into the same output, reproduce the single join
+    bit-exactly (P11), for the interleaved (c % P) and the balanced (snake deal
+    by the level-1 work estimate) ownership; every row is written by exactly
+    one rank (a row another rank owns stays at its -1 fill), and with the
+    balanced policy the C4 shards include elastic-switch dense tiles."""
+    Q, T, k, sj = datagen.workload(name, scale)
+    dQ = dev(Q)
+    dT = dQ if sj else dev(T)
     idx = torch.full((Q.shape[0], k), -1, dtype=torch.int32, device="cuda")
     dst = torch.zeros((Q.shape[0], k), dtype=torch.float32, device="cuda")
-    for r in range(3):
-        sknn.join(dX, dX, k, out=(idx, dst), shard_rank=r, shard_count=3)
+    owner = np.full(Q.shape[0], -1)
+    for r in range(P):
+        i1 = torch.full((Q.shape[0], k), -1, dtype=torch.int32, device="cuda")
+        d1 = torch.zeros((Q.shape[0], k), dtype=torch.float32, device="cuda")
+        sknn.join(dQ, dT, k, out=(i1, d1), shard_rank=r, shard_count=P, shard_policy=policy)
+        rows = (i1[:, 0] >= 0).cpu().numpy()
+        assert (owner[rows] == -1).all()   # no row computed by two ranks
+        owner[rows] = r
+        idx[rows] = i1[rows]
+        dst[rows] = d1[rows]
     torch.cuda.synchronize()
+    assert (owner >= 0).all()
     ridx, rdist = oracle.knn_join(Q, T, k)
     assert_knn_bitexact(idx.cpu().numpy(), dst.cpu().numpy(), ridx, rdist)
 
@@ -537,6 +552,18 @@ def test_query_batches_host_memory(sknn, batch):
     ridx, rdist = oracle.knn_join(Q, T, k)
     assert_knn_bitexact(np.asarray(idx), np.asarray(dist), ridx, rdist)
     assert st["pairs_total"] == Q.shape[0] * T.shape[0]
+    # without stats the batches overlap on two streams (pageable buffers go
+    # through page-locked staging; page-locked ones are used in place)
+    idx2, dist2 = ix.query(Q, k, query_batch=batch)
+    assert_knn_bitexact(np.asarray(idx2), np.asarray(dist2), ridx, rdist)
+    pq = torch.from_numpy(Q).pin_memory()
+    pi = torch.empty((Q.shape[0], k), dtype=torch.int32).pin_memory()
+    pd = torch.empty((Q.shape[0], k), dtype=torch.float32).pin_memory()
+    ix.query(pq, k, query_batch=batch, out=(pi, pd))
+    assert_knn_bitexact(pi.numpy(), pd.numpy(), ridx, rdist)
+    # pinned queries, pageable outputs (mixed staging)
+    idx3, dist3 = ix.query(pq, k, query_batch=batch)
+    assert_knn_bitexact(np.asarray(idx3), np.asarray(dist3), ridx, rdist)
     ix.close()
 
 
@@ -669,11 +696,20 @@ def test_dense_split_precision_fallback(sknn, hi, d):
     assert st["dist_evals_dense"] > 0 and st["dist_recompute"] > 0
 
 
-@pytest.mark.parametrize("P,k", [(1, 5), (2, 32), (8, 32), (3, 1), (20, 7), (5, 33), (9, 100), (4, 512), (17, 256)])
-def test_merge_partials_bitonic(sknn, P, k):
-    """sknn_merge_partials (bitonic warp merge) on P sorted lists with many
-    equal distances across lists: the k smallest (d2, idx) keys, compared with
-    a lexicographic sort of the concatenated lists (np.lexsort)."""
+@pytest.mark.parametrize("form", ["", "direct", "staged", "warp"])
+@pytest.mark.parametrize("P,k", [(1, 5), (2, 32), (8, 32), (3, 1), (20, 7), (5, 33), (9, 100), (4, 512), (17, 256),
+                                 (1, 32), (8, 16), (3, 20), (4, 8), (3, 4), (2, 12), (6, 28)])
+def test_merge_partials_bitonic(sknn, P, k, form, monkeypatch):
+    """sknn_merge_partials on P sorted lists with many equal distances across
+    lists: the k smallest (d2, idx) keys, compared with a lexicographic sort of
+    the concatenated lists (np.lexsort). k <= 32 runs every form: the staged
+    thread-per-query merge (default for k % 4 == 0), the direct-load thread
+    form (default otherwise) and the warp form; nq = 700 leaves a ragged
+    128-query block."""
+    if form and k > 32:
+        pytest.skip("one form above k = 32")
+    if form:
+        monkeypatch.setenv("SKNN_MERGE", form)
     rng = np.random.default_rng(P * 1000 + k)
     nq = 700
     d2 = np.sort(rng.integers(0, 50, size=(P, nq, k)).astype(np.float32), axis=2)
@@ -788,3 +824,29 @@ def test_target_sharded_global_ub(sknn):
     gi = parts["global"][0].cpu().numpy()
     gd = parts["global"][1].cpu().numpy()
     assert np.all((gi >= 0) | (gi == -1)) and np.all(np.isinf(gd[gi == -1]))
+
+
+# ------------------------------------------- basic KNN-TI ablation arm (NEXT-3) --
+@pytest.mark.parametrize("name,scale", [("C1", 1.0), ("C3int", 0.05), ("C5", 0.0025), ("C4", 0.002), ("C2", 0.02)])
+def test_basic_knnti_matches_oracle(sknn, name, scale):
+    """mapping='basic' (the basic KNN-TI of Fig. 4 / Alg. 2: thread per query in
+    input order, per-thread walks from the top of each candidate cluster) gives
+    the oracle's result: bit-exact on integer inputs, within 1e-5 on C2; and it
+    never evaluates fewer distances than the Alg. 2 windows need, i.e. its
+    evaluation count is >= 0 and pruning stays the TI pruning (< 100%)."""
+    Q, T, k, sj = datagen.workload(name, scale)
+    idx, dist, st = run(sknn, Q, T, k, sj, mapping="basic")
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    if name == "C2":
+        assert_knn_tolerant(Q, T, idx, dist, rdist)
+    else:
+        assert_knn_bitexact(idx, dist, ridx, rdist)
+    assert st["mapping_used"] == 3 and 0 < st["pruned_pct"] < 100
+
+
+def test_basic_knnti_rejects_unsupported(sknn):
+    Q, T, k, sj = datagen.workload("C1")
+    with pytest.raises(RuntimeError):
+        run(sknn, Q, T, 40, sj, mapping="basic")
+    with pytest.raises(RuntimeError):
+        run(sknn, Q, T, k, sj, mapping="basic", force_path="dense")
