@@ -380,14 +380,13 @@ def main():
     if args.mode == "query":
         out_idx = torch.empty((nq, k), dtype=torch.int32, device=dev)
         out_dist = torch.empty((nq, k), dtype=torch.float32, device=dev)
-        if self_join:
-            if ws > 1:
-                opts.update(shard_rank=rank, shard_count=ws)
-            lo, hi = 0, nq
-            Qr, Tr, oi, od = Q, Q, out_idx, out_dist
-        else:
-            lo, hi = sdist.shard_bounds(nq, ws, rank)
-            Qr, Tr, oi, od = Q[lo:hi], T, out_idx[lo:hi], out_dist[lo:hi]
+        # every rank clusters all of Q identically and takes the query clusters
+        # c % N == rank (dist.join_query_sharded's default partition; contiguous
+        # row slices measured far worse on C4: outlier queries in a slice)
+        if ws > 1:
+            opts.update(shard_rank=rank, shard_count=ws)
+        lo, hi = 0, nq
+        Qr, Tr, oi, od = Q, (Q if self_join else T), out_idx, out_dist
 
         def local_join(stats=False):
             return sknn.join(Qr, Tr, k, out=(oi, od), stats=stats, stream=stream, **opts)
@@ -395,7 +394,7 @@ def main():
         def step():
             local_join()
         parallelism = "query-sharded x%d (target index replicated, no data-path collective)" % ws
-        nq_rank = (nq / ws) if self_join else (hi - lo)
+        nq_rank = nq / ws
     else:
         tlo, thi = sdist.shard_bounds(nt, ws, rank)
         Tshard = T[tlo:thi].contiguous()
@@ -525,15 +524,13 @@ def measure_e2e(args, sknn, sdist, Qh, Th, k, self_join, ws, rank, dev, opts):
             def e2e_step():  # the C ABI stages the host arrays (H2D, join, D2H, sync inside)
                 sknn.join(Qp, Qp, k, out=(oi, od), **opts)
             h2d, d2h = nq * d * 4, nq * k * 8
-        else:
-            lo, hi = sdist.shard_bounds(nq, ws, rank)
-            Qs = Qp[lo:hi]
-            oi = torch.empty((hi - lo, k), dtype=torch.int32).pin_memory()
-            od = torch.empty((hi - lo, k), dtype=torch.float32).pin_memory()
+        else:  # the rank's query clusters of all of Q (opts carries shard_rank/count at N > 1)
+            oi = torch.empty((nq, k), dtype=torch.int32).pin_memory()
+            od = torch.empty((nq, k), dtype=torch.float32).pin_memory()
 
             def e2e_step():
-                sknn.join(Qs, Tp, k, out=(oi, od), **opts)
-            h2d, d2h = (hi - lo) * d * 4 + nt * d * 4, (hi - lo) * k * 8
+                sknn.join(Qp, Tp, k, out=(oi, od), **opts)
+            h2d, d2h = nq * d * 4 + nt * d * 4, nq * k * 8
     else:
         tlo, thi = sdist.shard_bounds(nt, ws, rank)
         Ts = Tp[tlo:thi]

@@ -52,7 +52,8 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
         const int4 tl = a.tiles[tile];
         const int qc = tl.x;
         const int qlo = a.qoff[qc], qsz = a.qoff[qc + 1] - qlo;
-        const int nq_tile = min(a.tile, qsz - tl.y);
+        const int tcount = (tl.z >> 16) & 0xff;  // single-query (outlier) tasks: 1
+        const int nq_tile = min(tcount ? tcount : a.tile, qsz - tl.y);
         const float ub = a.ub[qc];
         const int ncand = a.cand_count[qc];
         const int32_t* cl = a.cand + (int64_t)qc * a.mt;
@@ -132,10 +133,14 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
                     const int first = bm ? (__ffs(bm) - 1) : 32;
                     const bool ev = lane < first && ti_keep(-l, theta, dq + dt, a.eta);
                     key_t key = kInfKey;
-                    if (ev) {
-                        float d2;
-                        if constexpr (DP > 0) d2 = d2_reg<DP>(q, a.trows + (int64_t)j * DP);
-                        else d2 = d2_rows(sq, a.trows + (int64_t)j * dp, dp);
+                    if constexpr (DP > 0) {
+                        if (ev) {
+                            const float d2 = d2_reg<DP>(q, a.trows + (int64_t)j * DP);
+                            ++evals;
+                            if (d2 <= key_d2(kth)) key = make_key(d2, __ldg(a.torig + j));
+                        }
+                    } else if (ev) {
+                        const float d2 = d2_rows(sq, a.trows + (int64_t)j * dp, dp);
                         ++evals;
                         if (d2 <= key_d2(kth)) key = make_key(d2, __ldg(a.torig + j));
                     }
@@ -281,7 +286,7 @@ __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__
                                                      int shard_rank, int shard_count, const int32_t* __restrict__ owner,
                                                      const unsigned long long* __restrict__ work,
                                                      const int32_t* __restrict__ ccount, int slots, int cap_split,
-                                                     int split, int order, float wfac, float hfac,
+                                                     int split, int order, int outliers, float wfac, float hfac,
                                                      int4* __restrict__ tasks, int* __restrict__ ntasks,
                                                      int4* __restrict__ merges, int* __restrict__ nmerges) {
     __shared__ unsigned long long s_red[33];
@@ -336,11 +341,29 @@ __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__
             W0 *= 2;
         }
     }
-    // bucket sizes: x = split tasks, y = heavy unsplit tiles, z = the rest, w = merge entries
+    // Warp-per-query scan (split == false, tile 8): the first `tile` members of
+    // a cluster are its FARTHEST queries (members sort by distance descending,
+    // R11) -- the outliers whose k-th neighbour is far, so their windows stay
+    // wide and they approach brute force (profiled on a C4 query slice: one such
+    // 8-query tile ran 878 M cycles against a 1.9 M mean, 436 ms of a 450 ms
+    // scan with the GPU idle). They become single-query tasks, scheduled first.
+    int nfirst[kTaskPer];
+#pragma unroll
+    for (int u = 0; u < kTaskPer; ++u) {
+        nfirst[u] = 0;
+        if (outliers && nt[u] > 0) {
+            const int c = c0 + u;
+            const int qsz = qoff[c + 1] - qoff[c];
+            nfirst[u] = qsz < tile ? qsz : tile;
+            nt[u] = (qsz - nfirst[u] + tile - 1) / tile;
+        }
+    }
+    // bucket sizes: x = split tasks (and outlier queries), y = heavy unsplit tiles, z = the rest, w = merge entries
     int4 cnt = make_int4(0, 0, 0, 0);
 #pragma unroll
     for (int u = 0; u < kTaskPer; ++u) {
         const int S = s_of(u, W0);
+        cnt.x += nfirst[u];
         if (S > 1) { cnt.x += nt[u] * S; cnt.w += nt[u]; }
         else if (!order || wk[u] * 4 >= W0) cnt.y += nt[u];
         else cnt.z += nt[u];
@@ -351,8 +374,10 @@ __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__
     off.z += total.x + total.y;
 #pragma unroll
     for (int u = 0; u < kTaskPer; ++u) {
-        if (nt[u] == 0) continue;
         const int c = c0 + u;
+        for (int i = 0; i < nfirst[u]; ++i) tasks[off.x + i] = make_int4(c, i, (1 << 8) | (1 << 16), -1);
+        off.x += nfirst[u];
+        if (nt[u] == 0) continue;
         const int S = s_of(u, W0);
         if (S > 1) {
             for (int t = 0; t < nt[u]; ++t) {
@@ -366,7 +391,7 @@ __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__
             off.w += nt[u];
         } else {
             int& o = (!order || wk[u] * 4 >= W0) ? off.y : off.z;
-            for (int t = 0; t < nt[u]; ++t) tasks[o + t] = make_int4(c, t * tile, 1 << 8, -1);
+            for (int t = 0; t < nt[u]; ++t) tasks[o + t] = make_int4(c, nfirst[u] + t * tile, 1 << 8, -1);
             o += nt[u];
         }
     }
@@ -418,6 +443,7 @@ sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int s
     const int order = (eo && eo[0] == '0') ? 0 : 1;
     const char* ew = getenv("SKNN_SPLITW");  // piece size, x total work / resident warps
     const float wfac = ew ? (float)atof(ew) : 0.5f;
+    const char* eot = getenv("SKNN_OUTLIER_TASKS");  // ablation: 0 keeps 8-query first tiles (warp scan)
     const char* eh = getenv("SKNN_SPLITH");  // straggler threshold, x mean tile work
     const float hfac = eh ? (float)atof(eh) : 4.0f;
     // partial lists of split tasks: at most 2 x resident warps of them, <= 256 MB
@@ -426,7 +452,8 @@ sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int s
         const int64_t per_task = (int64_t)32 * k * sizeof(key_t);
         cap = (int)std::min<int64_t>(2 * (int64_t)slots, ((int64_t)256 << 20) / per_task);
     }
-    int64_t max_tiles = (qs.n + tile - 1) / tile + qs.m + cap;
+    // (+ tile per cluster: the single-query outlier tasks of the warp-per-query scan)
+    int64_t max_tiles = (qs.n + tile - 1) / tile + (int64_t)qs.m * (tile + 1) + cap;
     SKNN_TRY(cx.alloc_scratch((void**)&l1.tiles, sizeof(int4) * max_tiles));
     SKNN_TRY(cx.alloc_scratch((void**)&l1.ntiles, sizeof(int) * 2));
     SKNN_TRY(cx.alloc_scratch((void**)&l1.nmerges, sizeof(int)));
@@ -440,7 +467,10 @@ sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int s
     l1.tile = tile;
     k_make_tasks<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, l1.owner, l1.work,
                                              l1.cand_count,
-                                             slots, cap, split && cap > 0 ? 1 : 0, order, wfac, hfac, l1.tiles, l1.ntiles, l1.merges,
+                                             slots, cap, split && cap > 0 ? 1 : 0, order,
+                                             (tile == 8 && order && !scan_uses_bigk(k) && !(eot && eot[0] == '0')) ? 1 : 0,
+                                             wfac, hfac, l1.tiles,
+                                             l1.ntiles, l1.merges,
                                              l1.nmerges);
     cx.launched();
     if (getenv("SKNN_PLANDBG")) {  // diagnostics: the plan on stderr (synchronises)

@@ -6,10 +6,12 @@ SURVEY.md §8(e). Two modes:
   index and cluster metadata replicated"): every rank holds all of T. For a
   self-join every rank clusters T identically (seeded, deterministic sizes)
   and processes the query clusters c with c % P == rank
-  (``sknn_options.shard_rank/shard_count``); otherwise rank r takes the
-  contiguous query rows [r*nq/P, (r+1)*nq/P). No data-path collective; the
-  optional result assembly is one collective outside the join (an all-gather of
-  the row slices, or for a self-join one all-reduce of packed (dist, idx) keys).
+  (``sknn_options.shard_rank/shard_count``); a Q != T join does the same over
+  the clustering of all of Q (``partition="clusters"``, default) or takes the
+  contiguous query rows [r*nq/P, (r+1)*nq/P) (``partition="rows"``). No
+  data-path collective; the optional result assembly is one collective outside
+  the join (one all-reduce of packed (dist, idx) keys, or an all-gather of the
+  row slices).
 * Target sharding: rank r owns T[r*nt/P, (r+1)*nt/P), computes partial k-lists
   of ALL queries with squared distances and global indices (``out_squared``,
   ``index_base``), the partial lists are exchanged with one all-gather over
@@ -27,6 +29,8 @@ The local join and merge default to the CUDA library; tests may inject other
 callables to exercise the orchestration on CPU with the gloo backend.
 """
 from __future__ import annotations
+
+import math
 
 import torch
 import torch.distributed as dist
@@ -49,30 +53,45 @@ def _world(group):
 
 
 def join_query_sharded(Q, T, k: int, *, group=None, self_join: bool | None = None, gather: bool = True,
-                       local_join=None, **opts):
+                       local_join=None, partition: str = "clusters", **opts):
     """Query-sharded join. Returns (idx, dist) for the rank's rows (gather=False:
     full-size buffers with -1 / 0 in rows of other ranks) or the assembled
-    full result on every rank (gather=True, one collective)."""
+    full result on every rank (gather=True, one collective).
+
+    partition="clusters" (default): every rank clusters all of Q (identical,
+    deterministic) and takes the query clusters c % P == rank. "rows" (Q != T
+    only): rank r clusters and joins the contiguous rows [r nq/P, (r+1) nq/P)
+    -- no replicated query build, but measured on C4 (tools/shard_balance.py,
+    one GPU per rank's share) a rank's slice can hold outlier queries whose
+    near-brute-force scans run on one warp each (P = 8: 1.58 s max over ranks
+    vs 46 ms with cluster interleaving)."""
     world, rank = _world(group)
     local_join = local_join or _cuda_join
     if self_join is None:
         self_join = Q is T
     nq = Q.shape[0]
-    if self_join:
+    if self_join or partition == "clusters":
         idx = torch.full((nq, k), -1, dtype=torch.int32, device=Q.device)
         dst = torch.zeros((nq, k), dtype=torch.float32, device=Q.device)
-        local_join(Q, Q, k, out=(idx, dst), shard_rank=rank, shard_count=world, **opts)
+        local_join(Q, Q if self_join else T, k, out=(idx, dst), shard_rank=rank, shard_count=world, **opts)
     else:
         lo, hi = shard_bounds(nq, world, rank)
         idx = torch.full((nq, k), -1, dtype=torch.int32, device=Q.device)
         dst = torch.zeros((nq, k), dtype=torch.float32, device=Q.device)
         if hi > lo:
-            i, d = local_join(Q[lo:hi].contiguous(), T, k, **opts)[:2]
+            # cluster the slice as finely as the whole query set would be
+            # (floor(3 sqrt(nq)), P:L241): the default floor(3 sqrt(nq / P)) gives
+            # clusters sqrt(P) x wider, and on C4 at P = 8 a 5x larger dense-tile
+            # workload (measured: tools/diag_c4_slices.py)
+            lopts = dict(opts)
+            if world > 1 and not lopts.get("n_clusters_q"):
+                lopts["n_clusters_q"] = min(int(3.0 * math.sqrt(nq)), hi - lo)
+            i, d = local_join(Q[lo:hi].contiguous(), T, k, **lopts)[:2]
             idx[lo:hi] = i
             dst[lo:hi] = d
     if not gather or world == 1:
         return idx, dst
-    if not self_join:
+    if not self_join and partition != "clusters":
         # contiguous row slices: one all-gather of the (padded) slices
         splits = [shard_bounds(nq, world, r) for r in range(world)]
         cap = max(h - l for l, h in splits)
@@ -84,7 +103,7 @@ def join_query_sharded(Q, T, k: int, *, group=None, self_join: bool | None = Non
         dist.all_gather_into_tensor(allp, mine, group=group)
         out = torch.cat([allp[r * cap:r * cap + (h - l)] for r, (l, h) in enumerate(splits)])
         return out[:, :, 0].contiguous(), out[:, :, 1].contiguous().view(torch.float32)
-    # self-join, cluster-interleaved rows: each rank's rows hold (dist bits << 32 |
+    # cluster-interleaved rows: each rank's rows hold (dist bits << 32 |
     # idx + 1), every other row 0, so ONE all-reduce SUM assembles both arrays
     own = idx >= 0
     packed = torch.where(own, (dst.view(torch.int32).to(torch.int64) << 32) | (idx.to(torch.int64) + 1),

@@ -74,14 +74,16 @@ def _worker(rank, world, port, results):
         si_, sd_ = sdist.join_target_sharded(torch.from_numpy(Q2), torch.from_numpy(X[lo:hi]).contiguous(), k, lo,
                                              local_join=oracle_local_join, merge=host_merge, exchange="all_to_all",
                                              gather=False)
-        # query sharding, non-self join (contiguous rows)
+        # query sharding, non-self join: interleaved query clusters (default) and contiguous rows
         qi, qd = sdist.join_query_sharded(torch.from_numpy(Q), torch.from_numpy(X), k, self_join=False,
                                           local_join=oracle_local_join)
+        wi, wd = sdist.join_query_sharded(torch.from_numpy(Q), torch.from_numpy(X), k, self_join=False,
+                                          local_join=oracle_local_join, partition="rows")
         # query sharding, self join (cluster-interleaved rows, assembled by all-reduce)
         Xt = torch.from_numpy(X)
         si, sd = sdist.join_query_sharded(Xt, Xt, k, local_join=oracle_local_join)
         results[rank] = (i.numpy(), d.numpy(), qi.numpy(), qd.numpy(), si.numpy(), sd.numpy(),
-                         ai.numpy(), ad.numpy(), si_.numpy(), sd_.numpy())
+                         ai.numpy(), ad.numpy(), si_.numpy(), sd_.numpy(), wi.numpy(), wd.numpy())
     finally:
         dist.destroy_process_group()
 
@@ -112,7 +114,9 @@ def test_two_rank_gloo_matches_single_join():
     aidx, adist = oracle.knn_join(Q2, X, k)
     from paper_conf_icde_chends17_b200.dist import shard_bounds
     for r in range(world):
-        i, d, qi, qd, si, sd, ai, ad, ri, rd = results[r]
+        i, d, qi, qd, si, sd, ai, ad, ri, rd, wi, wd = results[r]
+        np.testing.assert_array_equal(wi, ridx)      # query-sharded by row slices, assembled
+        np.testing.assert_array_equal(wd, rdist)
         np.testing.assert_array_equal(ai, aidx)      # all-to-all exchange, assembled
         np.testing.assert_array_equal(ad, adist)
         lo, hi = shard_bounds(Q2.shape[0], world, r)
