@@ -168,6 +168,12 @@ def workload(name: str, scale: float = 1.0):
         else:
             X = c3_kegg(max(16, int(round(65_554 * scale))), d=d)
         return X, X, 16, True
+    if name in ("ARC", "DOR"):
+        # high-d shapes of Table III, not bench configs: arcene-like
+        # 100 x 10,000 (dense integer intensities 0..999, a few latent
+        # prototypes) and dorothea-like 1,950 x 100,000 (sparse binary, ~1%
+        # ones, rows near a few prototypes); integer-valued, self-joins, k = 8
+        return high_d(name, scale), None, 8, True
     cfg = CONFIGS[name.replace("int", "")]
     n = max(16, int(round(cfg["n"] * scale)))
     k = cfg["k"]
@@ -188,3 +194,18 @@ def workload(name: str, scale: float = 1.0):
     if name == "C5":
         return c5_blobs(n, which="Q"), c5_blobs(n, which="T"), k, False
     raise KeyError(name)
+
+
+def high_d(name: str, scale: float = 1.0, seed: int = 11) -> np.ndarray:
+    """ARC (arcene-like) or DOR (dorothea-like) rows; see workload()."""
+    rng = np.random.default_rng(seed)
+    if name == "ARC":
+        n, d = max(16, int(round(100 * scale))), 10_000
+        protos = rng.integers(0, 1000, size=(4, d))
+        X = protos[rng.integers(0, 4, size=n)] + rng.integers(-60, 61, size=(n, d))
+        return np.clip(X, 0, 999).astype(np.float32)
+    n, d = max(16, int(round(1950 * scale))), 100_000
+    protos = rng.random((8, d)) < 0.01
+    X = protos[rng.integers(0, 8, size=n)]
+    flip = rng.random((n, d)) < 0.002
+    return np.logical_xor(X, flip).astype(np.float32)

@@ -219,16 +219,23 @@ __global__ void __launch_bounds__(256) k_assign(const float* __restrict__ Xp, in
         }
     }
     const float* xrow = Xp + (active ? i : 0) * dp;
-    for (int c0 = 0; c0 < m; c0 += chunk) {
-        int cn = min(chunk, m - c0);
-        __syncthreads();
-        for (int e = threadIdx.x; e < cn * dp / 4; e += blockDim.x)
-            reinterpret_cast<float4*>(s_c)[e] = reinterpret_cast<const float4*>(centers + (int64_t)c0 * dp)[e];
-        __syncthreads();
+    const bool staged = chunk > 0;  // chunk 0: high d, centers read from global memory
+    const int step = staged ? chunk : m;
+    for (int c0 = 0; c0 < m; c0 += step) {
+        int cn = min(step, m - c0);
+        const float* s_c0 = s_c;
+        if (staged) {
+            __syncthreads();
+            for (int e = threadIdx.x; e < cn * dp / 4; e += blockDim.x)
+                reinterpret_cast<float4*>(s_c)[e] = reinterpret_cast<const float4*>(centers + (int64_t)c0 * dp)[e];
+            __syncthreads();
+        } else {
+            s_c0 = centers + (int64_t)c0 * dp;
+        }
         if (!active) continue;
         if constexpr (DP > 0) {
             for (int c = 0; c < cn; ++c) {
-                const float4* cc = reinterpret_cast<const float4*>(s_c + c * DP);
+                const float4* cc = reinterpret_cast<const float4*>(s_c0 + c * DP);
                 float s = 0.f;
 #pragma unroll
                 for (int j = 0; j < DP / 4; ++j) s = d2_acc4(s, q[j], cc[j]);
@@ -239,7 +246,7 @@ __global__ void __launch_bounds__(256) k_assign(const float* __restrict__ Xp, in
             int c = 0;
             for (; c + 4 <= cn; c += 4) {
                 float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
-                const float4* c4 = reinterpret_cast<const float4*>(s_c + c * dp);
+                const float4* c4 = reinterpret_cast<const float4*>(s_c0 + c * dp);
                 const int w = dp / 4;
                 for (int j = 0; j < w; ++j) {
                     float4 xv = x4[j];
@@ -254,7 +261,7 @@ __global__ void __launch_bounds__(256) k_assign(const float* __restrict__ Xp, in
                 if (s3 < best) { best = s3; bi = c0 + c + 3; }
             }
             for (; c < cn; ++c) {
-                const float4* c4 = reinterpret_cast<const float4*>(s_c + c * dp);
+                const float4* c4 = reinterpret_cast<const float4*>(s_c0 + c * dp);
                 float s = 0.f;
                 for (int j = 0; j < dp / 4; ++j) s = d2_acc4(s, x4[j], c4[j]);
                 if (s < best) { best = s; bi = c0 + c; }
@@ -825,10 +832,15 @@ __global__ void k_gather_side(const u64* __restrict__ keys, const float* __restr
 }
 
 // ------------------------------------------------------------ launcher --
+// centers per shared-memory chunk of the SIMT assignment; 0 = high d (a row
+// above 48 KB): the centers are read from global memory, no staging
 static int assign_chunk(int dp, int m, size_t* smem) {
     int chunk = int((48 * 1024) / (dp * sizeof(float)));
     if (chunk > m) chunk = m;
-    if (chunk < 1) chunk = 1;
+    if (chunk < 1) {
+        *smem = 0;
+        return 0;
+    }
     *smem = size_t(chunk) * dp * sizeof(float);
     return chunk;
 }

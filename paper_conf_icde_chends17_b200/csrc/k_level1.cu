@@ -188,7 +188,7 @@ __global__ void k_kth_member(const int4* __restrict__ tinfo, const float* __rest
 __global__ void __launch_bounds__(kL1Threads) k_level1(
     const float* __restrict__ qcent, const float* __restrict__ qrad, const int32_t* __restrict__ qoff,
     const float* __restrict__ tcent, const int4* __restrict__ tinfo, const float* __restrict__ tdk,
-    const float* __restrict__ tdist, int mt, int dp, int k, float eta, int keys_cap, int shard_rank,
+    const float* __restrict__ tdist, int mt, int dp, int row_in_smem, int k, float eta, int keys_cap, int shard_rank,
     int shard_count, int dense_mode, float dense_tau, const float* __restrict__ cq_o,
     const float* __restrict__ ct_o, float dense_eps, const float* __restrict__ ub_in, float* __restrict__ ub_out,
     int32_t* __restrict__ cand,
@@ -214,7 +214,11 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
         }
         return;
     }
-    for (int i = threadIdx.x; i < dp; i += blockDim.x) s_qc[i] = qcent[(int64_t)qc * dp + i];
+    // the query cluster's center row: staged in shared memory when it fits
+    // (row_in_smem, decided by the launcher), else read through L1 (high d)
+    const float* qrow = row_in_smem ? s_qc : qcent + (int64_t)qc * dp;
+    if (row_in_smem)
+        for (int i = threadIdx.x; i < dp; i += blockDim.x) s_qc[i] = qcent[(int64_t)qc * dp + i];
     if (threadIdx.x == 0) s_cnt = 0;
     __syncthreads();
     const float rq = qrad[qc];
@@ -234,7 +238,7 @@ __global__ void __launch_bounds__(kL1Threads) k_level1(
     for (int tc = threadIdx.x; tc < mt; tc += blockDim.x) {
         const float dmin = __int_as_float(__ldg(&tinfo[tc].w));  // +inf if empty
         const float dk = __ldg(tdk + tc);                        // +inf if fewer than k members
-        const float D = __fsqrt_rn(d2_rows(s_qc, tcent + (int64_t)tc * dp, dp));
+        const float D = __fsqrt_rn(d2_rows(qrow, tcent + (int64_t)tc * dp, dp));
         s_D[tc] = D;
         s_v[tc] = D + dmin;
         m1 = fminf(m1, D + dk);
@@ -423,6 +427,8 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
     cap = std::max(cap, kL1Vals);
     const int mt4 = (mt + 3) & ~3;  // s_keys holds the gathered bounds (<= kL1Vals) before phase 2
     size_t smem = sizeof(u64) * cap + sizeof(float) * (mt4 + std::max(mt4, kL1Vals) + dp);
+    const int row_in_smem = smem <= 200 * 1024 ? 1 : 0;  // high d: the center row stays in global memory
+    if (!row_in_smem) smem -= sizeof(float) * dp;
     if (smem > 227 * 1024) {
         set_last_error("level-1: too many target clusters for the shared-memory candidate sort");
         return SKNN_ERR_UNSUPPORTED;
@@ -433,7 +439,8 @@ sknn_status run_level1(Ctx& cx, const Side& qs, const Side& ts, const Level1Para
     k_kth_member<<<(mt + 255) / 256, 256, 0, cx.stream>>>(ts.tinfo, ts.dist, mt, p.k, tdk);
     cx.launched();
     k_level1<<<mq, kL1Threads, smem, cx.stream>>>(qs.centers, qs.radius, qs.off, ts.centers, ts.tinfo, tdk,
-                                                  ts.dist, mt, dp, p.k, p.eta, cap, p.shard_rank, p.shard_count,
+                                                  ts.dist, mt, dp, row_in_smem, p.k, p.eta, cap, p.shard_rank,
+                                                  p.shard_count,
                                                   p.dense_mode, p.dense_tau, p.dorg ? p.dorg->cq_o : nullptr,
                                                   p.dorg ? p.dorg->ct_o : nullptr, p.dorg ? p.dorg->eps : 0.f,
                                                   p.ub_in, out.ub, out.cand, out.cand_count, out.cand_D,

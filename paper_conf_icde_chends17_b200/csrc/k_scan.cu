@@ -42,7 +42,7 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int ntiles = *a.ntiles;
     const int dp = DP > 0 ? DP : a.dp;
-    float* sq = s_q + warp * (DP > 0 ? 0 : dp);
+    float* sq_s = s_q + warp * (DP > 0 || a.q_global ? 0 : dp);
     unsigned long long evals = 0, cevals = 0;
     for (;;) {
         int tile = 0;
@@ -63,11 +63,13 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
             if constexpr (DP > 0) {
 #pragma unroll
                 for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(a.qrows + (int64_t)qpos * DP) + c);
-            } else {
+            } else if (!a.q_global) {
                 __syncwarp();
-                for (int c = lane; c < dp; c += 32) sq[c] = a.qrows[(int64_t)qpos * dp + c];
+                for (int c = lane; c < dp; c += 32) sq_s[c] = a.qrows[(int64_t)qpos * dp + c];
                 __syncwarp();
             }
+            // runtime dp: the query row staged per warp, or (high d) read through L1
+            const float* sq = (DP == 0 && a.q_global) ? a.qrows + (int64_t)qpos * dp : sq_s;
             key_t mine = (lane < 32 - a.k) ? kNegKey : kInfKey;
             if (a.init_topk && a.dcount[qc] > 0 && lane >= 32 - a.k) mine = a.init_topk[(int64_t)qpos * a.k + lane - (32 - a.k)];
             key_t kth = __shfl_sync(0xffffffffu, mine, 31);
@@ -410,8 +412,11 @@ int occupancy_grid(Ctx& cx, const void* fn, int threads, size_t smem) {
 }
 
 template <int DP>
-static void launch_wpq(Ctx& cx, const ScanArgs& a) {
+static void launch_wpq(Ctx& cx, const ScanArgs& a_in) {
+    ScanArgs a = a_in;
     size_t smem = DP > 0 ? 0 : sizeof(float) * 8 * a.dp;
+    a.q_global = smem > 160 * 1024 ? 1 : 0;  // high d: query rows read through L1, no staging
+    if (a.q_global) smem = 0;
     if (smem > 48 * 1024) cudaFuncSetAttribute(k_scan_wpq<DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int grid = occupancy_grid(cx, (const void*)k_scan_wpq<DP>, 256, smem);
     if (a.probe_warps) {  // dry run: report resident warps for the task planner
@@ -732,12 +737,15 @@ __global__ void __launch_bounds__(256) k_brute(const float* __restrict__ Q, int6
                                                int64_t nt, int d, ScanArgs a) {
     extern __shared__ __align__(16) float s_qb[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    float* sq = s_qb + warp * d;
+    float* sq_s = s_qb + warp * (a.q_global ? 0 : d);
     unsigned long long evals = 0;
     for (int64_t qi = (int64_t)blockIdx.x * 8 + warp; qi < nq; qi += (int64_t)gridDim.x * 8) {
-        __syncwarp();
-        for (int c = lane; c < d; c += 32) sq[c] = Q[qi * d + c];
-        __syncwarp();
+        if (!a.q_global) {
+            __syncwarp();
+            for (int c = lane; c < d; c += 32) sq_s[c] = Q[qi * d + c];
+            __syncwarp();
+        }
+        const float* sq = a.q_global ? Q + qi * d : sq_s;  // high d: read through L1
         key_t mine = (lane < 32 - a.k) ? kNegKey : kInfKey;
         key_t kth = kInfKey;
         for (int64_t base = 0; base < nt; base += 32) {
@@ -773,6 +781,8 @@ sknn_status run_brute(Ctx& cx, const float* Q, int64_t nq, const float* T, int64
     a.k = p.k; a.out_squared = p.out_squared; a.index_base = p.index_base;
     a.out_idx = p.out_idx; a.out_dist = p.out_dist; a.counters = p.counters;
     size_t smem = sizeof(float) * 8 * d;
+    a.q_global = smem > 160 * 1024 ? 1 : 0;
+    if (a.q_global) smem = 0;
     if (smem > 48 * 1024) SKNN_CUDA(cudaFuncSetAttribute(k_brute, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int64_t blocks = (nq + 7) / 8;
     int grid = (int)std::min<int64_t>(blocks, (int64_t)cx.num_sms * 8);

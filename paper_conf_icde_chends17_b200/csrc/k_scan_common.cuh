@@ -45,6 +45,7 @@ struct ScanArgs {
     float* out_dist;
     Counters* counters;
     int* probe_warps;  // non-NULL: launchers only report resident warps (no launch)
+    int q_global;      // runtime-dp kernels: 1 = query rows read from global memory (too large to stage)
 };
 
 // First member position in [lo, hi) that is NOT in Alg. 2's `continue`

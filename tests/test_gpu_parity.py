@@ -850,3 +850,24 @@ def test_basic_knnti_rejects_unsupported(sknn):
         run(sknn, Q, T, 40, sj, mapping="basic")
     with pytest.raises(RuntimeError):
         run(sknn, Q, T, k, sj, mapping="basic", force_path="dense")
+
+
+# ------------------------------------------------ high d (NEXT-4, arcene/dor-like) --
+@pytest.mark.parametrize("d,n", [(300, 700), (1024, 600), (4096, 300), (10000, 150), (100000, 40)])
+def test_high_dimension_bitexact(sknn, d, n):
+    """Dimensions past the tensor-core kernels' K <= 256 (Table III's arcene
+    d = 10,000 and dorothea d = 100,000 shapes): sparse binary
+    rows (dorothea-like, ~1% ones) plus a dense integer block; every path the
+    dispatcher takes at this d (SIMT assignment, runtime-dp scans) is
+    bit-exact against the oracle, self-join and Q != T."""
+    rng = np.random.default_rng(d + n)
+    X = (rng.random((n, d)) < 0.01).astype(np.float32)
+    X[:, :8] = rng.integers(0, 4, size=(n, 8))
+    Q = (rng.random((n // 2, d)) < 0.01).astype(np.float32)
+    k = 8
+    idx, dist, _ = run(sknn, X, X, k, True)
+    ridx, rdist = oracle.knn_join(X, X, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    idx, dist, _ = run(sknn, Q, X, k, False)
+    ridx, rdist = oracle.knn_join(Q, X, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
