@@ -173,7 +173,8 @@ def workload(name: str, scale: float = 1.0):
         # 100 x 10,000 (dense integer intensities 0..999, a few latent
         # prototypes) and dorothea-like 1,950 x 100,000 (sparse binary, ~1%
         # ones, rows near a few prototypes); integer-valued, self-joins, k = 8
-        return high_d(name, scale), None, 8, True
+        X = high_d(name, scale)
+        return X, X, 8, True
     cfg = CONFIGS[name.replace("int", "")]
     n = max(16, int(round(cfg["n"] * scale)))
     k = cfg["k"]

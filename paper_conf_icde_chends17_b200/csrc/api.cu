@@ -446,7 +446,13 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     const int dp = (d + 3) & ~3;
     const bool self = qindex ? qindex == index : (index ? index_self_query(o, Q, nq, index) : (Q == T && nq == nt));
     int mapping = choose_mapping(o, di, nq, dp, k);
-    int path = o.force_path == SKNN_PATH_BRUTE ? SKNN_PATH_BRUTE : SKNN_PATH_SPARSE;
+    // dense-only (every pair, k_brute_tiled): forced, or auto at high d, where
+    // the TI filters keep most pairs and the scans' per-lane rows cost more
+    // than a tiled contraction (measured: arcene/dorothea shapes)
+    const bool dense_only = o.force_path == SKNN_PATH_BRUTE ||
+                            (o.force_path == SKNN_PATH_AUTO && dp >= kDenseOnlyDp && k <= 32 && !qindex &&
+                             o.shard_count <= 1 && !o.ub_in && o.mapping != SKNN_MAP_BASIC);
+    int path = dense_only ? SKNN_PATH_BRUTE : SKNN_PATH_SPARSE;
     Marks mk;
     int mq = 0, mt = 0;
     Counters host_c;
@@ -484,8 +490,8 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
             break;
         }
         if (path == SKNN_PATH_BRUTE) {
-            if (index) {
-                st = fail(SKNN_ERR_INVALID_ARG, "force_path = BRUTE is only available for sknn_join");
+            if (qindex) {
+                st = fail(SKNN_ERR_INVALID_ARG, "force_path = BRUTE is not available for sknn_join_indexed");
                 break;
             }
             ScanParams sp;
@@ -495,12 +501,20 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
             sp.out_idx = d_oidx;
             sp.out_dist = d_odist;
             sp.counters = counters;
-            mapping = SKNN_MAP_WARP;
             if (k > 32) {
                 st = fail(SKNN_ERR_UNSUPPORTED, "force_path = BRUTE supports k <= 32");
                 break;
             }
-            st = run_brute(cx, dQ, nq, dT, nt, d, sp);
+            const char* eb = getenv("SKNN_BRUTE");  // "warp": the warp-per-query anchor kernel (caller rows only)
+            if (eb && !strcmp(eb, "warp") && !index) {
+                mapping = SKNN_MAP_WARP;
+                st = run_brute(cx, dQ, nq, dT, nt, d, sp);
+            } else {
+                mapping = SKNN_MAP_THREAD;
+                // an index holds its rows permuted and padded to dp, with the original ids
+                st = index ? run_brute_tiled(cx, dQ, nq, d, index->t.rows, nt, index->t.dp, index->t.orig, d, sp)
+                           : run_brute_tiled(cx, dQ, nq, d, dT, nt, d, nullptr, d, sp);
+            }
             mk.bt = tm.mark();
             mk.scan = mk.bt;
             break;

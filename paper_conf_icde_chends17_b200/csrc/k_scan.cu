@@ -36,13 +36,13 @@ namespace sknn {
 // up to `tile` queries of one cluster from the atomic scheduler; no CTA
 // barriers. DP > 0: the query sits in registers of every lane; DP == 0:
 // runtime dp, the query is staged in shared memory per warp.
-template <int DP>
+template <int DP, bool QG = false>  // QG: (runtime dp only) query rows read from global memory (high d)
 __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
     extern __shared__ __align__(16) float s_q[];  // [8 warps x dp] when DP == 0
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int ntiles = *a.ntiles;
     const int dp = DP > 0 ? DP : a.dp;
-    float* sq_s = s_q + warp * (DP > 0 || a.q_global ? 0 : dp);
+    float* sq_s = s_q + warp * (DP > 0 || QG ? 0 : dp);
     unsigned long long evals = 0, cevals = 0;
     for (;;) {
         int tile = 0;
@@ -63,13 +63,13 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
             if constexpr (DP > 0) {
 #pragma unroll
                 for (int c = 0; c < DP / 4; ++c) q[c] = __ldg(reinterpret_cast<const float4*>(a.qrows + (int64_t)qpos * DP) + c);
-            } else if (!a.q_global) {
+            } else if constexpr (!QG) {
                 __syncwarp();
                 for (int c = lane; c < dp; c += 32) sq_s[c] = a.qrows[(int64_t)qpos * dp + c];
                 __syncwarp();
             }
             // runtime dp: the query row staged per warp, or (high d) read through L1
-            const float* sq = (DP == 0 && a.q_global) ? a.qrows + (int64_t)qpos * dp : sq_s;
+            const float* sq = QG ? a.qrows + (int64_t)qpos * dp : sq_s;
             key_t mine = (lane < 32 - a.k) ? kNegKey : kInfKey;
             if (a.init_topk && a.dcount[qc] > 0 && lane >= 32 - a.k) mine = a.init_topk[(int64_t)qpos * a.k + lane - (32 - a.k)];
             key_t kth = __shfl_sync(0xffffffffu, mine, 31);
@@ -412,11 +412,17 @@ int occupancy_grid(Ctx& cx, const void* fn, int threads, size_t smem) {
 }
 
 template <int DP>
-static void launch_wpq(Ctx& cx, const ScanArgs& a_in) {
-    ScanArgs a = a_in;
+static void launch_wpq(Ctx& cx, const ScanArgs& a) {
     size_t smem = DP > 0 ? 0 : sizeof(float) * 8 * a.dp;
-    a.q_global = smem > 160 * 1024 ? 1 : 0;  // high d: query rows read through L1, no staging
-    if (a.q_global) smem = 0;
+    if (DP == 0 && smem > 160 * 1024) {  // high d: query rows read through L1, no staging
+        const int grid = occupancy_grid(cx, (const void*)k_scan_wpq<0, true>, 256, 0);
+        if (a.probe_warps) {
+            *a.probe_warps = grid * (256 / 32);
+            return;
+        }
+        k_scan_wpq<0, true><<<grid, 256, 0, cx.stream>>>(a);
+        return;
+    }
     if (smem > 48 * 1024) cudaFuncSetAttribute(k_scan_wpq<DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int grid = occupancy_grid(cx, (const void*)k_scan_wpq<DP>, 256, smem);
     if (a.probe_warps) {  // dry run: report resident warps for the task planner

@@ -201,6 +201,11 @@ ScanArgs make_scan_args(const Side& qs, const Side& ts, const Level1& l1, const 
 sknn_status run_partial(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1, const ScanParams& p,
                         bool* fell_back);
 sknn_status run_brute(Ctx& cx, const float* Q, int64_t nq, const float* T, int64_t nt, int d, const ScanParams& p);
+// dense-only join (k_brute_tiled.cu): register-tiled SIMT contraction + fused top-k
+sknn_status run_brute_tiled(Ctx& cx, const float* Q, int64_t nq, int ldq, const float* T, int64_t nt, int ldt,
+                            const int32_t* torig, int d, const ScanParams& p);
+// dimensions from which auto takes the dense-only path (measured)
+constexpr int kDenseOnlyDp = 1024;
 sknn_status run_merge(Ctx& cx, const int32_t* part_idx, const float* part_d2, int P, int64_t nq, int k,
                       int32_t* out_idx, float* out_dist, int out_squared);
 

@@ -871,3 +871,42 @@ def test_high_dimension_bitexact(sknn, d, n):
     idx, dist, _ = run(sknn, Q, X, k, False)
     ridx, rdist = oracle.knn_join(Q, X, k)
     assert_knn_bitexact(idx, dist, ridx, rdist)
+
+
+@pytest.mark.parametrize("nq,nt,d,k", [(1, 1, 1, 1), (65, 63, 7, 5), (200, 3000, 130, 32), (700, 129, 2048, 8),
+                                       (33, 5000, 33, 17)])
+def test_dense_only_tiled_bitexact(sknn, nq, nt, d, k, monkeypatch):
+    """The dense-only path (k_brute_tiled: 64 x 64 register tiles, fused top-k,
+    target slices merged by sknn_merge_partials) on ragged shapes: bit-exact
+    against the oracle and against the warp-per-query anchor kernel
+    (SKNN_BRUTE=warp), with ties (small integer coordinates)."""
+    rng = np.random.default_rng(nq * 7 + nt + d)
+    Q = rng.integers(0, 3, size=(nq, d)).astype(np.float32)
+    T = rng.integers(0, 3, size=(nt, d)).astype(np.float32)
+    k = min(k, nt)
+    idx, dist, st = run(sknn, Q, T, k, False, force_path="brute")
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx, dist, ridx, rdist)
+    assert st["pruned_pct"] == 0.0
+    monkeypatch.setenv("SKNN_BRUTE", "warp")
+    i2, d2, _ = run(sknn, Q, T, k, False, force_path="brute")
+    assert_knn_bitexact(i2, d2, ridx, rdist)
+
+
+def test_dense_only_index_query_high_d(sknn):
+    """sknn_query against a prebuilt index at d >= 1024 takes the dense-only
+    path over the index's permuted rows (original ids through its map):
+    bit-exact, host batches included."""
+    rng = np.random.default_rng(5)
+    T = (rng.random((900, 1500)) < 0.02).astype(np.float32)
+    Q = (rng.random((300, 1500)) < 0.02).astype(np.float32)
+    k = 6
+    ix = sknn.build(dev(T))
+    idx, dist, st = ix.query(dev(Q), k, stats=True)
+    torch.cuda.synchronize()
+    ridx, rdist = oracle.knn_join(Q, T, k)
+    assert_knn_bitexact(idx.cpu().numpy(), dist.cpu().numpy(), ridx, rdist)
+    assert st["path_used"] == 3   # SKNN_PATH_BRUTE: every pair
+    i2, d2 = ix.query(Q, k, query_batch=100)
+    assert_knn_bitexact(np.asarray(i2), np.asarray(d2), ridx, rdist)
+    ix.close()
