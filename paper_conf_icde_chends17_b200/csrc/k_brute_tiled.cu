@@ -116,7 +116,7 @@ __global__ void __launch_bounds__(256) k_brute_tiled(const float* __restrict__ Q
                 if (q0 + r < nq && tj < t_hi) {
                     ++evals;
                     const key_t key = make_key(acc[u][v], torig ? __ldg(torig + tj) : (int)tj);
-                    if (key < kth) {
+                    if (key_lt(key, kth)) {
                         const int slot = atomicAdd(&s_cnt[r], 1);
                         if (slot < kBtBuf) s_buf[r][slot] = key;
                     }
@@ -132,7 +132,7 @@ __global__ void __launch_bounds__(256) k_brute_tiled(const float* __restrict__ Q
             key_t kth = __shfl_sync(0xffffffffu, mine[i], 31);
             for (int j = 0; j < n; ++j) {
                 const key_t key = s_buf[r][j];
-                if (key < kth) {
+                if (key_lt(key, kth)) {
                     mine[i] = warp_insert(mine[i], key, lane);
                     kth = __shfl_sync(0xffffffffu, mine[i], 31);
                 }

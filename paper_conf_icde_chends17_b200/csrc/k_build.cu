@@ -323,7 +323,7 @@ __global__ void __launch_bounds__(256) k_center_knn(const float* __restrict__ ce
     for (int base = 0; base < m; base += 32) {
         key_t key = next;
         next = batch_key(base + 32 + lane);
-        unsigned cm = __ballot_sync(0xffffffffu, key < kth);
+        unsigned cm = __ballot_sync(0xffffffffu, key_lt(key, kth));
         if (__popc(cm) <= 6) {  // few accepted keys: serial insertion
             while (cm) {
                 const int src = __ffs(cm) - 1;
@@ -331,7 +331,7 @@ __global__ void __launch_bounds__(256) k_center_knn(const float* __restrict__ ce
                 mine = warp_insert(mine, kk, lane);
                 kth = __shfl_sync(0xffffffffu, mine, 31);
                 cm &= ~(1u << src);
-                cm &= __ballot_sync(0xffffffffu, key < kth);
+                cm &= __ballot_sync(0xffffffffu, key_lt(key, kth));
             }
             continue;
         }

@@ -375,7 +375,7 @@ __global__ void __launch_bounds__(kDenseM, 1) k_dense(DenseArgs a) {
                     ++recomputed;
                     if (d2 <= key_d2(kth)) {
                         const key_t key = make_key(d2, __ldg(a.torig + jj));
-                        if (key < kth) {
+                        if (key_lt(key, kth)) {
                             top.insert(key);
                             kth = top.kth();
                             const float k2 = key_d2(kth);
@@ -651,7 +651,7 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
                             const float d2 = tj + na;  // exact (integer < 2^24)
                             if (d2 <= kth2) {
                                 const key_t key = make_key(d2, __ldg(a.torig + j0 + col + j));
-                                if (key < kth) {
+                                if (key_lt(key, kth)) {
                                     top.insert(key);
                                     kth = top.kth();
                                     if (key_d2(kth) < kth2) {
@@ -683,7 +683,7 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
             if (active && half == 0) {
                 for (int r = 0; r < a.k; ++r) {
                     const key_t key = orow[r];
-                    if (key < kth) {
+                    if (key_lt(key, kth)) {
                         top.insert(key);
                         kth = top.kth();
                     }

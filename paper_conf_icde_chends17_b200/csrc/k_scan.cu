@@ -146,14 +146,14 @@ __global__ void __launch_bounds__(256) k_scan_wpq(ScanArgs a) {
                         ++evals;
                         if (d2 <= key_d2(kth)) key = make_key(d2, __ldg(a.torig + j));
                     }
-                    unsigned cm = __ballot_sync(0xffffffffu, key < kth);
+                    unsigned cm = __ballot_sync(0xffffffffu, key_lt(key, kth));
                     while (cm) {
                         const int src = __ffs(cm) - 1;
                         const key_t kk = __shfl_sync(0xffffffffu, key, src);
                         mine = warp_insert(mine, kk, lane);
                         kth = __shfl_sync(0xffffffffu, mine, 31);
                         cm &= ~(1u << src);
-                        cm &= __ballot_sync(0xffffffffu, key < kth);
+                        cm &= __ballot_sync(0xffffffffu, key_lt(key, kth));
                     }
                     theta = fminf(ub, __fsqrt_ru(key_d2(kth)));
                     if (bm) break;
@@ -767,14 +767,14 @@ __global__ void __launch_bounds__(256) k_brute(const float* __restrict__ Q, int6
                 key = make_key(s, (int)j);
                 ++evals;
             }
-            unsigned cm = __ballot_sync(0xffffffffu, key < kth);
+            unsigned cm = __ballot_sync(0xffffffffu, key_lt(key, kth));
             while (cm) {
                 const int src = __ffs(cm) - 1;
                 const key_t kk = __shfl_sync(0xffffffffu, key, src);
                 mine = warp_insert(mine, kk, lane);
                 kth = __shfl_sync(0xffffffffu, mine, 31);
                 cm &= ~(1u << src);
-                cm &= __ballot_sync(0xffffffffu, key < kth);
+                cm &= __ballot_sync(0xffffffffu, key_lt(key, kth));
             }
         }
         if (lane >= 32 - a.k) write_result(a, (int)qi, lane - (32 - a.k), mine);

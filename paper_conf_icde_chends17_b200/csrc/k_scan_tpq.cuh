@@ -133,12 +133,12 @@ struct TopList<LIST_HEAP, KMAX, STRIDE> {
             int ci = l;
             if (l + 1 < n) {
                 const key_t c2 = s[(l + 1) * STRIDE];
-                if (c < c2) {
+                if (key_lt(c, c2)) {
                     c = c2;
                     ci = l + 1;
                 }
             }
-            if (!(key < c)) break;
+            if (!key_lt(key, c)) break;
             s[i * STRIDE] = c;
             i = ci;
         }
@@ -163,12 +163,12 @@ struct TopList<LIST_HEAP, KMAX, STRIDE> {
             int ci = l;
             if (!last || l + 1 < N) {
                 const key_t c2 = s[(l + 1) * STRIDE];
-                if (c < c2) {
+                if (key_lt(c, c2)) {
                     c = c2;
                     ci = l + 1;
                 }
             }
-            if (!(key < c)) break;
+            if (!key_lt(key, c)) break;
             s[i * STRIDE] = c;
             i = ci;
         }
@@ -287,7 +287,7 @@ __device__ __forceinline__ void tpq_tile(const ScanArgs& a, const int4 tl, key_t
             auto consider = [&](float d2, int jc) {
                 if (d2 <= kth_d2) {                                         // line 16 (distance part)
                     const key_t key = make_key(d2, __ldg(a.torig + jc));
-                    if (key < kth) {
+                    if (key_lt(key, kth)) {
                         ++ins;
                         kth = top.insert(key);
                         if (key_d2(kth) < kth_d2) {
@@ -458,7 +458,7 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
     auto flush = [&]() {
 #pragma unroll
         for (int b = 0; b < BUF; ++b) {
-            if (b < nb && buf[b] < kth) {
+            if (b < nb && key_lt(buf[b], kth)) {
                 ++ins;
                 kth = top.insert(buf[b]);
             }
@@ -472,7 +472,7 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
     auto consider = [&](float d2, int jc) {  // called by all 32 lanes
         if (active && d2 <= kth_d2) {                                // Alg. 2 line 16 (distance part)
             const key_t key = make_key(d2, __ldg(a.torig + jc));
-            if (key < kth) {
+            if (key_lt(key, kth)) {
                 if constexpr (BUF > 0) {
 #pragma unroll
                     for (int b = 0; b < BUF; ++b)
@@ -552,7 +552,7 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
                         if (u == v) d2 = dd[v];
                     if (d2 <= kth_d2) {  // re-checked: an earlier insert may have lowered the bound
                         const key_t key = make_key(d2, __ldg(a.torig + j0 + step * u));
-                        if (key < kth) {
+                        if (key_lt(key, kth)) {
                             ++ins;
                             kth = top.insert(key);
                             if (key_d2(kth) < kth_d2) {

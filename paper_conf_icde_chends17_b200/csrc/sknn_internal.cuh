@@ -28,6 +28,20 @@ constexpr key_t kNegKey = -1;
 __device__ __forceinline__ key_t make_key(float d2, int idx) {
     return (key_t(__float_as_uint(d2)) << 32) | key_t(uint32_t(idx));
 }
+// a < b for keys of which `a` is >= 0 (a real key or kInfKey) and `b` is a
+// key or the placeholder kNegKey. Read as IEEE doubles, keys >= 0 are finite
+// and non-negative (their top 11 bits are the float d2's bits 30..20, never all
+// ones for a finite or +inf d2) and order exactly like the integers, and -1 is
+// a NaN, so `a < -1` is false as for the integers: one DSETP (fp64 pipe)
+// instead of the 64-bit integer compare pair on the ALU pipe.
+// (SKNN_KEYCMP_INT builds the integer compare, for A/B timing.)
+__device__ __forceinline__ bool key_lt(key_t a, key_t b) {
+#ifdef SKNN_KEYCMP_INT
+    return a < b;
+#else
+    return __longlong_as_double(a) < __longlong_as_double(b);
+#endif
+}
 __device__ __forceinline__ float key_d2(key_t k) { return __uint_as_float(uint32_t(uint64_t(k) >> 32)); }
 __device__ __forceinline__ int key_idx(key_t k) { return int(uint32_t(uint64_t(k) & 0xffffffffu)); }
 
@@ -102,7 +116,7 @@ struct RegTopK {
     __device__ __forceinline__ void insert(key_t key) {
         bool c[KMAX];
 #pragma unroll
-        for (int i = 0; i < KMAX; ++i) c[i] = key < a[i];
+        for (int i = 0; i < KMAX; ++i) c[i] = key_lt(key, a[i]);
 #pragma unroll
         for (int i = KMAX - 1; i > 0; --i) a[i] = c[i - 1] ? a[i - 1] : (c[i] ? key : a[i]);
         a[0] = c[0] ? key : a[0];
@@ -115,7 +129,7 @@ struct RegTopK {
 // analogue of the paper's per-thread heaps merged at the end.
 __device__ __forceinline__ key_t warp_insert(key_t mine, key_t key, int lane) {
     key_t up = __shfl_up_sync(0xffffffffu, mine, 1);
-    if (key < mine) mine = (lane > 0 && key < up) ? up : key;
+    if (key_lt(key, mine)) mine = (lane > 0 && key_lt(key, up)) ? up : key;
     return mine;
 }
 
