@@ -206,23 +206,17 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
             float sc[32];
 #pragma unroll
             for (int j = 0; j < 32; ++j) sc[j] = __uint_as_float(v[j]);
-            float t[16];
-#pragma unroll
-            for (int j = 0; j < 16; ++j) t[j] = fminf(sc[j], sc[j + 16]);
-#pragma unroll
-            for (int w = 8; w > 0; w >>= 1)
-#pragma unroll
-                for (int j = 0; j < w; ++j) t[j] = fminf(t[j], t[j + w]);
+            const float mn = min_tree<32>(sc);  // 16 three-input FMNMX3 (was 31 FMNMX)
             // the lowest column holding a new best; a warp-uniform branch (the
             // compiler otherwise if-converts the 32-step search and runs it for
             // every block: ncu, 35% of the C5 pass's instructions)
-            const bool better = t[0] < best;
+            const bool better = mn < best;
             if (__any_sync(0xffffffffu, better)) {
                 if (better) {
                     int jm = 31;
 #pragma unroll
-                    for (int j = 31; j >= 0; --j) jm = (sc[j] == t[0]) ? j : jm;
-                    best = t[0];
+                    for (int j = 31; j >= 0; --j) jm = (sc[j] == mn) ? j : jm;
+                    best = mn;
                     bi = c * kTcN + col + jm;
                 }
             }

@@ -630,14 +630,7 @@ __global__ void __launch_bounds__(kExThreads, dense_exact_min_blocks(KMAX)) k_de
                         for (int j = 0; j < 16; ++j)
                             if (col + j >= nb) tt[j] = INF;
                     }
-                    float mn[8];
-#pragma unroll
-                    for (int j = 0; j < 8; ++j) mn[j] = fminf(tt[j], tt[j + 8]);
-#pragma unroll
-                    for (int w2 = 4; w2 > 0; w2 >>= 1)
-#pragma unroll
-                        for (int j = 0; j < w2; ++j) mn[j] = fminf(mn[j], mn[j + w2]);
-                    if (active && mn[0] <= thr) {
+                    if (active && min_tree<16>(tt) <= thr) {  // 8 FMNMX3 (was 15 FMNMX)
                         unsigned m = 0;
 #pragma unroll
                         for (int j = 0; j < 16; ++j) m |= (tt[j] <= thr ? 1u : 0u) << j;

@@ -533,7 +533,7 @@ __device__ __forceinline__ void union_tile(const ScanArgs& a, const int4 tl, key
                 // last member, so the minimum is still a real distance of the block)
                 float mn = dd[0];
 #pragma unroll
-                for (int u = 1; u < U; ++u) mn = fminf(mn, dd[u]);
+                for (int u = 1; u < U; u += 2) mn = (u + 1 < U) ? fmin3(mn, dd[u], dd[u + 1]) : fminf(mn, dd[u]);
                 if (active && mn <= kth_d2)
 #endif
                 {

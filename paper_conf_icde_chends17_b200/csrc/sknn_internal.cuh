@@ -97,6 +97,34 @@ __device__ __forceinline__ bool ti_keep(float lb, float theta, float mag, float 
     return lb <= theta + eta * (mag + theta);
 }
 
+// ------------------------------------------------------------ min trees --
+// sm_100 has a three-input float minimum (FMNMX3): a min over N values takes
+// about N/2 instructions instead of N - 1. min is exact and order-free, so
+// the result is the same value as any fminf chain (no NaNs reach these).
+__device__ __forceinline__ float fmin3(float a, float b, float c) {
+    float r;
+    asm("min.f32 %0, %1, %2, %3;" : "=f"(r) : "f"(a), "f"(b), "f"(c));
+    return r;
+}
+template <int N>
+__device__ __forceinline__ float min_tree(const float (&v)[N]) {
+    static_assert(N == 16 || N == 32, "min_tree: 16 or 32 values");
+    if constexpr (N == 32) {
+        float t[11];
+#pragma unroll
+        for (int j = 0; j < 10; ++j) t[j] = fmin3(v[3 * j], v[3 * j + 1], v[3 * j + 2]);
+        t[10] = fminf(v[30], v[31]);
+        const float u0 = fmin3(t[0], t[1], t[2]), u1 = fmin3(t[3], t[4], t[5]), u2 = fmin3(t[6], t[7], t[8]);
+        return fmin3(u0, u1, fmin3(u2, t[9], t[10]));
+    } else {
+        float t[6];
+#pragma unroll
+        for (int j = 0; j < 5; ++j) t[j] = fmin3(v[3 * j], v[3 * j + 1], v[3 * j + 2]);
+        t[5] = v[15];
+        return fmin3(fmin3(t[0], t[1], t[2]), fmin3(t[3], t[4], t[5]), t[5]);
+    }
+}
+
 // ---------------------------------------------------- register top-k -----
 // Sorted ascending array of KMAX keys held in registers (Fig. 8 / P:L629:
 // k*4 bytes <= th2 puts kNearests in registers). Slots [0, KMAX-k) hold the
