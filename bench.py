@@ -246,7 +246,8 @@ def roofline_of(st, stage, peaks, nq_r, nt, d, k, ws):
     scan (S9-S10): bytes = query rows once + target rows as the method's reuse
     unit fetches them (rows_loaded: once per warp tile and member for the
     warp-union walk; once per query tile and member for the warp-per-query
-    scan) + result rows + center row and bound inputs per (tile, candidate);
+    scan) + result rows + the bound inputs per (tile, candidate) + the center
+    row per (tile, candidate that passes the bound test);
     flops = 3d per evaluated distance and per candidate-center distance +
     log2 |tc| per (query, candidate) window search. Binding = larger fraction.
     dense (S11): tensor flops = 2 KP per (query, target) pair covered by a
@@ -268,7 +269,12 @@ def roofline_of(st, stage, peaks, nq_r, nt, d, k, ws):
             # coinciding: a lower bound of their union)
             Rl /= tile
             note = "warp-per-query scan: target rows counted once per 8-query tile (rows_loaded / 8)"
-        bytes_alg = 4.0 * dpad * nq_r + (4.0 * dpad + 4.0) * Rl + 8.0 * k * nq_r + (4.0 * dpad + 16.0) * P / tile
+        # per (tile, candidate): the 16-byte cluster summary and the 4-byte center
+        # distance D (every candidate is bound-tested); the center row only for
+        # the candidates that pass that test (center_evals, counted per query,
+        # shared by a tile's queries: C / tile)
+        bytes_alg = (4.0 * dpad * nq_r + (4.0 * dpad + 4.0) * Rl + 8.0 * k * nq_r + 20.0 * P / tile +
+                     4.0 * dpad * C / tile)
         flops = 3.0 * d * (E + C) + P * float(np.log2(max(2.0, nt / max(1, st["mt"]))))
         gbs = bytes_alg / (scan_ms / 1e3) / 1e9
         tfs = flops / (scan_ms / 1e3) / 1e12
