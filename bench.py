@@ -343,6 +343,8 @@ def main():
     ap.add_argument("--exchange", default="all_to_all", choices=["all_to_all", "all_gather"])
     ap.add_argument("--global-ub", action="store_true",
                     help="target mode: prune every shard with the global level-1 bound (all-reduce MIN)")
+    ap.add_argument("--prune-exchange", action="store_true",
+                    help="target mode, all_to_all: send only entries at or below the min-over-ranks k-th distance")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -415,9 +417,11 @@ def main():
                 local_join()
             else:
                 sdist.join_target_sharded(Q, Tshard, k, tlo, group=group, exchange=args.exchange, gather=False,
-                                          global_ub=args.global_ub, **opts)
-        parallelism = "target-sharded x%d (%s exchange of partial k-lists + exact merge%s)" % (
-            ws, args.exchange if ws > 1 else "no", ", global level-1 bound" if args.global_ub else "")
+                                          global_ub=args.global_ub,
+                                          prune=args.prune_exchange and args.exchange == "all_to_all", **opts)
+        parallelism = "target-sharded x%d (%s exchange of partial k-lists + exact merge%s%s)" % (
+            ws, args.exchange if ws > 1 else "no", ", global level-1 bound" if args.global_ub else "",
+            ", pruned by the min-over-ranks k-th" if args.prune_exchange else "")
         nq_rank = nq
 
     for _ in range(args.warmup):
@@ -551,7 +555,8 @@ def measure_e2e(args, sknn, sdist, Qh, Th, k, self_join, ws, rank, dev, opts):
             if ws == 1:
                 ri, rd = sknn.join(dQ, dT, k, stream=stream, **opts)
             else:
-                ri, rd = sdist.join_target_sharded(dQ, dT, k, tlo, exchange=args.exchange, gather=False, **opts)
+                ri, rd = sdist.join_target_sharded(dQ, dT, k, tlo, exchange=args.exchange, gather=False,
+                                                   prune=args.prune_exchange and args.exchange == "all_to_all", **opts)
             oi.copy_(ri, non_blocking=True)
             od.copy_(rd, non_blocking=True)
             torch.cuda.synchronize()

@@ -170,15 +170,57 @@ def target_shard_partials_global_ub(Q, T_shard, k: int, shard_offset: int, *, gr
     return join_indexed(qix, tix, k, out_squared=1, index_base=int(shard_offset), ub_in=ub, **opts)[:2]
 
 
+def _exchange_pruned(pidx, pd2, k, splits, rank, world, group):
+    """all_to_all of the partial lists with every entry above the query's
+    minimum over ranks of the local k-th squared distance dropped (NEXT-1).
+    Exact: the rank holding that minimum has k entries at or below it, so an
+    entry strictly above it is never among the k smallest keys; entries equal
+    to it are kept (ties are decided by the index in the merge). Returns the
+    receiver's [world, mine, k] lists padded with (+inf, -1), the merge's input."""
+    dev = pd2.device
+    nq = pd2.shape[0]
+    kth = pd2[:, k - 1].contiguous()  # sorted lists: the local k-th (+inf when short)
+    dist.all_reduce(kth, op=dist.ReduceOp.MIN, group=group)
+    keep = pd2 <= kth[:, None]
+    counts = keep.sum(1, dtype=torch.int32)
+    lo, hi = splits[rank]
+    mine = hi - lo
+    # per-query survivor counts of my rows from every rank (fixed sizes)
+    rcounts = torch.empty((world, mine), dtype=torch.int32, device=dev)
+    dist.all_to_all_single(rcounts.view(-1), counts, [mine] * world, [h - l for l, h in splits], group=group)
+    send_tot = [int(counts[l:h].sum()) for l, h in splits]
+    recv_tot = [int(x) for x in rcounts.sum(1).tolist()]
+    # survivors in row-major order, so each destination's block is contiguous
+    vals_d = pd2[keep].contiguous()
+    vals_i = pidx[keep].contiguous()
+    got_d = torch.empty(sum(recv_tot), dtype=torch.float32, device=dev)
+    got_i = torch.empty(sum(recv_tot), dtype=torch.int32, device=dev)
+    dist.all_to_all_single(got_d, vals_d, recv_tot, send_tot, group=group)
+    dist.all_to_all_single(got_i, vals_i, recv_tot, send_tot, group=group)
+    out_d = torch.full((world, mine, k), float("inf"), dtype=torch.float32, device=dev)
+    out_i = torch.full((world, mine, k), -1, dtype=torch.int32, device=dev)
+    if mine > 0:
+        c = rcounts.view(-1).to(torch.int64)                       # [world * mine] row lengths
+        row = torch.repeat_interleave(torch.arange(world * mine, device=dev), c)
+        start = torch.cumsum(c, 0) - c
+        col = torch.arange(row.numel(), device=dev) - start[row]
+        out_d.view(world * mine, k)[row, col] = got_d
+        out_i.view(world * mine, k)[row, col] = got_i
+    return out_i, out_d, int(sum(send_tot))
+
+
 def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, local_join=None, merge=None,
                         out_squared: bool = False, exchange: str = "all_gather", gather: bool = True,
-                        global_ub: bool = False, **opts):
+                        global_ub: bool = False, prune: bool = False, stats: dict | None = None, **opts):
     """Target-sharded join: local partial lists of every query against this
     rank's T_shard (global indices), exchanged and merged exactly.
     exchange="all_gather": every rank merges all nq rows (returns the full
     result). exchange="all_to_all": rank r merges only its rows
     shard_bounds(nq, P, r); gather=False returns that slice, gather=True the
-    full result assembled by one all-gather of the merged slices."""
+    full result assembled by one all-gather of the merged slices.
+    prune=True (all_to_all only, NEXT-1): one all-reduce MIN of the per-query
+    local k-th distances first, then only the entries at or below it travel
+    (variable-size all_to_all); `stats` (a dict) receives the entry counts."""
     world, rank = _world(group)
     local_join = local_join or _cuda_join
     merge = merge or _cuda_merge
@@ -209,10 +251,15 @@ def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, lo
     send = [(hi - lo) * k for lo, hi in splits]
     lo, hi = splits[rank]
     mine = hi - lo
-    recv_i = torch.empty((world, mine, k), dtype=torch.int32, device=Q.device)
-    recv_d = torch.empty((world, mine, k), dtype=torch.float32, device=Q.device)
-    dist.all_to_all_single(recv_i.view(-1), pidx.contiguous().view(-1), [mine * k] * world, send, group=group)
-    dist.all_to_all_single(recv_d.view(-1), pd2.contiguous().view(-1), [mine * k] * world, send, group=group)
+    if prune:
+        recv_i, recv_d, sent = _exchange_pruned(pidx, pd2, k, splits, rank, world, group)
+        if stats is not None:
+            stats.update(entries_sent=sent, entries_unpruned=nq * k)
+    else:
+        recv_i = torch.empty((world, mine, k), dtype=torch.int32, device=Q.device)
+        recv_d = torch.empty((world, mine, k), dtype=torch.float32, device=Q.device)
+        dist.all_to_all_single(recv_i.view(-1), pidx.contiguous().view(-1), [mine * k] * world, send, group=group)
+        dist.all_to_all_single(recv_d.view(-1), pd2.contiguous().view(-1), [mine * k] * world, send, group=group)
     if mine > 0:
         ri, rd = merge(recv_i, recv_d, k, out_squared=out_squared)
     else:

@@ -74,6 +74,11 @@ def _worker(rank, world, port, results):
         si_, sd_ = sdist.join_target_sharded(torch.from_numpy(Q2), torch.from_numpy(X[lo:hi]).contiguous(), k, lo,
                                              local_join=oracle_local_join, merge=host_merge, exchange="all_to_all",
                                              gather=False)
+        # all-to-all with the exchange pruned by the min-over-ranks k-th distance (NEXT-1)
+        pst = {}
+        pi_, pd_ = sdist.join_target_sharded(torch.from_numpy(Q2), torch.from_numpy(X[lo:hi]).contiguous(), k, lo,
+                                             local_join=oracle_local_join, merge=host_merge, exchange="all_to_all",
+                                             prune=True, stats=pst)
         # query sharding, non-self join: interleaved query clusters (default) and contiguous rows
         qi, qd = sdist.join_query_sharded(torch.from_numpy(Q), torch.from_numpy(X), k, self_join=False,
                                           local_join=oracle_local_join)
@@ -83,7 +88,8 @@ def _worker(rank, world, port, results):
         Xt = torch.from_numpy(X)
         si, sd = sdist.join_query_sharded(Xt, Xt, k, local_join=oracle_local_join)
         results[rank] = (i.numpy(), d.numpy(), qi.numpy(), qd.numpy(), si.numpy(), sd.numpy(),
-                         ai.numpy(), ad.numpy(), si_.numpy(), sd_.numpy(), wi.numpy(), wd.numpy())
+                         ai.numpy(), ad.numpy(), si_.numpy(), sd_.numpy(), wi.numpy(), wd.numpy(),
+                         pi_.numpy(), pd_.numpy(), pst["entries_sent"], pst["entries_unpruned"])
     finally:
         dist.destroy_process_group()
 
@@ -114,7 +120,10 @@ def test_two_rank_gloo_matches_single_join():
     aidx, adist = oracle.knn_join(Q2, X, k)
     from paper_conf_icde_chends17_b200.dist import shard_bounds
     for r in range(world):
-        i, d, qi, qd, si, sd, ai, ad, ri, rd, wi, wd = results[r]
+        i, d, qi, qd, si, sd, ai, ad, ri, rd, wi, wd, pi_, pd_, sent, unpruned = results[r]
+        np.testing.assert_array_equal(pi_, aidx)     # pruned all-to-all exchange, assembled: exact
+        np.testing.assert_array_equal(pd_, adist)
+        assert sent < unpruned                        # entries above the min k-th never travel
         np.testing.assert_array_equal(wi, ridx)      # query-sharded by row slices, assembled
         np.testing.assert_array_equal(wd, rdist)
         np.testing.assert_array_equal(ai, aidx)      # all-to-all exchange, assembled
