@@ -83,7 +83,11 @@ enum {
     SKNN_PATH_AUTO = 0,   /* adaptive scheme (Fig. 8 re-derived for B200)                 */
     SKNN_PATH_SPARSE = 1, /* TI filters + point-level scan only (Alg. 1 + Alg. 2)          */
     SKNN_PATH_DENSE = 2,  /* TI filters; every surviving cluster pair on the dense tile path */
-    SKNN_PATH_BRUTE = 3,  /* no filtering: every query against every target (the anchor)    */
+    SKNN_PATH_BRUTE = 3,  /* no filtering: every query against every target (the anchor and */
+                          /* the dense-only path): register-tiled SIMT contraction with a    */
+                          /* fused top-k, k <= 32; auto takes it at dp >= 1024 for sknn_join */
+                          /* and sknn_query (the index's permuted rows), where the TI filters */
+                          /* keep most pairs (Table IV arcene / dorothea)         */
     SKNN_PATH_PARTIAL = 4 /* TI filters; PARTIAL level-2 filter (§IV-B1): theta   */
                           /* fixed at the level-1 UB, every window member's distance stored  */
                           /* in a global survivor buffer, then a k-selection kernel; k <= 512 */

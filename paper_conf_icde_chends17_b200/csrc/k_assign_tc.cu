@@ -198,14 +198,15 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_assign_tc(const float* __rest
         // per 32 columns: the scores (straight from TMEM), their minimum by a
         // min tree (one FMNMX per score) and, only when it beats the running
         // best, the lowest column holding it (a strict running argmin)
-#pragma unroll 1
+        uint32_t v2[2][32];  // both 32-column blocks of this half, one TMEM round trip
+        tc::tmem_ld32x2(trow + (uint32_t)(buf * kTcN + half * 64), trow + (uint32_t)(buf * kTcN + half * 64 + 32),
+                        v2[0], v2[1]);
+#pragma unroll
         for (int cb = 0; cb < 2; ++cb) {
             const int col = half * 64 + cb * 32;
-            uint32_t v[32];
-            tc::tmem_ld32(trow + (uint32_t)(buf * kTcN + col), v);
             float sc[32];
 #pragma unroll
-            for (int j = 0; j < 32; ++j) sc[j] = __uint_as_float(v[j]);
+            for (int j = 0; j < 32; ++j) sc[j] = __uint_as_float(v2[cb][j]);
             const float mn = min_tree<32>(sc);  // 16 three-input FMNMX3 (was 31 FMNMX)
             // the lowest column holding a new best; a warp-uniform branch (the
             // compiler otherwise if-converts the 32-step search and runs it for
