@@ -465,9 +465,13 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
     Counters* counters = nullptr;
     Ctx cq;  // forked query-side build (Q != T joins)
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    // Q != T join with a forked query-side build: Q is staged on the forked
+    // stream after T's copy, so (host buffers) its host->device copy overlaps
+    // the target-side build instead of preceding it
+    const bool fork_q = !index && !self && !qindex && path != SKNN_PATH_BRUTE;
     do {
         const void* tmp;
-        if (!qindex) {
+        if (!qindex && !fork_q) {
             if ((st = stage_in(cx, Q, sizeof(float) * nq * d, &tmp, &q_host)) != SKNN_OK) break;
             dQ = (const float*)tmp;
         }
@@ -525,7 +529,6 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
         // stream concurrently with the target side (both are chains of mostly
         // small, latency-bound kernels; the joins and frees stay stream-ordered,
         // and a graph capture follows the fork/join events)
-        const bool fork_q = !index && !self && !qindex;
         if (fork_q) {
             cq.stream = side_stream(di.device);
             cq.device = cx.device;
@@ -537,6 +540,8 @@ static sknn_status run_join(const float* Q, int64_t nq, const float* T, int64_t 
                 st = fail(SKNN_ERR_CUDA, "fork of the query-side build failed");
                 break;
             }
+            if ((st = stage_in(cq, Q, sizeof(float) * nq * d, &tmp, &q_host)) != SKNN_OK) break;
+            dQ = (const float*)tmp;
             int m = det_lm_num(nq, o.n_clusters_q);
             NvtxRange r("sknn build query side (forked stream)");
             if ((st = build_side(cq, dQ, nq, d, m, o.landmark_trials, o.lloyd_iters, o.seed ^ 0x51ull, qs_local)) !=
