@@ -340,7 +340,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C2")
     ap.add_argument("--mode", default="query", choices=["query", "target"])
-    ap.add_argument("--exchange", default="all_to_all", choices=["all_to_all", "all_gather"])
+    ap.add_argument("--exchange", default="all_to_all", choices=["all_to_all", "all_gather", "peer"])
     ap.add_argument("--global-ub", action="store_true",
                     help="target mode: prune every shard with the global level-1 bound (all-reduce MIN)")
     ap.add_argument("--prune-exchange", action="store_true",

@@ -262,6 +262,21 @@ sknn_status sknn_merge_partials(const int32_t* part_idx, const float* part_d2,
                                 int32_t* out_idx, float* out_dist,
                                 int32_t out_squared, sknn_stream_t stream);
 
+/* The same merge reading the P lists from P separate buffers -- the fused
+ * peer-memory merge of the target-sharded mode (NEXT-1): rank r passes the
+ * device addresses of every rank's [nq_total x k] partial lists as mapped
+ * into its own address space (symmetric memory / CUDA IPC over NVLink; local
+ * buffers work the same) and merges its rows [row_lo, row_lo + nrows) into
+ * out_idx / out_dist [nrows x k], the remote lists read directly by the merge
+ * kernel -- no exchange collective. part_idx / part_d2 are HOST arrays of P
+ * pointers (1 <= P <= 16); the pointers are not classified (peer addresses
+ * belong to other devices); k <= 32. The caller orders the peers' writes
+ * before this call (e.g. a symmetric-memory barrier on `stream`). */
+sknn_status sknn_merge_partials_ptrs(const int32_t* const* part_idx, const float* const* part_d2,
+                                     int32_t P, int64_t nq_total, int64_t row_lo, int64_t nrows,
+                                     int32_t k, int32_t* out_idx, float* out_dist,
+                                     int32_t out_squared, sknn_stream_t stream);
+
 /* Free an index (after all queries using it completed). NULL is a no-op. */
 sknn_status sknn_index_free(sknn_index* index);
 

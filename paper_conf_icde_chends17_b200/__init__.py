@@ -31,7 +31,7 @@ MAX_K = 512
 
 # every symbol include/sknn.h declares (tests check the library exports them)
 ABI_SYMBOLS = ["sknn_options_default", "sknn_join", "sknn_join_ex", "sknn_build", "sknn_query",
-               "sknn_merge_partials", "sknn_index_free", "sknn_index_info", "sknn_index_export",
+               "sknn_merge_partials", "sknn_merge_partials_ptrs", "sknn_index_free", "sknn_index_info", "sknn_index_export",
                "sknn_debug_level1", "sknn_config_decide", "sknn_error_string", "sknn_last_error",
                "sknn_version", "sknn_index_arrays", "sknn_index_create", "sknn_join_indexed",
                "sknn_level1_bounds"]
@@ -115,6 +115,8 @@ def lib():
             L.sknn_query.argtypes = [_vp, _vp, _i64, _i32, _vp, _vp, ctypes.POINTER(Options),
                                      ctypes.POINTER(Stats), _vp]
             L.sknn_merge_partials.argtypes = [_vp, _vp, _i32, _i64, _i32, _vp, _vp, _i32, _vp]
+            L.sknn_merge_partials_ptrs.argtypes = [ctypes.POINTER(_vp), ctypes.POINTER(_vp), _i32, _i64, _i64, _i64,
+                                                   _i32, _vp, _vp, _i32, _vp]
             L.sknn_index_free.argtypes = [_vp]
             L.sknn_index_info.argtypes = [_vp, ctypes.POINTER(_i64), ctypes.POINTER(_i32), ctypes.POINTER(_i32),
                                           ctypes.POINTER(_i32), ctypes.POINTER(_i32)]
@@ -432,6 +434,29 @@ def merge_partials(part_idx, part_d2, k: int, *, out_squared: bool = False, stre
         _check(lib().sknn_merge_partials(part_idx.data_ptr(), part_d2.data_ptr(), P, nq, k,
                                          idx.data_ptr() if idx is not None else None, dist.data_ptr(),
                                          int(out_squared), _stream_ptr(stream, part_d2.device)))
+    return idx, dist
+
+
+def merge_partials_ptrs(idx_ptrs, d2_ptrs, nq_total: int, row_lo: int, nrows: int, k: int, *,
+                        out_squared: bool = False, stream=None, out=None, device=None):
+    """Merge the rows [row_lo, row_lo + nrows) of P partial-list buffers given
+    as device addresses (sknn_merge_partials_ptrs: e.g. symmetric-memory peer
+    buffers, each [nq_total, k] int32 indices / fp32 squared distances)."""
+    import torch
+    P = len(d2_ptrs)
+    assert len(idx_ptrs) == P
+    dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+    if out is not None:
+        idx, dist = out
+    else:
+        idx = torch.empty((nrows, k), dtype=torch.int32, device=dev)
+        dist = torch.empty((nrows, k), dtype=torch.float32, device=dev)
+    ip = (_vp * P)(*[int(x) for x in idx_ptrs])
+    dp_ = (_vp * P)(*[int(x) for x in d2_ptrs])
+    with _on_device(dev):
+        _check(lib().sknn_merge_partials_ptrs(ip, dp_, P, nq_total, row_lo, nrows, k,
+                                              idx.data_ptr() if idx is not None else None, dist.data_ptr(),
+                                              int(out_squared), _stream_ptr(stream, dev)))
     return idx, dist
 
 

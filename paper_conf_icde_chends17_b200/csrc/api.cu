@@ -1030,6 +1030,28 @@ sknn_status sknn_merge_partials(const int32_t* part_idx, const float* part_d2, i
     return run_merge(cx, part_idx, part_d2, P, nq, k, out_idx, out_dist, out_squared);
 }
 
+sknn_status sknn_merge_partials_ptrs(const int32_t* const* part_idx, const float* const* part_d2, int32_t P,
+                                     int64_t nq_total, int64_t row_lo, int64_t nrows, int32_t k, int32_t* out_idx,
+                                     float* out_dist, int32_t out_squared, sknn_stream_t stream) {
+    if (!part_idx || !part_d2 || !out_dist) return fail(SKNN_ERR_INVALID_ARG, "NULL pointer");
+    if (P <= 0 || P > kMaxPeerLists) return fail(SKNN_ERR_INVALID_ARG, "P must be in [1, 16]");
+    if (k <= 0 || nq_total < 0 || row_lo < 0 || nrows < 0 || row_lo + nrows > nq_total)
+        return fail(SKNN_ERR_INVALID_ARG, "bad k or row range");
+    if (k > 32) return fail(SKNN_ERR_UNSUPPORTED, "the peer-list merge keeps k <= 32");
+    for (int p = 0; p < P; ++p)
+        if (!part_idx[p] || !part_d2[p]) return fail(SKNN_ERR_INVALID_ARG, "NULL list pointer");
+    if (nrows == 0) return SKNN_OK;
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    if (classify(out_dist, di.device) != PTR_DEVICE || (out_idx && classify(out_idx, di.device) != PTR_DEVICE))
+        return fail(SKNN_ERR_NOT_DEVICE_PTR, "outputs must be device memory of the current device");
+    Ctx cx;
+    cx.stream = (cudaStream_t)stream;
+    cx.device = di.device;
+    cx.num_sms = di.num_sms;
+    return run_merge_ptrs(cx, part_idx, part_d2, P, row_lo, nrows, k, out_idx, out_dist, out_squared);
+}
+
 sknn_status sknn_index_free(sknn_index* ix) {
     if (!ix) return SKNN_OK;
     int cur = 0;

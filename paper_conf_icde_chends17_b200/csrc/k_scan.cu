@@ -1157,6 +1157,69 @@ __global__ void __launch_bounds__(128) k_merge_tpq_staged(const int32_t* __restr
     }
 }
 
+// Peer-buffer form (sknn_merge_partials_ptrs): list p of query row q at
+// d2[p] + q k -- each rank's buffer, read where it lives (over NVLink for a
+// peer's), by the thread that merges the query. Thread per query, k <= 32.
+struct PeerLists {
+    const int32_t* idx[kMaxPeerLists];
+    const float* d2[kMaxPeerLists];
+};
+
+template <int K>
+__global__ void __launch_bounds__(128) k_merge_tpq_ptrs(PeerLists L, int P, int64_t row_lo, int64_t nrows, int k,
+                                                        int32_t* __restrict__ out_idx, float* __restrict__ out_dist,
+                                                        int out_squared, int vec) {
+    for (int64_t qi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; qi < nrows; qi += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t row = (row_lo + qi) * k;
+        key_t A[K], B[K];
+        tmerge_load<K>(A, L.idx[0], L.d2[0], row, k, vec);
+        for (int p = 1; p < P; ++p) {
+            tmerge_load<K>(B, L.idx[p], L.d2[p], row, k, vec);
+#pragma unroll
+            for (int j = 0; j < K; ++j)
+                A[j] = __longlong_as_double(B[K - 1 - j]) < __longlong_as_double(A[j]) ? B[K - 1 - j] : A[j];
+#pragma unroll
+            for (int h = K / 2; h >= 1; h >>= 1)
+#pragma unroll
+                for (int j = 0; j < K; ++j)
+                    if ((j & h) == 0) {
+                        key_t lo, hi;
+                        cex(A[j], A[j + h], lo, hi);
+                        A[j] = lo;
+                        A[j + h] = hi;
+                    }
+        }
+#pragma unroll
+        for (int j = 0; j < K; ++j)
+            if (j < k) {
+                const float d2 = key_d2(A[j]);
+                out_dist[qi * k + j] = out_squared ? d2 : __fsqrt_rn(d2);
+                if (out_idx) out_idx[qi * k + j] = key_idx(A[j]);
+            }
+    }
+}
+
+sknn_status run_merge_ptrs(Ctx& cx, const int32_t* const* part_idx, const float* const* part_d2, int P,
+                           int64_t row_lo, int64_t nrows, int k, int32_t* out_idx, float* out_dist, int out_squared) {
+    PeerLists L{};
+    bool vec = (k % 4) == 0;
+    for (int p = 0; p < P; ++p) {
+        L.idx[p] = part_idx[p];
+        L.d2[p] = part_d2[p];
+        vec = vec && ((uintptr_t)part_idx[p] % 16) == 0 && ((uintptr_t)part_d2[p] % 16) == 0;
+    }
+    const int64_t blocks = (nrows + 127) / 128;
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)cx.num_sms * 8));
+#define SKNN_PMERGE(K) \
+    k_merge_tpq_ptrs<K><<<grid, 128, 0, cx.stream>>>(L, P, row_lo, nrows, k, out_idx, out_dist, out_squared, vec ? 1 : 0)
+    if (k <= 8) SKNN_PMERGE(8);
+    else if (k <= 16) SKNN_PMERGE(16);
+    else SKNN_PMERGE(32);
+#undef SKNN_PMERGE
+    cx.launched();
+    return cx.check_launch("merge (peer lists)");
+}
+
 sknn_status run_merge(Ctx& cx, const int32_t* part_idx, const float* part_d2, int P, int64_t nq, int k,
                       int32_t* out_idx, float* out_dist, int out_squared) {
     const char* env = getenv("SKNN_MERGE");  // study knob for k <= 32: "warp" | "direct" | "staged"

@@ -208,5 +208,9 @@ sknn_status run_brute_tiled(Ctx& cx, const float* Q, int64_t nq, int ldq, const 
 constexpr int kDenseOnlyDp = 1024;
 sknn_status run_merge(Ctx& cx, const int32_t* part_idx, const float* part_d2, int P, int64_t nq, int k,
                       int32_t* out_idx, float* out_dist, int out_squared);
+// merge of P lists in separate (possibly peer) buffers, rows [row_lo, row_lo + nrows)
+constexpr int kMaxPeerLists = 16;
+sknn_status run_merge_ptrs(Ctx& cx, const int32_t* const* part_idx, const float* const* part_d2, int P,
+                           int64_t row_lo, int64_t nrows, int k, int32_t* out_idx, float* out_dist, int out_squared);
 
 }  // namespace sknn

@@ -37,6 +37,7 @@ import torch.distributed as dist
 
 from . import join as _cuda_join
 from . import merge_partials as _cuda_merge
+from . import merge_partials_ptrs as _cuda_merge_ptrs
 
 
 def shard_bounds(n: int, world: int, rank: int):
@@ -209,6 +210,43 @@ def _exchange_pruned(pidx, pd2, k, splits, rank, world, group):
     return out_i, out_d, int(sum(send_tot))
 
 
+def _exchange_peer(Q, T_shard, k, shard_offset, group, world, rank, local_join, out_squared, gather, opts):
+    """exchange="peer" (NEXT-1, the fused peer-memory merge): every rank's
+    partial lists are written straight into symmetric-memory buffers (torch
+    symmetric memory over NVLink), one device-side barrier orders the writes,
+    and rank r's merge kernel reads its rows [r nq/P, (r+1) nq/P) of all P
+    buffers in place (sknn_merge_partials_ptrs) -- no exchange collective, the
+    transfer overlapped with the merge arithmetic thread by thread."""
+    import torch.distributed._symmetric_memory as symm_mem
+    nq = Q.shape[0]
+    pg = group if group is not None else dist.group.WORLD
+    bi = symm_mem.empty((nq, k), dtype=torch.int32, device=Q.device)
+    bd = symm_mem.empty((nq, k), dtype=torch.float32, device=Q.device)
+    local_join(Q, T_shard, k, out=(bi, bd), out_squared=1, index_base=int(shard_offset), **opts)
+    hi_ = symm_mem.rendezvous(bi, pg)
+    hd = symm_mem.rendezvous(bd, pg)
+    hd.barrier(channel=0)  # every rank's lists are written
+    splits = [shard_bounds(nq, world, r) for r in range(world)]
+    lo, hi = splits[rank]
+    ri, rd = _cuda_merge_ptrs(hi_.buffer_ptrs, hd.buffer_ptrs, nq, lo, hi - lo, k, out_squared=out_squared,
+                              device=Q.device)
+    hd.barrier(channel=0)  # every rank is done reading before the buffers are released
+    if not gather:
+        return ri, rd
+    cap = max(h - l for l, h in splits)
+    pad_i = torch.full((cap, k), -1, dtype=torch.int32, device=Q.device)
+    pad_d = torch.zeros((cap, k), dtype=torch.float32, device=Q.device)
+    pad_i[:hi - lo] = ri
+    pad_d[:hi - lo] = rd
+    all_i = torch.empty((world * cap, k), dtype=torch.int32, device=Q.device)
+    all_d = torch.empty((world * cap, k), dtype=torch.float32, device=Q.device)
+    dist.all_gather_into_tensor(all_i, pad_i, group=group)
+    dist.all_gather_into_tensor(all_d, pad_d, group=group)
+    out_i = torch.cat([all_i[r * cap:r * cap + (h - l)] for r, (l, h) in enumerate(splits)])
+    out_d = torch.cat([all_d[r * cap:r * cap + (h - l)] for r, (l, h) in enumerate(splits)])
+    return out_i, out_d
+
+
 def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, local_join=None, merge=None,
                         out_squared: bool = False, exchange: str = "all_gather", gather: bool = True,
                         global_ub: bool = False, prune: bool = False, stats: dict | None = None, **opts):
@@ -220,12 +258,16 @@ def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, lo
     full result assembled by one all-gather of the merged slices.
     prune=True (all_to_all only, NEXT-1): one all-reduce MIN of the per-query
     local k-th distances first, then only the entries at or below it travel
-    (variable-size all_to_all); `stats` (a dict) receives the entry counts."""
+    (variable-size all_to_all); `stats` (a dict) receives the entry counts.
+    exchange="peer" (NCCL + NVLink, k <= 32): the lists stay in symmetric
+    memory and each rank's merge kernel reads the peers' buffers directly."""
     world, rank = _world(group)
     local_join = local_join or _cuda_join
     merge = merge or _cuda_merge
     nq = Q.shape[0]
     kk = min(k, T_shard.shape[0])
+    if exchange == "peer" and world > 1 and not global_ub and kk == k:
+        return _exchange_peer(Q, T_shard, k, shard_offset, group, world, rank, local_join, out_squared, gather, opts)
     if global_ub:  # NEXT-1: prune every shard with the global level-1 bound
         pidx, pd2 = target_shard_partials_global_ub(Q, T_shard, kk, shard_offset, group=group, **opts)
     else:
@@ -237,6 +279,8 @@ def join_target_sharded(Q, T_shard, k: int, shard_offset: int, *, group=None, lo
         pd2 = torch.cat([pd2, pad_d], 1)
     if world == 1:  # one shard: its partial list is the result
         return merge(pidx.view(1, nq, k), pd2.view(1, nq, k), k, out_squared=out_squared)
+    if exchange == "peer":  # (world 1, global_ub or a shard smaller than k: the all-to-all path below)
+        exchange = "all_to_all"
     if exchange == "all_gather":
         all_i = torch.empty((world * nq, k), dtype=torch.int32, device=Q.device)
         all_d = torch.empty((world * nq, k), dtype=torch.float32, device=Q.device)

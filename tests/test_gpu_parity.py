@@ -367,8 +367,41 @@ def test_dist_nccl_world1(sknn):
         assert_knn_bitexact(i.cpu().numpy(), d.cpu().numpy(), ridx, rdist)
         i, d = sdist.join_query_sharded(dev(Q), dev(T), k, self_join=False)
         assert_knn_bitexact(i.cpu().numpy(), d.cpu().numpy(), ridx, rdist)
+        # the fused peer-memory merge's path on a world of one: symmetric-memory
+        # buffers, device barrier, merge kernel reading the (here local) buffer
+        try:
+            import torch.distributed._symmetric_memory as symm_mem
+            symm_mem.empty((4,), dtype=torch.float32, device="cuda")
+            peer_ok = True
+        except Exception:
+            peer_ok = False
+        if peer_ok:
+            i, d = sdist._exchange_peer(dev(Q), dev(T), k, 0, None, 1, 0, sknn.join, False, True, {})
+            torch.cuda.synchronize()
+            assert_knn_bitexact(i.cpu().numpy(), d.cpu().numpy(), ridx, rdist)
     finally:
         tdist.destroy_process_group()
+
+
+@pytest.mark.parametrize("P,k,nq,lo,n", [(1, 8, 500, 0, 500), (3, 32, 700, 129, 400), (8, 20, 1000, 999, 1),
+                                         (5, 16, 333, 0, 0), (16, 5, 257, 7, 250)])
+def test_merge_partials_ptrs_equals_stacked(sknn, P, k, nq, lo, n):
+    """sknn_merge_partials_ptrs (the peer-buffer merge of the fused NVLink
+    exchange) over P SEPARATE buffers, rows [lo, lo + n): bit-identical to the
+    stacked-array merge of the same lists (ties across lists included)."""
+    rng = np.random.default_rng(P * 31 + k)
+    d2 = np.sort(rng.integers(0, 40, size=(P, nq, k)).astype(np.float32), axis=2)
+    idx = (np.arange(k)[None, None, :] + np.arange(P)[:, None, None] * 10_000).astype(np.int32) + \
+        np.zeros((P, nq, k), np.int32)
+    bufs_i = [torch.from_numpy(idx[p].copy()).cuda() for p in range(P)]   # separate allocations
+    bufs_d = [torch.from_numpy(d2[p].copy()).cuda() for p in range(P)]
+    ri, rd = sknn.merge_partials(torch.from_numpy(idx).cuda(), torch.from_numpy(d2).cuda(), k)
+    if n == 0:
+        return
+    pi, pd = sknn.merge_partials_ptrs([b.data_ptr() for b in bufs_i], [b.data_ptr() for b in bufs_d], nq, lo, n, k)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(pi.cpu().numpy(), ri[lo:lo + n].cpu().numpy())
+    np.testing.assert_array_equal(pd.cpu().numpy().view(np.uint32), rd[lo:lo + n].cpu().numpy().view(np.uint32))
 
 
 def test_build_is_deterministic(sknn):
