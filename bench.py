@@ -343,6 +343,8 @@ def main():
     ap.add_argument("--exchange", default="all_to_all", choices=["all_to_all", "all_gather", "peer"])
     ap.add_argument("--global-ub", action="store_true",
                     help="target mode: prune every shard with the global level-1 bound (all-reduce MIN)")
+    ap.add_argument("--shard-q-build", action="store_true",
+                    help="target mode with --global-ub: the query clustering's final assignment split over the ranks")
     ap.add_argument("--prune-exchange", action="store_true",
                     help="target mode, all_to_all: send only entries at or below the min-over-ranks k-th distance")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -418,7 +420,8 @@ def main():
             else:
                 sdist.join_target_sharded(Q, Tshard, k, tlo, group=group, exchange=args.exchange, gather=False,
                                           global_ub=args.global_ub,
-                                          prune=args.prune_exchange and args.exchange == "all_to_all", **opts)
+                                          prune=args.prune_exchange and args.exchange == "all_to_all",
+                                          **(dict(opts, shard_q_build=True) if args.shard_q_build else opts))
         parallelism = "target-sharded x%d (%s exchange of partial k-lists + exact merge%s%s)" % (
             ws, args.exchange if ws > 1 else "no", ", global level-1 bound" if args.global_ub else "",
             ", pruned by the min-over-ranks k-th" if args.prune_exchange else "")

@@ -249,6 +249,27 @@ sknn_status sknn_query(const sknn_index* index, const float* Q, int64_t nq,
                        const sknn_options* opt, sknn_stats* stats,
                        sknn_stream_t stream);
 
+/* Sharded clustering of one point set (target-sharded mode: every rank holds
+ * all of Q; NEXT-1 "sharded Q clustering"). sknn_cluster_count: the m that
+ * sknn_build / the functions below use for n points (floor(3 sqrt(n)),
+ * clamped; opt->n_clusters_t overrides). sknn_build_assign_shard runs the
+ * landmark sampler and the Lloyd passes over all of T (deterministic: every
+ * rank computes the same centers) and the FINAL assignment of rows
+ * [row_lo, row_hi) only (row_lo % 8 == 0), writing centers_out [m x dp]
+ * (dp = d rounded up to 4), cid_out[row] and dist_out[row] (exact fp32
+ * member distances) for those rows; device pointers. After the ranks'
+ * rows are gathered, sknn_build_from_assignment turns the complete
+ * assignment into an index -- CSR, member sort, cluster summaries -- equal
+ * to the one sknn_build returns for the same T and options (P:L241,
+ * P:L317-331). Both synchronise `stream`. */
+int32_t sknn_cluster_count(int64_t n, const sknn_options* opt);
+sknn_status sknn_build_assign_shard(const float* T, int64_t nt, int32_t d, const sknn_options* opt,
+                                    int64_t row_lo, int64_t row_hi, float* centers_out,
+                                    int32_t* cid_out, float* dist_out, sknn_stream_t stream);
+sknn_status sknn_build_from_assignment(const float* T, int64_t nt, int32_t d, const sknn_options* opt,
+                                       const float* centers, int32_t m, const int32_t* cid,
+                                       const float* dist, sknn_index** out, sknn_stream_t stream);
+
 /* Merge P partial result lists into one (multi-GPU target-sharded mode;
  * the paper's merge of per-thread sorted heaps, generalised to
  * ranks). part_idx [P x nq x k] int32 global indices, part_d2 [P x nq x k]

@@ -31,7 +31,8 @@ MAX_K = 512
 
 # every symbol include/sknn.h declares (tests check the library exports them)
 ABI_SYMBOLS = ["sknn_options_default", "sknn_join", "sknn_join_ex", "sknn_build", "sknn_query",
-               "sknn_merge_partials", "sknn_merge_partials_ptrs", "sknn_index_free", "sknn_index_info", "sknn_index_export",
+               "sknn_merge_partials", "sknn_merge_partials_ptrs", "sknn_cluster_count", "sknn_build_assign_shard",
+               "sknn_build_from_assignment", "sknn_index_free", "sknn_index_info", "sknn_index_export",
                "sknn_debug_level1", "sknn_config_decide", "sknn_error_string", "sknn_last_error",
                "sknn_version", "sknn_index_arrays", "sknn_index_create", "sknn_join_indexed",
                "sknn_level1_bounds"]
@@ -115,6 +116,12 @@ def lib():
             L.sknn_query.argtypes = [_vp, _vp, _i64, _i32, _vp, _vp, ctypes.POINTER(Options),
                                      ctypes.POINTER(Stats), _vp]
             L.sknn_merge_partials.argtypes = [_vp, _vp, _i32, _i64, _i32, _vp, _vp, _i32, _vp]
+            L.sknn_cluster_count.argtypes = [_i64, ctypes.POINTER(Options)]
+            L.sknn_cluster_count.restype = _i32
+            L.sknn_build_assign_shard.argtypes = [_vp, _i64, _i32, ctypes.POINTER(Options), _i64, _i64, _vp, _vp, _vp,
+                                                  _vp]
+            L.sknn_build_from_assignment.argtypes = [_vp, _i64, _i32, ctypes.POINTER(Options), _vp, _i32, _vp, _vp,
+                                                     ctypes.POINTER(_vp), _vp]
             L.sknn_merge_partials_ptrs.argtypes = [ctypes.POINTER(_vp), ctypes.POINTER(_vp), _i32, _i64, _i64, _i64,
                                                    _i32, _vp, _vp, _i32, _vp]
             L.sknn_index_free.argtypes = [_vp]
@@ -271,6 +278,23 @@ class Index:
             _check(lib().sknn_build(tp, nt, d, ctypes.byref(o), ctypes.byref(self._handle),
                                     _stream_ptr(stream, tdev) if cuda else None))
         self.nt, self.d = nt, d
+
+    @classmethod
+    def from_assignment(cls, T, centers, cid, dist, stream=None, **opts):
+        """The index sknn_build would return, from a given clustering: centers
+        [m, dp] fp32, cid [n] int32, dist [n] fp32 member distances, all CUDA
+        (sknn_build_from_assignment; the sharded build of dist.py)."""
+        tp, nt, d, keep, cuda = _as_points(T)
+        self = cls.__new__(cls)
+        self._keep = keep
+        self._handle = ctypes.c_void_p()
+        o = make_options(**opts)
+        with _on_device(keep.device):
+            _check(lib().sknn_build_from_assignment(tp, nt, d, ctypes.byref(o), centers.data_ptr(), centers.shape[0],
+                                                    cid.data_ptr(), dist.data_ptr(), ctypes.byref(self._handle),
+                                                    _stream_ptr(stream, keep.device)))
+        self.nt, self.d = nt, d
+        return self
 
     @classmethod
     def create(cls, nt: int, d: int, mt: int, **opts):
@@ -458,6 +482,34 @@ def merge_partials_ptrs(idx_ptrs, d2_ptrs, nq_total: int, row_lo: int, nrows: in
                                               idx.data_ptr() if idx is not None else None, dist.data_ptr(),
                                               int(out_squared), _stream_ptr(stream, dev)))
     return idx, dist
+
+
+def cluster_count(n: int, **opts) -> int:
+    """m = the cluster count sknn_build uses for n points (sknn_cluster_count)."""
+    o = make_options(**opts)
+    return int(lib().sknn_cluster_count(n, ctypes.byref(o)))
+
+
+def build_assign_shard(T, row_lo: int, row_hi: int, *, out=None, stream=None, **opts):
+    """Seeding + Lloyd over all of T and the final assignment of rows
+    [row_lo, row_hi) (sknn_build_assign_shard). Returns (centers [m, dp],
+    cid [n], dist [n]); rows outside the range are left as given in `out`
+    (zeros when allocated here)."""
+    import torch
+    tp, nt, d, keep, cuda = _as_points(T)
+    m = cluster_count(nt, **opts)
+    dp = (d + 3) & ~3
+    if out is None:
+        centers = torch.empty((m, dp), dtype=torch.float32, device=keep.device)
+        cid = torch.zeros(nt, dtype=torch.int32, device=keep.device)
+        dist = torch.zeros(nt, dtype=torch.float32, device=keep.device)
+    else:
+        centers, cid, dist = out
+    o = make_options(**opts)
+    with _on_device(keep.device):
+        _check(lib().sknn_build_assign_shard(tp, nt, d, ctypes.byref(o), row_lo, row_hi, centers.data_ptr(),
+                                             cid.data_ptr(), dist.data_ptr(), _stream_ptr(stream, keep.device)))
+    return centers, cid, dist
 
 
 def config_decide(nq: int, nt: int, d: int, k: int, props: dict | None = None, r_factor: float = 0.25) -> dict:

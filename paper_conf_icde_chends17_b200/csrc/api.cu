@@ -764,8 +764,63 @@ sknn_status sknn_join_ex(const float* Q, int64_t nq, const float* T, int64_t nt,
     return run_join_graphed(Q, nq, T, nt, d, k, out_idx, out_dist, opt, stats, (cudaStream_t)stream);
 }
 
+static sknn_status build_index_impl(const float* T, int64_t nt, int32_t d, const sknn_options* opt, sknn_index** out,
+                                    sknn_stream_t stream_, const BuildShard* shard);
+
 sknn_status sknn_build(const float* T, int64_t nt, int32_t d, const sknn_options* opt, sknn_index** out,
                        sknn_stream_t stream_) {
+    return build_index_impl(T, nt, d, opt, out, stream_, nullptr);
+}
+
+int32_t sknn_cluster_count(int64_t n, const sknn_options* opt) {
+    const sknn_options o = merge_options(opt);
+    return n > 0 ? det_lm_num(n, o.n_clusters_t) : 0;
+}
+
+sknn_status sknn_build_from_assignment(const float* T, int64_t nt, int32_t d, const sknn_options* opt,
+                                       const float* centers, int32_t m, const int32_t* cid, const float* dist,
+                                       sknn_index** out, sknn_stream_t stream) {
+    if (!centers || !cid || !dist) return fail(SKNN_ERR_INVALID_ARG, "NULL pointer");
+    if (m != sknn_cluster_count(nt, opt)) return fail(SKNN_ERR_INVALID_ARG, "m differs from sknn_cluster_count");
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    if (classify(centers, di.device) != PTR_DEVICE || classify(cid, di.device) != PTR_DEVICE ||
+        classify(dist, di.device) != PTR_DEVICE)
+        return fail(SKNN_ERR_NOT_DEVICE_PTR, "centers, cid and dist must be device memory");
+    BuildShard sh;
+    sh.mode = 2;
+    sh.centers_in = centers;
+    sh.cid_in = cid;
+    sh.dist_in = dist;
+    return build_index_impl(T, nt, d, opt, out, stream, &sh);
+}
+
+sknn_status sknn_build_assign_shard(const float* T, int64_t nt, int32_t d, const sknn_options* opt, int64_t row_lo,
+                                    int64_t row_hi, float* centers_out, int32_t* cid_out, float* dist_out,
+                                    sknn_stream_t stream) {
+    if (!centers_out || !cid_out || !dist_out) return fail(SKNN_ERR_INVALID_ARG, "NULL pointer");
+    if (row_lo < 0 || row_hi < row_lo || row_hi > nt || (row_lo % 8) != 0)
+        return fail(SKNN_ERR_INVALID_ARG, "rows must satisfy 0 <= row_lo <= row_hi <= nt, row_lo % 8 == 0");
+    DevInfo di;
+    SKNN_TRY(device_info(di));
+    if (classify(centers_out, di.device) != PTR_DEVICE || classify(cid_out, di.device) != PTR_DEVICE ||
+        classify(dist_out, di.device) != PTR_DEVICE)
+        return fail(SKNN_ERR_NOT_DEVICE_PTR, "outputs must be device memory");
+    BuildShard sh;
+    sh.mode = 1;
+    sh.lo = row_lo;
+    sh.hi = row_hi;
+    sh.centers_out = centers_out;
+    sh.cid_out = cid_out;
+    sh.dist_out = dist_out;
+    sknn_index* tmp = nullptr;
+    sknn_status st = build_index_impl(T, nt, d, opt, &tmp, stream, &sh);
+    if (tmp) sknn_index_free(tmp);  // the partial side is not an index
+    return st;
+}
+
+static sknn_status build_index_impl(const float* T, int64_t nt, int32_t d, const sknn_options* opt, sknn_index** out,
+                                    sknn_stream_t stream_, const BuildShard* shard) {
     if (!out) return fail(SKNN_ERR_INVALID_ARG, "out is NULL");
     *out = nullptr;
     if (!T) return fail(SKNN_ERR_INVALID_ARG, "T is NULL");
@@ -790,7 +845,7 @@ sknn_status sknn_build(const float* T, int64_t nt, int32_t d, const sknn_options
         bool th;
         if ((st = stage_in(cx, T, sizeof(float) * nt * d, &dT, &th)) != SKNN_OK) break;
         int m = det_lm_num(nt, o.n_clusters_t);
-        st = build_side(cx, (const float*)dT, nt, d, m, o.landmark_trials, o.lloyd_iters, o.seed, ix->t);
+        st = build_side(cx, (const float*)dT, nt, d, m, o.landmark_trials, o.lloyd_iters, o.seed, ix->t, shard);
     } while (0);
     cx.free_scratch();
     if (st == SKNN_OK) {

@@ -363,7 +363,9 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
                                                      int32_t* __restrict__ cid_out, float* __restrict__ dist_out,
                                                      long long* __restrict__ sums, const double* __restrict__ fx,
                                                      int32_t* __restrict__ counts, int stride, int prev_stride,
-                                                     int nwalk, int32_t* __restrict__ rank_out) {
+                                                     int nwalk, int32_t* __restrict__ rank_out, int64_t base) {
+    // (base: the absolute row of row 0 -- a sharded final pass covers rows
+    // [base, base + n); cid_prev is valid at absolute multiples of prev_stride)
     const int dp = DP > 0 ? DP : dp_rt;
     const int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * stride;  // Lloyd passes subsample
     const unsigned live = __ballot_sync(0xffffffffu, i < n);  // lanes that reach the aggregated atomic
@@ -380,7 +382,7 @@ __global__ void __launch_bounds__(256) k_assign_walk(const float* __restrict__ X
     };
     int best;
     float bd;
-    if (cid_prev && i % prev_stride == 0) {
+    if (cid_prev && (i + base) % prev_stride == 0) {
         best = cid_prev[i];
         bd = dist2(best);
     } else {
@@ -862,8 +864,15 @@ static void launch_assign(Ctx& cx, const float* Xp, int64_t n, int dp, const flo
 }
 
 // Build one clustered side (Step 1). X is a device pointer [n x d].
+__global__ void k_histogram(const int32_t* __restrict__ cid, int64_t n, int32_t* __restrict__ counts) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(counts + cid[i], 1);
+}
+
 sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int trials, int lloyd, uint64_t seed,
-                       Side& out) {
+                       Side& out, const BuildShard* shard) {
+    const int mode = shard ? shard->mode : 0;
+    const bool from_asg = mode == 2;  // the clustering is given: no sampler, no Lloyd, no assignment
     const int dp = (d + 3) & ~3;
     out.n = n; out.d = d; out.dp = dp; out.m = m;
     cudaStream_t s = cx.stream;
@@ -900,8 +909,10 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     // landmark sampler
     int32_t* lidx;
     SKNN_TRY(cx.alloc_scratch((void**)&lidx, sizeof(int32_t) * trials * m0));
-    k_landmark_draw<<<dim3((m0 + 255) / 256, trials), 256, 0, s>>>(n, m0, trials, seed, lidx);
-    cx.launched();
+    if (!from_asg) {
+        k_landmark_draw<<<dim3((m0 + 255) / 256, trials), 256, 0, s>>>(n, m0, trials, seed, lidx);
+        cx.launched();
+    }
     const int nb = (m0 + kLmTile - 1) / kLmTile;
     const int ntile = nb * (nb + 1) / 2;
     double* partial;
@@ -911,10 +922,12 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         SKNN_CUDA(cudaFuncSetAttribute(k_landmark_sums, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lsm));
     // (measured and rejected: one CTA per (trial, 1/16 or 1/64 of the rows)
     // with the whole trial staged in shared memory -- C2 61 / 52 us vs 30 us)
-    k_landmark_sums<<<dim3(ntile, trials), 256, lsm, s>>>(Xp, dp, m0, lidx, nb, partial);
-    cx.launched();
-    k_landmark_pick<<<(m0 * dp + 511) / 512, 512, 0, s>>>(partial, ntile, trials, lidx, m0, Xp, dp, out.centers);
-    cx.launched();
+    if (!from_asg) {
+        k_landmark_sums<<<dim3(ntile, trials), 256, lsm, s>>>(Xp, dp, m0, lidx, nb, partial);
+        cx.launched();
+        k_landmark_pick<<<(m0 * dp + 511) / 512, 512, 0, s>>>(partial, ntile, trials, lidx, m0, Xp, dp, out.centers);
+        cx.launched();
+    }
 
     int32_t* cid;
     float* pdist;
@@ -944,17 +957,25 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     unsigned int* amax;
     SKNN_TRY(cx.alloc_scratch((void**)&fx, sizeof(double) + sizeof(unsigned int)));
     amax = reinterpret_cast<unsigned int*>(fx + 1);
-    if (lloyd > 0) {
+    if (lloyd > 0 && !from_asg) {
         SKNN_CUDA(cudaMemsetAsync(amax, 0, sizeof(unsigned int), s));
         k_absmax<<<(int)std::min<int64_t>((n * dp / 4 + 255) / 256, 148 * 2), 256, 0, s>>>(Xp, n * dp, amax);
         k_fx_scale<<<1, 1, 0, s>>>(amax, n, fx);
         cx.launched();
         cx.launched();
     }
+    const float* Xp_all = Xp;
     int graph_m = -1;
     int32_t* rank_o = nullptr;  // set for the final walk pass only
+    // rows the next assignment pass covers: all, or (mode 1, final pass) [alo, alo + an)
+    int64_t alo = 0, an = n;
     auto assign = [&](const int32_t* prev, int32_t* cid_o, float* dist_o, long long* sums_o, int mc, int stride,
                       int prev_stride) -> sknn_status {
+        const float* Xp = Xp_all + alo * dp;  // (alo is a multiple of every stride: 8)
+        const int64_t n = an;
+        if (prev) prev += alo;
+        if (cid_o) cid_o += alo;
+        if (dist_o) dist_o += alo;
         if (use_tc) return run_assign_tc(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, fx, counts, stride);
         if (!walk || mc <= kNbr) {
             launch_assign(cx, Xp, n, dp, out.centers, mc, cid_o, dist_o, sums_o, fx, counts);
@@ -980,14 +1001,14 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
 #define SKNN_WALK_CASE(D)                                                                                      \
     case D:                                                                                                    \
         k_assign_walk<D><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, mc, nbr, nentry, prev, cid_o, dist_o, sums_o, \
-                                              fx, counts, stride, prev_stride, nwalk, rank_o);                 \
+                                              fx, counts, stride, prev_stride, nwalk, rank_o, alo);                 \
         break;
             SKNN_WALK_CASE(4) SKNN_WALK_CASE(8) SKNN_WALK_CASE(12) SKNN_WALK_CASE(16)
             SKNN_WALK_CASE(20) SKNN_WALK_CASE(24) SKNN_WALK_CASE(28) SKNN_WALK_CASE(32)
 #undef SKNN_WALK_CASE
             default:
                 k_assign_walk<0><<<grid, 256, 0, s>>>(Xp, n, dp, out.centers, mc, nbr, nentry, prev, cid_o, dist_o,
-                                                      sums_o, fx, counts, stride, prev_stride, nwalk, rank_o);
+                                                      sums_o, fx, counts, stride, prev_stride, nwalk, rank_o, alo);
                 break;
         }
         cx.launched();
@@ -1001,7 +1022,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     // large and the warp-per-query scan's tail explode -- measured 25 -> 824 ms)
     const int sstride = dp <= 32 ? (int)std::max<int64_t>(1, std::min<int64_t>(8, n / (64LL * std::max(1, m0)))) : 1;
     int seed_stride = 1;
-    if (m0 < m) {
+    if (m0 < m && !from_asg) {
         SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
         if (sstride > 1) SKNN_CUDA(cudaMemsetAsync(pdist, 0, sizeof(float) * n, s));
         SKNN_TRY(assign(nullptr, cid, pdist, nullptr, m0, sstride, 1));
@@ -1036,7 +1057,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     // centers let a few clusters grow large and the scan's tail suffers)
     const int lstride = dp <= 32 ? (int)std::max<int64_t>(1, std::min<int64_t>(8, n / (64LL * m))) : 1;
     int prev_stride = seed_stride;  // cid entries valid at multiples of it
-    if (lloyd > 0) {
+    if (lloyd > 0 && !from_asg) {
         long long* sums;
         SKNN_TRY(cx.alloc_scratch((void**)&sums, sizeof(long long) * m * dp));
         SKNN_CUDA(cudaMemsetAsync(sums, 0, sizeof(long long) * m * dp, s));
@@ -1050,9 +1071,27 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
         }
     }
     // final assignment with exact member distances + histogram
-    if (lloyd <= 0) SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
-    if (walk) SKNN_TRY(cx.alloc_scratch((void**)&rank_o, sizeof(int32_t) * n));
-    SKNN_TRY(assign(prev, cid, pdist, nullptr, m, 1, prev_stride));
+    if (lloyd <= 0 || from_asg) SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
+    if (from_asg) {  // mode 2: the gathered clustering
+        SKNN_CUDA(cudaMemcpyAsync(out.centers, shard->centers_in, sizeof(float) * m * dp, cudaMemcpyDeviceToDevice, s));
+        SKNN_CUDA(cudaMemcpyAsync(cid, shard->cid_in, sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
+        SKNN_CUDA(cudaMemcpyAsync(pdist, shard->dist_in, sizeof(float) * n, cudaMemcpyDeviceToDevice, s));
+        k_histogram<<<(int)std::min<int64_t>((n + 255) / 256, 148 * 8), 256, 0, s>>>(cid, n, counts);
+        cx.launched();
+    } else if (mode == 1) {  // this rank's rows of the final assignment, then stop
+        alo = shard->lo;
+        an = shard->hi - shard->lo;
+        if (an > 0) SKNN_TRY(assign(prev, cid, pdist, nullptr, m, 1, prev_stride));
+        SKNN_CUDA(cudaMemcpyAsync(shard->centers_out, out.centers, sizeof(float) * m * dp, cudaMemcpyDeviceToDevice, s));
+        if (an > 0) {
+            SKNN_CUDA(cudaMemcpyAsync(shard->cid_out + alo, cid + alo, sizeof(int32_t) * an, cudaMemcpyDeviceToDevice, s));
+            SKNN_CUDA(cudaMemcpyAsync(shard->dist_out + alo, pdist + alo, sizeof(float) * an, cudaMemcpyDeviceToDevice, s));
+        }
+        return cx.check_launch("build_side (assignment shard)");
+    } else {
+        if (walk) SKNN_TRY(cx.alloc_scratch((void**)&rank_o, sizeof(int32_t) * n));
+        SKNN_TRY(assign(prev, cid, pdist, nullptr, m, 1, prev_stride));
+    }
     k_offsets<<<1, 1024, 0, s>>>(counts, m, out.off, cursor);
     cx.launched();
     unsigned long long* keys;

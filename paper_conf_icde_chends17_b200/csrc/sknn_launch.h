@@ -108,8 +108,23 @@ struct Ctx {
 // k_build.cu
 __global__ void k_offsets(const int32_t* __restrict__ counts, int m, int32_t* __restrict__ off,
                           int32_t* __restrict__ cursor);
+// Sharded query-side build (target-sharded mode, NEXT-1). mode 1: seeding +
+// Lloyd as usual (identical on every rank), then the final assignment of rows
+// [lo, hi) only, written to cid_out / dist_out (+ lo) with the centers to
+// centers_out; no CSR. mode 2: no clustering -- the centers and the complete
+// assignment (cid_in / dist_in, gathered from the ranks) become the side.
+struct BuildShard {
+    int mode = 0;
+    int64_t lo = 0, hi = 0;
+    float* centers_out = nullptr;
+    int32_t* cid_out = nullptr;
+    float* dist_out = nullptr;
+    const float* centers_in = nullptr;
+    const int32_t* cid_in = nullptr;
+    const float* dist_in = nullptr;
+};
 sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int trials, int lloyd, uint64_t seed,
-                       Side& out);
+                       Side& out, const BuildShard* shard = nullptr);
 
 // k_assign_tc.cu: nearest-center screen on the tensor cores
 bool assign_tc_supported(int dp);

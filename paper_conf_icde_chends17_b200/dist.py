@@ -151,6 +151,36 @@ def join_query_sharded_index(index, Q, k: int, *, group=None, out=None, **opts):
     return index.query(Q, k, out=out, self_query=1, shard_rank=rank, shard_count=world, **opts)
 
 
+def aligned_bounds(n: int, world: int, rank: int, align: int = 8):
+    """shard_bounds with every interior boundary rounded down to a multiple of
+    `align` (the sharded build's row ranges)."""
+    lo = (shard_bounds(n, world, rank)[0] // align) * align if rank > 0 else 0
+    hi = (shard_bounds(n, world, rank)[1] // align) * align if rank < world - 1 else n
+    return lo, hi
+
+
+def build_index_sharded(X, *, group=None, assign_shard=None, from_assignment=None, **opts):
+    """Cluster a point set every rank holds with the FINAL assignment pass
+    sharded (NEXT-1, SURVEY §8(e) "sharded Q clustering"): each rank runs the
+    landmark sampler and the Lloyd passes (deterministic, identical on every
+    rank, on strided samples for dp <= 32) and assigns only its rows
+    aligned_bounds(n, P, r) to the final centers (sknn_build_assign_shard);
+    one all-reduce SUM per array assembles the assignment (other ranks' rows
+    are zero) and every rank turns it into the same index
+    (sknn_build_from_assignment) -- identical to sknn_build's. The
+    functions may be injected (tests)."""
+    from . import Index, build_assign_shard
+    assign_shard = assign_shard or build_assign_shard
+    from_assignment = from_assignment or (lambda X_, c, i, d, **o: Index.from_assignment(X_, c, i, d, **o))
+    world, rank = _world(group)
+    lo, hi = aligned_bounds(X.shape[0], world, rank)
+    centers, cid, dst = assign_shard(X, lo, hi, **opts)
+    if world > 1:
+        dist.all_reduce(cid, op=dist.ReduceOp.SUM, group=group)
+        dist.all_reduce(dst, op=dist.ReduceOp.SUM, group=group)
+    return from_assignment(X, centers, cid, dst, **opts)
+
+
 def target_shard_partials_global_ub(Q, T_shard, k: int, shard_offset: int, *, group=None, qindex=None, **opts):
     """Partial k-lists of ALL queries against this rank's target shard, pruned
     with the GLOBAL level-1 bound: every rank clusters Q
@@ -162,8 +192,11 @@ def target_shard_partials_global_ub(Q, T_shard, k: int, shard_offset: int, *, gr
     than k real entries (+inf / -1 placeholders); the merged result is exact.
     Returns (idx, d2) with global indices."""
     from . import Index, join_indexed, level1_bounds
-    qix = qindex or Index(Q, **{kk: v for kk, v in opts.items() if kk in ("lloyd_iters", "landmark_trials", "seed",
-                                                                              "n_clusters_t")})
+    bopts = {kk: v for kk, v in opts.items() if kk in ("lloyd_iters", "landmark_trials", "seed", "n_clusters_t")}
+    shard_q = opts.pop("shard_q_build", False)
+    if qindex is None and shard_q:  # every rank clusters Q, the final assignment pass split over the ranks
+        qindex = build_index_sharded(Q, group=group, **bopts)
+    qix = qindex or Index(Q, **bopts)
     tix = Index(T_shard)
     ub = level1_bounds(qix, tix, k)
     if dist.is_initialized() and dist.get_world_size(group) > 1:

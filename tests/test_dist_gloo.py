@@ -79,6 +79,18 @@ def _worker(rank, world, port, results):
         pi_, pd_ = sdist.join_target_sharded(torch.from_numpy(Q2), torch.from_numpy(X[lo:hi]).contiguous(), k, lo,
                                              local_join=oracle_local_join, merge=host_merge, exchange="all_to_all",
                                              prune=True, stats=pst)
+        # sharded clustering (NEXT-1): each rank assigns its aligned rows, one all-reduce
+        # SUM per array assembles the assignment (CPU stand-in for the assignment)
+        def fake_assign(Xs, lo_, hi_, **_):
+            C = Xs[:4].clone()
+            d2 = ((Xs[:, None, :] - C[None]) ** 2).sum(-1)
+            ci = torch.zeros(Xs.shape[0], dtype=torch.int32)
+            di = torch.zeros(Xs.shape[0], dtype=torch.float32)
+            ci[lo_:hi_] = d2.argmin(1).int()[lo_:hi_]
+            di[lo_:hi_] = d2.min(1).values.sqrt()[lo_:hi_]
+            return C, ci, di
+        bi_, bd_ = sdist.build_index_sharded(torch.from_numpy(X), assign_shard=fake_assign,
+                                             from_assignment=lambda X_, c, i_, d_, **o: (i_.clone(), d_.clone()))
         # query sharding, non-self join: interleaved query clusters (default) and contiguous rows
         qi, qd = sdist.join_query_sharded(torch.from_numpy(Q), torch.from_numpy(X), k, self_join=False,
                                           local_join=oracle_local_join)
@@ -89,7 +101,8 @@ def _worker(rank, world, port, results):
         si, sd = sdist.join_query_sharded(Xt, Xt, k, local_join=oracle_local_join)
         results[rank] = (i.numpy(), d.numpy(), qi.numpy(), qd.numpy(), si.numpy(), sd.numpy(),
                          ai.numpy(), ad.numpy(), si_.numpy(), sd_.numpy(), wi.numpy(), wd.numpy(),
-                         pi_.numpy(), pd_.numpy(), pst["entries_sent"], pst["entries_unpruned"])
+                         pi_.numpy(), pd_.numpy(), pst["entries_sent"], pst["entries_unpruned"],
+                         bi_.numpy(), bd_.numpy())
     finally:
         dist.destroy_process_group()
 
@@ -120,7 +133,11 @@ def test_two_rank_gloo_matches_single_join():
     aidx, adist = oracle.knn_join(Q2, X, k)
     from paper_conf_icde_chends17_b200.dist import shard_bounds
     for r in range(world):
-        i, d, qi, qd, si, sd, ai, ad, ri, rd, wi, wd, pi_, pd_, sent, unpruned = results[r]
+        i, d, qi, qd, si, sd, ai, ad, ri, rd, wi, wd, pi_, pd_, sent, unpruned, bi_, bd_ = results[r]
+        Xt_ = torch.from_numpy(X)
+        d2_ = ((Xt_[:, None, :] - Xt_[:4][None]) ** 2).sum(-1)
+        np.testing.assert_array_equal(bi_, d2_.argmin(1).int().numpy())   # sharded assignment, assembled
+        np.testing.assert_array_equal(bd_, d2_.min(1).values.sqrt().numpy())
         np.testing.assert_array_equal(pi_, aidx)     # pruned all-to-all exchange, assembled: exact
         np.testing.assert_array_equal(pd_, adist)
         assert sent < unpruned                        # entries above the min k-th never travel

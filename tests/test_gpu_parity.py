@@ -943,3 +943,34 @@ def test_dense_only_index_query_high_d(sknn):
     i2, d2 = ix.query(Q, k, query_batch=100)
     assert_knn_bitexact(np.asarray(i2), np.asarray(d2), ridx, rdist)
     ix.close()
+
+
+@pytest.mark.parametrize("name,scale,P", [("C5", 0.01, 3), ("C2", 0.05, 4), ("C4", 0.01, 2), ("C1", 1.0, 5)])
+def test_sharded_build_equals_build(sknn, name, scale, P):
+    """Sharded clustering (NEXT-1): P ranks' final-assignment shards
+    (sknn_build_assign_shard on aligned row ranges, simulated one after the
+    other on one GPU), summed as the all-reduce would, then
+    sknn_build_from_assignment: the index is identical to sknn_build's (every
+    exported array), through the tensor-core assignment (C4, C5) and the
+    graph walk (C1, C2), ragged and 8-aligned shard boundaries."""
+    from paper_conf_icde_chends17_b200.dist import aligned_bounds
+    Q, T, k, sj = datagen.workload(name, scale)
+    X = dev(Q)
+    ref = sknn.build(X).export()
+    cid_sum = torch.zeros(X.shape[0], dtype=torch.int32, device="cuda")
+    dist_sum = torch.zeros(X.shape[0], dtype=torch.float32, device="cuda")
+    centers = None
+    for r in range(P):
+        lo, hi = aligned_bounds(X.shape[0], P, r)
+        c, i, d = sknn.build_assign_shard(X, lo, hi)
+        cid_sum += i
+        dist_sum += d
+        if centers is None:
+            centers = c
+        else:
+            assert torch.equal(c, centers)   # every rank computes the same centers
+    ix = sknn.Index.from_assignment(X, centers, cid_sum, dist_sum)
+    got = ix.export()
+    for key in ref:
+        np.testing.assert_array_equal(got[key], ref[key])
+    ix.close()
