@@ -1020,7 +1020,10 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     // C5 build 21.2 -> 17.1 ms for both sides, C3 join 3.94 -> 3.65 ms)
     // (dp <= 32 only: at d = 128 (C4) the sampled seeding let a few clusters grow
     // large and the warp-per-query scan's tail explode -- measured 25 -> 824 ms)
-    const int sstride = dp <= 32 ? (int)std::max<int64_t>(1, std::min<int64_t>(8, n / (64LL * std::max(1, m0)))) : 1;
+    // (study knob SKNN_SUBSAMPLE_HIGHD=1: strided seeding / Lloyd passes also above dp 32)
+    static const bool sub_highd = getenv("SKNN_SUBSAMPLE_HIGHD") != nullptr;
+    const bool subsample = dp <= 32 || sub_highd;
+    const int sstride = subsample ? (int)std::max<int64_t>(1, std::min<int64_t>(8, n / (64LL * std::max(1, m0)))) : 1;
     int seed_stride = 1;
     if (m0 < m && !from_asg) {
         SKNN_CUDA(cudaMemsetAsync(counts, 0, sizeof(int32_t) * m, s));
@@ -1055,7 +1058,7 @@ sknn_status build_side(Ctx& cx, const float* X, int64_t n, int d, int m, int tri
     // the centers only have to be good, not exact (mini-batch k-means)
     // (measured: neutral-to-better for dp <= 32; at d = 128 (C4) the subsampled
     // centers let a few clusters grow large and the scan's tail suffers)
-    const int lstride = dp <= 32 ? (int)std::max<int64_t>(1, std::min<int64_t>(8, n / (64LL * m))) : 1;
+    const int lstride = subsample ? (int)std::max<int64_t>(1, std::min<int64_t>(8, n / (64LL * m))) : 1;
     int prev_stride = seed_stride;  // cid entries valid at multiples of it
     if (lloyd > 0 && !from_asg) {
         long long* sums;
