@@ -314,8 +314,22 @@ static sknn_status query_core(Ctx& cx, const Side& qs, const Side& ts, int k, co
     const bool partial = o.force_path == SKNN_PATH_PARTIAL;
     // the partial filter's passes take 32 queries per warp task (thread per query)
     const int tile = partial ? 32 : scan_tile_size(mapping, ts.dp, k);
+    // Fig. 8: threads per query = nearest power of two of
+    // r * max_cur / |Q| when |Q| < r * max_cur -- applied as the minimum split
+    // of the thread-per-query scan's tiles (several warps per tile of queries)
+    int fig8 = 1;
+    {
+        int dev = 0, sms = 148, mt_sm = 2048;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaDeviceGetAttribute(&mt_sm, cudaDevAttrMaxThreadsPerMultiProcessor, dev);
+        const double rmax = (double)o.r_factor * sms * mt_sm;
+        const int64_t nq_eff = qs.n / std::max(1, shard_count);
+        if (nq_eff > 0 && (double)nq_eff < rmax) fig8 = 1 << (int)lround(log2(rmax / (double)nq_eff));
+    }
     if (!basic)
-        SKNN_TRY(run_tiles(cx, qs, tile, k, scan_resident_warps(cx, mapping, ts.dp, k), shard_rank, shard_count, l1));
+        SKNN_TRY(run_tiles(cx, qs, tile, k, scan_resident_warps(cx, mapping, ts.dp, k), shard_rank, shard_count, l1,
+                           fig8));
     mk.l1 = tm.mark();
     key_t* init_topk = nullptr;
     if (lp.dense_mode != 1) {

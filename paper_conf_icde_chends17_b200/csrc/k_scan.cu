@@ -288,7 +288,8 @@ __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__
                                                      int shard_rank, int shard_count, const int32_t* __restrict__ owner,
                                                      const unsigned long long* __restrict__ work,
                                                      const int32_t* __restrict__ ccount, int slots, int cap_split,
-                                                     int split, int order, int outliers, float wfac, float hfac,
+                                                     int split, int order, int outliers, int min_split,
+                                                     float wfac, float hfac,
                                                      int4* __restrict__ tasks, int* __restrict__ ntasks,
                                                      int4* __restrict__ merges, int* __restrict__ nmerges) {
     __shared__ unsigned long long s_red[33];
@@ -324,10 +325,17 @@ __global__ void __launch_bounds__(1024) k_make_tasks(const int32_t* __restrict__
     const unsigned long long H = (unsigned long long)fmax(per_slot, hfac * mean);
     unsigned long long W0 = (unsigned long long)(per_slot * wfac);
     if (W0 < 64) W0 = 64;
+    // min_split (Fig. 8): with fewer queries than r * max_cur every
+    // tile is split into at least that many candidate-interleaved tasks -- the
+    // paper's "several threads per query", here several warps per query tile
     auto s_of = [&](int u, unsigned long long w0) -> int {
-        if (!split || nt[u] == 0 || wk[u] <= H) return 1;
-        unsigned long long s = (wk[u] + w0 - 1) / w0;
-        s = s < 32 ? (s > 2 ? s : 2) : 32;
+        if (!split || nt[u] == 0) return 1;
+        unsigned long long s = 1;
+        if (wk[u] > H) {
+            s = (wk[u] + w0 - 1) / w0;
+            s = s < 32 ? (s > 2 ? s : 2) : 32;
+        }
+        if (s < (unsigned long long)min_split) s = (unsigned long long)min_split;
         return (int)(s < (unsigned long long)ncc[u] ? s : (unsigned long long)ncc[u]);
     };
     if (split) {
@@ -447,7 +455,7 @@ bool scan_uses_tpq(int mapping, int dp, int k) {
 int scan_tile_size(int mapping, int dp, int k) { return scan_uses_tpq(mapping, dp, k) ? 32 : 8; }
 
 sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int shard_rank, int shard_count,
-                      Level1& l1) {
+                      Level1& l1, int fig8_width) {
     const char* ev = getenv("SKNN_SPLIT");  // ablation: SKNN_SPLIT=0 disables tile splitting
     const bool split = tile == 32 && !(ev && ev[0] == '0');  // thread-per-query scan only
     const char* eo = getenv("SKNN_TASKORDER");  // ablation: SKNN_TASKORDER=0 keeps cluster order
@@ -476,10 +484,16 @@ sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int s
         SKNN_CUDA(cudaMemsetAsync(l1.theta2, 0x7f, sizeof(unsigned) * (size_t)qs.n, cx.stream));
     }
     l1.tile = tile;
+    // Fig. 8 width, only while every tile's split fits the partial-list buffer
+    int min_split = (split && cap > 0) ? std::min(fig8_width, 32) : 1;
+    const char* ef = getenv("SKNN_FIG8");  // ablation: SKNN_FIG8=0 ignores the Fig. 8 width
+    if (ef && ef[0] == '0') min_split = 1;
+    while (min_split > 1 && ((qs.n + tile - 1) / tile + qs.m) * (int64_t)min_split > cap) min_split >>= 1;
     k_make_tasks<<<1, 1024, 0, cx.stream>>>(qs.off, qs.m, tile, shard_rank, shard_count, l1.owner, l1.work,
                                              l1.cand_count,
                                              slots, cap, split && cap > 0 ? 1 : 0, order,
                                              (tile == 8 && order && !scan_uses_bigk(k) && !(eot && eot[0] == '0')) ? 1 : 0,
+                                             min_split,
                                              wfac, hfac, l1.tiles,
                                              l1.ntiles, l1.merges,
                                              l1.nmerges);

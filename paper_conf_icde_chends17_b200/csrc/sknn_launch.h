@@ -188,7 +188,7 @@ sknn_status run_dense(Ctx& cx, const Side& qs, const Side& ts, const Level1& l1,
 // k_scan.cu: tiles of `tile` queries of one query cluster (thread-data remapping)
 // level-2 task list; slots = resident warps of the scan kernel (scan_resident_warps)
 sknn_status run_tiles(Ctx& cx, const Side& qs, int tile, int k, int slots, int shard_rank, int shard_count,
-                      Level1& l1);
+                      Level1& l1, int fig8_width = 1);
 int scan_resident_warps(Ctx& cx, int mapping, int dp, int k);
 int scan_tile_size(int mapping, int dp, int k);
 bool scan_uses_tpq(int mapping, int dp, int k);
